@@ -1,0 +1,97 @@
+"""Pins for oracle/score.py, oracle/sizes.py, oracle/hrcs.py, oracle/scheduler.py."""
+import math
+
+import numpy as np
+import pytest
+
+from oracle import hrcs, scheduler, sizes
+from oracle.score import score, softmax, topk
+
+
+# ----------------------------------------------------------------- score
+def test_softmax_closed_form():
+    s = softmax(np.log([1.0, 2.0, 3.0]))          # exp(z_i) = 1, 2, 3 -> s = i / 6
+    np.testing.assert_allclose(s, [1 / 6, 2 / 6, 3 / 6], rtol=1e-15)
+
+
+def test_softmax_shift_invariance_and_extremes():
+    z = np.array([1000.0, 1000.0, -1000.0])       # max subtraction keeps this finite
+    np.testing.assert_allclose(softmax(z), [0.5, 0.5, 0.0], atol=1e-300)
+
+
+def test_score_uses_identifier_rows():
+    rows = np.array([[1.0, 0.0], [0.0, 2.0], [1.0, 1.0]])
+    hf = np.array([0.5, 0.25])
+    z, s, top = score(rows, hf, k=2)
+    np.testing.assert_allclose(z, [0.5, 0.5, 0.75])
+    assert list(top) == [2, 0]                    # tie between 0 and 1 -> lower index first
+
+
+def test_topk_tie_rule():
+    assert list(topk(np.array([0.2, 0.3, 0.3, 0.2]), 4)) == [1, 2, 0, 3]
+
+
+# ------------------------------------------------------------------ sizes (Table 2)
+@pytest.mark.parametrize("kv,d,L,expected", [(2, 128, 28, 28672), (4, 128, 28, 57344), (8, 64, 16, 32768)])
+def test_table2_bytes_per_token(kv, d, L, expected):
+    assert sizes.kv_bytes_per_token(kv, d, L) == expected
+
+
+def test_kv_size_examples():
+    # a 1000-token Qwen2-1.5B user occupies ~29 MB; 10^8 such users ~2.9 PB
+    user = sizes.prefix_bytes(1000, 2, 128, 28)
+    assert round(user / 1e6) == 29
+    assert round(1e8 * round(user / 1e6) * 1e6 / 1e15, 1) == 2.9
+    # P:273 / P:427: 1M (10M) items x 10 tokens ~ 287 GB (2.87 TB)
+    assert round(sizes.prefix_bytes(10 * 10 ** 6, 2, 128, 28) / 1e9) == 287
+    assert round(sizes.prefix_bytes(10 * 10 ** 7, 2, 128, 28) / 1e12, 2) == 2.87
+    # one 16-token page of all 28 layers: 16 x 28672 B
+    assert sizes.page_bytes(16, 2, 128, 28) == 458752
+
+
+# ---------------------------------------------------------------- HRCS (Algorithm 1)
+def test_rmax_paper_formula_by_hand():
+    # alpha*t = 0.2 s; 0.2 * 100 tok/s * 3 / (10 * 5 * 4) = 0.3
+    assert math.isclose(hrcs.rmax_paper(B=100, t=2, alpha=0.1, c=10, tau_i=5, N=4), 0.3)
+    assert hrcs.rmax_paper(B=100, t=2, alpha=0.1, c=10, tau_i=5, N=1) == 0.0
+
+
+def test_replication_ratio_hand_cases():
+    F = [0.5, 0.3, 0.1, 0.1]
+    assert hrcs.replication_ratio(F, 0.25) == 2 / 4     # CDF .5, .8 >= .75
+    assert hrcs.replication_ratio(F, 1.0) == 1 / 4      # R_max >= 1 -> first item
+    assert hrcs.replication_ratio(F, 5.0) == 1 / 4
+    assert hrcs.replication_ratio(F, 0.0) == 1.0        # nothing may cross the network
+    assert hrcs.replication_ratio([1, 3, 2, 4], 0.35) == 2 / 4   # unnormalised, unsorted input
+
+
+def test_place_round_robin_by_hotness():
+    F = [0.05, 0.4, 0.05, 0.3, 0.1, 0.1]
+    rep, owner = hrcs.place(F, 2 / 6, 2)
+    assert rep == [1, 3]
+    assert owner == {4: 0, 5: 1, 0: 0, 2: 1}                      # ties -> lower id first
+
+
+def test_compute_replication_ratio_end_to_end():
+    r = hrcs.compute_replication_ratio(B=100, F=[0.5, 0.3, 0.1, 0.1], tau_u=1000, tau_i=5,
+                                       alpha=0.1, c=10, N=4, t=2)
+    assert r == 2 / 4                                   # R_max = 0.3 -> CDF .8 >= .7 at i = 2
+
+
+# ----------------------------------------------------------- scheduler
+def test_cache_agnostic_rule():
+    assert scheduler.cache_agnostic(4096, 3200) == "UP"
+    assert scheduler.cache_agnostic(512, 3200) == "IP"
+    assert scheduler.cache_agnostic(3200, 3200) == "UP"
+
+
+def test_hotness_aware_rule():
+    assert scheduler.hotness_aware(4096, 3200, 5.0, [1.0, 7.0]) == "UP"
+    assert scheduler.hotness_aware(4096, 3200, 0.5, [1.0, 7.0]) == "IP"
+    assert scheduler.hotness_aware(512, 3200, 99.0, [1.0]) == "IP"
+    assert scheduler.hotness_aware(4096, 3200, 0.0, []) == "UP"        # empty C_u
+
+
+def test_window_similarity():
+    assert scheduler.window_similarity(3, 3) == 1.0
+    assert scheduler.window_similarity(3, 1) == 0.5
