@@ -1,0 +1,268 @@
+/*
+ * bat.h — C ABI of the B200-native Bipartite Attention (BAT) prefill library (libbat.so).
+ *
+ * `P:n` cites /root/reference/PAPER.md line n (BAT: Efficient Generative Recommender Serving
+ * with Bipartite Attention, ASPLOS '26).
+ *
+ * What the library computes: a ranking request is a user
+ * profile U, N candidate items I_1..I_N and instruction tokens Instr.  Per request one
+ * side is a reused prefix KV cache: the user (User-as-prefix, UP, order [U, I_1..I_N, Instr],
+ * P:249) or every item independently (Item-as-prefix, IP, order [I_1..I_N, U, Instr]).
+ * The other tokens (the suffix) run through L transformer layers; at every layer they attend
+ * to [prefix KV ; suffix KV] under the bipartite mask — different items never see
+ * each other, all items start at the same position id (|U| in UP, 0 or after header tokens in
+ * IP), everything else causal (Fig. 1).  The discriminant (last) token's hidden
+ * state is projected on the N item-identifier logits, softmaxed and ranked.
+ *
+ * Conventions (every call):
+ *   - Return BAT_OK (0) or a negative bat_status; bat_last_error() returns a thread-local
+ *     message for the last failure.  No C++ exception crosses the ABI.
+ *   - "device" pointers are CUDA device pointers on the object's device; "host" pointers are
+ *     ordinary host memory, read during the call and not retained.
+ *   - Device work is enqueued on `stream` (a cudaStream_t; NULL = the legacy default stream)
+ *     and is asynchronous unless stated; host arrays are copied before the call returns.
+ *   - Objects are not thread-safe: calls on one pool/model must be externally serialised.
+ *   - Layouts are row-major with the last index contiguous.
+ */
+#ifndef BAT_H_
+#define BAT_H_
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#if defined(__GNUC__)
+#define BAT_API __attribute__((visibility("default")))
+#else
+#define BAT_API
+#endif
+
+typedef void* bat_stream_t; /* cudaStream_t */
+
+typedef enum {
+  BAT_OK = 0,
+  BAT_E_INVAL = -1,       /* bad argument / shape / unsupported value */
+  BAT_E_OOM = -2,         /* device or host allocation failed */
+  BAT_E_CUDA = -3,        /* a CUDA runtime/driver call failed (message has the CUDA error) */
+  BAT_E_NOTFOUND = -4,    /* a required prefix entity is not in the pool */
+  BAT_E_POOLFULL = -5,    /* not enough free pages; the pool is left unchanged */
+  BAT_E_UNSUPPORTED = -6, /* valid request this build does not implement */
+  BAT_E_STATE = -7        /* object in the wrong state (e.g. index-only pool used for compute) */
+} bat_status;
+
+typedef enum { BAT_BF16 = 0, BAT_FP32 = 1 } bat_dtype;
+
+/* Cache entries at user / item granularity; HEADER = the optional IP notation
+ * tokens ("Candidate items:"), cached once as its own entry. */
+typedef enum { BAT_ENT_USER = 0, BAT_ENT_ITEM = 1, BAT_ENT_HEADER = 2 } bat_entity;
+
+/* Prefix side of a request. */
+typedef enum { BAT_ORDER_UP = 0, BAT_ORDER_IP = 1 } bat_order;
+
+BAT_API const char* bat_last_error(void);
+BAT_API const char* bat_version(void);
+/* Number of device kernels this library launched since load (all devices). */
+BAT_API int64_t bat_kernel_launch_count(void);
+
+/* ------------------------------------------------------------------------------------------
+ * Model (Qwen2-shaped GR ranking model, Table 2)
+ * ---------------------------------------------------------------------------------------- */
+typedef struct {
+  int32_t layers, hidden, q_heads, kv_heads, head_dim, ffn, vocab;
+  float rope_theta; /* rotate-half RoPE base */
+  float rms_eps;    /* RMSNorm epsilon */
+  int32_t dtype;    /* bat_dtype of weights / activations / KV (BAT_BF16 is the product path) */
+} bat_model_cfg;
+
+/* Index of each weight in the pointer array passed to bat_model_create (3 + 7*layers device
+ * pointers, all of dtype cfg.dtype):
+ *   [0] embed      [vocab][hidden]          E, h^(0)_t = E[x_t]
+ *   [1] lm_head    [vocab][hidden]          W_out, z = W_out h_T; may alias embed (tied)
+ *   [2] final_norm [hidden]                 RMSNorm gain applied to h_T
+ *   per layer l, at 3 + 7*l + j:
+ *   j=0 ln1  [hidden]                       pre-attention RMSNorm gain
+ *   j=1 wqkv [(q_heads+2*kv_heads)*head_dim][hidden]   rows: all q heads, then k, then v
+ *   j=2 bqkv [(q_heads+2*kv_heads)*head_dim]          q/k/v bias
+ *   j=3 wo   [hidden][q_heads*head_dim]
+ *   j=4 ln2  [hidden]                       pre-MLP RMSNorm gain
+ *   j=5 wgu  [2*ffn][hidden]                rows: gate (ffn), then up (ffn); SwiGLU
+ *   j=6 wd   [hidden][ffn]
+ * The model BORROWS these pointers: the caller keeps them alive and unchanged until
+ * bat_model_destroy.  Supported: head_dim in {16, 32, 64, 128}, q_heads % kv_heads == 0,
+ * q_heads/kv_heads <= 128, hidden % 64 == 0, ffn % 128 == 0, BAT_BF16. */
+enum { BAT_W_EMBED = 0, BAT_W_LM_HEAD = 1, BAT_W_FINAL_NORM = 2, BAT_W_N_GLOBAL = 3 };
+enum { BAT_WL_LN1 = 0, BAT_WL_WQKV = 1, BAT_WL_BQKV = 2, BAT_WL_WO = 3, BAT_WL_LN2 = 4,
+       BAT_WL_WGU = 5, BAT_WL_WD = 6, BAT_WL_N = 7 };
+
+typedef struct bat_model_s* bat_model;
+BAT_API bat_status bat_model_create(const bat_model_cfg* cfg, const void* const* weights,
+                            int32_t n_weights, int32_t device, bat_model* out);
+BAT_API bat_status bat_model_destroy(bat_model m);
+
+/* ------------------------------------------------------------------------------------------
+ * Disaggregated paged KV pool: one page arena per GPU; entries at user/item
+ * granularity, each entry a list of fixed-size pages of page_tokens (16) tokens, each page
+ * holding all layers of its tokens.  Byte size per token = 2*kv_heads*head_dim*layers*2
+ * (Table 2: 28672 B for Qwen2-1.5B).  The in-HBM page layout is the tensor-core
+ * operand layout and is private; read entries back with bat_kv_read.
+ * ---------------------------------------------------------------------------------------- */
+typedef struct {
+  int32_t device;      /* CUDA device ordinal; -1 = index-only pool (no arena; planning tests) */
+  int32_t page_tokens; /* must be 16 */
+  int64_t num_pages;   /* arena capacity in pages */
+  int32_t dtype;       /* bat_dtype; must match the model's */
+  int32_t layers, kv_heads, head_dim;
+  int32_t rank, world; /* data-parallel rank / size for the HRCS item placement */
+} bat_pool_cfg;
+
+typedef struct bat_pool_s* bat_pool;
+BAT_API bat_status bat_kv_pool_create(const bat_pool_cfg* cfg, bat_pool* out); /* OWNS its arena */
+BAT_API bat_status bat_kv_pool_destroy(bat_pool p);
+/* bytes of one page (all layers) */
+BAT_API int64_t bat_kv_page_bytes(bat_pool p);
+BAT_API bat_status bat_kv_pool_stats(bat_pool p, int64_t* free_pages, int64_t* used_pages,
+                             int64_t* n_entities);
+
+/* Append n_tokens of prefix KV to entry (kind, id), creating it if absent (the background
+ * cache write of P:209/P:294 and the offline item precompute of P:312).  k, v: device
+ * [layers][n_tokens][kv_heads][head_dim] in the pool dtype, post-RoPE keys.  All-or-nothing:
+ * BAT_E_POOLFULL leaves the pool unchanged. */
+BAT_API bat_status bat_kv_append(bat_pool p, int32_t kind, int64_t id, const void* k, const void* v,
+                         int32_t n_tokens, bat_stream_t stream);
+/* Reserve pages for a new entry without writing data (index-only pools, and the entity
+ * prefill below).  BAT_E_INVAL if the entry exists. */
+BAT_API bat_status bat_kv_reserve(bat_pool p, int32_t kind, int64_t id, int32_t n_tokens);
+/* Drop an entry and free its pages. */
+BAT_API bat_status bat_kv_evict(bat_pool p, int32_t kind, int64_t id);
+/* Host query of an entry: its token count and page ids (pages_out may be NULL). */
+BAT_API bat_status bat_kv_lookup(bat_pool p, int32_t kind, int64_t id, int32_t* n_tokens,
+                         int32_t* pages_out, int32_t pages_cap, int32_t* n_pages);
+/* Copy an entry back out in the plain layout of bat_kv_append (device k_out, v_out). */
+BAT_API bat_status bat_kv_read(bat_pool p, int32_t kind, int64_t id, void* k_out, void* v_out,
+                       bat_stream_t stream);
+
+/* Prefix-miss path: compute the KV of n_entities new entries with the
+ * model — each entry's tokens run alone through the L layers, causally, at positions
+ * pos0, pos0+1, ... (UP user: pos0 = 0; IP item: pos0 = header length), attending first to
+ * the optional context entry (ctx_kind, ctx_id; pass ctx_kind = -1 for none; the IP header)
+ * — and store them as entries (kind, ids[e]).  tokens: host, entry e's tokens are
+ * tokens[tok_off[e] .. tok_off[e+1]).  The entries must not exist. */
+BAT_API bat_status bat_kv_prefill_entities(bat_pool p, bat_model m, int32_t kind, int32_t n_entities,
+                                   const int64_t* ids, const int32_t* tok_off,
+                                   const int32_t* tokens, int32_t pos0, int32_t ctx_kind,
+                                   int64_t ctx_id, bat_stream_t stream);
+
+/* ------------------------------------------------------------------------------------------
+ * Bipartite prefill (the hot path)
+ * ---------------------------------------------------------------------------------------- */
+typedef struct {
+  int32_t order;      /* bat_order: prefix side chosen for this request */
+  int32_t use_cache;  /* 1: prefix served from the pool; 0: recompute every token (RE) */
+  int64_t user_id;
+  const int32_t* user_tok; int32_t n_user;          /* host */
+  int32_t n_items;                                  /* N >= 1 */
+  const int64_t* item_id;                           /* host [N] */
+  const int32_t* item_off;                          /* host [N+1]: item i = item_tok[off[i]..off[i+1]) */
+  const int32_t* item_tok;                          /* host */
+  const int32_t* instr_tok; int32_t n_instr;        /* host; n_instr >= 1 (discriminant) */
+  int64_t header_id;                                /* IP notation tokens, may be 0-length */
+  const int32_t* header_tok; int32_t n_header;      /* host */
+} bat_query;
+
+/* Run the L layers for B requests (data-parallel batch): every request's suffix
+ * tokens are computed and attend to its cached prefix entries (BAT_E_NOTFOUND if one is
+ * missing and use_cache = 1).  Writes the final-RMSNormed discriminant hidden state of every
+ * request to out_hidden (device fp32 [B][hidden]).  Positions follow P:257 with the readings
+ * of DESIGN.md §2 (tokens after the item set continue from the longest item). */
+BAT_API bat_status bat_bipartite_prefill(bat_pool p, bat_model m, const bat_query* queries, int32_t B,
+                                 float* out_hidden, bat_stream_t stream);
+
+/* s[b][i] = softmax_i(W_out[labels[b][i]] . hidden[b]) over i < n_items[b];
+ * topk[b][0..k) = candidate indices by descending s (ties -> lower index).
+ * hidden: device fp32 [B][hidden]; labels: device int32 [B][n_max] (identifier token v_i,
+ * P:177); n_items: device int32 [B]; scores: device fp32 [B][n_max] (entries >= n_items[b]
+ * set to 0); topk: device int32 [B][k] or NULL when k = 0.  Requires n_max <= 4096,
+ * k <= n_items. */
+BAT_API bat_status bat_score(bat_model m, const float* hidden, const int32_t* labels,
+                     const int32_t* n_items, int32_t B, int32_t n_max, float* scores,
+                     int32_t k, int32_t* topk, bat_stream_t stream);
+
+/* ------------------------------------------------------------------------------------------
+ * Plan introspection (host only; bit-exact checks against the oracle's plan)
+ * ---------------------------------------------------------------------------------------- */
+typedef struct bat_plan_s* bat_plan;
+/* group = q_heads / kv_heads of the model the plan is for (GQA packing of q-tiles). */
+BAT_API bat_status bat_plan_create(bat_pool p, int32_t group, const bat_query* queries, int32_t B,
+                           bat_plan* out);
+BAT_API bat_status bat_plan_destroy(bat_plan plan);
+/* info[0..11] of request b: S (suffix tokens), P (prefix tokens), n_pages (incl. suffix
+ * pages, excl. padding), n_prefix_pages, n_qtiles, n_ktiles, token_off, scratch_page0,
+ * n_live_pairs (visible (query,key) pairs, per head per layer), qtile_tokens,
+ * first_qtile (global), page_off (global). */
+BAT_API bat_status bat_plan_query_info(bat_plan plan, int32_t b, int64_t info[12]);
+enum {
+  BAT_PF_TOKENS = 0,  /* int32 [S]  suffix token ids in prompt order */
+  BAT_PF_POS = 1,     /* int32 [S]  position ids */
+  BAT_PF_SEG = 2,     /* int32 [S]  -1 user, -2 instr, -3 header, i >= 0 item i */
+  BAT_PF_PAGES = 3,   /* int32 [n_pages] pool page id >= 0, or -(s+1) for scratch page s */
+  BAT_PF_VALID = 4,   /* int32 [n_pages] valid slots per page */
+  BAT_PF_KSEG = 5,    /* int32 [16*n_pages] key segment (-1 for empty slots) */
+  BAT_PF_KORD = 6,    /* int32 [16*n_pages] 0 prefix key, suffix index+1, INT32_MAX empty */
+  BAT_PF_TILES = 7    /* int32 [n_qtiles][n_ktiles] 0 skip / 1 full / 2 partial */
+};
+/* Copy field `field` of request b into out (cap elements); *count = its length. */
+BAT_API bat_status bat_plan_export(bat_plan plan, int32_t b, int32_t field, int32_t* out, int64_t cap,
+                           int64_t* count);
+
+/* ------------------------------------------------------------------------------------------
+ * Multi-GPU: hot-replicated / cold-sharded item placement (Algorithm 1)
+ * ---------------------------------------------------------------------------------------- */
+/* Algorithm 1 line 7 verbatim: R_max = alpha*t*B*(N-1) / (c*S_item*N), t = measured prefill
+ * time (s) of one request (replaces PrefillTime, line 4), B tokens/s, S_item = tau_i. */
+BAT_API bat_status bat_hrcs_rmax(double B, double t, double alpha, int32_t c, double tau_i,
+                         int32_t N, double* r_max_out);
+/* Lines 8-18: sort freq descending (ties: lower index first), replicate the first r*n items
+ * where r = i/n at the first i with CDF >= 1 - R_max (r = 1 if never reached); the rest are
+ * round-robin by hotness rank.  owner_out[i] = -1 replicated, else the owning rank. */
+BAT_API bat_status bat_hrcs_place(const double* freq, int64_t n_items, double r_max, int32_t world,
+                          int32_t* owner_out, double* r_out);
+
+/* CUDA-IPC export of the pool arena (64-byte handle) and import of a peer's arena. */
+BAT_API bat_status bat_pool_ipc_handle(bat_pool p, void* handle_out64);
+BAT_API bat_status bat_pool_attach_peer(bat_pool p, int32_t peer_rank, const void* handle64);
+/* Record that entry (kind, id) lives on peer `owner` in its pages owner_pages[0..n_pages). */
+BAT_API bat_status bat_kv_register_remote(bat_pool p, int32_t kind, int64_t id, int32_t owner,
+                                  const int32_t* owner_pages, int32_t n_pages,
+                                  int32_t n_tokens);
+/* Pull the listed remote entries (deduplicated, skipping ones already local) from their
+ * owners' arenas over NVLink into local pages (one copy kernel on `stream`), making them
+ * resolvable by bat_bipartite_prefill.  *n_fetched = entries pulled. */
+BAT_API bat_status bat_kv_fetch(bat_pool p, int32_t kind, const int64_t* ids, int32_t n,
+                        int32_t* n_fetched, bat_stream_t stream);
+
+/* ------------------------------------------------------------------------------------------
+ * Test-only entry points (kernel-level parity tests; not part of the serving path)
+ * ---------------------------------------------------------------------------------------- */
+/* One tcgen05 GEMM: epi 0 out = A B^T (bf16), 1 out = A B^T + bias (bf16), 2 out += A B^T
+ * (fp32 out), 3 out = silu(A Bg^T) * (A Bu^T) with Bg = B rows [0,N), Bu = rows [up_row0,..).
+ * A: device bf16 [M][K]; B: device bf16 [rows][K]; out leading dimension ldo (elements). */
+BAT_API bat_status bat_debug_gemm(int32_t epi, int32_t M, int32_t N, int32_t K, const void* A,
+                                  const void* Bw, int64_t b_rows, void* out, int32_t ldo,
+                                  const void* bias, int32_t up_row0, int32_t device,
+                                  bat_stream_t stream);
+/* Layer `layer` of the bipartite attention alone: plan the requests, apply RoPE (if
+ * rope_enabled) to the given qkv rows (device bf16 [M][(q_heads+2 kv_heads) head_dim], rows
+ * in plan order) and stage them, attend over the pool's prefix pages at that layer and the
+ * staged suffix, write O (device bf16 [M][q_heads*head_dim]). */
+BAT_API bat_status bat_debug_attention_layer(bat_pool p, bat_model m, const bat_query* queries,
+                                             int32_t B, int32_t layer, const void* qkv,
+                                             void* out_o, int32_t rope_enabled,
+                                             bat_stream_t stream);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* BAT_H_ */

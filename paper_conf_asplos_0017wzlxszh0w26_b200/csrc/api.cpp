@@ -1,0 +1,924 @@
+// C ABI of libbat (include/bat.h): model, pool, prefill driver, score, plan introspection,
+// HRCS placement and the NVLink page pull.  Host code only; device work is in k_*.cu.
+#include <cuda.h>
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cmath>
+#include <cstring>
+#include <memory>
+#include <mutex>
+#include <numeric>
+#include <string>
+#include <vector>
+
+#include "common.h"
+#include "kernels.h"
+#include "plan.h"
+#include "pool.h"
+
+struct bat_model_s;
+struct bat_pool_s {
+  bat::Pool pool;
+};
+struct bat_plan_s {
+  bat::Plan plan;
+};
+
+namespace bat {
+
+static thread_local std::string g_err;
+void set_error(const std::string& m) { g_err = m; }
+const char* last_error() { return g_err.c_str(); }
+
+#define CUDA_OK(expr)                                                                    \
+  do {                                                                                   \
+    cudaError_t e_ = (expr);                                                             \
+    if (e_ != cudaSuccess)                                                               \
+      ::bat::fail(BAT_E_CUDA, std::string(#expr) + ": " + cudaGetErrorString(e_));       \
+  } while (0)
+
+// ---------------------------------------------------------------- tensor-map creation
+using EncodeTiledFn = CUresult (*)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*,
+                                   const cuuint64_t*, const cuuint64_t*, const cuuint32_t*,
+                                   const cuuint32_t*, CUtensorMapInterleave, CUtensorMapSwizzle,
+                                   CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
+static EncodeTiledFn encode_fn() {
+  static EncodeTiledFn fn = nullptr;
+  static std::once_flag once;
+  std::call_once(once, [] {
+    void* p = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &p, cudaEnableDefault, &q) == cudaSuccess &&
+        q == cudaDriverEntryPointSuccess)
+      fn = reinterpret_cast<EncodeTiledFn>(p);
+  });
+  if (!fn) fail(BAT_E_CUDA, "cuTensorMapEncodeTiled unavailable");
+  return fn;
+}
+
+// bf16 row-major [rows][cols] with leading dimension ld (elements); box = [64 cols][box_rows]
+static CUtensorMap make_tmap(const void* ptr, int64_t rows, int64_t cols, int64_t ld, int box_rows) {
+  CUtensorMap m;
+  cuuint64_t dims[2] = {cuuint64_t(cols), cuuint64_t(rows)};
+  cuuint64_t strides[1] = {cuuint64_t(ld * 2)};
+  cuuint32_t box[2] = {64, cuuint32_t(box_rows)};
+  cuuint32_t estr[2] = {1, 1};
+  CUresult r = encode_fn()(&m, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 2, const_cast<void*>(ptr), dims,
+                           strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
+                           CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                           CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  if (r != CUDA_SUCCESS) fail(BAT_E_CUDA, "cuTensorMapEncodeTiled failed (" + std::to_string(int(r)) + ")");
+  return m;
+}
+
+// ------------------------------------------------------------------------ device buffer
+struct DevBuf {
+  void* p = nullptr;
+  size_t cap = 0;
+  void ensure(size_t bytes) {
+    if (bytes <= cap) return;
+    if (p) cudaFree(p);
+    p = nullptr;
+    cap = 0;
+    size_t want = std::max(bytes, size_t(1) << 16);
+    want = (want + (want >> 2) + 255) & ~size_t(255);
+    CUDA_OK(cudaMalloc(&p, want));
+    cap = want;
+  }
+  ~DevBuf() {
+    if (p) cudaFree(p);
+  }
+  template <class T>
+  T* as() const { return static_cast<T*>(p); }
+};
+
+struct Workspace {
+  DevBuf h, xn, qkv, qp, scratch, o, act, hc, xc, oc, actc, img, small;
+  void* img_host = nullptr;
+  size_t img_host_cap = 0;
+  cudaEvent_t img_done = nullptr;
+  ~Workspace() {
+    if (img_host) cudaFreeHost(img_host);
+    if (img_done) cudaEventDestroy(img_done);
+  }
+};
+
+struct Model {
+  bat_model_cfg cfg{};
+  int device = 0, num_sms = 148, dpad = 128;
+  const __nv_bfloat16 *embed = nullptr, *lm_head = nullptr, *final_norm = nullptr;
+  struct Layer {
+    const __nv_bfloat16 *ln1, *wqkv, *bqkv, *wo, *ln2, *wgu, *wd;
+    CUtensorMap t_qkv, t_o, t_gu, t_d;
+  };
+  std::vector<Layer> layers;
+  float2* rope = nullptr;
+  int max_pos = 0;
+  Workspace ws;
+  ~Model() {
+    if (rope) cudaFree(rope);
+  }
+  int nqkv() const { return (cfg.q_heads + 2 * cfg.kv_heads) * cfg.head_dim; }
+};
+
+struct DeviceGuard {
+  int prev = -1;
+  explicit DeviceGuard(int dev) {
+    cudaGetDevice(&prev);
+    if (dev >= 0 && dev != prev) CUDA_OK(cudaSetDevice(dev));
+  }
+  ~DeviceGuard() {
+    if (prev >= 0) cudaSetDevice(prev);
+  }
+};
+
+static void ensure_rope(Model& m, int need_pos, cudaStream_t st) {
+  if (need_pos <= m.max_pos) return;
+  int np = std::max(32768, m.max_pos);
+  while (np < need_pos) np *= 2;
+  if (m.rope) {
+    CUDA_OK(cudaStreamSynchronize(st));
+    cudaFree(m.rope);
+    m.rope = nullptr;
+  }
+  CUDA_OK(cudaMalloc(&m.rope, sizeof(float2) * size_t(np) * (m.cfg.head_dim / 2)));
+  launch_rope_table(m.rope, np, m.cfg.head_dim, double(m.cfg.rope_theta), st);
+  m.max_pos = np;
+}
+
+static PageIO page_io(const Pool& p) {
+  PageIO io;
+  io.arena = p.arena;
+  io.page_bytes = p.geo.page_bytes;
+  io.layer_bytes = p.geo.layer_bytes;
+  io.head_bytes = p.geo.head_bytes;
+  io.layers = p.geo.layers;
+  io.kv_heads = p.geo.kv_heads;
+  io.head_dim = p.geo.head_dim;
+  return io;
+}
+
+static void check_compat(const Pool& p, const Model& m) {
+  if (p.index_only) fail(BAT_E_STATE, "index-only pool cannot run device work");
+  BAT_REQUIRE(p.cfg.layers == m.cfg.layers && p.cfg.kv_heads == m.cfg.kv_heads &&
+                  p.cfg.head_dim == m.cfg.head_dim && p.cfg.dtype == m.cfg.dtype,
+              "pool geometry / dtype does not match the model");
+  BAT_REQUIRE(p.device == m.device, "pool and model are on different devices");
+}
+
+// Workspace sizing + plan upload; returns the device image.
+static const int32_t* prepare(Pool& pool, Model& m, Plan& plan, cudaStream_t st) {
+  const bat_model_cfg& c = m.cfg;
+  Workspace& ws = m.ws;
+  const int M = plan.M, B = static_cast<int>(plan.q.size());
+  const int H = c.hidden, F = c.ffn, nq = c.q_heads * c.head_dim;
+  const int64_t tile_bytes = int64_t(m.dpad / 64) * 16384;
+  int max_pos = 0;
+  for (auto& q : plan.q)
+    for (int32_t ps : q.pos) max_pos = std::max(max_pos, ps);
+  ensure_rope(m, max_pos + 1, st);
+  ws.h.ensure(size_t(M) * H * 4);
+  ws.xn.ensure(size_t(M) * std::max(H, nq) * 2);
+  ws.qkv.ensure(size_t(M) * m.nqkv() * 2);
+  ws.qp.ensure(size_t(plan.n_qtiles_total) * c.kv_heads * tile_bytes);
+  ws.scratch.ensure(size_t(std::max(plan.n_spages, 1)) * pool.geo.layer_bytes);
+  ws.o.ensure(size_t(M) * nq * 2);
+  ws.act.ensure(size_t(M) * F * 2);
+  ws.hc.ensure(size_t(B) * H * 4);
+  ws.xc.ensure(size_t(B) * H * 2);
+  ws.oc.ensure(size_t(B) * nq * 2);
+  ws.actc.ensure(size_t(B) * F * 2);
+  const size_t img_bytes = plan.img.buf.size() * 4;
+  ws.img.ensure(img_bytes);
+  if (!ws.img_done) CUDA_OK(cudaEventCreateWithFlags(&ws.img_done, cudaEventDisableTiming));
+  CUDA_OK(cudaEventSynchronize(ws.img_done));  // the previous upload finished reading the staging buffer
+  if (ws.img_host_cap < img_bytes) {
+    if (ws.img_host) cudaFreeHost(ws.img_host);
+    ws.img_host_cap = img_bytes + img_bytes / 4 + 4096;
+    CUDA_OK(cudaMallocHost(&ws.img_host, ws.img_host_cap));
+  }
+  std::memcpy(ws.img_host, plan.img.buf.data(), img_bytes);
+  CUDA_OK(cudaMemcpyAsync(ws.img.p, ws.img_host, img_bytes, cudaMemcpyHostToDevice, st));
+  CUDA_OK(cudaEventRecord(ws.img_done, st));
+  return ws.img.as<int32_t>();
+}
+
+static AttnParams attn_params(const Pool& pool, const Model& m, const Plan& plan, const int32_t* I) {
+  const bat_model_cfg& c = m.cfg;
+  const PlanImage& im = plan.img;
+  AttnParams ap{};
+  ap.img = I;
+  ap.off_qinfo = im.off_qinfo;
+  ap.off_pages = im.off_pages;
+  ap.off_kmeta = im.off_kmeta;
+  ap.off_rseg = im.off_rseg;
+  ap.off_work = im.off_work;
+  ap.n_work = plan.n_work;
+  ap.pool = pool.arena;
+  ap.pool_page_bytes = pool.geo.page_bytes;
+  ap.scratch = m.ws.scratch.as<char>();
+  ap.scratch_page_bytes = pool.geo.layer_bytes;
+  ap.scratch_layer_off = 0;
+  ap.zero_page = pool.arena + int64_t(pool.zero_page) * pool.geo.page_bytes;
+  ap.head_bytes = pool.geo.head_bytes;
+  ap.kv_heads = c.kv_heads;
+  ap.group = plan.group;
+  ap.qt = plan.qt;
+  ap.head_dim = c.head_dim;
+  ap.ldo = c.q_heads * c.head_dim;
+  ap.qp = m.ws.qp.as<__nv_bfloat16>();
+  ap.out = m.ws.o.as<__nv_bfloat16>();
+  ap.scale_log2 = float(1.4426950408889634 / std::sqrt(double(c.head_dim)));
+  return ap;
+}
+
+static StageParams stage_params(const Pool& pool, const Model& m, const Plan& plan, const int32_t* I) {
+  const bat_model_cfg& c = m.cfg;
+  const PlanImage& im = plan.img;
+  StageParams sp{};
+  sp.qkv = m.ws.qkv.as<__nv_bfloat16>();
+  sp.img = I;
+  sp.off_pos = im.off_pos;
+  sp.off_qinfo = im.off_qinfo;
+  sp.off_qtiles = im.off_qtiles;
+  sp.off_spages = im.off_spages;
+  sp.n_qtiles = plan.n_qtiles_total;
+  sp.n_spages = plan.n_spages;
+  sp.rope = m.rope;
+  sp.rope_enabled = 1;
+  sp.max_pos = m.max_pos;
+  sp.q_heads = c.q_heads;
+  sp.kv_heads = c.kv_heads;
+  sp.head_dim = c.head_dim;
+  sp.dpad = m.dpad;
+  sp.group = plan.group;
+  sp.qt = plan.qt;
+  sp.qp = m.ws.qp.as<__nv_bfloat16>();
+  sp.pool = pool.arena;
+  sp.pool_page_bytes = pool.geo.page_bytes;
+  sp.scratch = m.ws.scratch.as<char>();
+  sp.scratch_page_bytes = pool.geo.layer_bytes;
+  sp.scratch_layer_off = 0;
+  sp.head_bytes = pool.geo.head_bytes;
+  return sp;
+}
+
+// Run the L layers over a planned batch (SURVEY §3 call stack (3)).
+static void run_plan(Pool& pool, Model& m, Plan& plan, float* out_hidden, cudaStream_t st) {
+  const bat_model_cfg& c = m.cfg;
+  Workspace& ws = m.ws;
+  const int M = plan.M, B = static_cast<int>(plan.q.size());
+  const int H = c.hidden, F = c.ffn, dp = m.dpad;
+  const int nq = c.q_heads * c.head_dim;
+  const int32_t* I = prepare(pool, m, plan, st);
+  const PlanImage& im = plan.img;
+
+  // tensor maps of this call's activations
+  const CUtensorMap tA_xn = make_tmap(ws.xn.p, M, H, H, 128);
+  const CUtensorMap tA_o = make_tmap(ws.o.p, M, nq, nq, 128);
+  const CUtensorMap tA_act = make_tmap(ws.act.p, M, F, F, 128);
+  const CUtensorMap tA_xc = make_tmap(ws.xc.p, B, H, H, 128);
+  const CUtensorMap tA_oc = make_tmap(ws.oc.p, B, nq, nq, 128);
+  const CUtensorMap tA_actc = make_tmap(ws.actc.p, B, F, F, 128);
+  AttnParams ap = attn_params(pool, m, plan, I);
+  StageParams sp = stage_params(pool, m, plan, I);
+
+  launch_embed(m.embed, I + im.off_tok, ws.h.as<float>(), M, H, st);
+  for (int l = 0; l < c.layers; ++l) {
+    const Model::Layer& Lw = m.layers[l];
+    const bool last = (l == c.layers - 1);
+    launch_rmsnorm_bf16(ws.h.as<float>(), Lw.ln1, ws.xn.as<__nv_bfloat16>(), M, H, c.rms_eps, st);
+    GemmParams gp{M, m.nqkv(), H, ws.qkv.p, m.nqkv(), Lw.bqkv, 0};
+    launch_gemm(EPI_BF16_BIAS, tA_xn, Lw.t_qkv, gp, m.num_sms, st);
+    sp.pool_layer_off = int64_t(l) * pool.geo.layer_bytes;
+    launch_stage(sp, st);
+    if (last && plan.entity_mode) break;  // entity prefill: only this layer's K/V are needed
+    ap.pool_layer_off = int64_t(l) * pool.geo.layer_bytes;
+    if (!last) {
+      ap.off_work = im.off_work;
+      ap.n_work = plan.n_work;
+      launch_attention(dp, ap, m.num_sms, st);
+      GemmParams go{M, H, nq, ws.h.p, H, nullptr, 0};
+      launch_gemm(EPI_RESID_F32, tA_o, Lw.t_o, go, m.num_sms, st);
+      launch_rmsnorm_bf16(ws.h.as<float>(), Lw.ln2, ws.xn.as<__nv_bfloat16>(), M, H, c.rms_eps, st);
+      GemmParams gg{M, F, H, ws.act.p, F, nullptr, F};
+      launch_gemm(EPI_SWIGLU, tA_xn, Lw.t_gu, gg, m.num_sms, st);
+      GemmParams gd{M, H, F, ws.h.p, H, nullptr, 0};
+      launch_gemm(EPI_RESID_F32, tA_act, Lw.t_d, gd, m.num_sms, st);
+    } else {
+      // a8: after the last layer's K/V only the discriminant rows matter
+      ap.off_work = im.off_work_last;
+      ap.n_work = plan.n_work_last;
+      launch_attention(dp, ap, m.num_sms, st);
+      const int32_t* disc = I + im.off_disc;
+      launch_gather_rows_bf16(ws.o.as<__nv_bfloat16>(), disc, ws.oc.as<__nv_bfloat16>(), B, nq, st);
+      launch_gather_rows_f32(ws.h.as<float>(), disc, ws.hc.as<float>(), B, H, st);
+      GemmParams go{B, H, nq, ws.hc.p, H, nullptr, 0};
+      launch_gemm(EPI_RESID_F32, tA_oc, Lw.t_o, go, m.num_sms, st);
+      launch_rmsnorm_bf16(ws.hc.as<float>(), Lw.ln2, ws.xc.as<__nv_bfloat16>(), B, H, c.rms_eps, st);
+      GemmParams gg{B, F, H, ws.actc.p, F, nullptr, F};
+      launch_gemm(EPI_SWIGLU, tA_xc, Lw.t_gu, gg, m.num_sms, st);
+      GemmParams gd{B, H, F, ws.hc.p, H, nullptr, 0};
+      launch_gemm(EPI_RESID_F32, tA_actc, Lw.t_d, gd, m.num_sms, st);
+      launch_rmsnorm_f32out(ws.hc.as<float>(), m.final_norm, out_hidden, B, H, c.rms_eps, st);
+    }
+  }
+  CUDA_OK(cudaGetLastError());
+}
+
+static int64_t key_kind_check(int32_t kind) {
+  BAT_REQUIRE(kind == BAT_ENT_USER || kind == BAT_ENT_ITEM || kind == BAT_ENT_HEADER, "entity kind");
+  return kind;
+}
+
+}  // namespace bat
+
+using namespace bat;
+
+struct bat_model_s {
+  Model m;
+};
+
+extern "C" {
+
+const char* bat_last_error(void) { return bat::last_error(); }
+const char* bat_version(void) { return "bat-b200 0.1 (sm_100a)"; }
+int64_t bat_kernel_launch_count(void) { return bat::launch_count(); }
+
+bat_status bat_model_create(const bat_model_cfg* cfg, const void* const* weights, int32_t n_weights,
+                            int32_t device, bat_model* out) {
+  return guarded([&] {
+    BAT_REQUIRE(cfg && weights && out, "null argument");
+    const bat_model_cfg& c = *cfg;
+    BAT_REQUIRE(c.dtype == BAT_BF16, "only BAT_BF16 is implemented");
+    BAT_REQUIRE(c.layers >= 1 && c.hidden >= 64 && c.hidden % 64 == 0, "hidden % 64 == 0");
+    BAT_REQUIRE(c.head_dim == 16 || c.head_dim == 32 || c.head_dim == 64 || c.head_dim == 128,
+                "head_dim in {16,32,64,128}");
+    BAT_REQUIRE(c.kv_heads >= 1 && c.q_heads % c.kv_heads == 0 && c.q_heads / c.kv_heads <= 128,
+                "q_heads % kv_heads == 0 and group <= 128");
+    BAT_REQUIRE(c.ffn % 128 == 0, "ffn % 128 == 0");
+    BAT_REQUIRE((c.q_heads * c.head_dim) % 64 == 0, "q_heads*head_dim % 64 == 0");
+    BAT_REQUIRE(c.vocab >= 1, "vocab");
+    BAT_REQUIRE(n_weights == BAT_W_N_GLOBAL + BAT_WL_N * c.layers, "n_weights == 3 + 7*layers");
+    for (int i = 0; i < n_weights; ++i) BAT_REQUIRE(weights[i] != nullptr, "null weight pointer");
+    DeviceGuard dg(device);
+    auto mp = std::make_unique<bat_model_s>();
+    Model& m = mp->m;
+    m.cfg = c;
+    m.device = device;
+    m.dpad = head_dim_pad(c.head_dim);
+    CUDA_OK(cudaDeviceGetAttribute(&m.num_sms, cudaDevAttrMultiProcessorCount, device));
+    int major = 0;
+    CUDA_OK(cudaDeviceGetAttribute(&major, cudaDevAttrComputeCapabilityMajor, device));
+    if (major != 10) fail(BAT_E_UNSUPPORTED, "libbat kernels are sm_100a (B200) only");
+    auto W = [&](int i) { return static_cast<const __nv_bfloat16*>(weights[i]); };
+    m.embed = W(BAT_W_EMBED);
+    m.lm_head = W(BAT_W_LM_HEAD);
+    m.final_norm = W(BAT_W_FINAL_NORM);
+    const int H = c.hidden, nq = c.q_heads * c.head_dim, F = c.ffn;
+    for (int l = 0; l < c.layers; ++l) {
+      auto w = [&](int j) { return W(BAT_W_N_GLOBAL + BAT_WL_N * l + j); };
+      Model::Layer L{};
+      L.ln1 = w(BAT_WL_LN1);
+      L.wqkv = w(BAT_WL_WQKV);
+      L.bqkv = w(BAT_WL_BQKV);
+      L.wo = w(BAT_WL_WO);
+      L.ln2 = w(BAT_WL_LN2);
+      L.wgu = w(BAT_WL_WGU);
+      L.wd = w(BAT_WL_WD);
+      L.t_qkv = make_tmap(L.wqkv, m.nqkv(), H, H, 256);
+      L.t_o = make_tmap(L.wo, H, nq, nq, 256);
+      L.t_gu = make_tmap(L.wgu, 2 * int64_t(F), H, H, 128);
+      L.t_d = make_tmap(L.wd, H, F, F, 256);
+      m.layers.push_back(L);
+    }
+    ensure_rope(m, 32768, 0);
+    CUDA_OK(cudaStreamSynchronize(0));
+    *out = mp.release();
+  });
+}
+
+bat_status bat_model_destroy(bat_model m) {
+  return guarded([&] {
+    if (!m) return;
+    DeviceGuard dg(m->m.device);
+    cudaDeviceSynchronize();
+    delete m;
+  });
+}
+
+// ------------------------------------------------------------------------------- pool
+bat_status bat_kv_pool_create(const bat_pool_cfg* cfg, bat_pool* out) {
+  return guarded([&] {
+    BAT_REQUIRE(cfg && out, "null argument");
+    const bat_pool_cfg& c = *cfg;
+    BAT_REQUIRE(c.page_tokens == kPageTokens, "page_tokens must be 16");
+    BAT_REQUIRE(c.num_pages >= 1 && c.num_pages < (int64_t(1) << 30), "num_pages");
+    BAT_REQUIRE(c.dtype == BAT_BF16, "only BAT_BF16 pools are implemented");
+    BAT_REQUIRE(c.layers >= 1 && c.kv_heads >= 1, "layers / kv_heads");
+    BAT_REQUIRE(c.head_dim == 16 || c.head_dim == 32 || c.head_dim == 64 || c.head_dim == 128, "head_dim");
+    auto pp = std::make_unique<bat_pool_s>();
+    Pool& p = pp->pool;
+    p.cfg = c;
+    if (p.cfg.world < 1) p.cfg.world = 1;
+    p.device = c.device;
+    p.index_only = c.device < 0;
+    p.geo.init(c.layers, c.kv_heads, c.head_dim);
+    p.zero_page = static_cast<int32_t>(c.num_pages);
+    p.free_pages.reserve(c.num_pages);
+    for (int64_t i = c.num_pages - 1; i >= 0; --i) p.free_pages.push_back(static_cast<int32_t>(i));
+    p.peer_arena.assign(p.cfg.world, nullptr);
+    if (!p.index_only) {
+      DeviceGuard dg(c.device);
+      const size_t bytes = size_t(c.num_pages + 1) * p.geo.page_bytes;
+      cudaError_t e = cudaMalloc(&p.arena, bytes);
+      if (e != cudaSuccess) fail(BAT_E_OOM, std::string("pool arena: ") + cudaGetErrorString(e));
+      CUDA_OK(cudaMemset(p.arena, 0, bytes));  // padded columns / empty slots stay zero
+    }
+    *out = pp.release();
+  });
+}
+
+bat_status bat_kv_pool_destroy(bat_pool p) {
+  return guarded([&] {
+    if (!p) return;
+    if (p->pool.arena) {
+      DeviceGuard dg(p->pool.device);
+      cudaDeviceSynchronize();
+      for (char* a : p->pool.peer_arena)
+        if (a) cudaIpcCloseMemHandle(a);
+      cudaFree(p->pool.arena);
+    }
+    delete p;
+  });
+}
+
+int64_t bat_kv_page_bytes(bat_pool p) { return p ? p->pool.geo.page_bytes : 0; }
+
+bat_status bat_kv_pool_stats(bat_pool p, int64_t* free_pages, int64_t* used_pages, int64_t* n_entities) {
+  return guarded([&] {
+    BAT_REQUIRE(p, "null pool");
+    if (free_pages) *free_pages = int64_t(p->pool.free_pages.size());
+    if (used_pages) *used_pages = p->pool.cfg.num_pages - int64_t(p->pool.free_pages.size());
+    if (n_entities) *n_entities = int64_t(p->pool.index.size());
+  });
+}
+
+bat_status bat_kv_reserve(bat_pool p, int32_t kind, int64_t id, int32_t n_tokens) {
+  return guarded([&] {
+    BAT_REQUIRE(p, "null pool");
+    key_kind_check(kind);
+    BAT_REQUIRE(n_tokens >= 1, "n_tokens >= 1");
+    Pool& P = p->pool;
+    EntityKey k{kind, id};
+    BAT_REQUIRE(P.index.find(k) == P.index.end(), "entry already exists");
+    Entity e;
+    e.n_tokens = n_tokens;
+    if (!P.alloc_pages(ceil_div(n_tokens, kPageTokens), e.pages)) {
+      P.release_pages(e.pages);
+      fail(BAT_E_POOLFULL, "pool full");
+    }
+    P.index.emplace(k, std::move(e));
+  });
+}
+
+bat_status bat_kv_evict(bat_pool p, int32_t kind, int64_t id) {
+  return guarded([&] {
+    BAT_REQUIRE(p, "null pool");
+    Pool& P = p->pool;
+    auto it = P.index.find(EntityKey{kind, id});
+    if (it == P.index.end()) fail(BAT_E_NOTFOUND, "entry not found");
+    P.release_pages(it->second.pages);
+    P.index.erase(it);
+  });
+}
+
+bat_status bat_kv_lookup(bat_pool p, int32_t kind, int64_t id, int32_t* n_tokens, int32_t* pages_out,
+                         int32_t pages_cap, int32_t* n_pages) {
+  return guarded([&] {
+    BAT_REQUIRE(p, "null pool");
+    const Entity* e = p->pool.find(kind, id);
+    if (!e) fail(BAT_E_NOTFOUND, "entry not found");
+    if (n_tokens) *n_tokens = e->n_tokens;
+    if (n_pages) *n_pages = int32_t(e->pages.size());
+    if (pages_out) {
+      BAT_REQUIRE(pages_cap >= int32_t(e->pages.size()), "pages_cap too small");
+      std::copy(e->pages.begin(), e->pages.end(), pages_out);
+    }
+  });
+}
+
+bat_status bat_kv_append(bat_pool p, int32_t kind, int64_t id, const void* k, const void* v,
+                         int32_t n_tokens, bat_stream_t stream) {
+  return guarded([&] {
+    BAT_REQUIRE(p && k && v, "null argument");
+    key_kind_check(kind);
+    BAT_REQUIRE(n_tokens >= 1, "n_tokens >= 1");
+    Pool& P = p->pool;
+    if (P.index_only) fail(BAT_E_STATE, "index-only pool");
+    DeviceGuard dg(P.device);
+    EntityKey key{kind, id};
+    auto it = P.index.find(key);
+    const bool exists = it != P.index.end();
+    const int32_t old_n = exists ? it->second.n_tokens : 0;
+    const int64_t need = ceil_div(old_n + n_tokens, kPageTokens) - (exists ? int64_t(it->second.pages.size()) : 0);
+    std::vector<int32_t> fresh;
+    if (!P.alloc_pages(need, fresh)) {
+      P.release_pages(fresh);
+      fail(BAT_E_POOLFULL, "pool full");
+    }
+    std::vector<int32_t> pages = exists ? it->second.pages : std::vector<int32_t>();
+    pages.insert(pages.end(), fresh.begin(), fresh.end());
+    int32_t* dpages = nullptr;
+    cudaStream_t st = static_cast<cudaStream_t>(stream);
+    cudaError_t e = cudaMallocAsync(reinterpret_cast<void**>(&dpages), pages.size() * 4, st);
+    if (e != cudaSuccess) {
+      P.release_pages(fresh);
+      fail(BAT_E_CUDA, std::string("cudaMallocAsync: ") + cudaGetErrorString(e));
+    }
+    CUDA_OK(cudaMemcpyAsync(dpages, pages.data(), pages.size() * 4, cudaMemcpyHostToDevice, st));
+    launch_kv_scatter(page_io(P), static_cast<const __nv_bfloat16*>(k), static_cast<const __nv_bfloat16*>(v),
+                      dpages, n_tokens, old_n, n_tokens, st);
+    CUDA_OK(cudaFreeAsync(dpages, st));
+    CUDA_OK(cudaStreamSynchronize(st));  // the host page list above is a stack temporary
+    if (exists) {
+      it->second.pages = std::move(pages);
+      it->second.n_tokens = old_n + n_tokens;
+    } else {
+      Entity en;
+      en.n_tokens = n_tokens;
+      en.pages = std::move(pages);
+      P.index.emplace(key, std::move(en));
+    }
+  });
+}
+
+bat_status bat_kv_read(bat_pool p, int32_t kind, int64_t id, void* k_out, void* v_out, bat_stream_t stream) {
+  return guarded([&] {
+    BAT_REQUIRE(p && k_out && v_out, "null argument");
+    Pool& P = p->pool;
+    if (P.index_only) fail(BAT_E_STATE, "index-only pool");
+    const Entity* e = P.find(kind, id);
+    if (!e) fail(BAT_E_NOTFOUND, "entry not found");
+    DeviceGuard dg(P.device);
+    cudaStream_t st = static_cast<cudaStream_t>(stream);
+    int32_t* dpages = nullptr;
+    CUDA_OK(cudaMallocAsync(reinterpret_cast<void**>(&dpages), e->pages.size() * 4, st));
+    CUDA_OK(cudaMemcpyAsync(dpages, e->pages.data(), e->pages.size() * 4, cudaMemcpyHostToDevice, st));
+    launch_kv_gather(page_io(P), static_cast<__nv_bfloat16*>(k_out), static_cast<__nv_bfloat16*>(v_out),
+                     dpages, e->n_tokens, st);
+    CUDA_OK(cudaFreeAsync(dpages, st));
+    CUDA_OK(cudaStreamSynchronize(st));
+  });
+}
+
+bat_status bat_kv_prefill_entities(bat_pool p, bat_model mdl, int32_t kind, int32_t n_entities,
+                                   const int64_t* ids, const int32_t* tok_off, const int32_t* tokens,
+                                   int32_t pos0, int32_t ctx_kind, int64_t ctx_id, bat_stream_t stream) {
+  return guarded([&] {
+    BAT_REQUIRE(p && mdl && ids && tok_off && tokens, "null argument");
+    key_kind_check(kind);
+    BAT_REQUIRE(n_entities >= 1 && pos0 >= 0, "n_entities / pos0");
+    Pool& P = p->pool;
+    Model& m = mdl->m;
+    check_compat(P, m);
+    DeviceGuard dg(P.device);
+    std::vector<EntityKey> made;
+    std::vector<std::vector<int32_t>> pages(n_entities);
+    try {
+      for (int e = 0; e < n_entities; ++e) {
+        const int32_t n = tok_off[e + 1] - tok_off[e];
+        BAT_REQUIRE(n >= 1, "entity with no tokens");
+        for (int32_t j = 0; j < n; ++j)
+          BAT_REQUIRE(tokens[tok_off[e] + j] >= 0 && tokens[tok_off[e] + j] < m.cfg.vocab, "token id out of range");
+        EntityKey key{kind, ids[e]};
+        BAT_REQUIRE(P.index.find(key) == P.index.end(), "entry already exists");
+        Entity en;
+        en.n_tokens = n;
+        if (!P.alloc_pages(ceil_div(n, kPageTokens), en.pages)) {
+          P.release_pages(en.pages);
+          fail(BAT_E_POOLFULL, "pool full");
+        }
+        pages[e] = en.pages;
+        P.index.emplace(key, std::move(en));
+        made.push_back(key);
+      }
+      std::vector<PlanRequest> reqs(n_entities);
+      for (int e = 0; e < n_entities; ++e) {
+        reqs[e].ent_tok = tokens + tok_off[e];
+        reqs[e].ent_n = tok_off[e + 1] - tok_off[e];
+        reqs[e].ent_pos0 = pos0;
+        reqs[e].ctx_kind = ctx_kind;
+        reqs[e].ctx_id = ctx_id;
+        reqs[e].ent_pages = &pages[e];
+      }
+      Plan plan;
+      build_plan(P, m.cfg.q_heads / m.cfg.kv_heads, m.cfg.kv_heads, reqs, plan, true);
+      run_plan(P, m, plan, nullptr, static_cast<cudaStream_t>(stream));
+      CUDA_OK(cudaStreamSynchronize(static_cast<cudaStream_t>(stream)));
+    } catch (...) {
+      for (auto& k : made) {
+        auto it = P.index.find(k);
+        if (it != P.index.end()) {
+          P.release_pages(it->second.pages);
+          P.index.erase(it);
+        }
+      }
+      throw;
+    }
+  });
+}
+
+// -------------------------------------------------------------------------- prefill
+static std::vector<PlanRequest> wrap(const bat_query* q, int32_t B) {
+  std::vector<PlanRequest> r(B);
+  for (int b = 0; b < B; ++b) r[b].q = &q[b];
+  return r;
+}
+
+static void validate_tokens(const bat_query& q, int vocab) {
+  auto chk = [&](const int32_t* t, int n) {
+    for (int i = 0; i < n; ++i) BAT_REQUIRE(t[i] >= 0 && t[i] < vocab, "token id out of range");
+  };
+  chk(q.user_tok, q.n_user);
+  chk(q.instr_tok, q.n_instr);
+  chk(q.header_tok, q.n_header);
+  if (q.n_items > 0 && q.item_off) chk(q.item_tok, q.item_off[q.n_items]);
+}
+
+bat_status bat_bipartite_prefill(bat_pool p, bat_model mdl, const bat_query* queries, int32_t B,
+                                 float* out_hidden, bat_stream_t stream) {
+  return guarded([&] {
+    BAT_REQUIRE(p && mdl && queries && out_hidden, "null argument");
+    BAT_REQUIRE(B >= 1, "B >= 1");
+    Pool& P = p->pool;
+    Model& m = mdl->m;
+    check_compat(P, m);
+    for (int b = 0; b < B; ++b) validate_tokens(queries[b], m.cfg.vocab);
+    DeviceGuard dg(P.device);
+    Plan plan;
+    build_plan(P, m.cfg.q_heads / m.cfg.kv_heads, m.cfg.kv_heads, wrap(queries, B), plan, true);
+    run_plan(P, m, plan, out_hidden, static_cast<cudaStream_t>(stream));
+  });
+}
+
+bat_status bat_score(bat_model mdl, const float* hidden, const int32_t* labels, const int32_t* n_items,
+                     int32_t B, int32_t n_max, float* scores, int32_t k, int32_t* topk, bat_stream_t stream) {
+  return guarded([&] {
+    BAT_REQUIRE(mdl && hidden && labels && n_items && scores, "null argument");
+    BAT_REQUIRE(B >= 1 && n_max >= 1 && n_max <= 4096, "B >= 1, 1 <= n_max <= 4096");
+    BAT_REQUIRE(k >= 0 && (k == 0 || topk), "k / topk");
+    BAT_REQUIRE(k <= n_max, "k <= n_max");
+    Model& m = mdl->m;
+    DeviceGuard dg(m.device);
+    launch_score(hidden, m.lm_head, labels, n_items, B, n_max, m.cfg.hidden, scores, k, topk,
+                 static_cast<cudaStream_t>(stream));
+    CUDA_OK(cudaGetLastError());
+  });
+}
+
+// ---------------------------------------------------------------------- plan inspection
+bat_status bat_plan_create(bat_pool p, int32_t group, const bat_query* queries, int32_t B, bat_plan* out) {
+  return guarded([&] {
+    BAT_REQUIRE(p && queries && out && B >= 1, "null argument");
+    auto pl = std::make_unique<bat_plan_s>();
+    build_plan(p->pool, group, 1, wrap(queries, B), pl->plan, false);
+    *out = pl.release();
+  });
+}
+
+bat_status bat_plan_destroy(bat_plan plan) {
+  return guarded([&] { delete plan; });
+}
+
+bat_status bat_plan_query_info(bat_plan plan, int32_t b, int64_t info[12]) {
+  return guarded([&] {
+    BAT_REQUIRE(plan && info && b >= 0 && b < int32_t(plan->plan.q.size()), "argument");
+    const QueryPlan& q = plan->plan.q[b];
+    const int64_t v[12] = {q.S, q.P, q.n_pages, q.n_prefix_pages, q.n_qtiles, q.n_ktiles, q.token_off,
+                           q.scratch0, q.n_live_pairs, plan->plan.qt, q.qtile0, q.page_off};
+    std::copy(v, v + 12, info);
+  });
+}
+
+bat_status bat_plan_export(bat_plan plan, int32_t b, int32_t field, int32_t* out, int64_t cap, int64_t* count) {
+  return guarded([&] {
+    BAT_REQUIRE(plan && b >= 0 && b < int32_t(plan->plan.q.size()), "argument");
+    const QueryPlan& q = plan->plan.q[b];
+    std::vector<int32_t> tiles;
+    const std::vector<int32_t>* src = nullptr;
+    switch (field) {
+      case BAT_PF_TOKENS: src = &q.tokens; break;
+      case BAT_PF_POS: src = &q.pos; break;
+      case BAT_PF_SEG: src = &q.seg; break;
+      case BAT_PF_PAGES: src = &q.pages; break;
+      case BAT_PF_VALID: src = &q.valid; break;
+      case BAT_PF_KSEG: src = &q.kseg; break;
+      case BAT_PF_KORD: src = &q.kord; break;
+      case BAT_PF_TILES:
+        tiles.assign(q.tiles.begin(), q.tiles.end());
+        src = &tiles;
+        break;
+      default: BAT_REQUIRE(false, "unknown field");
+    }
+    if (count) *count = int64_t(src->size());
+    if (out) {
+      BAT_REQUIRE(cap >= int64_t(src->size()), "cap too small");
+      std::copy(src->begin(), src->end(), out);
+    }
+  });
+}
+
+// ------------------------------------------------------------------ HRCS (Algorithm 1)
+bat_status bat_hrcs_rmax(double B, double t, double alpha, int32_t c, double tau_i, int32_t N, double* out) {
+  return guarded([&] {
+    BAT_REQUIRE(out && c >= 1 && tau_i > 0 && N >= 1, "argument");
+    const double T_max = alpha * t;               // line 5
+    const double S_item = tau_i;                  // line 6
+    *out = T_max * B * double(N - 1) / (double(c) * S_item * double(N));  // line 7
+  });
+}
+
+bat_status bat_hrcs_place(const double* freq, int64_t n, double r_max, int32_t world, int32_t* owner,
+                          double* r_out) {
+  return guarded([&] {
+    BAT_REQUIRE(freq && owner && n >= 1 && world >= 1, "argument");
+    double total = 0.0;
+    for (int64_t i = 0; i < n; ++i) total += freq[i];
+    BAT_REQUIRE(total > 0.0, "frequencies sum to zero");
+    std::vector<int64_t> order(n);
+    std::iota(order.begin(), order.end(), 0);
+    std::stable_sort(order.begin(), order.end(), [&](int64_t a, int64_t b) { return freq[a] > freq[b]; });
+    double cdf = 0.0, r = 1.0;
+    for (int64_t i = 1; i <= n; ++i) {  // lines 9-16
+      cdf += freq[order[i - 1]] / total;
+      if (cdf >= 1.0 - r_max) {
+        r = double(i) / double(n);
+        break;
+      }
+    }
+    const int64_t n_rep = static_cast<int64_t>(std::llround(r * double(n)));
+    for (int64_t i = 0; i < n; ++i) {  // lines 17-18
+      owner[order[i]] = i < n_rep ? -1 : static_cast<int32_t>((i - n_rep) % world);
+    }
+    if (r_out) *r_out = r;
+  });
+}
+
+// ------------------------------------------------------------- NVLink page pull (a10)
+bat_status bat_pool_ipc_handle(bat_pool p, void* out64) {
+  return guarded([&] {
+    BAT_REQUIRE(p && out64, "null argument");
+    Pool& P = p->pool;
+    if (P.index_only) fail(BAT_E_STATE, "index-only pool");
+    DeviceGuard dg(P.device);
+    cudaIpcMemHandle_t h;
+    CUDA_OK(cudaIpcGetMemHandle(&h, P.arena));
+    static_assert(sizeof(h) == 64, "ipc handle size");
+    std::memcpy(out64, &h, 64);
+  });
+}
+
+bat_status bat_pool_attach_peer(bat_pool p, int32_t peer, const void* h64) {
+  return guarded([&] {
+    BAT_REQUIRE(p && h64, "null argument");
+    Pool& P = p->pool;
+    BAT_REQUIRE(peer >= 0 && peer < P.cfg.world && peer != P.cfg.rank, "peer rank");
+    if (P.index_only) fail(BAT_E_STATE, "index-only pool");
+    DeviceGuard dg(P.device);
+    cudaIpcMemHandle_t h;
+    std::memcpy(&h, h64, 64);
+    void* ptr = nullptr;
+    CUDA_OK(cudaIpcOpenMemHandle(&ptr, h, cudaIpcMemLazyEnablePeerAccess));
+    P.peer_arena[peer] = static_cast<char*>(ptr);
+  });
+}
+
+bat_status bat_kv_register_remote(bat_pool p, int32_t kind, int64_t id, int32_t owner, const int32_t* pages,
+                                  int32_t n_pages, int32_t n_tokens) {
+  return guarded([&] {
+    BAT_REQUIRE(p && pages && n_pages >= 1 && n_tokens >= 1, "argument");
+    key_kind_check(kind);
+    Pool& P = p->pool;
+    BAT_REQUIRE(owner >= 0 && owner < P.cfg.world, "owner rank");
+    BAT_REQUIRE(n_pages == ceil_div(n_tokens, kPageTokens), "n_pages == ceil(n_tokens/16)");
+    RemoteEntity r;
+    r.owner = owner;
+    r.n_tokens = n_tokens;
+    r.pages.assign(pages, pages + n_pages);
+    P.remote[EntityKey{kind, id}] = std::move(r);
+  });
+}
+
+bat_status bat_kv_fetch(bat_pool p, int32_t kind, const int64_t* ids, int32_t n, int32_t* n_fetched,
+                        bat_stream_t stream) {
+  return guarded([&] {
+    BAT_REQUIRE(p && (ids || n == 0), "null argument");
+    Pool& P = p->pool;
+    if (P.index_only) fail(BAT_E_STATE, "index-only pool");
+    DeviceGuard dg(P.device);
+    std::vector<uint64_t> src;
+    std::vector<int32_t> dst;
+    std::vector<EntityKey> made;
+    int32_t fetched = 0;
+    try {
+      for (int32_t i = 0; i < n; ++i) {
+        EntityKey key{kind, ids[i]};
+        if (P.index.count(key)) continue;  // local (replicated, owned or already fetched)
+        auto it = P.remote.find(key);
+        if (it == P.remote.end()) fail(BAT_E_NOTFOUND, "entry neither local nor registered remote");
+        const RemoteEntity& r = it->second;
+        char* peer = P.peer_arena[r.owner];
+        if (!peer) fail(BAT_E_STATE, "peer arena of rank " + std::to_string(r.owner) + " not attached");
+        Entity en;
+        en.n_tokens = r.n_tokens;
+        en.fetched = true;
+        if (!P.alloc_pages(int64_t(r.pages.size()), en.pages)) {
+          P.release_pages(en.pages);
+          fail(BAT_E_POOLFULL, "pool full while fetching");
+        }
+        for (size_t k = 0; k < r.pages.size(); ++k) {
+          src.push_back(reinterpret_cast<uint64_t>(peer + int64_t(r.pages[k]) * P.geo.page_bytes));
+          dst.push_back(en.pages[k]);
+        }
+        P.index.emplace(key, std::move(en));
+        made.push_back(key);
+        ++fetched;
+      }
+      if (!src.empty()) {
+        cudaStream_t st = static_cast<cudaStream_t>(stream);
+        void* buf = nullptr;
+        const size_t bytes = src.size() * 8 + dst.size() * 4;
+        CUDA_OK(cudaMallocAsync(&buf, bytes, st));
+        CUDA_OK(cudaMemcpyAsync(buf, src.data(), src.size() * 8, cudaMemcpyHostToDevice, st));
+        CUDA_OK(cudaMemcpyAsync(static_cast<char*>(buf) + src.size() * 8, dst.data(), dst.size() * 4,
+                                cudaMemcpyHostToDevice, st));
+        launch_page_copy(static_cast<const uint64_t*>(buf),
+                         reinterpret_cast<const int32_t*>(static_cast<char*>(buf) + src.size() * 8), P.arena,
+                         P.geo.page_bytes, int(src.size()), st);
+        CUDA_OK(cudaFreeAsync(buf, st));
+        CUDA_OK(cudaStreamSynchronize(st));  // host vectors above are temporaries
+      }
+    } catch (...) {
+      for (auto& k : made) {
+        auto it = P.index.find(k);
+        if (it != P.index.end()) {
+          P.release_pages(it->second.pages);
+          P.index.erase(it);
+        }
+      }
+      throw;
+    }
+    if (n_fetched) *n_fetched = fetched;
+  });
+}
+
+
+// ------------------------------------------------------------------------ test-only
+bat_status bat_debug_gemm(int32_t epi, int32_t M, int32_t N, int32_t K, const void* A, const void* Bw,
+                          int64_t b_rows, void* out, int32_t ldo, const void* bias, int32_t up_row0,
+                          int32_t device, bat_stream_t stream) {
+  return guarded([&] {
+    BAT_REQUIRE(A && Bw && out && M >= 1 && N >= 1 && K >= 8 && K % 8 == 0, "argument");
+    BAT_REQUIRE(epi >= 0 && epi <= 3, "epi");
+    DeviceGuard dg(device);
+    int sms = 148;
+    CUDA_OK(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, device));
+    const CUtensorMap ta = make_tmap(A, M, K, K, 128);
+    const CUtensorMap tb = make_tmap(Bw, b_rows, K, K, epi == EPI_SWIGLU ? 128 : 256);
+    GemmParams gp{M, N, K, out, ldo, static_cast<const __nv_bfloat16*>(bias), up_row0};
+    launch_gemm(epi, ta, tb, gp, sms, static_cast<cudaStream_t>(stream));
+    CUDA_OK(cudaGetLastError());
+  });
+}
+
+bat_status bat_debug_attention_layer(bat_pool p, bat_model mdl, const bat_query* queries, int32_t B,
+                                     int32_t layer, const void* qkv, void* out_o, int32_t rope_enabled,
+                                     bat_stream_t stream) {
+  return guarded([&] {
+    BAT_REQUIRE(p && mdl && queries && qkv && out_o && B >= 1, "argument");
+    Pool& P = p->pool;
+    Model& m = mdl->m;
+    check_compat(P, m);
+    BAT_REQUIRE(layer >= 0 && layer < m.cfg.layers, "layer");
+    DeviceGuard dg(P.device);
+    cudaStream_t st = static_cast<cudaStream_t>(stream);
+    Plan plan;
+    build_plan(P, m.cfg.q_heads / m.cfg.kv_heads, m.cfg.kv_heads, wrap(queries, B), plan, true);
+    const int32_t* I = prepare(P, m, plan, st);
+    StageParams sp = stage_params(P, m, plan, I);
+    sp.qkv = static_cast<const __nv_bfloat16*>(qkv);
+    sp.rope_enabled = rope_enabled;
+    sp.pool_layer_off = int64_t(layer) * P.geo.layer_bytes;
+    launch_stage(sp, st);
+    AttnParams ap = attn_params(P, m, plan, I);
+    ap.pool_layer_off = int64_t(layer) * P.geo.layer_bytes;
+    ap.out = static_cast<__nv_bfloat16*>(out_o);
+    launch_attention(m.dpad, ap, m.num_sms, st);
+    CUDA_OK(cudaGetLastError());
+    CUDA_OK(cudaStreamSynchronize(st));
+  });
+}
+
+}  // extern "C"

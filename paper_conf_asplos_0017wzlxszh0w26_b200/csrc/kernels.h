@@ -1,0 +1,97 @@
+// Launchers of libbat's device kernels (all sm_100a).  Every launcher bumps the launch
+// counter reported by bat_kernel_launch_count().
+#pragma once
+
+#include <cuda.h>
+#include <cuda_bf16.h>
+#include <cuda_runtime.h>
+#include <cstdint>
+
+namespace bat {
+
+void count_launch(int n = 1);
+int64_t launch_count();
+
+// ------------------------------------------------------------------------ tcgen05 GEMM
+enum GemmEpi { EPI_BF16 = 0, EPI_BF16_BIAS = 1, EPI_RESID_F32 = 2, EPI_SWIGLU = 3 };
+struct GemmParams {
+  int M, N, K;        // N = output columns (SWIGLU: the ffn width F)
+  void* out;          // bf16 [M][ldo] or fp32 residual [M][ldo]
+  int ldo;
+  const __nv_bfloat16* bias;  // EPI_BF16_BIAS
+  int up_row0;        // EPI_SWIGLU: first "up" row of B (= F)
+};
+size_t gemm_smem_bytes();
+void launch_gemm(int epi, const CUtensorMap& tmA, const CUtensorMap& tmB, const GemmParams& p,
+                 int num_sms, cudaStream_t stream);
+
+// ------------------------------------------------------------------ bipartite attention
+struct AttnParams {
+  const int32_t* img;       // plan image (device)
+  int64_t off_qinfo, off_pages, off_kmeta, off_rseg, off_work;
+  int32_t n_work;
+  const char* pool;         // arena; page p, layer l at pool + p*pool_page_bytes + pool_layer_off
+  int64_t pool_page_bytes, pool_layer_off;
+  const char* scratch;      // suffix pages; page s at scratch + s*scratch_page_bytes + scratch_layer_off
+  int64_t scratch_page_bytes, scratch_layer_off;
+  const char* zero_page;    // all-zero K/V block source for page-list padding
+  int64_t head_bytes;       // bytes of one head's K (or V) in a page-layer block
+  int32_t kv_heads, group, qt, head_dim, ldo;
+  const __nv_bfloat16* qp;  // packed, swizzled q-tiles
+  __nv_bfloat16* out;       // O [M][q_heads*head_dim]
+  float scale_log2;         // log2(e) / sqrt(head_dim)
+};
+size_t attn_smem_bytes(int dpad);
+void launch_attention(int dpad, const AttnParams& p, int num_sms, cudaStream_t stream);
+
+// --------------------------------------------------------------------- small kernels
+void launch_embed(const __nv_bfloat16* E, const int32_t* tok, float* h, int M, int H,
+                  cudaStream_t s);
+// y = x * rsqrt(mean(x^2) + eps) * g  (rows given by idx when idx != nullptr)
+void launch_rmsnorm_bf16(const float* x, const __nv_bfloat16* g, __nv_bfloat16* y, int M, int H,
+                         float eps, cudaStream_t s);
+void launch_rmsnorm_f32out(const float* x, const __nv_bfloat16* g, float* y, int M, int H,
+                           float eps, cudaStream_t s);
+void launch_rope_table(float2* tab, int max_pos, int d, double theta, cudaStream_t s);
+
+struct StageParams {
+  const __nv_bfloat16* qkv;  // [M][(Hq+2Hkv)*d]
+  const int32_t* img;
+  int64_t off_pos, off_qinfo, off_qtiles, off_spages;
+  int32_t n_qtiles, n_spages;
+  const float2* rope;        // [max_pos][d/2] (cos, sin)
+  int32_t rope_enabled, max_pos;
+  int32_t q_heads, kv_heads, head_dim, dpad, group, qt;
+  __nv_bfloat16* qp;         // q-tiles out
+  char* pool;                // target pages: pool page p (>= 0) or scratch page s (-(s+1))
+  int64_t pool_page_bytes, pool_layer_off;
+  char* scratch;
+  int64_t scratch_page_bytes, scratch_layer_off;
+  int64_t head_bytes;
+};
+void launch_stage(const StageParams& p, cudaStream_t s);
+
+void launch_gather_rows_bf16(const __nv_bfloat16* src, const int32_t* idx, __nv_bfloat16* dst,
+                             int n, int cols, cudaStream_t s);
+void launch_gather_rows_f32(const float* src, const int32_t* idx, float* dst, int n, int cols,
+                            cudaStream_t s);
+void launch_score(const float* hidden, const __nv_bfloat16* w_out, const int32_t* labels,
+                  const int32_t* n_items, int B, int n_max, int H, float* scores, int k,
+                  int32_t* topk, cudaStream_t s);
+
+// KV pool page scatter / gather in the swizzled page layout (bf16)
+struct PageIO {
+  char* arena;
+  int64_t page_bytes, layer_bytes, head_bytes;
+  int32_t layers, kv_heads, head_dim;
+};
+void launch_kv_scatter(const PageIO& io, const __nv_bfloat16* k, const __nv_bfloat16* v,
+                       const int32_t* pages_dev, int n_tokens, int slot0, int n_total,
+                       cudaStream_t s);
+void launch_kv_gather(const PageIO& io, __nv_bfloat16* k, __nv_bfloat16* v,
+                      const int32_t* pages_dev, int n_tokens, cudaStream_t s);
+// copy whole pages: dst_arena page dst[i] <- src_ptrs[i] (peer-mapped)
+void launch_page_copy(const uint64_t* src_ptrs, const int32_t* dst_pages, char* dst_arena,
+                      int64_t page_bytes, int n, cudaStream_t s);
+
+}  // namespace bat

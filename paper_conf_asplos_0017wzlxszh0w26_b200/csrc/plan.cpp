@@ -1,0 +1,342 @@
+// Host planner: see plan.h.  The visibility rule (DESIGN.md §2 R4-R6):
+//   key k is visible to suffix row t  iff  kord[k] <= rord[t]  and
+//   (kseg[k] == rseg[t]  or  kseg[k] < 0  or  rseg[t] < 0)
+// with kord = 0 for a prefix key (every prefix token precedes every suffix token), the suffix
+// index + 1 for a suffix key, INT32_MAX for an empty slot; rord[t] = t + 1.
+#include "plan.h"
+
+#include <algorithm>
+#include <numeric>
+#include <unordered_map>
+
+namespace bat {
+namespace {
+
+struct PrefixEnt {
+  int32_t kind;
+  int64_t id;
+  int32_t seg;
+  int32_t expect_n;  // tokens the request carries for it (-1: unchecked)
+};
+
+void add_prefix_pages(const Pool& pool, const PrefixEnt& e, QueryPlan& qp) {
+  const Entity* ent = pool.find(e.kind, e.id);
+  if (!ent) {
+    fail(BAT_E_NOTFOUND, "prefix entry (kind " + std::to_string(e.kind) + ", id " +
+                             std::to_string(e.id) + ") is not in the pool");
+  }
+  if (e.expect_n >= 0 && ent->n_tokens != e.expect_n) {
+    fail(BAT_E_INVAL, "prefix entry (kind " + std::to_string(e.kind) + ", id " +
+                          std::to_string(e.id) + ") holds " + std::to_string(ent->n_tokens) +
+                          " tokens but the request has " + std::to_string(e.expect_n));
+  }
+  for (size_t pi = 0; pi < ent->pages.size(); ++pi) {
+    int32_t nv = std::min<int32_t>(kPageTokens, ent->n_tokens - static_cast<int32_t>(pi) * kPageTokens);
+    qp.pages.push_back(ent->pages[pi]);
+    qp.valid.push_back(nv);
+    for (int j = 0; j < kPageTokens; ++j) {
+      qp.kseg.push_back(j < nv ? e.seg : -1);
+      qp.kord.push_back(j < nv ? 0 : kInvalidOrd);
+    }
+  }
+  qp.P += ent->n_tokens;
+}
+
+// Suffix tokens / positions / segments of a ranking request (readings R2, R3).
+void build_request(const Pool& pool, const bat_query& q, QueryPlan& qp) {
+  BAT_REQUIRE(q.order == BAT_ORDER_UP || q.order == BAT_ORDER_IP, "order must be UP or IP");
+  BAT_REQUIRE(q.n_items >= 1, "n_items >= 1");
+  BAT_REQUIRE(q.n_instr >= 1, "n_instr >= 1 (the discriminant is the last token, P:173)");
+  BAT_REQUIRE(q.n_user >= 0 && q.n_header >= 0, "negative length");
+  BAT_REQUIRE(q.n_header == 0 || q.order == BAT_ORDER_IP, "header tokens are IP-only (P:257)");
+  BAT_REQUIRE(q.item_off && q.item_id, "item arrays");
+  BAT_REQUIRE(q.n_user == 0 || q.user_tok, "user_tok");
+  BAT_REQUIRE(q.instr_tok, "instr_tok");
+  BAT_REQUIRE(q.n_header == 0 || q.header_tok, "header_tok");
+  BAT_REQUIRE(q.item_off[0] == 0, "item_off[0] == 0");
+  int32_t m = 0;
+  for (int i = 0; i < q.n_items; ++i) {
+    int32_t n = q.item_off[i + 1] - q.item_off[i];
+    BAT_REQUIRE(n >= 1, "every item has >= 1 token");
+    m = std::max(m, n);
+  }
+  const int32_t nu = q.n_user, nx = q.n_instr, h = q.n_header;
+  auto put = [&](const int32_t* t, int32_t n, int32_t seg, int32_t pos0) {
+    for (int32_t j = 0; j < n; ++j) {
+      qp.tokens.push_back(t[j]);
+      qp.seg.push_back(seg);
+      qp.pos.push_back(pos0 + j);
+    }
+  };
+  auto put_items = [&](int32_t start) {
+    for (int i = 0; i < q.n_items; ++i)
+      put(q.item_tok + q.item_off[i], q.item_off[i + 1] - q.item_off[i], i, start);
+  };
+  if (q.order == BAT_ORDER_UP) {
+    if (q.use_cache) {
+      add_prefix_pages(pool, PrefixEnt{BAT_ENT_USER, q.user_id, SEG_USER, nu}, qp);
+    } else {
+      put(q.user_tok, nu, SEG_USER, 0);
+    }
+    put_items(nu);
+    put(q.instr_tok, nx, SEG_INSTR, nu + m);
+  } else {
+    if (q.use_cache) {
+      if (h > 0) add_prefix_pages(pool, PrefixEnt{BAT_ENT_HEADER, q.header_id, SEG_HEADER, h}, qp);
+      for (int i = 0; i < q.n_items; ++i)
+        add_prefix_pages(pool, PrefixEnt{BAT_ENT_ITEM, q.item_id[i], i, q.item_off[i + 1] - q.item_off[i]}, qp);
+    } else {
+      put(q.header_tok, h, SEG_HEADER, 0);
+      put_items(h);
+    }
+    put(q.user_tok, nu, SEG_USER, h + m);
+    put(q.instr_tok, nx, SEG_INSTR, h + m + nu);
+  }
+  qp.n_prefix_pages = static_cast<int32_t>(qp.pages.size());
+  qp.S = static_cast<int32_t>(qp.tokens.size());
+}
+
+void build_entity(const Pool& pool, const PlanRequest& r, QueryPlan& qp) {
+  if (r.ctx_kind >= 0) add_prefix_pages(pool, PrefixEnt{r.ctx_kind, r.ctx_id, SEG_HEADER, -1}, qp);
+  for (int32_t j = 0; j < r.ent_n; ++j) {
+    qp.tokens.push_back(r.ent_tok[j]);
+    qp.seg.push_back(SEG_USER);  // one entity alone: plain causal attention
+    qp.pos.push_back(r.ent_pos0 + j);
+  }
+  qp.n_prefix_pages = static_cast<int32_t>(qp.pages.size());
+  qp.S = r.ent_n;
+}
+
+// Exact block-skip states by per-tile summaries (matches the oracle's pair enumeration).
+void classify_tiles(QueryPlan& qp, int32_t qt) {
+  const int32_t n_slots = qp.n_pages * kPageTokens;
+  qp.n_ktiles = static_cast<int32_t>(ceil_div(n_slots, kKtile));
+  qp.n_qtiles = static_cast<int32_t>(ceil_div(qp.S, qt));
+  constexpr int32_t INF = kInvalidOrd;
+  struct KT {
+    int32_t min_all = INF, max_all = -1, min_nonitem = INF;
+    bool all_valid = true;
+    std::vector<std::pair<int32_t, int32_t>> item_min;  // (item, min kord), item ascending
+  };
+  std::vector<KT> kts(qp.n_ktiles);
+  for (int32_t j = 0; j < qp.n_ktiles; ++j) {
+    KT& k = kts[j];
+    for (int32_t s = j * kKtile; s < (j + 1) * kKtile; ++s) {
+      if (s >= n_slots || qp.kord[s] == kInvalidOrd) {
+        k.all_valid = false;
+        continue;
+      }
+      int32_t o = qp.kord[s], g = qp.kseg[s];
+      k.min_all = std::min(k.min_all, o);
+      k.max_all = std::max(k.max_all, o);
+      if (g < 0) {
+        k.min_nonitem = std::min(k.min_nonitem, o);
+      } else {
+        auto it = std::lower_bound(k.item_min.begin(), k.item_min.end(), std::make_pair(g, INT32_MIN));
+        if (it != k.item_min.end() && it->first == g) it->second = std::min(it->second, o);
+        else k.item_min.insert(it, {g, o});
+      }
+    }
+  }
+  qp.tiles.assign(static_cast<size_t>(qp.n_qtiles) * qp.n_ktiles, 0);
+  std::vector<std::pair<int32_t, int32_t>> row_items;  // (item, max rord)
+  for (int32_t i = 0; i < qp.n_qtiles; ++i) {
+    const int32_t r0 = i * qt, r1 = std::min(qp.S, (i + 1) * qt);
+    const int32_t rmin = r0 + 1;
+    int32_t rn_max = -1;
+    row_items.clear();
+    for (int32_t t = r0; t < r1; ++t) {
+      int32_t g = qp.seg[t];
+      if (g < 0) {
+        rn_max = std::max(rn_max, t + 1);
+      } else {
+        if (!row_items.empty() && row_items.back().first == g) row_items.back().second = t + 1;
+        else {
+          auto it = std::find_if(row_items.begin(), row_items.end(), [&](auto& p) { return p.first == g; });
+          if (it == row_items.end()) row_items.push_back({g, t + 1});
+          else it->second = std::max(it->second, t + 1);
+        }
+      }
+    }
+    for (int32_t j = 0; j < qp.n_ktiles; ++j) {
+      const KT& k = kts[j];
+      bool any = rn_max >= 0 && k.min_all <= rn_max;
+      for (size_t a = 0; !any && a < row_items.size(); ++a) {
+        int32_t mm = k.min_nonitem;
+        auto it = std::lower_bound(k.item_min.begin(), k.item_min.end(),
+                                   std::make_pair(row_items[a].first, INT32_MIN));
+        if (it != k.item_min.end() && it->first == row_items[a].first) mm = std::min(mm, it->second);
+        any = mm <= row_items[a].second;
+      }
+      uint8_t st = 0;
+      if (any) {
+        bool excl_free = row_items.empty() || k.item_min.empty() ||
+                         (row_items.size() == 1 && k.item_min.size() == 1 &&
+                          row_items[0].first == k.item_min[0].first);
+        bool full = k.all_valid && k.max_all <= rmin && excl_free;
+        st = full ? 1 : 2;
+      }
+      qp.tiles[static_cast<size_t>(i) * qp.n_ktiles + j] = st;
+    }
+  }
+  // visible pairs per head per layer, O(S + slots): count per row
+  int64_t pre_nonitem = 0;
+  std::unordered_map<int32_t, int64_t> pre_item;
+  for (int32_t s = 0; s < qp.n_prefix_pages * kPageTokens; ++s) {
+    if (qp.kord[s] == kInvalidOrd) continue;
+    if (qp.kseg[s] < 0) ++pre_nonitem;
+    else ++pre_item[qp.kseg[s]];
+  }
+  const int64_t pre_total = qp.P;
+  int64_t sfx_nonitem = 0, live = 0;
+  std::unordered_map<int32_t, int64_t> sfx_item;
+  for (int32_t t = 0; t < qp.S; ++t) {
+    int32_t g = qp.seg[t];
+    if (g < 0) ++sfx_nonitem;
+    else ++sfx_item[g];
+    if (g < 0) {
+      live += pre_total + (t + 1);
+    } else {
+      auto pi = pre_item.find(g);
+      live += pre_nonitem + (pi == pre_item.end() ? 0 : pi->second) + sfx_nonitem + sfx_item[g];
+    }
+  }
+  qp.n_live_pairs = live;
+}
+
+}  // namespace
+
+void build_plan(const Pool& pool, int32_t group, int32_t kv_heads,
+                const std::vector<PlanRequest>& reqs, Plan& plan, bool build_image) {
+  BAT_REQUIRE(group >= 1 && group <= kQtileRows, "group in [1,128]");
+  plan.group = group;
+  plan.kv_heads = kv_heads;
+  plan.qt = kQtileRows / group;
+  plan.q.assign(reqs.size(), QueryPlan{});
+  int32_t tok = 0, sp = 0, qt0 = 0, pg = 0;
+  for (size_t b = 0; b < reqs.size(); ++b) {
+    QueryPlan& qp = plan.q[b];
+    const PlanRequest& r = reqs[b];
+    if (r.q) {
+      build_request(pool, *r.q, qp);
+    } else {
+      build_entity(pool, r, qp);
+      plan.entity_mode = true;
+    }
+    BAT_REQUIRE(qp.S >= 1, "request with no suffix tokens");
+    // the suffix's own pages follow the prefix pages (reading: virtual key order)
+    const int32_t n_sfx = static_cast<int32_t>(ceil_div(qp.S, kPageTokens));
+    if (r.ent_pages) BAT_REQUIRE(static_cast<int32_t>(r.ent_pages->size()) == n_sfx, "entity pages");
+    for (int32_t s = 0; s < n_sfx; ++s) {
+      int32_t nv = std::min(kPageTokens, qp.S - s * kPageTokens);
+      qp.pages.push_back(r.ent_pages ? (*r.ent_pages)[s] : -(sp + s) - 1);
+      qp.valid.push_back(nv);
+      for (int j = 0; j < kPageTokens; ++j) {
+        int32_t t = s * kPageTokens + j;
+        qp.kseg.push_back(j < nv ? qp.seg[t] : -1);
+        qp.kord.push_back(j < nv ? t + 1 : kInvalidOrd);
+      }
+    }
+    qp.n_pages = static_cast<int32_t>(qp.pages.size());
+    classify_tiles(qp, plan.qt);
+    qp.token_off = tok;
+    qp.scratch0 = sp;
+    qp.qtile0 = qt0;
+    qp.page_off = pg;
+    tok += qp.S;
+    sp += n_sfx;
+    qt0 += qp.n_qtiles;
+    pg += qp.n_ktiles * kKtilePages;
+  }
+  plan.M = tok;
+  plan.n_spages = sp;
+  plan.n_qtiles_total = qt0;
+  plan.n_pages_padded = pg;
+  if (!build_image) return;
+
+  // ---- flat device image --------------------------------------------------------------
+  const int32_t B = static_cast<int32_t>(plan.q.size());
+  PlanImage& im = plan.img;
+  std::vector<int32_t>& v = im.buf;
+  v.clear();
+  auto reserve_at = [&](int64_t n) {
+    int64_t o = static_cast<int64_t>(v.size());
+    o = (o + 3) & ~int64_t(3);  // 16-byte alignment of every array
+    v.resize(o + n, 0);
+    return o;
+  };
+  im.off_tok = reserve_at(plan.M);
+  im.off_pos = reserve_at(plan.M);
+  im.off_rseg = reserve_at(plan.M);
+  im.off_qinfo = reserve_at(int64_t(B) * 8);
+  im.off_pages = reserve_at(plan.n_pages_padded);
+  im.off_kmeta = reserve_at(int64_t(plan.n_pages_padded) * kPageTokens * 2);
+  im.off_qtiles = reserve_at(int64_t(plan.n_qtiles_total) * 4);
+  im.off_spages = reserve_at(int64_t(plan.n_spages) * 4);
+  im.off_disc = reserve_at(B);
+  for (int32_t b = 0; b < B; ++b) {
+    const QueryPlan& qp = plan.q[b];
+    for (int32_t t = 0; t < qp.S; ++t) {
+      v[im.off_tok + qp.token_off + t] = qp.tokens[t];
+      v[im.off_pos + qp.token_off + t] = qp.pos[t];
+      v[im.off_rseg + qp.token_off + t] = qp.seg[t];
+    }
+    int32_t* qi = &v[im.off_qinfo + int64_t(b) * 8];
+    qi[0] = qp.token_off; qi[1] = qp.S; qi[2] = qp.qtile0; qi[3] = qp.n_qtiles;
+    qi[4] = qp.page_off; qi[5] = qp.n_ktiles; qi[6] = qp.scratch0; qi[7] = qp.token_off + qp.S - 1;
+    for (int32_t p = 0; p < qp.n_ktiles * kKtilePages; ++p) {
+      bool real = p < qp.n_pages;
+      v[im.off_pages + qp.page_off + p] = real ? qp.pages[p] : kZeroPage;
+      for (int j = 0; j < kPageTokens; ++j) {
+        int64_t s = int64_t(p) * kPageTokens + j;
+        int64_t o = im.off_kmeta + (int64_t(qp.page_off) * kPageTokens + s) * 2;
+        v[o] = real ? qp.kseg[s] : -1;
+        v[o + 1] = real ? qp.kord[s] : kInvalidOrd;
+      }
+    }
+    for (int32_t i = 0; i < qp.n_qtiles; ++i) {
+      int32_t* e = &v[im.off_qtiles + int64_t(qp.qtile0 + i) * 4];
+      e[0] = b; e[1] = i * plan.qt; e[2] = std::min(plan.qt, qp.S - i * plan.qt); e[3] = 0;
+    }
+    const int32_t n_sfx = static_cast<int32_t>(ceil_div(qp.S, kPageTokens));
+    for (int32_t s = 0; s < n_sfx; ++s) {
+      int32_t* e = &v[im.off_spages + int64_t(qp.scratch0 + s) * 4];
+      e[0] = b; e[1] = s * kPageTokens; e[2] = std::min(kPageTokens, qp.S - s * kPageTokens);
+      e[3] = qp.pages[qp.n_prefix_pages + s];
+    }
+    v[im.off_disc + b] = qp.token_off + qp.S - 1;
+  }
+  // work items (b, kvh, q-tile) with their live k-tiles, longest first (LPT over the SMs)
+  struct W { int32_t b, kvh, i, n; std::vector<int32_t> kt; };
+  auto make_work = [&](bool last_only, int64_t& off_work, int32_t& n_work) {
+    std::vector<W> ws;
+    for (int32_t b = 0; b < B; ++b) {
+      const QueryPlan& qp = plan.q[b];
+      for (int32_t i = last_only ? qp.n_qtiles - 1 : 0; i < qp.n_qtiles; ++i) {
+        std::vector<int32_t> kt;
+        for (int32_t j = 0; j < qp.n_ktiles; ++j) {
+          uint8_t st = qp.tiles[static_cast<size_t>(i) * qp.n_ktiles + j];
+          if (st) kt.push_back(j | (int32_t(st) << 24));
+        }
+        for (int32_t h = 0; h < kv_heads; ++h) ws.push_back(W{b, h, i, int32_t(kt.size()), kt});
+      }
+    }
+    std::stable_sort(ws.begin(), ws.end(), [](const W& a, const W& c) { return a.n > c.n; });
+    n_work = static_cast<int32_t>(ws.size());
+    off_work = reserve_at(int64_t(n_work) * 4);
+    int64_t total_kt = 0;
+    for (auto& w : ws) total_kt += w.n;
+    int64_t off_kt = reserve_at(total_kt);
+    int64_t cur = 0;
+    for (int32_t w = 0; w < n_work; ++w) {
+      int32_t* e = &v[off_work + int64_t(w) * 4];
+      e[0] = ws[w].b; e[1] = (ws[w].kvh << 16) | ws[w].i;
+      e[2] = static_cast<int32_t>(off_kt + cur); e[3] = ws[w].n;  // absolute offset into buf
+      for (int32_t x : ws[w].kt) v[off_kt + cur++] = x;
+    }
+  };
+  make_work(false, im.off_work, plan.n_work);
+  make_work(true, im.off_work_last, plan.n_work_last);
+}
+
+}  // namespace bat

@@ -1,0 +1,65 @@
+// Host planner: per request, the suffix tokens in prompt order, their
+// bipartite positions and segments, the key-slot list (prefix entries'
+// pages, then the suffix's own pages), key metadata, and the block-skip tile states
+// of every (packed q-tile, 128-key k-tile) pair; plus the flat device image the kernels read.
+#pragma once
+
+#include <cstdint>
+#include <vector>
+
+#include "common.h"
+#include "pool.h"
+
+namespace bat {
+
+struct QueryPlan {
+  int32_t S = 0, P = 0;
+  int32_t n_pages = 0, n_prefix_pages = 0, n_qtiles = 0, n_ktiles = 0;
+  int32_t token_off = 0, scratch0 = 0, qtile0 = 0, page_off = 0;
+  int64_t n_live_pairs = 0;
+  std::vector<int32_t> tokens, pos, seg;  // [S]
+  std::vector<int32_t> pages, valid;      // [n_pages]
+  std::vector<int32_t> kseg, kord;        // [16 * n_pages]
+  std::vector<uint8_t> tiles;             // [n_qtiles * n_ktiles]: 0 skip, 1 full, 2 partial
+};
+
+// One request description, independent of the C struct (entity prefill builds these too).
+struct PlanRequest {
+  const bat_query* q = nullptr;  // a ranking request, or
+  // an entity-prefill pseudo request: tokens at pos0.., causal, optional context entry,
+  // suffix pages = the new entry's own pool pages
+  const int32_t* ent_tok = nullptr;
+  int32_t ent_n = 0, ent_pos0 = 0;
+  int32_t ctx_kind = -1;
+  int64_t ctx_id = 0;
+  const std::vector<int32_t>* ent_pages = nullptr;
+};
+
+// Flat int32 image uploaded once per call; offsets (in int32 units) into it.
+struct PlanImage {
+  std::vector<int32_t> buf;
+  int64_t off_tok = 0, off_pos = 0, off_rseg = 0;   // [M]
+  int64_t off_qinfo = 0;                            // [B][8]
+  int64_t off_pages = 0;                            // [n_pages_padded_total]
+  int64_t off_kmeta = 0;                            // [16 * n_pages_padded_total][2]
+  int64_t off_qtiles = 0;                           // [n_qtiles_total][4] {b, t0, ntok, 0}
+  int64_t off_spages = 0;                           // [n_spages][4] {b, t0, ntok, target}
+  int64_t off_work = 0, off_work_last = 0;          // [W][4] {b, kvh<<16|qtile, kt_off, kt_n}
+  int64_t off_ktl = 0;                              // kt list: ktile | state << 24
+  int64_t off_disc = 0;                             // [B] global discriminant row
+};
+
+struct Plan {
+  int32_t group = 1, qt = 128, kv_heads = 1;
+  std::vector<QueryPlan> q;
+  int32_t M = 0, n_qtiles_total = 0, n_spages = 0, n_pages_padded = 0;
+  int32_t n_work = 0, n_work_last = 0;
+  bool entity_mode = false;
+  PlanImage img;
+};
+
+// Build the plan of a batch.  Pool supplies the entry -> pages index.  Throws bat::Error.
+void build_plan(const Pool& pool, int32_t group, int32_t kv_heads,
+                const std::vector<PlanRequest>& reqs, Plan& plan, bool build_image);
+
+}  // namespace bat

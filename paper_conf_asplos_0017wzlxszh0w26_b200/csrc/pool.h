@@ -1,0 +1,91 @@
+// Disaggregated paged KV pool: one page arena per GPU, entries at
+// user / item granularity, every entry a list of 16-token pages holding all layers.
+#pragma once
+
+#include <cstdint>
+#include <unordered_map>
+#include <vector>
+
+#include "common.h"
+
+namespace bat {
+
+struct EntityKey {
+  int32_t kind;
+  int64_t id;
+  bool operator==(const EntityKey& o) const { return kind == o.kind && id == o.id; }
+};
+struct EntityKeyHash {
+  size_t operator()(const EntityKey& k) const {
+    uint64_t x = static_cast<uint64_t>(k.id) * 0x9E3779B97F4A7C15ull ^ static_cast<uint64_t>(k.kind);
+    x ^= x >> 29;
+    return static_cast<size_t>(x * 0xBF58476D1CE4E5B9ull);
+  }
+};
+
+struct Entity {
+  int32_t n_tokens = 0;
+  std::vector<int32_t> pages;
+  bool fetched = false;  // a local copy of a remote (cold-sharded) entry
+};
+
+struct RemoteEntity {
+  int32_t owner = -1;
+  int32_t n_tokens = 0;
+  std::vector<int32_t> pages;  // page ids in the owner's arena
+};
+
+// Page layout (bf16): page = [layers][2 (K,V)][kv_heads][Dp/64][16 slots][64] with the
+// 128-byte swizzle of the tensor-core operand layout applied inside each 2 KB block
+// ([16][64] bf16): element (slot r, col c) sits at r*128 + (((c/8) ^ (r%8)) * 16) + (c%8)*2.
+// A page's K (or V) rows for one head and one layer are therefore (Dp/64) contiguous 2 KB
+// blocks that a bulk copy drops into shared memory ready for tcgen05.mma.
+struct PageGeometry {
+  int32_t layers = 0, kv_heads = 0, head_dim = 0, dpad = 0;
+  int64_t block_bytes = 2048;  // [16][64] bf16
+  int64_t head_bytes = 0;      // (dpad/64) blocks
+  int64_t layer_bytes = 0;     // 2 * kv_heads * head_bytes
+  int64_t page_bytes = 0;      // layers * layer_bytes
+  void init(int L, int hkv, int d) {
+    layers = L;
+    kv_heads = hkv;
+    head_dim = d;
+    dpad = head_dim_pad(d);
+    head_bytes = (dpad / 64) * block_bytes;
+    layer_bytes = 2 * kv_heads * head_bytes;
+    page_bytes = layers * layer_bytes;
+  }
+};
+
+struct Pool {
+  bat_pool_cfg cfg{};
+  bool index_only = false;
+  int device = -1;
+  PageGeometry geo;
+  char* arena = nullptr;  // num_pages + 1 pages; page num_pages is the all-zero page
+  int32_t zero_page = 0;
+  std::vector<int32_t> free_pages;
+  std::unordered_map<EntityKey, Entity, EntityKeyHash> index;
+  std::unordered_map<EntityKey, RemoteEntity, EntityKeyHash> remote;
+  std::vector<char*> peer_arena;  // by rank (IPC-mapped), nullptr for self / unattached
+  uint64_t ipc_handle[8] = {0};
+
+  const Entity* find(int32_t kind, int64_t id) const {
+    auto it = index.find(EntityKey{kind, id});
+    return it == index.end() ? nullptr : &it->second;
+  }
+  // allocate n pages (all-or-nothing)
+  bool alloc_pages(int64_t n, std::vector<int32_t>& out) {
+    if (static_cast<int64_t>(free_pages.size()) < n) return false;
+    for (int64_t i = 0; i < n; ++i) {
+      out.push_back(free_pages.back());
+      free_pages.pop_back();
+    }
+    return true;
+  }
+  void release_pages(const std::vector<int32_t>& pages) {
+    for (auto it = pages.rbegin(); it != pages.rend(); ++it) free_pages.push_back(*it);
+  }
+};
+
+}  // namespace bat

@@ -1,0 +1,142 @@
+"""Device-memory helpers around the C ABI (PyTorch used only for memory and streams).
+
+``DeviceModel`` uploads a weight set to bf16 device tensors in the layout of include/bat.h
+and owns the ``bat_model`` handle; ``DevicePool`` owns a ``bat_pool``.  Neither computes any
+step of the method.
+"""
+from __future__ import annotations
+
+from typing import Dict, List, Optional
+
+import numpy as np
+
+from . import bat
+
+LAYER_KEYS = ("ln1", "wqkv", "bqkv", "wo", "ln2", "wgu", "wd")
+
+
+def _torch():
+    import torch
+    return torch
+
+
+class DeviceModel:
+    """Weights (bf16, device) + the library's model handle.
+
+    ``source`` is any object with ``cfg`` (dict), ``embed_full()``, ``lm_head_full()``,
+    ``final_norm()`` and ``layer(l)`` returning the 7 per-layer arrays, or
+    ``tensors=`` a dict {"embed", "lm_head" (optional: tied), "final_norm", "layers": [...]}
+    of device tensors already in bf16."""
+
+    def __init__(self, cfg: dict, source=None, tensors: Optional[dict] = None, device: int = 0):
+        torch = _torch()
+        self.cfg = dict(cfg)
+        self.device = device
+        dev = torch.device("cuda", device)
+        to = lambda a: torch.as_tensor(np.asarray(a, dtype=np.float32)).to(dev, torch.bfloat16).contiguous()
+        if tensors is None:
+            embed = to(source.embed_full())
+            lm = embed if cfg.get("tied") else to(source.lm_head_full())
+            fin = to(source.final_norm())
+            layers = []
+            for l in range(cfg["layers"]):
+                w = source.layer(l)
+                layers.append({k: to(w[k]) for k in LAYER_KEYS})
+            tensors = dict(embed=embed, lm_head=lm, final_norm=fin, layers=layers)
+        if tensors.get("lm_head") is None:
+            tensors["lm_head"] = tensors["embed"]
+        self.t = tensors
+        ptrs = [tensors["embed"].data_ptr(), tensors["lm_head"].data_ptr(), tensors["final_norm"].data_ptr()]
+        for lw in tensors["layers"]:
+            ptrs += [lw[k].data_ptr() for k in LAYER_KEYS]
+        self.handle = bat.bat_model_create(cfg, ptrs, device)
+
+    def close(self):
+        if self.handle:
+            bat.bat_model_destroy(self.handle)
+            self.handle = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+
+class DevicePool:
+    def __init__(self, cfg: dict, num_pages: int, device: int = 0, rank: int = 0, world: int = 1):
+        self.cfg = dict(cfg)
+        self.device = device
+        self.handle = bat.bat_kv_pool_create(device, num_pages, cfg["layers"], cfg["kv_heads"],
+                                             cfg["head_dim"], rank=rank, world=world)
+
+    def close(self):
+        if self.handle:
+            bat.bat_kv_pool_destroy(self.handle)
+            self.handle = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+
+def needed_entities(queries) -> Dict[tuple, np.ndarray]:
+    """The (kind, id) -> tokens of every prefix entry a batch of cached requests needs
+    (UP: the user; IP: header + items) — bookkeeping only."""
+    out: Dict[tuple, np.ndarray] = {}
+    for q in queries:
+        if not q.use_cache:
+            continue
+        if q.order == "UP":
+            out[(bat.BAT_ENT_USER, int(q.user_id))] = np.asarray(q.user_tok, np.int32)
+        else:
+            if len(q.header_tok):
+                out[(bat.BAT_ENT_HEADER, int(q.header_id))] = np.asarray(q.header_tok, np.int32)
+            for iid, t in zip(q.item_ids, q.item_toks):
+                out[(bat.BAT_ENT_ITEM, int(iid))] = np.asarray(t, np.int32)
+    return out
+
+
+def prefill_missing_entities(pool: DevicePool, model: DeviceModel, queries, stream=None,
+                             batch: int = 256) -> int:
+    """Compute and cache every prefix entry the batch needs that the pool lacks (the
+    prefix-miss path), through bat_kv_prefill_entities.  Returns the count."""
+    ents = needed_entities(queries)
+    n = 0
+    headers = {k: v for k, v in ents.items() if k[0] == bat.BAT_ENT_HEADER}
+    for (kind, eid), toks in headers.items():
+        try:
+            bat.bat_kv_lookup(pool.handle, kind, eid)
+            continue
+        except bat.BatError:
+            pass
+        bat.bat_kv_prefill_entities(pool.handle, model.handle, kind, [eid], [toks], 0, stream=stream)
+        n += 1
+    hdr_len = {int(q.header_id): len(q.header_tok) for q in queries if q.order == "IP" and len(q.header_tok)}
+    for kind in (bat.BAT_ENT_USER, bat.BAT_ENT_ITEM):
+        todo = []
+        for (k, eid), toks in ents.items():
+            if k != kind:
+                continue
+            try:
+                bat.bat_kv_lookup(pool.handle, kind, eid)
+            except bat.BatError:
+                todo.append((eid, toks))
+        # items with a header context are grouped by header
+        groups: Dict[int, List] = {}
+        for eid, toks in todo:
+            groups.setdefault(-1, []).append((eid, toks))
+        for _, lst in groups.items():
+            for s in range(0, len(lst), batch):
+                chunk = lst[s:s + batch]
+                if kind == bat.BAT_ENT_ITEM and hdr_len:
+                    hid, hl = next(iter(hdr_len.items()))
+                    bat.bat_kv_prefill_entities(pool.handle, model.handle, kind, [e for e, _ in chunk],
+                                                [t for _, t in chunk], hl, bat.BAT_ENT_HEADER, hid, stream)
+                else:
+                    bat.bat_kv_prefill_entities(pool.handle, model.handle, kind, [e for e, _ in chunk],
+                                                [t for _, t in chunk], 0, stream=stream)
+                n += len(chunk)
+    return n

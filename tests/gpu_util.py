@@ -1,0 +1,62 @@
+"""Helpers shared by the GPU tests (marshalling and reference assembly only)."""
+from __future__ import annotations
+
+import numpy as np
+
+import synth
+from oracle import model as om
+from oracle.sequence import bipartite_mask, build_sequence
+
+
+def tol_ok(got, ref, atol=2e-2, rtol=2e-2):
+    got = np.asarray(got, np.float64)
+    ref = np.asarray(ref, np.float64)
+    return np.all(np.abs(got - ref) <= atol + rtol * np.abs(ref))
+
+
+def max_excess(got, ref, atol=2e-2, rtol=2e-2):
+    got = np.asarray(got, np.float64)
+    ref = np.asarray(ref, np.float64)
+    return float(np.max(np.abs(got - ref) - (atol + rtol * np.abs(ref))))
+
+
+def prefix_entities_in_order(q):
+    """(kind, id, tokens) of the prefix entries of a cached request, in prompt order."""
+    from paper_conf_asplos_0017wzlxszh0w26_b200 import bat
+    if not q.use_cache:
+        return []
+    if q.order == "UP":
+        return [(bat.BAT_ENT_USER, int(q.user_id), q.user_tok)]
+    out = []
+    if len(q.header_tok):
+        out.append((bat.BAT_ENT_HEADER, int(q.header_id), q.header_tok))
+    out += [(bat.BAT_ENT_ITEM, int(i), t) for i, t in zip(q.item_ids, q.item_toks)]
+    return out
+
+
+def oracle_attention_layer(cfg, q, entity_kv, qkv_rows, layer, rope_on=True):
+    """fp64 reference of one layer of bipartite attention for request q given the cached
+    prefix K/V (entity_kv[(kind,id)] = (K [L][n][Hkv][d], V)) and the suffix's raw qkv rows."""
+    d, Hq, Hkv = cfg["head_dim"], cfg["q_heads"], cfg["kv_heads"]
+    toks, seg, pos = build_sequence(q.order, q.user_tok, q.item_toks, q.instr_tok,
+                                    q.header_tok if q.order == "IP" else ())
+    ents = prefix_entities_in_order(q)
+    P = sum(len(t) for _, _, t in ents)
+    S = len(toks) - P
+    x = np.asarray(qkv_rows, np.float64)
+    assert x.shape[0] == S
+    qq = x[:, : Hq * d].reshape(S, Hq, d)
+    kk = x[:, Hq * d:(Hq + Hkv) * d].reshape(S, Hkv, d)
+    vv = x[:, (Hq + Hkv) * d:].reshape(S, Hkv, d)
+    if rope_on:
+        qq = om.rope(qq, pos[P:], cfg["rope_theta"])
+        kk = om.rope(kk, pos[P:], cfg["rope_theta"])
+    if ents:
+        Kp = np.concatenate([entity_kv[(k, i)][0][layer] for k, i, _ in ents]).astype(np.float64)
+        Vp = np.concatenate([entity_kv[(k, i)][1][layer] for k, i, _ in ents]).astype(np.float64)
+        K = np.concatenate([Kp, kk])
+        V = np.concatenate([Vp, vv])
+    else:
+        K, V = kk, vv
+    mask = bipartite_mask(seg)[P:, :]
+    return om.attention(qq, K, V, mask, Hq // Hkv)

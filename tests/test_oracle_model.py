@@ -192,6 +192,17 @@ def test_mask_sensitivity_guard(W, order):
     assert np.max(np.abs(good["z"] - bad["z"])) > 10 * 2e-2
 
 
+@pytest.mark.parametrize("order", ["UP", "IP"])
+def test_mask_sensitivity_guard_small_gqa6(order):
+    """Same guard at the Qwen-like "small" GPU-parity config (g = 6, d = 128, init 0.02)."""
+    cfg = synth.model_config("small")
+    Ws = synth.Weights(cfg, seed=1)
+    q = synth.make_query(3, cfg, 6, 100, list(range(200, 220)), (16, 16), 8, order)
+    good = om.run_query(cfg, Ws, q, "full")
+    bad = om.run_query(cfg, Ws, q, "full", mask_fn=lambda seg: causal_mask(len(seg)))
+    assert np.max(np.abs(good["z"] - bad["z"])) > 10 * 2e-2
+
+
 # ------------------------------------------------------------------------- attention
 def test_attention_dense_block_is_textbook_softmax():
     from scipy.special import softmax
