@@ -191,18 +191,42 @@ BAT_API bat_status bat_score(bat_model m, const float* hidden, const int32_t* la
                      int32_t k, int32_t* topk, bat_stream_t stream);
 
 /* ------------------------------------------------------------------------------------------
- * Plan introspection (host only; bit-exact checks against the oracle's plan)
+ * Planned execution: build (host) + upload (device, async on `stream`) the plan of a batch
+ * once, then run it any number of times — the same computation as bat_bipartite_prefill
+ * without the per-call planning and H2D upload.  The plan must be destroyed with
+ * bat_plan_destroy; it is invalidated when a referenced pool entry is evicted.
  * ---------------------------------------------------------------------------------------- */
 typedef struct bat_plan_s* bat_plan;
+BAT_API bat_status bat_plan_build(bat_pool p, bat_model m, const bat_query* queries, int32_t B,
+                                  bat_stream_t stream, bat_plan* out);
+BAT_API bat_status bat_prefill_plan(bat_pool p, bat_model m, bat_plan plan, float* out_hidden,
+                                    bat_stream_t stream);
+
+/* ------------------------------------------------------------------------------------------
+ * Kernel timing (CUDA events recorded on the launch stream around every kernel of the
+ * prefill, grouped by class).  bat_profile_read synchronises on the recorded events.
+ * ---------------------------------------------------------------------------------------- */
+enum { BAT_K_EMBED = 0, BAT_K_RMSNORM = 1, BAT_K_GEMM_QKV = 2, BAT_K_STAGE = 3, BAT_K_ATTN = 4,
+       BAT_K_GEMM_O = 5, BAT_K_GEMM_GU = 6, BAT_K_GEMM_DOWN = 7, BAT_K_OTHER = 8, BAT_K_N = 9 };
+BAT_API bat_status bat_profile_enable(bat_model m, int32_t on);
+/* Accumulated since the last reset: total ms, launches, algorithmic FLOPs (GEMMs 2MNK;
+ * attention 4 * head_dim * q_heads * visible pairs) and algorithmic bytes of class cls. */
+BAT_API bat_status bat_profile_read(bat_model m, int32_t cls, double* total_ms, int64_t* launches,
+                                    double* flops, double* bytes);
+BAT_API bat_status bat_profile_reset(bat_model m);
+
+/* ------------------------------------------------------------------------------------------
+ * Plan introspection (host only; bit-exact checks against the oracle's plan)
+ * ---------------------------------------------------------------------------------------- */
 /* group = q_heads / kv_heads of the model the plan is for (GQA packing of q-tiles). */
 BAT_API bat_status bat_plan_create(bat_pool p, int32_t group, const bat_query* queries, int32_t B,
                            bat_plan* out);
 BAT_API bat_status bat_plan_destroy(bat_plan plan);
-/* info[0..11] of request b: S (suffix tokens), P (prefix tokens), n_pages (incl. suffix
+/* info[0..12] of request b: S (suffix tokens), P (prefix tokens), n_pages (incl. suffix
  * pages, excl. padding), n_prefix_pages, n_qtiles, n_ktiles, token_off, scratch_page0,
  * n_live_pairs (visible (query,key) pairs, per head per layer), qtile_tokens,
- * first_qtile (global), page_off (global). */
-BAT_API bat_status bat_plan_query_info(bat_plan plan, int32_t b, int64_t info[12]);
+ * first_qtile (global), page_off (global), n_live_pairs of the last q-tile's rows. */
+BAT_API bat_status bat_plan_query_info(bat_plan plan, int32_t b, int64_t info[13]);
 enum {
   BAT_PF_TOKENS = 0,  /* int32 [S]  suffix token ids in prompt order */
   BAT_PF_POS = 1,     /* int32 [S]  position ids */
@@ -257,6 +281,9 @@ BAT_API bat_status bat_debug_gemm(int32_t epi, int32_t M, int32_t N, int32_t K, 
  * rope_enabled) to the given qkv rows (device bf16 [M][(q_heads+2 kv_heads) head_dim], rows
  * in plan order) and stage them, attend over the pool's prefix pages at that layer and the
  * staged suffix, write O (device bf16 [M][q_heads*head_dim]). */
+/* Attach another in-process pool's arena as peer `peer_rank` (single-GPU tests of the
+ * NVLink page pull; multi-process code uses bat_pool_ipc_handle / bat_pool_attach_peer). */
+BAT_API bat_status bat_debug_attach_peer_pool(bat_pool p, int32_t peer_rank, bat_pool other);
 BAT_API bat_status bat_debug_attention_layer(bat_pool p, bat_model m, const bat_query* queries,
                                              int32_t B, int32_t layer, const void* qkv,
                                              void* out_o, int32_t rope_enabled,

@@ -101,6 +101,13 @@ def lib() -> ctypes.CDLL:
         "bat_pool_attach_peer": (S, [c_void_p, c_int32, c_void_p]),
         "bat_kv_register_remote": (S, [c_void_p, c_int32, c_int64, c_int32, POINTER(c_int32), c_int32, c_int32]),
         "bat_kv_fetch": (S, [c_void_p, c_int32, POINTER(c_int64), c_int32, POINTER(c_int32), c_void_p]),
+        "bat_plan_build": (S, [c_void_p, c_void_p, POINTER(bat_query), c_int32, c_void_p, POINTER(c_void_p)]),
+        "bat_prefill_plan": (S, [c_void_p, c_void_p, c_void_p, c_void_p, c_void_p]),
+        "bat_profile_enable": (S, [c_void_p, c_int32]),
+        "bat_profile_read": (S, [c_void_p, c_int32, POINTER(c_double), POINTER(c_int64), POINTER(c_double),
+                                 POINTER(c_double)]),
+        "bat_profile_reset": (S, [c_void_p]),
+        "bat_debug_attach_peer_pool": (S, [c_void_p, c_int32, c_void_p]),
         "bat_debug_gemm": (S, [c_int32, c_int32, c_int32, c_int32, c_void_p, c_void_p, c_int64, c_void_p,
                                c_int32, c_void_p, c_int32, c_int32, c_void_p]),
         "bat_debug_attention_layer": (S, [c_void_p, c_void_p, POINTER(bat_query), c_int32, c_int32, c_void_p,
@@ -120,7 +127,9 @@ EXPORTED = ("bat_last_error", "bat_version", "bat_kernel_launch_count", "bat_mod
             "bat_kv_read", "bat_kv_prefill_entities", "bat_bipartite_prefill", "bat_score",
             "bat_plan_create", "bat_plan_destroy", "bat_plan_query_info", "bat_plan_export",
             "bat_hrcs_rmax", "bat_hrcs_place", "bat_pool_ipc_handle", "bat_pool_attach_peer",
-            "bat_kv_register_remote", "bat_kv_fetch", "bat_debug_gemm", "bat_debug_attention_layer")
+            "bat_kv_register_remote", "bat_kv_fetch", "bat_debug_gemm", "bat_debug_attention_layer",
+            "bat_plan_build", "bat_prefill_plan", "bat_profile_enable", "bat_profile_read",
+            "bat_profile_reset", "bat_debug_attach_peer_pool")
 
 
 def _check(status: int) -> None:
@@ -300,11 +309,11 @@ def bat_plan_destroy(plan: int) -> None:
 
 
 PLAN_INFO_KEYS = ("S", "P", "n_pages", "n_prefix_pages", "n_qtiles", "n_ktiles", "token_off",
-                  "scratch0", "n_live_pairs", "qtile_tokens", "qtile0", "page_off")
+                  "scratch0", "n_live_pairs", "qtile_tokens", "qtile0", "page_off", "n_live_pairs_last")
 
 
 def bat_plan_query_info(plan: int, b: int) -> dict:
-    info = (c_int64 * 12)()
+    info = (c_int64 * 13)()
     _check(lib().bat_plan_query_info(plan, b, info))
     return dict(zip(PLAN_INFO_KEYS, [int(x) for x in info]))
 
@@ -315,6 +324,39 @@ def bat_plan_export(plan: int, b: int, field: int) -> np.ndarray:
     out = np.zeros(max(n.value, 1), dtype=np.int32)
     _check(lib().bat_plan_export(plan, b, field, _i32p(out), len(out), byref(n)))
     return out[: n.value]
+
+
+# ---------------------------------------------------------------- planned execution
+def bat_plan_build(pool: int, model: int, queries: QueryArray, stream=None) -> int:
+    out = c_void_p()
+    _check(lib().bat_plan_build(pool, model, queries.arr, len(queries), _vp(stream), byref(out)))
+    return out.value
+
+
+def bat_prefill_plan(pool: int, model: int, plan: int, out_hidden, stream=None) -> None:
+    _check(lib().bat_prefill_plan(pool, model, plan, _vp(out_hidden), _vp(stream)))
+
+
+# ------------------------------------------------------------------------ profiling
+K_CLASSES = ("embed", "rmsnorm", "gemm_qkv", "stage", "attention", "gemm_o", "gemm_gate_up",
+             "gemm_down", "other")
+
+
+def bat_profile_enable(model: int, on: bool = True) -> None:
+    _check(lib().bat_profile_enable(model, 1 if on else 0))
+
+
+def bat_profile_read(model: int) -> dict:
+    out = {}
+    for i, name in enumerate(K_CLASSES):
+        ms, n, fl, by = c_double(), c_int64(), c_double(), c_double()
+        _check(lib().bat_profile_read(model, i, byref(ms), byref(n), byref(fl), byref(by)))
+        out[name] = dict(ms=ms.value, launches=n.value, flops=fl.value, bytes=by.value)
+    return out
+
+
+def bat_profile_reset(model: int) -> None:
+    _check(lib().bat_profile_reset(model))
 
 
 # ------------------------------------------------------------------- HRCS / multi-GPU
@@ -368,3 +410,7 @@ def bat_debug_attention_layer(pool: int, model: int, queries: QueryArray, layer:
                               rope_enabled: bool = True, stream=None) -> None:
     _check(lib().bat_debug_attention_layer(pool, model, queries.arr, len(queries), layer, _vp(qkv),
                                            _vp(out_o), 1 if rope_enabled else 0, _vp(stream)))
+
+
+def bat_debug_attach_peer_pool(pool: int, peer: int, other: int) -> None:
+    _check(lib().bat_debug_attach_peer_pool(pool, peer, other))

@@ -23,6 +23,11 @@ struct bat_pool_s {
 };
 struct bat_plan_s {
   bat::Plan plan;
+  void* dev_img = nullptr;  // device copy of plan.img (bat_plan_build)
+  int device = -1;
+  ~bat_plan_s() {
+    if (dev_img) cudaFree(dev_img);
+  }
 };
 
 namespace bat {
@@ -104,7 +109,72 @@ struct Workspace {
   }
 };
 
+// CUDA-event timing of every launch of the prefill, grouped by kernel class
+struct Profiler {
+  bool on = false;
+  struct Rec {
+    cudaEvent_t a, b;
+    int cls;
+    double flops, bytes;
+  };
+  std::vector<Rec> recs;
+  std::vector<cudaEvent_t> spare;
+  double ms[BAT_K_N] = {0}, flops[BAT_K_N] = {0}, bytes[BAT_K_N] = {0};
+  int64_t n[BAT_K_N] = {0};
+  cudaEvent_t ev() {
+    if (!spare.empty()) {
+      cudaEvent_t e = spare.back();
+      spare.pop_back();
+      return e;
+    }
+    cudaEvent_t e;
+    CUDA_OK(cudaEventCreate(&e));
+    return e;
+  }
+  void begin(cudaStream_t st) {
+    if (!on) return;
+    Rec r{ev(), nullptr, 0, 0, 0};
+    CUDA_OK(cudaEventRecord(r.a, st));
+    recs.push_back(r);
+  }
+  void end(cudaStream_t st, int cls, double fl, double by) {
+    if (!on) return;
+    Rec& r = recs.back();
+    r.b = ev();
+    r.cls = cls;
+    r.flops = fl;
+    r.bytes = by;
+    CUDA_OK(cudaEventRecord(r.b, st));
+  }
+  void collect() {
+    for (Rec& r : recs) {
+      CUDA_OK(cudaEventSynchronize(r.b));
+      float t = 0;
+      CUDA_OK(cudaEventElapsedTime(&t, r.a, r.b));
+      ms[r.cls] += t;
+      flops[r.cls] += r.flops;
+      bytes[r.cls] += r.bytes;
+      n[r.cls] += 1;
+      spare.push_back(r.a);
+      spare.push_back(r.b);
+    }
+    recs.clear();
+  }
+  void reset() {
+    collect();
+    for (int i = 0; i < BAT_K_N; ++i) ms[i] = flops[i] = bytes[i] = 0, n[i] = 0;
+  }
+  ~Profiler() {
+    for (Rec& r : recs) {
+      cudaEventDestroy(r.a);
+      if (r.b) cudaEventDestroy(r.b);
+    }
+    for (cudaEvent_t e : spare) cudaEventDestroy(e);
+  }
+};
+
 struct Model {
+  Profiler prof;
   bat_model_cfg cfg{};
   int device = 0, num_sms = 148, dpad = 128;
   const __nv_bfloat16 *embed = nullptr, *lm_head = nullptr, *final_norm = nullptr;
@@ -168,7 +238,8 @@ static void check_compat(const Pool& p, const Model& m) {
 }
 
 // Workspace sizing + plan upload; returns the device image.
-static const int32_t* prepare(Pool& pool, Model& m, Plan& plan, cudaStream_t st) {
+static const int32_t* prepare(Pool& pool, Model& m, Plan& plan, cudaStream_t st,
+                              const int32_t* dev_img = nullptr) {
   const bat_model_cfg& c = m.cfg;
   Workspace& ws = m.ws;
   const int M = plan.M, B = static_cast<int>(plan.q.size());
@@ -189,6 +260,7 @@ static const int32_t* prepare(Pool& pool, Model& m, Plan& plan, cudaStream_t st)
   ws.xc.ensure(size_t(B) * H * 2);
   ws.oc.ensure(size_t(B) * nq * 2);
   ws.actc.ensure(size_t(B) * F * 2);
+  if (dev_img) return dev_img;
   const size_t img_bytes = plan.img.buf.size() * 4;
   ws.img.ensure(img_bytes);
   if (!ws.img_done) CUDA_OK(cudaEventCreateWithFlags(&ws.img_done, cudaEventDisableTiming));
@@ -265,13 +337,27 @@ static StageParams stage_params(const Pool& pool, const Model& m, const Plan& pl
 }
 
 // Run the L layers over a planned batch (SURVEY §3 call stack (3)).
-static void run_plan(Pool& pool, Model& m, Plan& plan, float* out_hidden, cudaStream_t st) {
+static void run_plan(Pool& pool, Model& m, Plan& plan, float* out_hidden, cudaStream_t st,
+                     const int32_t* dev_img = nullptr) {
   const bat_model_cfg& c = m.cfg;
   Workspace& ws = m.ws;
   const int M = plan.M, B = static_cast<int>(plan.q.size());
   const int H = c.hidden, F = c.ffn, dp = m.dpad;
   const int nq = c.q_heads * c.head_dim;
-  const int32_t* I = prepare(pool, m, plan, st);
+  const int32_t* I = prepare(pool, m, plan, st, dev_img);
+  Profiler& pf = m.prof;
+  const double d_ = c.head_dim, Hq_ = c.q_heads, Hkv_ = c.kv_heads;
+  auto gemm_fb = [&](int Mr, int N, int K, int out_bytes) {
+    return std::make_pair(2.0 * Mr * N * K, 2.0 * (double(Mr) * K + double(N) * K) + double(out_bytes) * Mr * N);
+  };
+  double live_all = 0, live_last = 0, kv_slots = 0;
+  for (auto& q : plan.q) {
+    live_all += double(q.n_live_pairs);
+    live_last += double(q.n_live_pairs_last);
+    kv_slots += double(q.n_pages) * kPageTokens;
+  }
+  const double attn_fl = 4.0 * d_ * Hq_ * live_all, attn_fl_last = 4.0 * d_ * Hq_ * live_last;
+  const double attn_by = 2.0 * 2.0 * M * Hq_ * d_ + 2.0 * 2.0 * kv_slots * Hkv_ * d_;
   const PlanImage& im = plan.img;
 
   // tensor maps of this call's activations
@@ -284,44 +370,83 @@ static void run_plan(Pool& pool, Model& m, Plan& plan, float* out_hidden, cudaSt
   AttnParams ap = attn_params(pool, m, plan, I);
   StageParams sp = stage_params(pool, m, plan, I);
 
+  pf.begin(st);
   launch_embed(m.embed, I + im.off_tok, ws.h.as<float>(), M, H, st);
+  pf.end(st, BAT_K_EMBED, 0, 6.0 * M * H);
   for (int l = 0; l < c.layers; ++l) {
     const Model::Layer& Lw = m.layers[l];
     const bool last = (l == c.layers - 1);
+    pf.begin(st);
     launch_rmsnorm_bf16(ws.h.as<float>(), Lw.ln1, ws.xn.as<__nv_bfloat16>(), M, H, c.rms_eps, st);
+    pf.end(st, BAT_K_RMSNORM, 0, 6.0 * M * H);
     GemmParams gp{M, m.nqkv(), H, ws.qkv.p, m.nqkv(), Lw.bqkv, 0};
+    auto fq = gemm_fb(M, m.nqkv(), H, 2);
+    pf.begin(st);
     launch_gemm(EPI_BF16_BIAS, tA_xn, Lw.t_qkv, gp, m.num_sms, st);
+    pf.end(st, BAT_K_GEMM_QKV, fq.first, fq.second);
     sp.pool_layer_off = int64_t(l) * pool.geo.layer_bytes;
+    pf.begin(st);
     launch_stage(sp, st);
+    pf.end(st, BAT_K_STAGE, 0, 4.0 * M * m.nqkv());
     if (last && plan.entity_mode) break;  // entity prefill: only this layer's K/V are needed
     ap.pool_layer_off = int64_t(l) * pool.geo.layer_bytes;
     if (!last) {
       ap.off_work = im.off_work;
       ap.n_work = plan.n_work;
+      pf.begin(st);
       launch_attention(dp, ap, m.num_sms, st);
+      pf.end(st, BAT_K_ATTN, attn_fl, attn_by);
       GemmParams go{M, H, nq, ws.h.p, H, nullptr, 0};
+      auto fo = gemm_fb(M, H, nq, 8);
+      pf.begin(st);
       launch_gemm(EPI_RESID_F32, tA_o, Lw.t_o, go, m.num_sms, st);
+      pf.end(st, BAT_K_GEMM_O, fo.first, fo.second);
+      pf.begin(st);
       launch_rmsnorm_bf16(ws.h.as<float>(), Lw.ln2, ws.xn.as<__nv_bfloat16>(), M, H, c.rms_eps, st);
+      pf.end(st, BAT_K_RMSNORM, 0, 6.0 * M * H);
       GemmParams gg{M, F, H, ws.act.p, F, nullptr, F};
+      auto fg = gemm_fb(M, 2 * F, H, 1);
+      pf.begin(st);
       launch_gemm(EPI_SWIGLU, tA_xn, Lw.t_gu, gg, m.num_sms, st);
+      pf.end(st, BAT_K_GEMM_GU, fg.first, fg.second);
       GemmParams gd{M, H, F, ws.h.p, H, nullptr, 0};
+      auto fd = gemm_fb(M, H, F, 8);
+      pf.begin(st);
       launch_gemm(EPI_RESID_F32, tA_act, Lw.t_d, gd, m.num_sms, st);
+      pf.end(st, BAT_K_GEMM_DOWN, fd.first, fd.second);
     } else {
       // a8: after the last layer's K/V only the discriminant rows matter
       ap.off_work = im.off_work_last;
       ap.n_work = plan.n_work_last;
+      pf.begin(st);
       launch_attention(dp, ap, m.num_sms, st);
+      pf.end(st, BAT_K_ATTN, attn_fl_last, attn_by);
       const int32_t* disc = I + im.off_disc;
+      pf.begin(st);
       launch_gather_rows_bf16(ws.o.as<__nv_bfloat16>(), disc, ws.oc.as<__nv_bfloat16>(), B, nq, st);
       launch_gather_rows_f32(ws.h.as<float>(), disc, ws.hc.as<float>(), B, H, st);
+      pf.end(st, BAT_K_OTHER, 0, 2.0 * B * (2.0 * nq + 4.0 * H));
       GemmParams go{B, H, nq, ws.hc.p, H, nullptr, 0};
+      auto fo = gemm_fb(B, H, nq, 8);
+      pf.begin(st);
       launch_gemm(EPI_RESID_F32, tA_oc, Lw.t_o, go, m.num_sms, st);
+      pf.end(st, BAT_K_GEMM_O, fo.first, fo.second);
+      pf.begin(st);
       launch_rmsnorm_bf16(ws.hc.as<float>(), Lw.ln2, ws.xc.as<__nv_bfloat16>(), B, H, c.rms_eps, st);
+      pf.end(st, BAT_K_RMSNORM, 0, 6.0 * B * H);
       GemmParams gg{B, F, H, ws.actc.p, F, nullptr, F};
+      auto fg = gemm_fb(B, 2 * F, H, 1);
+      pf.begin(st);
       launch_gemm(EPI_SWIGLU, tA_xc, Lw.t_gu, gg, m.num_sms, st);
+      pf.end(st, BAT_K_GEMM_GU, fg.first, fg.second);
       GemmParams gd{B, H, F, ws.hc.p, H, nullptr, 0};
+      auto fd = gemm_fb(B, H, F, 8);
+      pf.begin(st);
       launch_gemm(EPI_RESID_F32, tA_actc, Lw.t_d, gd, m.num_sms, st);
+      pf.end(st, BAT_K_GEMM_DOWN, fd.first, fd.second);
+      pf.begin(st);
       launch_rmsnorm_f32out(ws.hc.as<float>(), m.final_norm, out_hidden, B, H, c.rms_eps, st);
+      pf.end(st, BAT_K_OTHER, 0, 8.0 * B * H);
     }
   }
   CUDA_OK(cudaGetLastError());
@@ -429,6 +554,7 @@ bat_status bat_kv_pool_create(const bat_pool_cfg* cfg, bat_pool* out) {
     p.free_pages.reserve(c.num_pages);
     for (int64_t i = c.num_pages - 1; i >= 0; --i) p.free_pages.push_back(static_cast<int32_t>(i));
     p.peer_arena.assign(p.cfg.world, nullptr);
+    p.peer_ipc.assign(p.cfg.world, 0);
     if (!p.index_only) {
       DeviceGuard dg(c.device);
       const size_t bytes = size_t(c.num_pages + 1) * p.geo.page_bytes;
@@ -446,8 +572,8 @@ bat_status bat_kv_pool_destroy(bat_pool p) {
     if (p->pool.arena) {
       DeviceGuard dg(p->pool.device);
       cudaDeviceSynchronize();
-      for (char* a : p->pool.peer_arena)
-        if (a) cudaIpcCloseMemHandle(a);
+      for (size_t r = 0; r < p->pool.peer_arena.size(); ++r)
+        if (p->pool.peer_arena[r] && p->pool.peer_ipc[r]) cudaIpcCloseMemHandle(p->pool.peer_arena[r]);
       cudaFree(p->pool.arena);
     }
     delete p;
@@ -692,13 +818,13 @@ bat_status bat_plan_destroy(bat_plan plan) {
   return guarded([&] { delete plan; });
 }
 
-bat_status bat_plan_query_info(bat_plan plan, int32_t b, int64_t info[12]) {
+bat_status bat_plan_query_info(bat_plan plan, int32_t b, int64_t info[13]) {
   return guarded([&] {
     BAT_REQUIRE(plan && info && b >= 0 && b < int32_t(plan->plan.q.size()), "argument");
     const QueryPlan& q = plan->plan.q[b];
-    const int64_t v[12] = {q.S, q.P, q.n_pages, q.n_prefix_pages, q.n_qtiles, q.n_ktiles, q.token_off,
-                           q.scratch0, q.n_live_pairs, plan->plan.qt, q.qtile0, q.page_off};
-    std::copy(v, v + 12, info);
+    const int64_t v[13] = {q.S, q.P, q.n_pages, q.n_prefix_pages, q.n_qtiles, q.n_ktiles, q.token_off,
+                           q.scratch0, q.n_live_pairs, plan->plan.qt, q.qtile0, q.page_off, q.n_live_pairs_last};
+    std::copy(v, v + 13, info);
   });
 }
 
@@ -792,6 +918,7 @@ bat_status bat_pool_attach_peer(bat_pool p, int32_t peer, const void* h64) {
     void* ptr = nullptr;
     CUDA_OK(cudaIpcOpenMemHandle(&ptr, h, cudaIpcMemLazyEnablePeerAccess));
     P.peer_arena[peer] = static_cast<char*>(ptr);
+    P.peer_ipc[peer] = 1;
   });
 }
 
@@ -921,4 +1048,80 @@ bat_status bat_debug_attention_layer(bat_pool p, bat_model mdl, const bat_query*
   });
 }
 
+
+// ------------------------------------------------------------------ planned execution
+bat_status bat_plan_build(bat_pool p, bat_model mdl, const bat_query* queries, int32_t B, bat_stream_t stream,
+                          bat_plan* out) {
+  return guarded([&] {
+    BAT_REQUIRE(p && mdl && queries && out && B >= 1, "null argument");
+    Pool& P = p->pool;
+    Model& m = mdl->m;
+    check_compat(P, m);
+    for (int b = 0; b < B; ++b) validate_tokens(queries[b], m.cfg.vocab);
+    DeviceGuard dg(P.device);
+    auto pl = std::make_unique<bat_plan_s>();
+    build_plan(P, m.cfg.q_heads / m.cfg.kv_heads, m.cfg.kv_heads, wrap(queries, B), pl->plan, true);
+    const size_t bytes = pl->plan.img.buf.size() * 4;
+    CUDA_OK(cudaMalloc(&pl->dev_img, bytes));
+    CUDA_OK(cudaMemcpyAsync(pl->dev_img, pl->plan.img.buf.data(), bytes, cudaMemcpyHostToDevice,
+                            static_cast<cudaStream_t>(stream)));
+    CUDA_OK(cudaStreamSynchronize(static_cast<cudaStream_t>(stream)));
+    pl->device = P.device;
+    *out = pl.release();
+  });
+}
+
+bat_status bat_prefill_plan(bat_pool p, bat_model mdl, bat_plan plan, float* out_hidden, bat_stream_t stream) {
+  return guarded([&] {
+    BAT_REQUIRE(p && mdl && plan && out_hidden, "null argument");
+    BAT_REQUIRE(plan->dev_img, "plan was not built with bat_plan_build");
+    Pool& P = p->pool;
+    Model& m = mdl->m;
+    check_compat(P, m);
+    BAT_REQUIRE(!plan->plan.entity_mode && plan->plan.kv_heads == m.cfg.kv_heads, "plan / model mismatch");
+    DeviceGuard dg(P.device);
+    run_plan(P, m, plan->plan, out_hidden, static_cast<cudaStream_t>(stream),
+             static_cast<const int32_t*>(plan->dev_img));
+  });
+}
+
+// ----------------------------------------------------------------------- profiling
+bat_status bat_profile_enable(bat_model mdl, int32_t on) {
+  return guarded([&] {
+    BAT_REQUIRE(mdl, "null model");
+    mdl->m.prof.on = on != 0;
+  });
+}
+
+bat_status bat_profile_read(bat_model mdl, int32_t cls, double* total_ms, int64_t* launches, double* flops,
+                            double* bytes) {
+  return guarded([&] {
+    BAT_REQUIRE(mdl && cls >= 0 && cls < BAT_K_N, "argument");
+    DeviceGuard dg(mdl->m.device);
+    Profiler& pf = mdl->m.prof;
+    pf.collect();
+    if (total_ms) *total_ms = pf.ms[cls];
+    if (launches) *launches = pf.n[cls];
+    if (flops) *flops = pf.flops[cls];
+    if (bytes) *bytes = pf.bytes[cls];
+  });
+}
+
+bat_status bat_profile_reset(bat_model mdl) {
+  return guarded([&] {
+    BAT_REQUIRE(mdl, "null model");
+    DeviceGuard dg(mdl->m.device);
+    mdl->m.prof.reset();
+  });
+}
+
+bat_status bat_debug_attach_peer_pool(bat_pool p, int32_t peer, bat_pool other) {
+  return guarded([&] {
+    BAT_REQUIRE(p && other, "null argument");
+    Pool& P = p->pool;
+    BAT_REQUIRE(peer >= 0 && peer < P.cfg.world && peer != P.cfg.rank, "peer rank");
+    BAT_REQUIRE(other->pool.geo.page_bytes == P.geo.page_bytes, "page geometry differs");
+    P.peer_arena[peer] = other->pool.arena;
+  });
+}
 }  // extern "C"

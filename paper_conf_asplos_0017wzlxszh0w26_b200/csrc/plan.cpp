@@ -188,20 +188,25 @@ void classify_tiles(QueryPlan& qp, int32_t qt) {
     else ++pre_item[qp.kseg[s]];
   }
   const int64_t pre_total = qp.P;
-  int64_t sfx_nonitem = 0, live = 0;
+  int64_t sfx_nonitem = 0, live = 0, live_last = 0;
   std::unordered_map<int32_t, int64_t> sfx_item;
+  const int32_t last_tile0 = (qp.n_qtiles - 1) * qt;
   for (int32_t t = 0; t < qp.S; ++t) {
     int32_t g = qp.seg[t];
     if (g < 0) ++sfx_nonitem;
     else ++sfx_item[g];
+    int64_t row;
     if (g < 0) {
-      live += pre_total + (t + 1);
+      row = pre_total + (t + 1);
     } else {
       auto pi = pre_item.find(g);
-      live += pre_nonitem + (pi == pre_item.end() ? 0 : pi->second) + sfx_nonitem + sfx_item[g];
+      row = pre_nonitem + (pi == pre_item.end() ? 0 : pi->second) + sfx_nonitem + sfx_item[g];
     }
+    live += row;
+    if (t >= last_tile0) live_last += row;
   }
   qp.n_live_pairs = live;
+  qp.n_live_pairs_last = live_last;
 }
 
 }  // namespace

@@ -16,7 +16,8 @@ struct QueryPlan {
   int32_t S = 0, P = 0;
   int32_t n_pages = 0, n_prefix_pages = 0, n_qtiles = 0, n_ktiles = 0;
   int32_t token_off = 0, scratch0 = 0, qtile0 = 0, page_off = 0;
-  int64_t n_live_pairs = 0;
+  int64_t n_live_pairs = 0;       // visible (row, key) pairs per head per layer
+  int64_t n_live_pairs_last = 0;  // ... of the rows in the last q-tile (last-layer trim)
   std::vector<int32_t> tokens, pos, seg;  // [S]
   std::vector<int32_t> pages, valid;      // [n_pages]
   std::vector<int32_t> kseg, kord;        // [16 * n_pages]

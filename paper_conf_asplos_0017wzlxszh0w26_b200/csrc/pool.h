@@ -68,6 +68,7 @@ struct Pool {
   std::unordered_map<EntityKey, Entity, EntityKeyHash> index;
   std::unordered_map<EntityKey, RemoteEntity, EntityKeyHash> remote;
   std::vector<char*> peer_arena;  // by rank (IPC-mapped), nullptr for self / unattached
+  std::vector<uint8_t> peer_ipc;  // 1 if peer_arena[r] came from cudaIpcOpenMemHandle
   uint64_t ipc_handle[8] = {0};
 
   const Entity* find(int32_t kind, int64_t id) const {

@@ -246,17 +246,21 @@ def distinct_label_items(seed: int, cfg: dict, n_items: int, rng: np.random.Gene
     seen_items, seen_labels = set(), set()
     while len(chosen) < n_items:
         if weights is None:
-            i = int(rng.integers(0, corpus))
+            draw = rng.integers(0, corpus, size=2 * n_items)
         else:
-            i = int(rng.choice(corpus, p=weights))
-        if i in seen_items:
-            continue
-        lab = item_label(seed, i, V)
-        if lab in seen_labels:
-            continue
-        seen_items.add(i)
-        seen_labels.add(lab)
-        chosen.append(i)
+            draw = rng.choice(corpus, size=2 * n_items, p=weights)
+        for i in draw:
+            i = int(i)
+            if len(chosen) == n_items:
+                break
+            if i in seen_items:
+                continue
+            lab = item_label(seed, i, V)
+            if lab in seen_labels:
+                continue
+            seen_items.add(i)
+            seen_labels.add(lab)
+            chosen.append(i)
     return np.array(chosen, dtype=np.int64)
 
 
