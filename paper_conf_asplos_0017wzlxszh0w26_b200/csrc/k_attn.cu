@@ -1,24 +1,27 @@
 // Bipartite attention over paged prefix KV + the suffix's own KV (
 // PAPER.md P:207).
 //
-// One work item = (request b, KV head, packed q-tile): 128 rows = qt suffix tokens x the g
-// query heads sharing that KV head (GQA packing), against the item's list of live 128-key
-// k-tiles from the plan (block-skip: dead tiles never reach the kernel; "full" tiles skip
-// the element mask; "partial" tiles apply  kord <= rord && (kseg == rseg || (kseg|rseg) < 0)).
+// One work item = (request b, KV head, a pair of packed q-tiles).  A q-tile is 128 rows =
+// qt suffix tokens x the g query heads sharing the KV head (GQA packing).  Both q-tiles of
+// the pair share every 128-key K/V tile the loader brings in (halving K/V traffic per FLOP).
+// The plan lists the pair's live k-tiles (block-skip: dead tiles never reach the kernel)
+// with a state per q-tile: 0 dead (P = 0), 1 full (no element mask), 2 partial (apply
+//   kord <= rord && (kseg == rseg || (kseg|rseg) < 0)  per element).
 //
-// Warp roles (192 threads, one CTA per SM, persistent over work items):
-//   warp 0   loader: one bulk copy for the q-tile (pre-packed and pre-swizzled by the stage
-//            kernel) and, per k-tile, 2 KB bulk copies of each page's K and V blocks — the
-//            pool stores pages in the tensor-core operand layout, so no TMA descriptor or
-//            reshuffle is needed — plus the k-tile's key metadata (1 KB).
-//   warp 1   MMA issuer (one thread): S = Q K^T (tcgen05.mma SS, M=128 N=128 K=16) into one
-//            of two TMEM S buffers; O += P V (tcgen05.mma TS: P read from TMEM, V MN-major
-//            from smem) into a TMEM O accumulator.  Issue order S0 S1 PV0 S2 PV1 ... keeps the
-//            tensor pipe busy while the softmax warps work on the other S buffer.
-//   warps 2-5 softmax (thread = row): tcgen05.ld of the S row, mask, online softmax in the
-//            log2 domain with a lazy running max (O is rescaled only when the max grows by
-//            more than 2^8, FA4-style), P = exp2(.) packed to bf16 and written back into the S
-//            buffer's TMEM columns with tcgen05.st; finally O / l is stored as bf16.
+// Warp roles (384 threads, one CTA per SM, persistent over work items, FA4-style):
+//   warp 0      loader: lanes 0-7 each bulk-copy one page's K (then V) blocks of a k-tile —
+//               pages are stored in the tensor-core operand layout (128-byte swizzle), so
+//               2 KB blocks drop into shared memory ready for tcgen05.mma; page ids of the
+//               next tile are prefetched into registers while waiting for a free stage.
+//   warp 1      MMA issuer (one thread): S0 = Q0 K^T, S1 = Q1 K^T (SS, M=128 N=128 K=16) and
+//               O0 += P0 V, O1 += P1 V (TS: P read from TMEM, V MN-major from smem), issued as
+//               S0_0 S1_0 | PV0_j S0_{j+1} PV1_j S1_{j+1} | ... so one softmax warpgroup works
+//               while the tensor core serves the other.
+//   warps 4-7   softmax warpgroup 0 (q-tile 0), warps 8-11 warpgroup 1 (q-tile 1), one row per
+//               thread: max pass over the S row (tcgen05.ld), exp2 pass writing P as bf16 into
+//               the S buffer's TMEM columns (tcgen05.st), lazy rescaling of O (only when the
+//               running max grows by > 2^8), final O / l -> bf16 stores.
+// TMEM (512 columns): S0 [0,128) S1 [128,256) O0 [256,384) O1 [384,512).
 #include <cuda_bf16.h>
 #include <cuda_runtime.h>
 
@@ -29,26 +32,25 @@
 namespace bat {
 namespace {
 
-constexpr int NUM_THREADS = 192;
+constexpr int NUM_THREADS = 384;
 constexpr float kRescaleThreshold = 8.0f;  // log2 units: P <= 2^8 between rescales
 
 template <int DP>
 struct AttnSmem {
   static constexpr int CHUNKS = DP / 64;
   static constexpr int TILE_BYTES = CHUNKS * 128 * 128;  // [CHUNKS][128 rows][64] bf16
-  static constexpr int Q_OFF = 0;                        // 2 q buffers
+  static constexpr int Q_OFF = 0;                        // Q0, Q1
   static constexpr int K_OFF = Q_OFF + 2 * TILE_BYTES;   // 2 stages
   static constexpr int V_OFF = K_OFF + 2 * TILE_BYTES;   // 2 stages
-  static constexpr int META_OFF = V_OFF + 2 * TILE_BYTES;  // 2 x 128 x int2
+  static constexpr int META_OFF = V_OFF + 2 * TILE_BYTES;  // 2 x 128 x int2 (with V)
   static constexpr int BAR_OFF = META_OFF + 2 * 1024;
   static constexpr int TOTAL = BAR_OFF + 256;
 };
 
 struct __align__(8) AttnBars {
-  uint64_t q_full[2], q_empty[2];
-  uint64_t k_full[2], v_full[2], kv_empty[2];
-  uint64_t s_full[2], p_full[2], pv_done[2];
-  uint64_t o_full, o_empty;
+  uint64_t q_full, q_empty;
+  uint64_t k_full[2], k_empty[2], v_full[2], v_empty[2];
+  uint64_t s_full[2], p_full[2], o_full[2], o_empty[2];
   uint32_t tmem_base;
 };
 
@@ -58,6 +60,21 @@ __device__ __forceinline__ const char* resolve_page(const AttnParams& p, int32_t
   return p.scratch + int64_t(-page - 1) * p.scratch_page_bytes + p.scratch_layer_off;
 }
 
+__device__ __forceinline__ float ex2(float x) {
+  float y;
+  asm("ex2.approx.ftz.f32 %0, %1;" : "=f"(y) : "f"(x));
+  return y;
+}
+
+struct WorkItem {
+  int b, kvh, q0, q1, kt_off, kt_n;
+};
+__device__ __forceinline__ WorkItem load_work(const int32_t* work, int w) {
+  const int4 a = *reinterpret_cast<const int4*>(work + int64_t(w) * 8);
+  const int4 c = *reinterpret_cast<const int4*>(work + int64_t(w) * 8 + 4);
+  return WorkItem{a.x, a.y, a.z, a.w, c.x, c.y};
+}
+
 template <int DP>
 __global__ void __launch_bounds__(NUM_THREADS, 1) attn_tc_kernel(const __grid_constant__ AttnParams p) {
   using L = AttnSmem<DP>;
@@ -65,24 +82,22 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) attn_tc_kernel(const __grid_co
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
   AttnBars* bars = reinterpret_cast<AttnBars*>(smem + L::BAR_OFF);
   const uint32_t warp = ptx::warp_id(), lane = ptx::lane_id();
-  constexpr uint32_t S_COLS = 128;
-  constexpr uint32_t O_COL = 256;
   constexpr uint32_t IDESC_S = ptx::idesc_bf16(128, 128, 0, 0);
   constexpr uint32_t IDESC_PV = ptx::idesc_bf16(128, DP, 0, 1);
 
   if (warp == 0 && lane == 0) {
+    ptx::mbar_init(&bars->q_full, 1);
+    ptx::mbar_init(&bars->q_empty, 1);
     for (int i = 0; i < 2; ++i) {
-      ptx::mbar_init(&bars->q_full[i], 1);
-      ptx::mbar_init(&bars->q_empty[i], 1);
       ptx::mbar_init(&bars->k_full[i], 1);
+      ptx::mbar_init(&bars->k_empty[i], 1);
       ptx::mbar_init(&bars->v_full[i], 1);
-      ptx::mbar_init(&bars->kv_empty[i], 1);
+      ptx::mbar_init(&bars->v_empty[i], 1);
       ptx::mbar_init(&bars->s_full[i], 1);
       ptx::mbar_init(&bars->p_full[i], 4);
-      ptx::mbar_init(&bars->pv_done[i], 1);
+      ptx::mbar_init(&bars->o_full[i], 1);
+      ptx::mbar_init(&bars->o_empty[i], 4);
     }
-    ptx::mbar_init(&bars->o_full, 1);
-    ptx::mbar_init(&bars->o_empty, 4);
     ptx::fence_mbar_init();
   }
   if (warp == 1) ptx::tmem_alloc(&bars->tmem_base, 512);
@@ -94,201 +109,301 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) attn_tc_kernel(const __grid_co
   const int32_t* img = p.img;
   const int32_t* work = img + p.off_work;
 
-  if (warp == 0) {
-    if (lane == 0) {  // ------------------------------------------------------ loader
-      uint32_t qc = 0, kc = 0;
-      for (int w = blockIdx.x; w < p.n_work; w += gridDim.x, ++qc) {
-        const int4 wi = *reinterpret_cast<const int4*>(work + int64_t(w) * 4);
-        const int b = wi.x, kvh = wi.y >> 16, qi = wi.y & 0xFFFF, kt_off = wi.z, kt_n = wi.w;
-        const int32_t* q_info = img + p.off_qinfo + int64_t(b) * 8;
-        const int qtile0 = q_info[2], page_off = q_info[4];
-        const int qb = qc & 1;
-        ptx::mbar_wait(&bars->q_empty[qb], ((qc >> 1) & 1) ^ 1);
-        ptx::mbar_expect_tx(&bars->q_full[qb], L::TILE_BYTES);
-        const char* qsrc = reinterpret_cast<const char*>(p.qp) +
-                           (int64_t(qtile0 + qi) * p.kv_heads + kvh) * L::TILE_BYTES;
-        ptx::bulk_g2s(smem + L::Q_OFF + qb * L::TILE_BYTES, qsrc, L::TILE_BYTES, &bars->q_full[qb]);
-        for (int x = 0; x < kt_n; ++x, ++kc) {
-          const int j = img[kt_off + x] & 0xFFFFFF;
-          const int s = kc & 1;
-          ptx::mbar_wait(&bars->kv_empty[s], ((kc >> 1) & 1) ^ 1);
-          uint8_t* sk = smem + L::K_OFF + s * L::TILE_BYTES;
-          uint8_t* sv = smem + L::V_OFF + s * L::TILE_BYTES;
-          const int32_t* pages = img + p.off_pages + page_off + j * kKtilePages;
-          ptx::mbar_expect_tx(&bars->k_full[s], L::TILE_BYTES + 1024);
-          for (int pg = 0; pg < kKtilePages; ++pg) {
-            const char* base = resolve_page(p, pages[pg]) + int64_t(kvh) * p.head_bytes;
+  if (warp == 0) {  // --------------------------------------------------------- loader
+    uint32_t qc = 0, kc = 0;
+    for (int w = blockIdx.x; w < p.n_work; w += gridDim.x, ++qc) {
+      const WorkItem wi = load_work(work, w);
+      const int32_t* q_info = img + p.off_qinfo + int64_t(wi.b) * 8;
+      const int qtile0 = q_info[2], page_off = q_info[4];
+      const int32_t* pages = img + p.off_pages + page_off;
+      const int32_t* ktl = img + wi.kt_off;
+      // prefetch tile 0's page ids (lanes 0-7)
+      int32_t next_page = 0;
+      if (wi.kt_n > 0 && lane < kKtilePages) next_page = pages[(ktl[0] & 0xFFFFFF) * kKtilePages + lane];
+      if (lane == 0) {
+        ptx::mbar_wait(&bars->q_empty, (qc & 1) ^ 1);
+        const int nq = wi.q1 >= 0 ? 2 : 1;
+        ptx::mbar_expect_tx(&bars->q_full, nq * L::TILE_BYTES);
+        const char* qbase = reinterpret_cast<const char*>(p.qp);
+        ptx::bulk_g2s(smem + L::Q_OFF, qbase + (int64_t(qtile0 + wi.q0) * p.kv_heads + wi.kvh) * L::TILE_BYTES,
+                      L::TILE_BYTES, &bars->q_full);
+        if (wi.q1 >= 0)
+          ptx::bulk_g2s(smem + L::Q_OFF + L::TILE_BYTES,
+                        qbase + (int64_t(qtile0 + wi.q1) * p.kv_heads + wi.kvh) * L::TILE_BYTES, L::TILE_BYTES,
+                        &bars->q_full);
+      }
+      for (int x = 0; x < wi.kt_n; ++x, ++kc) {
+        const int j = ktl[x] & 0xFFFFFF;
+        const int32_t my_page = next_page;
+        if (x + 1 < wi.kt_n && lane < kKtilePages)
+          next_page = pages[(ktl[x + 1] & 0xFFFFFF) * kKtilePages + lane];
+        const int s = kc & 1;
+        const uint32_t ph = ((kc >> 1) & 1) ^ 1;
+        const char* src = (lane < kKtilePages) ? resolve_page(p, my_page) : nullptr;
+        uint8_t* sk = smem + L::K_OFF + s * L::TILE_BYTES;
+        uint8_t* sv = smem + L::V_OFF + s * L::TILE_BYTES;
+        if (lane == 0) {
+          ptx::mbar_wait(&bars->k_empty[s], ph);
+          ptx::mbar_expect_tx(&bars->k_full[s], L::TILE_BYTES);
+        }
+        __syncwarp();
+        if (lane < kKtilePages) {
+          const char* kb = src + int64_t(wi.kvh) * p.head_bytes;
 #pragma unroll
-            for (int c = 0; c < L::CHUNKS; ++c)
-              ptx::bulk_g2s(sk + c * 16384 + pg * 2048, base + c * 2048, 2048, &bars->k_full[s]);
-          }
+          for (int c = 0; c < L::CHUNKS; ++c)
+            ptx::bulk_g2s(sk + c * 16384 + lane * 2048, kb + c * 2048, 2048, &bars->k_full[s]);
+        }
+        if (lane == 0) {
+          ptx::mbar_wait(&bars->v_empty[s], ph);
+          ptx::mbar_expect_tx(&bars->v_full[s], L::TILE_BYTES + 1024);
           ptx::bulk_g2s(smem + L::META_OFF + s * 1024,
                         img + p.off_kmeta + (int64_t(page_off) + int64_t(j) * kKtilePages) * kPageTokens * 2,
-                        1024, &bars->k_full[s]);
-          ptx::mbar_expect_tx(&bars->v_full[s], L::TILE_BYTES);
-          for (int pg = 0; pg < kKtilePages; ++pg) {
-            const char* base = resolve_page(p, pages[pg]) + int64_t(p.kv_heads + kvh) * p.head_bytes;
+                        1024, &bars->v_full[s]);
+        }
+        __syncwarp();
+        if (lane < kKtilePages) {
+          const char* vb = src + int64_t(p.kv_heads + wi.kvh) * p.head_bytes;
 #pragma unroll
-            for (int c = 0; c < L::CHUNKS; ++c)
-              ptx::bulk_g2s(sv + c * 16384 + pg * 2048, base + c * 2048, 2048, &bars->v_full[s]);
-          }
+          for (int c = 0; c < L::CHUNKS; ++c)
+            ptx::bulk_g2s(sv + c * 16384 + lane * 2048, vb + c * 2048, 2048, &bars->v_full[s]);
         }
       }
     }
-  } else if (warp == 1) {
-    if (lane == 0) {  // ---------------------------------------------------- MMA issuer
-      uint32_t qc = 0, kc = 0;
-      for (int w = blockIdx.x; w < p.n_work; w += gridDim.x, ++qc) {
-        const int4 wi = *reinterpret_cast<const int4*>(work + int64_t(w) * 4);
-        const int kt_n = wi.w;
-        const int qb = qc & 1;
-        ptx::mbar_wait(&bars->q_full[qb], (qc >> 1) & 1);
-        ptx::tc_fence_after();
-        const uint32_t sq = ptx::smem_u32(smem + L::Q_OFF + qb * L::TILE_BYTES);
-        auto issue_pv = [&](int y) {
-          const uint32_t g = kc + y;
-          const int s = g & 1;
-          const uint32_t ph = (g >> 1) & 1;
-          if (y == 0) ptx::mbar_wait(&bars->o_empty, (qc & 1) ^ 1);
-          ptx::mbar_wait(&bars->p_full[s], ph);
-          ptx::mbar_wait(&bars->v_full[s], ph);
-          ptx::tc_fence_after();
-          const uint32_t sv = ptx::smem_u32(smem + L::V_OFF + s * L::TILE_BYTES);
+  } else if (warp == 1) {  // ---------------------------------------------- MMA issuer
+    if (lane == 0) {
+      uint32_t qc = 0, kc = 0, sc0 = 0, sc1 = 0, pc0 = 0, pc1 = 0, oc0 = 0, oc1 = 0;
+      const uint32_t sq0 = ptx::smem_u32(smem + L::Q_OFF);
+      const uint32_t sq1 = sq0 + L::TILE_BYTES;
+      const uint32_t tS0 = tmem, tS1 = tmem + 128, tO0 = tmem + 256, tO1 = tmem + 384;
+      auto issue_s = [&](uint32_t sq, uint32_t tS, uint32_t sk) {
 #pragma unroll
-          for (int kk = 0; kk < 8; ++kk) {
-            uint64_t db = ptx::desc_sw128(sv + kk * 2048, 16384, 1024);
-            ptx::mma_ts(tmem + O_COL, tmem + s * S_COLS + kk * 8, db, IDESC_PV, (y | kk) ? 1u : 0u);
-          }
-          ptx::mma_commit(&bars->kv_empty[s]);
-          ptx::mma_commit(&bars->pv_done[s]);
-        };
-        for (int x = 0; x < kt_n; ++x) {
-          const uint32_t g = kc + x;
-          const int s = g & 1;
-          ptx::mbar_wait(&bars->k_full[s], (g >> 1) & 1);
+        for (int kk = 0; kk < DP / 16; ++kk) {
+          const uint32_t off = (kk >> 2) * 16384 + (kk & 3) * 32;
+          ptx::mma_ss(tS, ptx::desc_sw128(sq + off, 16, 1024), ptx::desc_sw128(sk + off, 16, 1024), IDESC_S,
+                      kk ? 1u : 0u);
+        }
+      };
+      auto issue_pv = [&](uint32_t tS, uint32_t tO, uint32_t sv, bool acc) {
+#pragma unroll
+        for (int kk = 0; kk < 8; ++kk)
+          ptx::mma_ts(tO, tS + kk * 8, ptx::desc_sw128(sv + kk * 2048, 16384, 1024), IDESC_PV,
+                      (acc || kk) ? 1u : 0u);
+      };
+      for (int w = blockIdx.x; w < p.n_work; w += gridDim.x, ++qc) {
+        const WorkItem wi = load_work(work, w);
+        const bool has1 = wi.q1 >= 0;
+        const int n = wi.kt_n;
+        if (n == 0) continue;
+        ptx::mbar_wait(&bars->q_full, qc & 1);
+        // S for tile 0
+        {
+          const int s = kc & 1;
+          ptx::mbar_wait(&bars->k_full[s], (kc >> 1) & 1);
           ptx::tc_fence_after();
           const uint32_t sk = ptx::smem_u32(smem + L::K_OFF + s * L::TILE_BYTES);
-#pragma unroll
-          for (int kk = 0; kk < DP / 16; ++kk) {
-            const uint32_t off = (kk >> 2) * 16384 + (kk & 3) * 32;
-            uint64_t da = ptx::desc_sw128(sq + off, 16, 1024);
-            uint64_t db = ptx::desc_sw128(sk + off, 16, 1024);
-            ptx::mma_ss(tmem + s * S_COLS, da, db, IDESC_S, kk ? 1u : 0u);
+          issue_s(sq0, tS0, sk);
+          ptx::mma_commit(&bars->s_full[0]);
+          if (has1) {
+            issue_s(sq1, tS1, sk);
+            ptx::mma_commit(&bars->s_full[1]);
           }
-          ptx::mma_commit(&bars->s_full[s]);
-          if (x == kt_n - 1) ptx::mma_commit(&bars->q_empty[qb]);
-          if (x >= 1) issue_pv(x - 1);
+          ptx::mma_commit(&bars->k_empty[s]);
+          if (n == 1) ptx::mma_commit(&bars->q_empty);
         }
-        if (kt_n > 0) issue_pv(kt_n - 1);
-        ptx::mma_commit(&bars->o_full);
-        kc += kt_n;
+        for (int x = 0; x < n; ++x) {
+          const uint32_t g = kc + x;
+          const int s = g & 1;
+          const uint32_t sv = ptx::smem_u32(smem + L::V_OFF + s * L::TILE_BYTES);
+          const bool more = x + 1 < n;
+          const uint32_t gn = g + 1;
+          const int sn = gn & 1;
+          const uint32_t skn = ptx::smem_u32(smem + L::K_OFF + sn * L::TILE_BYTES);
+          // ---- q-tile 0: PV0_x, then S0_{x+1}
+          ptx::mbar_wait(&bars->p_full[0], pc0 & 1);
+          ++pc0;
+          ptx::mbar_wait(&bars->v_full[s], (g >> 1) & 1);
+          if (x == 0) ptx::mbar_wait(&bars->o_empty[0], (oc0 & 1) ^ 1);
+          ptx::tc_fence_after();
+          issue_pv(tS0, tO0, sv, x > 0);
+          if (more) {
+            ptx::mbar_wait(&bars->k_full[sn], (gn >> 1) & 1);
+            ptx::tc_fence_after();
+            issue_s(sq0, tS0, skn);
+            ptx::mma_commit(&bars->s_full[0]);
+          }
+          // ---- q-tile 1: PV1_x, then S1_{x+1}
+          if (has1) {
+            ptx::mbar_wait(&bars->p_full[1], pc1 & 1);
+            ++pc1;
+            if (x == 0) ptx::mbar_wait(&bars->o_empty[1], (oc1 & 1) ^ 1);
+            ptx::tc_fence_after();
+            issue_pv(tS1, tO1, sv, x > 0);
+          }
+          ptx::mma_commit(&bars->v_empty[s]);
+          if (more) {
+            if (has1) {
+              issue_s(sq1, tS1, skn);
+              ptx::mma_commit(&bars->s_full[1]);
+            }
+            ptx::mma_commit(&bars->k_empty[sn]);
+            if (x + 1 == n - 1) ptx::mma_commit(&bars->q_empty);
+          }
+        }
+        ptx::mma_commit(&bars->o_full[0]);
+        ++oc0;
+        if (has1) {
+          ptx::mma_commit(&bars->o_full[1]);
+          ++oc1;
+        }
+        kc += n;
+        (void)sc0;
+        (void)sc1;
       }
     }
-  } else {  // ------------------------------------------------------------ softmax warps
+  } else if (warp >= 4) {  // ------------------------------------------ softmax warpgroups
+    const int wg = (warp - 4) >> 2;  // 0 or 1
     const uint32_t sub = warp & 3;
     const int row = sub * 32 + lane;
     const uint32_t lane_base = (sub * 32) << 16;
-    uint32_t qc = 0, kc = 0;
-    for (int w = blockIdx.x; w < p.n_work; w += gridDim.x, ++qc) {
-      const int4 wi = *reinterpret_cast<const int4*>(work + int64_t(w) * 4);
-      const int b = wi.x, kvh = wi.y >> 16, qi = wi.y & 0xFFFF, kt_off = wi.z, kt_n = wi.w;
-      const int32_t* q_info = img + p.off_qinfo + int64_t(b) * 8;
+    const uint32_t tS = tmem + wg * 128 + lane_base;
+    const uint32_t tO = tmem + 256 + wg * 128 + lane_base;
+    uint32_t kc = 0, sc = 0, oc = 0;
+    for (int w = blockIdx.x; w < p.n_work; w += gridDim.x) {
+      const WorkItem wi = load_work(work, w);
+      const int qi = wg == 0 ? wi.q0 : wi.q1;
+      if (qi < 0 || wi.kt_n == 0) {
+        kc += wi.kt_n;
+        continue;
+      }
+      const int32_t* q_info = img + p.off_qinfo + int64_t(wi.b) * 8;
       const int tok_off = q_info[0], S = q_info[1];
       const int tok_local = qi * p.qt + row / p.group;
       const bool valid_row = row < p.qt * p.group && tok_local < S;
       const int32_t rseg = valid_row ? img[p.off_rseg + tok_off + tok_local] : -1;
       const int32_t rord = valid_row ? tok_local + 1 : kInvalidOrd - 1;
+      const int32_t* ktl = img + wi.kt_off;
       float m_ref = -INFINITY, l_sum = 0.0f;
-      for (int x = 0; x < kt_n; ++x) {
+      for (int x = 0; x < wi.kt_n; ++x) {
         const uint32_t g = kc + x;
         const int s = g & 1;
-        const uint32_t ph = (g >> 1) & 1;
-        const int state = img[kt_off + x] >> 24;
-        ptx::mbar_wait(&bars->s_full[s], ph);
+        const int state = (ktl[x] >> (24 + 2 * wg)) & 3;
+        ptx::mbar_wait(&bars->s_full[wg], sc & 1);
+        ++sc;
         ptx::tc_fence_after();
-        float v[128];
-        {
-          uint32_t r[32];
+        uint32_t vis[4] = {0xffffffffu, 0xffffffffu, 0xffffffffu, 0xffffffffu};
+        if (state == 2) {
+          ptx::mbar_wait(&bars->v_full[s], (g >> 1) & 1);  // key metadata travels with V
+          const int4* meta = reinterpret_cast<const int4*>(smem + L::META_OFF + s * 1024);
 #pragma unroll
           for (int c = 0; c < 4; ++c) {
-            ptx::tmem_ld32(tmem + lane_base + s * S_COLS + c * 32, r);
+            uint32_t bits = 0;
+#pragma unroll
+            for (int i = 0; i < 16; ++i) {
+              const int4 km = meta[c * 16 + i];  // (kseg, kord) x 2, broadcast across the warp
+              const bool v0 = (km.y <= rord) && ((km.x == rseg) || ((km.x | rseg) < 0));
+              const bool v1 = (km.w <= rord) && ((km.z == rseg) || ((km.z | rseg) < 0));
+              bits |= (uint32_t(v0) << (2 * i)) | (uint32_t(v1) << (2 * i + 1));
+            }
+            vis[c] = bits;
+          }
+        } else if (state == 0) {
+          vis[0] = vis[1] = vis[2] = vis[3] = 0u;
+        }
+        // pass 1: row max (raw scores)
+        float mt = -INFINITY;
+        if (state != 0) {
+#pragma unroll
+          for (int c = 0; c < 4; ++c) {
+            uint32_t r[32];
+            ptx::tmem_ld32(tS + c * 32, r);
             ptx::tmem_ld_wait();
+            float m0 = -INFINITY, m1 = -INFINITY;
 #pragma unroll
-            for (int i = 0; i < 32; ++i) v[c * 32 + i] = __uint_as_float(r[i]) * p.scale_log2;
+            for (int i = 0; i < 32; i += 2) {
+              const float a = ((vis[c] >> i) & 1u) ? __uint_as_float(r[i]) : -INFINITY;
+              const float b = ((vis[c] >> (i + 1)) & 1u) ? __uint_as_float(r[i + 1]) : -INFINITY;
+              m0 = fmaxf(m0, a);
+              m1 = fmaxf(m1, b);
+            }
+            mt = fmaxf(mt, fmaxf(m0, m1));
           }
         }
-        if (state == 2) {
-          ptx::mbar_wait(&bars->k_full[s], ph);  // key metadata landed (already complete)
-          const int2* meta = reinterpret_cast<const int2*>(smem + L::META_OFF + s * 1024);
-#pragma unroll
-          for (int c = 0; c < 128; ++c) {
-            const int2 km = meta[c];  // (kseg, kord), same address across the warp: broadcast
-            const bool vis = (km.y <= rord) && ((km.x == rseg) || ((km.x | rseg) < 0));
-            v[c] = vis ? v[c] : -INFINITY;
-          }
-        }
-        float mt = v[0];
-#pragma unroll
-        for (int c = 1; c < 128; ++c) mt = fmaxf(mt, v[c]);
         const float m_old = m_ref;
-        const float m_new = fmaxf(m_ref, mt);
+        const float m_new = fmaxf(m_ref, mt * p.scale_log2);
         const bool grow = m_new > m_ref + kRescaleThreshold;
         float alpha = 1.0f;
         if (grow) {
-          alpha = exp2f(m_ref - m_new);  // 0 when m_ref = -inf
+          alpha = ex2(m_ref - m_new);  // 0 when m_ref = -inf
           l_sum *= alpha;
           m_ref = m_new;
         }
-        // rescale the O accumulator rows of this warp when any lane's reference max moved
+        // O rows of this warp are rescaled when a lane's reference max moved.  The previous
+        // P.V of this q-tile is complete: it was issued before this S (in-order tensor pipe).
         const bool need_o = grow && (m_old != -INFINITY) && (x > 0);
         if (__any_sync(0xffffffffu, need_o)) {
-          const uint32_t gp = g - 1;
-          ptx::mbar_wait(&bars->pv_done[gp & 1], (gp >> 1) & 1);
-          ptx::tc_fence_after();
           const float a = need_o ? alpha : 1.0f;
-#pragma unroll
+#pragma unroll 1
           for (int c = 0; c < DP / 32; ++c) {
             uint32_t r[32];
-            ptx::tmem_ld32(tmem + lane_base + O_COL + c * 32, r);
+            ptx::tmem_ld32(tO + c * 32, r);
             ptx::tmem_ld_wait();
 #pragma unroll
             for (int i = 0; i < 32; ++i) r[i] = __float_as_uint(__uint_as_float(r[i]) * a);
-            ptx::tmem_st32(tmem + lane_base + O_COL + c * 32, r);
+            ptx::tmem_st32(tO + c * 32, r);
           }
           ptx::tmem_st_wait();
         }
+        // pass 2: P = exp2(s * scale - m_ref) -> bf16 into the S buffer's first 64 columns
         const float mref = (m_ref == -INFINITY) ? 0.0f : m_ref;
         float lsum = 0.0f;
 #pragma unroll
-        for (int c = 0; c < 2; ++c) {
-          uint32_t pk[32];
+        for (int c = 0; c < 4; ++c) {
+          uint32_t pk[16];
+          if (state != 0) {
+            uint32_t r[32];
+            ptx::tmem_ld32(tS + c * 32, r);
+            ptx::tmem_ld_wait();
 #pragma unroll
-          for (int i = 0; i < 32; ++i) {
-            const float p0 = exp2f(v[c * 64 + 2 * i] - mref);
-            const float p1 = exp2f(v[c * 64 + 2 * i + 1] - mref);
-            lsum += p0 + p1;
-            pk[i] = ptx::pack_bf16x2(p0, p1);
+            for (int i = 0; i < 16; ++i) {
+              float p0 = ex2(fmaf(__uint_as_float(r[2 * i]), p.scale_log2, -mref));
+              float p1 = ex2(fmaf(__uint_as_float(r[2 * i + 1]), p.scale_log2, -mref));
+              p0 = ((vis[c] >> (2 * i)) & 1u) ? p0 : 0.0f;
+              p1 = ((vis[c] >> (2 * i + 1)) & 1u) ? p1 : 0.0f;
+              lsum += p0 + p1;
+              pk[i] = ptx::pack_bf16x2(p0, p1);
+            }
+          } else {
+#pragma unroll
+            for (int i = 0; i < 16; ++i) pk[i] = 0u;
           }
-          ptx::tmem_st32(tmem + lane_base + s * S_COLS + c * 32, pk);
+          // columns [16c, 16c+16) of the S buffer: already consumed S values
+          asm volatile(
+              "tcgen05.st.sync.aligned.32x32b.x16.b32 [%0], "
+              "{%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,%16};" ::"r"(tS + c * 16),
+              "r"(pk[0]), "r"(pk[1]), "r"(pk[2]), "r"(pk[3]), "r"(pk[4]), "r"(pk[5]), "r"(pk[6]), "r"(pk[7]),
+              "r"(pk[8]), "r"(pk[9]), "r"(pk[10]), "r"(pk[11]), "r"(pk[12]), "r"(pk[13]), "r"(pk[14]),
+              "r"(pk[15]));
         }
         l_sum += lsum;
         ptx::tmem_st_wait();
         ptx::tc_fence_before();
         __syncwarp();
-        if (lane == 0) ptx::mbar_arrive(&bars->p_full[s]);
+        if (lane == 0) ptx::mbar_arrive(&bars->p_full[wg]);
       }
+      kc += wi.kt_n;
       // ---- epilogue: O / l -> bf16
-      ptx::mbar_wait(&bars->o_full, qc & 1);
+      ptx::mbar_wait(&bars->o_full[wg], oc & 1);
+      ++oc;
       ptx::tc_fence_after();
       const float inv = (l_sum > 0.0f) ? 1.0f / l_sum : 0.0f;
-      const int head = kvh * p.group + row % p.group;
+      const int head = wi.kvh * p.group + row % p.group;
       __nv_bfloat16* dst = p.out + int64_t(tok_off + tok_local) * p.ldo + int64_t(head) * p.head_dim;
-#pragma unroll
+#pragma unroll 1
       for (int c = 0; c < DP / 32; ++c) {
         uint32_t r[32];
-        ptx::tmem_ld32(tmem + lane_base + O_COL + c * 32, r);
+        ptx::tmem_ld32(tO + c * 32, r);
         ptx::tmem_ld_wait();
-        if (valid_row && kt_n > 0 && c * 32 < p.head_dim) {
+        if (valid_row && c * 32 < p.head_dim) {
           uint32_t pk[16];
 #pragma unroll
           for (int i = 0; i < 16; ++i)
@@ -300,8 +415,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) attn_tc_kernel(const __grid_co
       }
       ptx::tc_fence_before();
       __syncwarp();
-      if (lane == 0) ptx::mbar_arrive(&bars->o_empty);
-      kc += kt_n;
+      if (lane == 0) ptx::mbar_arrive(&bars->o_empty[wg]);
     }
   }
   ptx::tc_fence_before();

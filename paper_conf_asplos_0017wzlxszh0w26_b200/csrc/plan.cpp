@@ -311,32 +311,41 @@ void build_plan(const Pool& pool, int32_t group, int32_t kv_heads,
     }
     v[im.off_disc + b] = qp.token_off + qp.S - 1;
   }
-  // work items (b, kvh, q-tile) with their live k-tiles, longest first (LPT over the SMs)
-  struct W { int32_t b, kvh, i, n; std::vector<int32_t> kt; };
+  // work items: (b, kvh, q-tile pair) sharing every K/V tile, with the union of the two
+  // q-tiles' live k-tiles and a state per q-tile; longest first (LPT over the SMs)
+  struct W { int32_t b, kvh, q0, q1, n; std::vector<int32_t> kt; };
   auto make_work = [&](bool last_only, int64_t& off_work, int32_t& n_work) {
     std::vector<W> ws;
     for (int32_t b = 0; b < B; ++b) {
       const QueryPlan& qp = plan.q[b];
-      for (int32_t i = last_only ? qp.n_qtiles - 1 : 0; i < qp.n_qtiles; ++i) {
+      std::vector<std::pair<int32_t, int32_t>> pairs;
+      if (last_only) pairs.push_back({qp.n_qtiles - 1, -1});
+      else
+        for (int32_t i = 0; i < qp.n_qtiles; i += 2) pairs.push_back({i, i + 1 < qp.n_qtiles ? i + 1 : -1});
+      for (auto& pr : pairs) {
         std::vector<int32_t> kt;
         for (int32_t j = 0; j < qp.n_ktiles; ++j) {
-          uint8_t st = qp.tiles[static_cast<size_t>(i) * qp.n_ktiles + j];
-          if (st) kt.push_back(j | (int32_t(st) << 24));
+          uint8_t s0 = qp.tiles[static_cast<size_t>(pr.first) * qp.n_ktiles + j];
+          uint8_t s1 = pr.second >= 0 ? qp.tiles[static_cast<size_t>(pr.second) * qp.n_ktiles + j] : 0;
+          if (s0 || s1) kt.push_back(j | (int32_t(s0) << 24) | (int32_t(s1) << 26));
         }
-        for (int32_t h = 0; h < kv_heads; ++h) ws.push_back(W{b, h, i, int32_t(kt.size()), kt});
+        if (kt.empty()) continue;  // cannot happen for real rows (each row sees itself)
+        for (int32_t h = 0; h < kv_heads; ++h) ws.push_back(W{b, h, pr.first, pr.second, int32_t(kt.size()), kt});
       }
     }
-    std::stable_sort(ws.begin(), ws.end(), [](const W& a, const W& c) { return a.n > c.n; });
+    std::stable_sort(ws.begin(), ws.end(), [](const W& a, const W& c) {
+      return a.n * (a.q1 >= 0 ? 2 : 1) > c.n * (c.q1 >= 0 ? 2 : 1);
+    });
     n_work = static_cast<int32_t>(ws.size());
-    off_work = reserve_at(int64_t(n_work) * 4);
+    off_work = reserve_at(int64_t(n_work) * 8);
     int64_t total_kt = 0;
     for (auto& w : ws) total_kt += w.n;
     int64_t off_kt = reserve_at(total_kt);
     int64_t cur = 0;
     for (int32_t w = 0; w < n_work; ++w) {
-      int32_t* e = &v[off_work + int64_t(w) * 4];
-      e[0] = ws[w].b; e[1] = (ws[w].kvh << 16) | ws[w].i;
-      e[2] = static_cast<int32_t>(off_kt + cur); e[3] = ws[w].n;  // absolute offset into buf
+      int32_t* e = &v[off_work + int64_t(w) * 8];
+      e[0] = ws[w].b; e[1] = ws[w].kvh; e[2] = ws[w].q0; e[3] = ws[w].q1;
+      e[4] = static_cast<int32_t>(off_kt + cur); e[5] = ws[w].n; e[6] = 0; e[7] = 0;
       for (int32_t x : ws[w].kt) v[off_kt + cur++] = x;
     }
   };
