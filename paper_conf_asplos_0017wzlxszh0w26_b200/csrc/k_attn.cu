@@ -34,6 +34,9 @@ namespace {
 
 constexpr int NUM_THREADS = 384;
 constexpr float kRescaleThreshold = 8.0f;  // log2 units: P <= 2^8 between rescales
+#ifndef BAT_POLY_PAIRS
+#define BAT_POLY_PAIRS 6  // of every 16 column pairs, exp2 on the FMA pipe (rest: MUFU)
+#endif
 
 template <int DP>
 struct AttnSmem {
@@ -64,6 +67,54 @@ __device__ __forceinline__ float ex2(float x) {
   float y;
   asm("ex2.approx.ftz.f32 %0, %1;" : "=f"(y) : "f"(x));
   return y;
+}
+
+// ---- packed f32x2 math (FFMA2 / FADD2) and 3-input max (FMNMX3), sm_100a
+__device__ __forceinline__ uint64_t pk2(float a, float b) {
+  uint64_t r;
+  asm("mov.b64 %0, {%1, %2};" : "=l"(r) : "f"(a), "f"(b));
+  return r;
+}
+__device__ __forceinline__ void up2(uint64_t v, float& a, float& b) {
+  asm("mov.b64 {%0, %1}, %2;" : "=f"(a), "=f"(b) : "l"(v));
+}
+__device__ __forceinline__ uint64_t ffma2(uint64_t a, uint64_t b, uint64_t c) {
+  uint64_t d;
+  asm("fma.rn.f32x2 %0, %1, %2, %3;" : "=l"(d) : "l"(a), "l"(b), "l"(c));
+  return d;
+}
+__device__ __forceinline__ uint64_t fadd2(uint64_t a, uint64_t b) {
+  uint64_t d;
+  asm("add.f32x2 %0, %1, %2;" : "=l"(d) : "l"(a), "l"(b));
+  return d;
+}
+__device__ __forceinline__ float fmax3(float a, float b, float c) {
+  float d;
+  asm("max.f32 %0, %1, %2, %3;" : "=f"(d) : "f"(a), "f"(b), "f"(c));
+  return d;
+}
+// 2^x for a pair on the FMA pipe (offloads the MUFU): x = j + f, j = rint(x) by the
+// 1.5*2^23 trick, 2^f on [-0.5, 0.5] by a degree-3 minimax polynomial (rel. err 1.1e-4, far
+// below the bf16 rounding of P), exponent inserted with an integer multiply-add.
+__device__ __forceinline__ uint64_t exp2_poly2(uint64_t x) {
+  float x0, x1;
+  up2(x, x0, x1);
+  x = pk2(fmaxf(x0, -127.0f), fmaxf(x1, -127.0f));
+  const uint64_t magic = pk2(12582912.0f, 12582912.0f);
+  const uint64_t t = fadd2(x, magic);
+  const uint64_t jf = fadd2(t, pk2(-12582912.0f, -12582912.0f));
+  float j0, j1;
+  up2(jf, j0, j1);
+  const uint64_t f = fadd2(x, pk2(-j0, -j1));
+  uint64_t p = ffma2(pk2(0.05592204f, 0.05592204f), f, pk2(0.24264008f, 0.24264008f));
+  p = ffma2(p, f, pk2(0.69312103f, 0.69312103f));
+  p = ffma2(p, f, pk2(0.99992448f, 0.99992448f));
+  float p0, p1, t0, t1;
+  up2(p, p0, p1);
+  up2(t, t0, t1);
+  const uint32_t r0 = __float_as_uint(p0) + (__float_as_uint(t0) << 23);
+  const uint32_t r1 = __float_as_uint(p1) + (__float_as_uint(t1) << 23);
+  return pk2(__uint_as_float(r0), __uint_as_float(r1));
 }
 
 struct WorkItem {
@@ -306,18 +357,32 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) attn_tc_kernel(const __grid_co
             }
             vis[c] = bits;
           }
-        } else if (state == 0) {
-          vis[0] = vis[1] = vis[2] = vis[3] = 0u;
         }
-        // pass 1: row max (raw scores)
+        // pass 1: row max of the raw scores (4 independent FMNMX3 chains)
         float mt = -INFINITY;
-        if (state != 0) {
+        if (state == 1) {
 #pragma unroll
           for (int c = 0; c < 4; ++c) {
             uint32_t r[32];
             ptx::tmem_ld32(tS + c * 32, r);
             ptx::tmem_ld_wait();
-            float m0 = -INFINITY, m1 = -INFINITY;
+            float m0 = mt, m1 = -INFINITY, m2 = -INFINITY, m3 = -INFINITY;
+#pragma unroll
+            for (int i = 0; i < 32; i += 8) {
+              m0 = fmax3(m0, __uint_as_float(r[i]), __uint_as_float(r[i + 1]));
+              m1 = fmax3(m1, __uint_as_float(r[i + 2]), __uint_as_float(r[i + 3]));
+              m2 = fmax3(m2, __uint_as_float(r[i + 4]), __uint_as_float(r[i + 5]));
+              m3 = fmax3(m3, __uint_as_float(r[i + 6]), __uint_as_float(r[i + 7]));
+            }
+            mt = fmaxf(fmax3(m0, m1, m2), m3);
+          }
+        } else if (state == 2) {
+#pragma unroll
+          for (int c = 0; c < 4; ++c) {
+            uint32_t r[32];
+            ptx::tmem_ld32(tS + c * 32, r);
+            ptx::tmem_ld_wait();
+            float m0 = mt, m1 = -INFINITY;
 #pragma unroll
             for (int i = 0; i < 32; i += 2) {
               const float a = ((vis[c] >> i) & 1u) ? __uint_as_float(r[i]) : -INFINITY;
@@ -325,7 +390,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) attn_tc_kernel(const __grid_co
               m0 = fmaxf(m0, a);
               m1 = fmaxf(m1, b);
             }
-            mt = fmaxf(mt, fmaxf(m0, m1));
+            mt = fmaxf(m0, m1);
           }
         }
         const float m_old = m_ref;
@@ -353,9 +418,11 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) attn_tc_kernel(const __grid_co
           }
           ptx::tmem_st_wait();
         }
-        // pass 2: P = exp2(s * scale - m_ref) -> bf16 into the S buffer's first 64 columns
+        // pass 2: P = exp2(s * scale - m_ref) -> bf16 into the S buffer's first 64 columns;
+        // 6 of every 16 column pairs on the FMA pipe (polynomial), the rest on the MUFU.
         const float mref = (m_ref == -INFINITY) ? 0.0f : m_ref;
-        float lsum = 0.0f;
+        const uint64_t sc2 = pk2(p.scale_log2, p.scale_log2), nm2 = pk2(-mref, -mref);
+        uint64_t acc0 = pk2(0.0f, 0.0f), acc1 = acc0;
 #pragma unroll
         for (int c = 0; c < 4; ++c) {
           uint32_t pk[16];
@@ -365,11 +432,24 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) attn_tc_kernel(const __grid_co
             ptx::tmem_ld_wait();
 #pragma unroll
             for (int i = 0; i < 16; ++i) {
-              float p0 = ex2(fmaf(__uint_as_float(r[2 * i]), p.scale_log2, -mref));
-              float p1 = ex2(fmaf(__uint_as_float(r[2 * i + 1]), p.scale_log2, -mref));
-              p0 = ((vis[c] >> (2 * i)) & 1u) ? p0 : 0.0f;
-              p1 = ((vis[c] >> (2 * i + 1)) & 1u) ? p1 : 0.0f;
-              lsum += p0 + p1;
+              const uint64_t xv = ffma2(pk2(__uint_as_float(r[2 * i]), __uint_as_float(r[2 * i + 1])), sc2, nm2);
+              uint64_t e;
+              if (i < BAT_POLY_PAIRS) {
+                e = exp2_poly2(xv);
+              } else {
+                float x0, x1;
+                up2(xv, x0, x1);
+                e = pk2(ex2(x0), ex2(x1));
+              }
+              float p0, p1;
+              up2(e, p0, p1);
+              if (state == 2) {
+                p0 = ((vis[c] >> (2 * i)) & 1u) ? p0 : 0.0f;
+                p1 = ((vis[c] >> (2 * i + 1)) & 1u) ? p1 : 0.0f;
+                e = pk2(p0, p1);
+              }
+              if (i & 1) acc1 = fadd2(acc1, e);
+              else acc0 = fadd2(acc0, e);
               pk[i] = ptx::pack_bf16x2(p0, p1);
             }
           } else {
@@ -383,6 +463,13 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) attn_tc_kernel(const __grid_co
               "r"(pk[0]), "r"(pk[1]), "r"(pk[2]), "r"(pk[3]), "r"(pk[4]), "r"(pk[5]), "r"(pk[6]), "r"(pk[7]),
               "r"(pk[8]), "r"(pk[9]), "r"(pk[10]), "r"(pk[11]), "r"(pk[12]), "r"(pk[13]), "r"(pk[14]),
               "r"(pk[15]));
+        }
+        float lsum;
+        {
+          float a0, a1, b0, b1;
+          up2(acc0, a0, a1);
+          up2(acc1, b0, b1);
+          lsum = (a0 + a1) + (b0 + b1);
         }
         l_sum += lsum;
         ptx::tmem_st_wait();

@@ -8,7 +8,8 @@ inputs.  The recipe is stated in DESIGN.md §"Input recipe" and follows SURVEY.m
 
 * weights N(0, 0.02) for every matrix and bias of the Qwen-width models (the token
   embedding included: an N(0,1) embedding hides mask bugs, SURVEY §8(c) issue 11b) and
-  N(0, 1/H) for the narrow tiny config (H=64); RMSNorm gains 1 + N(0, 0.1);
+  for the narrow tiny config (H=64) N(0, 1/H) for the embedding and attention matrices and
+  N(0, 0.05^2) for the MLP matrices; RMSNorm gains 1 + N(0, 0.1);
   every value rounded to bf16 (RNE) so that both sides use exactly the same numbers;
 * token ids uniform in [0, vocab); item tokens and identifier labels are a function of
   the item id (the same item has the same tokens in every query, which is what makes its
@@ -118,6 +119,9 @@ class Weights:
         # tiny config, where 0.02 leaves attention so flat that a wrong mask moves the
         # logits by less than 10x the bf16 tolerance (tests/test_oracle_model.py guard)
         self.std = float(std) if std is not None else (0.02 if H >= 512 else 1.0 / np.sqrt(H))
+        # tiny: MLP matrices N(0, 0.05^2) — with fan-in MLP weights the 2-layer net amplifies
+        # bf16 rounding to ~1.5x the 2e-2 tolerance on hf (emulated in numpy; R12)
+        self.mlp_std = self.std if (std is not None or H >= 512) else 0.05
         # tiny (H=64): a tied 0.02 head gives logit std ~0.16; use N(0, 1/sqrt(H)) untied
         self.lm_std = (1.0 / np.sqrt(H)) if H < 512 else self.std
         self._cache: Dict[int, dict] = {}
@@ -159,8 +163,8 @@ class Weights:
             bqkv=gen_rows(s, _TAG["bqkv"], l, 1, nqkv, sd)[0],
             wo=gen_rows(s, _TAG["wo"], l, H, Hq * d, sd),
             ln2=gen_rows(s, _TAG["ln2"], l, 1, H, 0.1, 1.0)[0],
-            wgu=gen_rows(s, _TAG["wgu"], l, 2 * F, H, sd),
-            wd=gen_rows(s, _TAG["wd"], l, H, F, sd),
+            wgu=gen_rows(s, _TAG["wgu"], l, 2 * F, H, self.mlp_std),
+            wd=gen_rows(s, _TAG["wd"], l, H, F, self.mlp_std),
         )
         if c["layers"] * H <= 4096:  # small models: keep in memory
             self._cache[l] = w

@@ -118,6 +118,9 @@ def _attention_case(B, cfg_name, queries_fn, layer=1, seed=0):
         ref = oracle_attention_layer(cfg, q, ekv, qkv_np[off:off + s], layer)
         got = out_np[off:off + s].reshape(ref.shape)
         worst = max(worst, max_excess(got, ref))
+        err = np.abs(got - ref)
+        print(f"attention layer {cfg_name} {q.order} cache={q.use_cache}: max|err| {err.max():.4g} "
+              f"mean|err| {err.mean():.3g} max|ref| {np.abs(ref).max():.3g} excess {worst:.4g}")
         off += s
     pool.close()
     model.close()

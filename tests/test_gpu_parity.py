@@ -78,6 +78,7 @@ def _check(cfg, W, queries, out, k=3):
                 assert out["topk"][b, r] == ref["topk"][r], (b, r)
             else:
                 break
+    print("worst excess over tolerance:", {k: round(v, 5) for k, v in worst.items()})
     for name, v in worst.items():
         assert v <= 0, (name, v)
     return worst
