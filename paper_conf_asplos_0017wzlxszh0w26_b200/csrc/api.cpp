@@ -5,6 +5,8 @@
 
 #include <algorithm>
 #include <cmath>
+#include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <memory>
 #include <mutex>
@@ -1042,9 +1044,29 @@ bat_status bat_debug_attention_layer(bat_pool p, bat_model mdl, const bat_query*
     AttnParams ap = attn_params(P, m, plan, I);
     ap.pool_layer_off = int64_t(layer) * P.geo.layer_bytes;
     ap.out = static_cast<__nv_bfloat16*>(out_o);
+    const char* tl = std::getenv("BAT_ATTN_TIMELINE");  // debug: clock64 timeline of CTA 0
+    long long* dbg = nullptr;
+    if (tl) {
+      CUDA_OK(cudaMalloc(&dbg, 16 * 64 * sizeof(long long)));
+      CUDA_OK(cudaMemsetAsync(dbg, 0, 16 * 64 * sizeof(long long), st));
+      ap.dbg = dbg;
+    }
     launch_attention(m.dpad, ap, m.num_sms, st);
     CUDA_OK(cudaGetLastError());
     CUDA_OK(cudaStreamSynchronize(st));
+    if (dbg) {
+      std::vector<long long> h(16 * 64);
+      CUDA_OK(cudaMemcpy(h.data(), dbg, h.size() * sizeof(long long), cudaMemcpyDeviceToHost));
+      FILE* f = std::fopen(tl, "w");
+      if (f) {
+        for (int e = 0; e < 16; ++e) {
+          for (int x = 0; x < 64; ++x) std::fprintf(f, "%lld ", h[e * 64 + x]);
+          std::fprintf(f, "\n");
+        }
+        std::fclose(f);
+      }
+      cudaFree(dbg);
+    }
   });
 }
 

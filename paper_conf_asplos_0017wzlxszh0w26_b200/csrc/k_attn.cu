@@ -35,7 +35,7 @@ namespace {
 constexpr int NUM_THREADS = 384;
 constexpr float kRescaleThreshold = 8.0f;  // log2 units: P <= 2^8 between rescales
 #ifndef BAT_POLY_PAIRS
-#define BAT_POLY_PAIRS 6  // of every 16 column pairs, exp2 on the FMA pipe (rest: MUFU)
+#define BAT_POLY_PAIRS 4  // of every 16 column pairs, exp2 on the FMA pipe (rest: MUFU)
 #endif
 
 template <int DP>
@@ -117,6 +117,11 @@ __device__ __forceinline__ uint64_t exp2_poly2(uint64_t x) {
   return pk2(__uint_as_float(r0), __uint_as_float(r1));
 }
 
+#define DBG(ev, x)                                                                       \
+  do {                                                                                   \
+    if (p.dbg && blockIdx.x == 0 && (x) < 64 && dbg_first) p.dbg[(ev) * 64 + (x)] = clock64(); \
+  } while (0)
+
 struct WorkItem {
   int b, kvh, q0, q1, kt_off, kt_n;
 };
@@ -124,6 +129,159 @@ __device__ __forceinline__ WorkItem load_work(const int32_t* work, int w) {
   const int4 a = *reinterpret_cast<const int4*>(work + int64_t(w) * 8);
   const int4 c = *reinterpret_cast<const int4*>(work + int64_t(w) * 8 + 4);
   return WorkItem{a.x, a.y, a.z, a.w, c.x, c.y};
+}
+
+// ---- softmax passes over one 128-column S row held in TMEM (one row per thread) ----------
+// Row max of the raw scores; MASKED applies the visibility bits.
+template <bool MASKED>
+__device__ __forceinline__ float row_max(uint32_t tS, const uint32_t (&vis)[4]) {
+  float mt = -INFINITY;
+#pragma unroll
+  for (int c = 0; c < 4; c += 2) {
+    uint32_t r[32], q[32];
+    ptx::tmem_ld32(tS + c * 32, r);
+    ptx::tmem_ld32(tS + (c + 1) * 32, q);
+    ptx::tmem_ld_wait();
+    if (MASKED) {
+#pragma unroll
+      for (int i = 0; i < 32; ++i) {
+        r[i] = ((vis[c] >> i) & 1u) ? r[i] : 0xff800000u;  // -inf
+        q[i] = ((vis[c + 1] >> i) & 1u) ? q[i] : 0xff800000u;
+      }
+    }
+    float m0 = mt, m1 = -INFINITY, m2 = -INFINITY, m3 = -INFINITY;
+#pragma unroll
+    for (int i = 0; i < 32; i += 4) {
+      m0 = fmax3(m0, __uint_as_float(r[i]), __uint_as_float(r[i + 1]));
+      m1 = fmax3(m1, __uint_as_float(r[i + 2]), __uint_as_float(r[i + 3]));
+      m2 = fmax3(m2, __uint_as_float(q[i]), __uint_as_float(q[i + 1]));
+      m3 = fmax3(m3, __uint_as_float(q[i + 2]), __uint_as_float(q[i + 3]));
+    }
+    mt = fmaxf(fmax3(m0, m1, m2), m3);
+  }
+  return mt;
+}
+
+// P = exp2(s * scale - mref) written as bf16 pairs into the row's first 64 TMEM columns
+// (columns [16c, 16c+16) after S columns [32c, 32c+32) were read); returns the row sum.
+template <bool MASKED>
+__device__ __forceinline__ float row_exp(uint32_t tS, const uint32_t (&vis)[4], uint64_t sc2, uint64_t nm2) {
+  uint64_t acc0 = pk2(0.0f, 0.0f), acc1 = acc0;
+  uint32_t ra[32], rb[32];
+  ptx::tmem_ld32(tS, ra);
+  ptx::tmem_ld_wait();
+#pragma unroll
+  for (int c = 0; c < 4; ++c) {
+    uint32_t (&r)[32] = (c & 1) ? rb : ra;
+    uint32_t (&rn)[32] = (c & 1) ? ra : rb;
+    if (c < 3) ptx::tmem_ld32(tS + (c + 1) * 32, rn);  // in flight while chunk c computes
+    uint32_t pk[16];
+#pragma unroll
+    for (int i = 0; i < 16; ++i) {
+      const uint64_t xv = ffma2(pk2(__uint_as_float(r[2 * i]), __uint_as_float(r[2 * i + 1])), sc2, nm2);
+      uint64_t e;
+      if (i < BAT_POLY_PAIRS) {
+        e = exp2_poly2(xv);
+      } else {
+        float x0, x1;
+        up2(xv, x0, x1);
+        e = pk2(ex2(x0), ex2(x1));
+      }
+      float p0, p1;
+      up2(e, p0, p1);
+      if (MASKED) {
+        p0 = ((vis[c] >> (2 * i)) & 1u) ? p0 : 0.0f;
+        p1 = ((vis[c] >> (2 * i + 1)) & 1u) ? p1 : 0.0f;
+        e = pk2(p0, p1);
+      }
+      if (i & 1) acc1 = fadd2(acc1, e);
+      else acc0 = fadd2(acc0, e);
+      pk[i] = ptx::pack_bf16x2(p0, p1);
+    }
+    // P columns [16c, 16c+16): S columns already consumed (chunk c+1 reads [32c+32, 32c+64))
+    asm volatile(
+        "tcgen05.st.sync.aligned.32x32b.x16.b32 [%0], "
+        "{%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,%16};" ::"r"(tS + c * 16),
+        "r"(pk[0]), "r"(pk[1]), "r"(pk[2]), "r"(pk[3]), "r"(pk[4]), "r"(pk[5]), "r"(pk[6]), "r"(pk[7]),
+        "r"(pk[8]), "r"(pk[9]), "r"(pk[10]), "r"(pk[11]), "r"(pk[12]), "r"(pk[13]), "r"(pk[14]),
+        "r"(pk[15]));
+    if (c < 3) ptx::tmem_ld_wait();
+  }
+  float a0, a1, b0, b1;
+  up2(acc0, a0, a1);
+  up2(acc1, b0, b1);
+  return (a0 + a1) + (b0 + b1);
+}
+
+// Single-pass variant against the current reference max: computes all of P in registers and
+// tracks the row's largest exponent; P is written to TMEM only if no visible exponent exceeds
+// `limit` (the lazy-rescale threshold) — the common case once the running max has settled.
+// Returns false (nothing written, S intact) when the caller must take the two-pass path.
+template <bool MASKED>
+__device__ __forceinline__ bool row_exp_opt(uint32_t tS, const uint32_t (&vis)[4], uint64_t sc2, uint64_t nm2,
+                                            float limit, float& lsum) {
+  uint64_t acc0 = pk2(0.0f, 0.0f), acc1 = acc0;
+  uint32_t pk[64];
+  float xm0 = -INFINITY, xm1 = -INFINITY;
+#pragma unroll
+  for (int c = 0; c < 4; ++c) {
+    uint32_t r[32];
+    ptx::tmem_ld32(tS + c * 32, r);
+    ptx::tmem_ld_wait();
+#pragma unroll
+    for (int i = 0; i < 16; ++i) {
+      uint64_t xv = ffma2(pk2(__uint_as_float(r[2 * i]), __uint_as_float(r[2 * i + 1])), sc2, nm2);
+      float x0, x1;
+      up2(xv, x0, x1);
+      if (MASKED) {
+        x0 = ((vis[c] >> (2 * i)) & 1u) ? x0 : -INFINITY;
+        x1 = ((vis[c] >> (2 * i + 1)) & 1u) ? x1 : -INFINITY;
+        xv = pk2(x0, x1);
+      }
+      if (i & 1) xm1 = fmax3(xm1, x0, x1);
+      else xm0 = fmax3(xm0, x0, x1);
+      uint64_t e;
+      if (i < BAT_POLY_PAIRS) {
+        e = exp2_poly2(xv);
+        if (MASKED) {  // the polynomial clamps at -127: re-zero masked lanes
+          float p0, p1;
+          up2(e, p0, p1);
+          e = pk2(x0 == -INFINITY ? 0.0f : p0, x1 == -INFINITY ? 0.0f : p1);
+        }
+      } else {
+        e = pk2(ex2(x0), ex2(x1));  // ex2(-inf) = 0
+      }
+      float p0, p1;
+      up2(e, p0, p1);
+      if (i & 1) acc1 = fadd2(acc1, e);
+      else acc0 = fadd2(acc0, e);
+      pk[c * 16 + i] = ptx::pack_bf16x2(p0, p1);
+    }
+  }
+  const bool ok = fmaxf(xm0, xm1) <= limit;
+  if (!__all_sync(0xffffffffu, ok)) return false;
+#pragma unroll
+  for (int c = 0; c < 4; ++c)
+    asm volatile(
+        "tcgen05.st.sync.aligned.32x32b.x16.b32 [%0], "
+        "{%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,%16};" ::"r"(tS + c * 16),
+        "r"(pk[c * 16 + 0]), "r"(pk[c * 16 + 1]), "r"(pk[c * 16 + 2]), "r"(pk[c * 16 + 3]), "r"(pk[c * 16 + 4]),
+        "r"(pk[c * 16 + 5]), "r"(pk[c * 16 + 6]), "r"(pk[c * 16 + 7]), "r"(pk[c * 16 + 8]), "r"(pk[c * 16 + 9]),
+        "r"(pk[c * 16 + 10]), "r"(pk[c * 16 + 11]), "r"(pk[c * 16 + 12]), "r"(pk[c * 16 + 13]),
+        "r"(pk[c * 16 + 14]), "r"(pk[c * 16 + 15]));
+  float a0, a1, b0, b1;
+  up2(acc0, a0, a1);
+  up2(acc1, b0, b1);
+  lsum = (a0 + a1) + (b0 + b1);
+  return true;
+}
+
+__device__ __forceinline__ void row_zero_p(uint32_t tS) {
+#pragma unroll
+  for (int c = 0; c < 4; ++c)
+    asm volatile(
+        "tcgen05.st.sync.aligned.32x32b.x16.b32 [%0], "
+        "{%1,%1,%1,%1,%1,%1,%1,%1,%1,%1,%1,%1,%1,%1,%1,%1};" ::"r"(tS + c * 16), "r"(0u));
 }
 
 template <int DP>
@@ -193,8 +351,11 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) attn_tc_kernel(const __grid_co
         const char* src = (lane < kKtilePages) ? resolve_page(p, my_page) : nullptr;
         uint8_t* sk = smem + L::K_OFF + s * L::TILE_BYTES;
         uint8_t* sv = smem + L::V_OFF + s * L::TILE_BYTES;
+        const bool dbg_first = (qc == 0);
         if (lane == 0) {
+          DBG(0, x);
           ptx::mbar_wait(&bars->k_empty[s], ph);
+          DBG(1, x);
           ptx::mbar_expect_tx(&bars->k_full[s], L::TILE_BYTES);
         }
         __syncwarp();
@@ -206,6 +367,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) attn_tc_kernel(const __grid_co
         }
         if (lane == 0) {
           ptx::mbar_wait(&bars->v_empty[s], ph);
+          DBG(2, x);
           ptx::mbar_expect_tx(&bars->v_full[s], L::TILE_BYTES + 1024);
           ptx::bulk_g2s(smem + L::META_OFF + s * 1024,
                         img + p.off_kmeta + (int64_t(page_off) + int64_t(j) * kKtilePages) * kPageTokens * 2,
@@ -261,23 +423,28 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) attn_tc_kernel(const __grid_co
           ptx::mma_commit(&bars->k_empty[s]);
           if (n == 1) ptx::mma_commit(&bars->q_empty);
         }
+        const bool dbg_first = (qc == 0);
         for (int x = 0; x < n; ++x) {
           const uint32_t g = kc + x;
           const int s = g & 1;
           const uint32_t sv = ptx::smem_u32(smem + L::V_OFF + s * L::TILE_BYTES);
+          DBG(3, x);
           const bool more = x + 1 < n;
           const uint32_t gn = g + 1;
           const int sn = gn & 1;
           const uint32_t skn = ptx::smem_u32(smem + L::K_OFF + sn * L::TILE_BYTES);
           // ---- q-tile 0: PV0_x, then S0_{x+1}
           ptx::mbar_wait(&bars->p_full[0], pc0 & 1);
+          DBG(4, x);
           ++pc0;
           ptx::mbar_wait(&bars->v_full[s], (g >> 1) & 1);
+          DBG(5, x);
           if (x == 0) ptx::mbar_wait(&bars->o_empty[0], (oc0 & 1) ^ 1);
           ptx::tc_fence_after();
           issue_pv(tS0, tO0, sv, x > 0);
           if (more) {
             ptx::mbar_wait(&bars->k_full[sn], (gn >> 1) & 1);
+            DBG(6, x);
             ptx::tc_fence_after();
             issue_s(sq0, tS0, skn);
             ptx::mma_commit(&bars->s_full[0]);
@@ -285,6 +452,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) attn_tc_kernel(const __grid_co
           // ---- q-tile 1: PV1_x, then S1_{x+1}
           if (has1) {
             ptx::mbar_wait(&bars->p_full[1], pc1 & 1);
+            DBG(7, x);
             ++pc1;
             if (x == 0) ptx::mbar_wait(&bars->o_empty[1], (oc1 & 1) ^ 1);
             ptx::tc_fence_after();
@@ -338,7 +506,10 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) attn_tc_kernel(const __grid_co
         const uint32_t g = kc + x;
         const int s = g & 1;
         const int state = (ktl[x] >> (24 + 2 * wg)) & 3;
+        const bool dbg_first = (kc == 0) && row == 0;
+        DBG(8 + 4 * wg, x);
         ptx::mbar_wait(&bars->s_full[wg], sc & 1);
+        DBG(9 + 4 * wg, x);
         ++sc;
         ptx::tc_fence_after();
         uint32_t vis[4] = {0xffffffffu, 0xffffffffu, 0xffffffffu, 0xffffffffu};
@@ -358,41 +529,24 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) attn_tc_kernel(const __grid_co
             vis[c] = bits;
           }
         }
-        // pass 1: row max of the raw scores (4 independent FMNMX3 chains)
-        float mt = -INFINITY;
-        if (state == 1) {
-#pragma unroll
-          for (int c = 0; c < 4; ++c) {
-            uint32_t r[32];
-            ptx::tmem_ld32(tS + c * 32, r);
-            ptx::tmem_ld_wait();
-            float m0 = mt, m1 = -INFINITY, m2 = -INFINITY, m3 = -INFINITY;
-#pragma unroll
-            for (int i = 0; i < 32; i += 8) {
-              m0 = fmax3(m0, __uint_as_float(r[i]), __uint_as_float(r[i + 1]));
-              m1 = fmax3(m1, __uint_as_float(r[i + 2]), __uint_as_float(r[i + 3]));
-              m2 = fmax3(m2, __uint_as_float(r[i + 4]), __uint_as_float(r[i + 5]));
-              m3 = fmax3(m3, __uint_as_float(r[i + 6]), __uint_as_float(r[i + 7]));
-            }
-            mt = fmaxf(fmax3(m0, m1, m2), m3);
-          }
-        } else if (state == 2) {
-#pragma unroll
-          for (int c = 0; c < 4; ++c) {
-            uint32_t r[32];
-            ptx::tmem_ld32(tS + c * 32, r);
-            ptx::tmem_ld_wait();
-            float m0 = mt, m1 = -INFINITY;
-#pragma unroll
-            for (int i = 0; i < 32; i += 2) {
-              const float a = ((vis[c] >> i) & 1u) ? __uint_as_float(r[i]) : -INFINITY;
-              const float b = ((vis[c] >> (i + 1)) & 1u) ? __uint_as_float(r[i + 1]) : -INFINITY;
-              m0 = fmaxf(m0, a);
-              m1 = fmaxf(m1, b);
-            }
-            mt = fmaxf(m0, m1);
-          }
+        // fast path: one pass against the settled reference max
+        bool done = false;
+        float lsum = 0.0f;
+        if (state == 0) {
+          row_zero_p(tS);
+          done = true;
+        } else if (__all_sync(0xffffffffu, m_ref != -INFINITY)) {  // warp-uniform: .sync.aligned ops
+          const float mref0 = m_ref;
+          const uint64_t sc2 = pk2(p.scale_log2, p.scale_log2), nm2 = pk2(-mref0, -mref0);
+          done = (state == 1) ? row_exp_opt<false>(tS, vis, sc2, nm2, kRescaleThreshold, lsum)
+                              : row_exp_opt<true>(tS, vis, sc2, nm2, kRescaleThreshold, lsum);
         }
+        DBG(10 + 4 * wg, x);
+        if (!done) {
+        // slow path, pass 1: row max of the raw scores
+        float mt = -INFINITY;
+        if (state == 1) mt = row_max<false>(tS, vis);
+        else if (state == 2) mt = row_max<true>(tS, vis);
         const float m_old = m_ref;
         const float m_new = fmaxf(m_ref, mt * p.scale_log2);
         const bool grow = m_new > m_ref + kRescaleThreshold;
@@ -419,63 +573,18 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) attn_tc_kernel(const __grid_co
           ptx::tmem_st_wait();
         }
         // pass 2: P = exp2(s * scale - m_ref) -> bf16 into the S buffer's first 64 columns;
-        // 6 of every 16 column pairs on the FMA pipe (polynomial), the rest on the MUFU.
+        // BAT_POLY_PAIRS of every 16 column pairs on the FMA pipe (polynomial), rest on MUFU.
         const float mref = (m_ref == -INFINITY) ? 0.0f : m_ref;
         const uint64_t sc2 = pk2(p.scale_log2, p.scale_log2), nm2 = pk2(-mref, -mref);
-        uint64_t acc0 = pk2(0.0f, 0.0f), acc1 = acc0;
-#pragma unroll
-        for (int c = 0; c < 4; ++c) {
-          uint32_t pk[16];
-          if (state != 0) {
-            uint32_t r[32];
-            ptx::tmem_ld32(tS + c * 32, r);
-            ptx::tmem_ld_wait();
-#pragma unroll
-            for (int i = 0; i < 16; ++i) {
-              const uint64_t xv = ffma2(pk2(__uint_as_float(r[2 * i]), __uint_as_float(r[2 * i + 1])), sc2, nm2);
-              uint64_t e;
-              if (i < BAT_POLY_PAIRS) {
-                e = exp2_poly2(xv);
-              } else {
-                float x0, x1;
-                up2(xv, x0, x1);
-                e = pk2(ex2(x0), ex2(x1));
-              }
-              float p0, p1;
-              up2(e, p0, p1);
-              if (state == 2) {
-                p0 = ((vis[c] >> (2 * i)) & 1u) ? p0 : 0.0f;
-                p1 = ((vis[c] >> (2 * i + 1)) & 1u) ? p1 : 0.0f;
-                e = pk2(p0, p1);
-              }
-              if (i & 1) acc1 = fadd2(acc1, e);
-              else acc0 = fadd2(acc0, e);
-              pk[i] = ptx::pack_bf16x2(p0, p1);
-            }
-          } else {
-#pragma unroll
-            for (int i = 0; i < 16; ++i) pk[i] = 0u;
-          }
-          // columns [16c, 16c+16) of the S buffer: already consumed S values
-          asm volatile(
-              "tcgen05.st.sync.aligned.32x32b.x16.b32 [%0], "
-              "{%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,%16};" ::"r"(tS + c * 16),
-              "r"(pk[0]), "r"(pk[1]), "r"(pk[2]), "r"(pk[3]), "r"(pk[4]), "r"(pk[5]), "r"(pk[6]), "r"(pk[7]),
-              "r"(pk[8]), "r"(pk[9]), "r"(pk[10]), "r"(pk[11]), "r"(pk[12]), "r"(pk[13]), "r"(pk[14]),
-              "r"(pk[15]));
-        }
-        float lsum;
-        {
-          float a0, a1, b0, b1;
-          up2(acc0, a0, a1);
-          up2(acc1, b0, b1);
-          lsum = (a0 + a1) + (b0 + b1);
+        if (state == 1) lsum = row_exp<false>(tS, vis, sc2, nm2);
+        else if (state == 2) lsum = row_exp<true>(tS, vis, sc2, nm2);
         }
         l_sum += lsum;
         ptx::tmem_st_wait();
         ptx::tc_fence_before();
         __syncwarp();
         if (lane == 0) ptx::mbar_arrive(&bars->p_full[wg]);
+        DBG(11 + 4 * wg, x);
       }
       kc += wi.kt_n;
       // ---- epilogue: O / l -> bf16

@@ -40,6 +40,7 @@ struct AttnParams {
   const __nv_bfloat16* qp;  // packed, swizzled q-tiles
   __nv_bfloat16* out;       // O [M][q_heads*head_dim]
   float scale_log2;         // log2(e) / sqrt(head_dim)
+  long long* dbg;           // optional timeline (clock64) of CTA 0's first work item
 };
 size_t attn_smem_bytes(int dpad);
 void launch_attention(int dpad, const AttnParams& p, int num_sms, cudaStream_t stream);
