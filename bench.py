@@ -447,8 +447,14 @@ def main():
     dom = max(prof, key=lambda k: prof[k]["ms"])
     dp = prof[dom]
     achieved = dp["flops"] / (dp["ms"] / 1e3) / 1e12 if dp["ms"] > 0 else 0.0
+    traffic = None
+    tp = os.path.join(ROOT, "profiles", "ncu_traffic.json")
+    if os.path.exists(tp) and B == 64:  # captured at this batch (layer-0 launch, one ncu --set full)
+        traffic = json.load(open(tp))["dram_bytes_per_launch"].get(dom)
     roof = dict(kernel=dom, bound="tensor", achieved=achieved, peak=pk["bf16_sus"], unit="TFLOP/s",
-                frac=achieved / pk["bf16_sus"], traffic=None,
+                frac=achieved / pk["bf16_sus"], traffic=traffic,
+                traffic_unit="DRAM bytes per launch (ncu dram__bytes_read.sum + dram__bytes_write.sum)",
+                algorithmic_bytes_per_launch=dp["bytes"] / max(1, dp["launches"]),
                 peak_note=f"bf16 sustained, {pk['src']} (kernel timed inside the step)",
                 share_of_step=dp["ms"] / max(1e-9, sum(v["ms"] for v in prof.values())))
     at = prof["attention"]
