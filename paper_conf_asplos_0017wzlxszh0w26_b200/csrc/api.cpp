@@ -64,14 +64,18 @@ static EncodeTiledFn encode_fn() {
   return fn;
 }
 
-// bf16 row-major [rows][cols] with leading dimension ld (elements); box = [64 cols][box_rows]
-static CUtensorMap make_tmap(const void* ptr, int64_t rows, int64_t cols, int64_t ld, int box_rows) {
+// row-major [rows][cols] with leading dimension ld (elements); box = [128 bytes of cols][box_rows],
+// 128-byte swizzle (bf16: 64 columns; fp32: 32 columns)
+static CUtensorMap make_tmap(const void* ptr, int64_t rows, int64_t cols, int64_t ld, int box_rows,
+                             bool f32 = false) {
   CUtensorMap m;
+  const int esz = f32 ? 4 : 2;
   cuuint64_t dims[2] = {cuuint64_t(cols), cuuint64_t(rows)};
-  cuuint64_t strides[1] = {cuuint64_t(ld * 2)};
-  cuuint32_t box[2] = {64, cuuint32_t(box_rows)};
+  cuuint64_t strides[1] = {cuuint64_t(ld * esz)};
+  cuuint32_t box[2] = {cuuint32_t(128 / esz), cuuint32_t(box_rows)};
   cuuint32_t estr[2] = {1, 1};
-  CUresult r = encode_fn()(&m, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 2, const_cast<void*>(ptr), dims,
+  CUresult r = encode_fn()(&m, f32 ? CU_TENSOR_MAP_DATA_TYPE_FLOAT32 : CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 2,
+                           const_cast<void*>(ptr), dims,
                            strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
                            CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
                            CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
@@ -369,6 +373,12 @@ static void run_plan(Pool& pool, Model& m, Plan& plan, float* out_hidden, cudaSt
   const CUtensorMap tA_xc = make_tmap(ws.xc.p, B, H, H, 128);
   const CUtensorMap tA_oc = make_tmap(ws.oc.p, B, nq, nq, 128);
   const CUtensorMap tA_actc = make_tmap(ws.actc.p, B, F, F, 128);
+  // outputs (epilogue TMA store / reduce-add, 32-row boxes)
+  const CUtensorMap tC_qkv = make_tmap(ws.qkv.p, M, m.nqkv(), m.nqkv(), 32);
+  const CUtensorMap tC_h = make_tmap(ws.h.p, M, H, H, 32, true);
+  const CUtensorMap tC_act = make_tmap(ws.act.p, M, F, F, 32);
+  const CUtensorMap tC_hc = make_tmap(ws.hc.p, B, H, H, 32, true);
+  const CUtensorMap tC_actc = make_tmap(ws.actc.p, B, F, F, 32);
   AttnParams ap = attn_params(pool, m, plan, I);
   StageParams sp = stage_params(pool, m, plan, I);
 
@@ -384,7 +394,7 @@ static void run_plan(Pool& pool, Model& m, Plan& plan, float* out_hidden, cudaSt
     GemmParams gp{M, m.nqkv(), H, ws.qkv.p, m.nqkv(), Lw.bqkv, 0};
     auto fq = gemm_fb(M, m.nqkv(), H, 2);
     pf.begin(st);
-    launch_gemm(EPI_BF16_BIAS, tA_xn, Lw.t_qkv, gp, m.num_sms, st);
+    launch_gemm(EPI_BF16_BIAS, tA_xn, Lw.t_qkv, tC_qkv, gp, m.num_sms, st);
     pf.end(st, BAT_K_GEMM_QKV, fq.first, fq.second);
     sp.pool_layer_off = int64_t(l) * pool.geo.layer_bytes;
     pf.begin(st);
@@ -401,7 +411,7 @@ static void run_plan(Pool& pool, Model& m, Plan& plan, float* out_hidden, cudaSt
       GemmParams go{M, H, nq, ws.h.p, H, nullptr, 0};
       auto fo = gemm_fb(M, H, nq, 8);
       pf.begin(st);
-      launch_gemm(EPI_RESID_F32, tA_o, Lw.t_o, go, m.num_sms, st);
+      launch_gemm(EPI_RESID_F32, tA_o, Lw.t_o, tC_h, go, m.num_sms, st);
       pf.end(st, BAT_K_GEMM_O, fo.first, fo.second);
       pf.begin(st);
       launch_rmsnorm_bf16(ws.h.as<float>(), Lw.ln2, ws.xn.as<__nv_bfloat16>(), M, H, c.rms_eps, st);
@@ -409,12 +419,12 @@ static void run_plan(Pool& pool, Model& m, Plan& plan, float* out_hidden, cudaSt
       GemmParams gg{M, F, H, ws.act.p, F, nullptr, F};
       auto fg = gemm_fb(M, 2 * F, H, 1);
       pf.begin(st);
-      launch_gemm(EPI_SWIGLU, tA_xn, Lw.t_gu, gg, m.num_sms, st);
+      launch_gemm(EPI_SWIGLU, tA_xn, Lw.t_gu, tC_act, gg, m.num_sms, st);
       pf.end(st, BAT_K_GEMM_GU, fg.first, fg.second);
       GemmParams gd{M, H, F, ws.h.p, H, nullptr, 0};
       auto fd = gemm_fb(M, H, F, 8);
       pf.begin(st);
-      launch_gemm(EPI_RESID_F32, tA_act, Lw.t_d, gd, m.num_sms, st);
+      launch_gemm(EPI_RESID_F32, tA_act, Lw.t_d, tC_h, gd, m.num_sms, st);
       pf.end(st, BAT_K_GEMM_DOWN, fd.first, fd.second);
     } else {
       // a8: after the last layer's K/V only the discriminant rows matter
@@ -431,7 +441,7 @@ static void run_plan(Pool& pool, Model& m, Plan& plan, float* out_hidden, cudaSt
       GemmParams go{B, H, nq, ws.hc.p, H, nullptr, 0};
       auto fo = gemm_fb(B, H, nq, 8);
       pf.begin(st);
-      launch_gemm(EPI_RESID_F32, tA_oc, Lw.t_o, go, m.num_sms, st);
+      launch_gemm(EPI_RESID_F32, tA_oc, Lw.t_o, tC_hc, go, m.num_sms, st);
       pf.end(st, BAT_K_GEMM_O, fo.first, fo.second);
       pf.begin(st);
       launch_rmsnorm_bf16(ws.hc.as<float>(), Lw.ln2, ws.xc.as<__nv_bfloat16>(), B, H, c.rms_eps, st);
@@ -439,12 +449,12 @@ static void run_plan(Pool& pool, Model& m, Plan& plan, float* out_hidden, cudaSt
       GemmParams gg{B, F, H, ws.actc.p, F, nullptr, F};
       auto fg = gemm_fb(B, 2 * F, H, 1);
       pf.begin(st);
-      launch_gemm(EPI_SWIGLU, tA_xc, Lw.t_gu, gg, m.num_sms, st);
+      launch_gemm(EPI_SWIGLU, tA_xc, Lw.t_gu, tC_actc, gg, m.num_sms, st);
       pf.end(st, BAT_K_GEMM_GU, fg.first, fg.second);
       GemmParams gd{B, H, F, ws.hc.p, H, nullptr, 0};
       auto fd = gemm_fb(B, H, F, 8);
       pf.begin(st);
-      launch_gemm(EPI_RESID_F32, tA_actc, Lw.t_d, gd, m.num_sms, st);
+      launch_gemm(EPI_RESID_F32, tA_actc, Lw.t_d, tC_hc, gd, m.num_sms, st);
       pf.end(st, BAT_K_GEMM_DOWN, fd.first, fd.second);
       pf.begin(st);
       launch_rmsnorm_f32out(ws.hc.as<float>(), m.final_norm, out_hidden, B, H, c.rms_eps, st);
@@ -1016,8 +1026,9 @@ bat_status bat_debug_gemm(int32_t epi, int32_t M, int32_t N, int32_t K, const vo
     CUDA_OK(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, device));
     const CUtensorMap ta = make_tmap(A, M, K, K, 128);
     const CUtensorMap tb = make_tmap(Bw, b_rows, K, K, epi == EPI_SWIGLU ? 128 : 256);
+    const CUtensorMap tc = make_tmap(out, M, N, ldo, 32, epi == EPI_RESID_F32);
     GemmParams gp{M, N, K, out, ldo, static_cast<const __nv_bfloat16*>(bias), up_row0};
-    launch_gemm(epi, ta, tb, gp, sms, static_cast<cudaStream_t>(stream));
+    launch_gemm(epi, ta, tb, tc, gp, sms, static_cast<cudaStream_t>(stream));
     CUDA_OK(cudaGetLastError());
   });
 }

@@ -1,6 +1,7 @@
 // tcgen05 GEMM for the dense projections of every layer:
 //   C[M,N] = A[M,K] * B[N,K]^T, A = bf16 activations (K-major), B = bf16 weights [N][K]
-// with the layer's elementwise work fused into the epilogue:
+// with the layer's elementwise work fused into the epilogue, written back through 128B-swizzled
+// shared-memory staging and TMA (tile store, or TMA reduce-add for the fp32 residual stream):
 //   EPI_BF16_BIAS  qkv = a*Wqkv^T + b             (bf16 out)
 //   EPI_RESID_F32  h  += o*Wo^T  /  h += act*Wd^T (fp32 residual stream, in place)
 //   EPI_SWIGLU     act = silu(x*Wg^T) * (x*Wu^T)  (the B tile holds 128 gate + 128 up rows)
@@ -32,7 +33,9 @@ struct __align__(8) GemmSmemBars {
   uint32_t tmem_base;
 };
 
-constexpr size_t kGemmSmem = 1024 /*align slack*/ + STAGES * STAGE_BYTES + sizeof(GemmSmemBars);
+constexpr int STG_BYTES = 4096;  // per-warp epilogue staging buffer: [32 rows][128 B], 128B-swizzled
+constexpr int STG_OFF = STAGES * STAGE_BYTES;
+constexpr size_t kGemmSmem = 1024 /*align slack*/ + STAGES * STAGE_BYTES + 4 * 2 * STG_BYTES + sizeof(GemmSmemBars);
 
 __device__ __forceinline__ void tile_coords(int t, int num_m, int num_n, int& m, int& n) {
   const int per_group = GROUP_M * num_n;
@@ -48,10 +51,10 @@ __device__ __forceinline__ float silu(float x) { return x / (1.0f + __expf(-x));
 template <int EPI>
 __global__ void __launch_bounds__(NUM_THREADS, 1)
 gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
-               GemmParams p) {
+               const __grid_constant__ CUtensorMap tmC, GemmParams p) {
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
-  GemmSmemBars* bars = reinterpret_cast<GemmSmemBars*>(smem + STAGES * STAGE_BYTES);
+  GemmSmemBars* bars = reinterpret_cast<GemmSmemBars*>(smem + STG_OFF + 4 * 2 * STG_BYTES);
   const uint32_t warp = ptx::warp_id(), lane = ptx::lane_id();
 
   const int out_bn = (EPI == EPI_SWIGLU) ? BN / 2 : BN;  // output columns per tile
@@ -72,6 +75,7 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
     ptx::fence_mbar_init();
     ptx::prefetch_tmap(&tmA);
     ptx::prefetch_tmap(&tmB);
+    ptx::prefetch_tmap(&tmC);
   }
   if (warp == 1) ptx::tmem_alloc(&bars->tmem_base, 512);
   ptx::tc_fence_before();
@@ -131,8 +135,30 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
       }
     }
   } else {  // ------------------------------ epilogue warps 2..5
+    // TMEM -> registers -> (bias / SwiGLU) -> 128B-swizzled smem staging -> TMA store (bf16)
+    // or TMA reduce-add (fp32 residual).  Coalesced, asynchronous, double-buffered per warp.
     const uint32_t sub = warp & 3;  // TMEM sub-partition this warp may access
-    const int row_in_tile = sub * 32 + lane;
+    uint8_t* stg = smem + STG_OFF + (warp - 2) * 2 * STG_BYTES;
+    int sbuf = 0;
+    auto stage_row = [&](uint8_t* buf, int chunk16, uint32_t a, uint32_t b, uint32_t c, uint32_t d) {
+      ptx::st_shared_v4(buf + lane * 128 + ((chunk16 ^ (lane & 7)) << 4), a, b, c, d);
+    };
+    auto next_buf = [&]() -> uint8_t* {
+      uint8_t* buf = stg + sbuf * STG_BYTES;
+      if (lane == 0) ptx::bulk_wait_read<1>();  // the group that last used this buffer is done
+      __syncwarp();
+      return buf;
+    };
+    auto flush = [&](uint8_t* buf, int col, int row) {
+      ptx::fence_proxy_async_smem();
+      __syncwarp();
+      if (lane == 0) {
+        if (EPI == EPI_RESID_F32) ptx::tma_reduce_add_2d(&tmC, buf, col, row);
+        else ptx::tma_store_2d(&tmC, buf, col, row);
+        ptx::bulk_commit();
+      }
+      sbuf ^= 1;
+    };
     int acc = 0;
     uint32_t acc_phase = 0;
     for (int t = blockIdx.x; t < num_tiles; t += gridDim.x) {
@@ -141,17 +167,17 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
       ptx::mbar_wait(&bars->tfull[acc], acc_phase);
       ptx::tc_fence_after();
       const uint32_t tbase = tmem + ((sub * 32) << 16) + acc * BN;
-      const int row = m * BM + row_in_tile;
-      const bool row_ok = row < p.M;
+      const int row0 = m * BM + sub * 32;
       if (EPI == EPI_SWIGLU) {
 #pragma unroll 1
-        for (int c = 0; c < BN / 2; c += 32) {
-          uint32_t g[32], u[32];
-          ptx::tmem_ld32(tbase + c, g);
-          ptx::tmem_ld32(tbase + BN / 2 + c, u);
-          ptx::tmem_ld_wait();
-          const int col = n * (BN / 2) + c;
-          if (row_ok && col < p.N) {
+        for (int c = 0; c < BN / 2; c += 64) {  // 64 output columns per staging buffer
+          uint8_t* buf = next_buf();
+#pragma unroll
+          for (int h = 0; h < 2; ++h) {
+            uint32_t g[32], u[32];
+            ptx::tmem_ld32(tbase + c + 32 * h, g);
+            ptx::tmem_ld32(tbase + BN / 2 + c + 32 * h, u);
+            ptx::tmem_ld_wait();
             uint32_t pk[16];
 #pragma unroll
             for (int i = 0; i < 16; ++i) {
@@ -159,46 +185,46 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
               float u0 = __uint_as_float(u[2 * i]), u1 = __uint_as_float(u[2 * i + 1]);
               pk[i] = ptx::pack_bf16x2(silu(g0) * u0, silu(g1) * u1);
             }
-            uint4* dst = reinterpret_cast<uint4*>(static_cast<__nv_bfloat16*>(p.out) + size_t(row) * p.ldo + col);
 #pragma unroll
-            for (int i = 0; i < 4; ++i) dst[i] = make_uint4(pk[4 * i], pk[4 * i + 1], pk[4 * i + 2], pk[4 * i + 3]);
+            for (int j = 0; j < 4; ++j) stage_row(buf, 4 * h + j, pk[4 * j], pk[4 * j + 1], pk[4 * j + 2], pk[4 * j + 3]);
           }
+          flush(buf, n * (BN / 2) + c, row0);
         }
-      } else {
+      } else if (EPI == EPI_RESID_F32) {
 #pragma unroll 1
-        for (int c = 0; c < BN; c += 32) {
+        for (int c = 0; c < BN; c += 32) {  // 32 fp32 columns per staging buffer
+          uint8_t* buf = next_buf();
           uint32_t r[32];
           ptx::tmem_ld32(tbase + c, r);
           ptx::tmem_ld_wait();
-          const int col = n * BN + c;
-          if (row_ok && col < p.N) {
-            if (EPI == EPI_RESID_F32) {
-              float4* dst = reinterpret_cast<float4*>(static_cast<float*>(p.out) + size_t(row) * p.ldo + col);
 #pragma unroll
-              for (int i = 0; i < 8; ++i) {
-                float4 h = dst[i];
-                h.x += __uint_as_float(r[4 * i]);
-                h.y += __uint_as_float(r[4 * i + 1]);
-                h.z += __uint_as_float(r[4 * i + 2]);
-                h.w += __uint_as_float(r[4 * i + 3]);
-                dst[i] = h;
+          for (int j = 0; j < 8; ++j) stage_row(buf, j, r[4 * j], r[4 * j + 1], r[4 * j + 2], r[4 * j + 3]);
+          flush(buf, n * BN + c, row0);
+        }
+      } else {
+#pragma unroll 1
+        for (int c = 0; c < BN; c += 64) {  // 64 bf16 columns per staging buffer
+          uint8_t* buf = next_buf();
+#pragma unroll
+          for (int h = 0; h < 2; ++h) {
+            uint32_t r[32];
+            ptx::tmem_ld32(tbase + c + 32 * h, r);
+            ptx::tmem_ld_wait();
+            const int col = n * BN + c + 32 * h;
+            uint32_t pk[16];
+#pragma unroll
+            for (int i = 0; i < 16; ++i) {
+              float v0 = __uint_as_float(r[2 * i]), v1 = __uint_as_float(r[2 * i + 1]);
+              if (EPI == EPI_BF16_BIAS && col + 2 * i + 1 < p.N) {
+                v0 += __bfloat162float(p.bias[col + 2 * i]);
+                v1 += __bfloat162float(p.bias[col + 2 * i + 1]);
               }
-            } else {
-              uint32_t pk[16];
-#pragma unroll
-              for (int i = 0; i < 16; ++i) {
-                float v0 = __uint_as_float(r[2 * i]), v1 = __uint_as_float(r[2 * i + 1]);
-                if (EPI == EPI_BF16_BIAS) {
-                  v0 += __bfloat162float(p.bias[col + 2 * i]);
-                  v1 += __bfloat162float(p.bias[col + 2 * i + 1]);
-                }
-                pk[i] = ptx::pack_bf16x2(v0, v1);
-              }
-              uint4* dst = reinterpret_cast<uint4*>(static_cast<__nv_bfloat16*>(p.out) + size_t(row) * p.ldo + col);
-#pragma unroll
-              for (int i = 0; i < 4; ++i) dst[i] = make_uint4(pk[4 * i], pk[4 * i + 1], pk[4 * i + 2], pk[4 * i + 3]);
+              pk[i] = ptx::pack_bf16x2(v0, v1);
             }
+#pragma unroll
+            for (int j = 0; j < 4; ++j) stage_row(buf, 4 * h + j, pk[4 * j], pk[4 * j + 1], pk[4 * j + 2], pk[4 * j + 3]);
           }
+          flush(buf, n * BN + c, row0);
         }
       }
       ptx::tc_fence_before();
@@ -206,6 +232,8 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
       if (lane == 0) ptx::mbar_arrive(&bars->tempty[acc]);
       if (++acc == 2) { acc = 0; acc_phase ^= 1; }
     }
+    if (lane == 0) ptx::bulk_wait<0>();
+    __syncwarp();
   }
   ptx::tc_fence_before();
   __syncthreads();
@@ -216,8 +244,8 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
 
 size_t gemm_smem_bytes() { return kGemmSmem; }
 
-void launch_gemm(int epi, const CUtensorMap& tmA, const CUtensorMap& tmB, const GemmParams& p,
-                 int num_sms, cudaStream_t stream) {
+void launch_gemm(int epi, const CUtensorMap& tmA, const CUtensorMap& tmB, const CUtensorMap& tmC,
+                 const GemmParams& p, int num_sms, cudaStream_t stream) {
   const int out_bn = (epi == EPI_SWIGLU) ? BN / 2 : BN;
   const int tiles = ((p.M + BM - 1) / BM) * ((p.N + out_bn - 1) / out_bn);
   const int grid = tiles < num_sms ? tiles : num_sms;
@@ -231,7 +259,7 @@ void launch_gemm(int epi, const CUtensorMap& tmA, const CUtensorMap& tmB, const 
                            static_cast<int>(kGemmSmem));                                        \
       attr = true;                                                                              \
     }                                                                                           \
-    gemm_tc_kernel<E><<<grid, NUM_THREADS, kGemmSmem, stream>>>(tmA, tmB, p);                  \
+    gemm_tc_kernel<E><<<grid, NUM_THREADS, kGemmSmem, stream>>>(tmA, tmB, tmC, p);             \
     break;                                                                                      \
   }
     BAT_GEMM_CASE(EPI_BF16)

@@ -22,8 +22,10 @@ struct GemmParams {
   int up_row0;        // EPI_SWIGLU: first "up" row of B (= F)
 };
 size_t gemm_smem_bytes();
-void launch_gemm(int epi, const CUtensorMap& tmA, const CUtensorMap& tmB, const GemmParams& p,
-                 int num_sms, cudaStream_t stream);
+// tmC: output tensor map — bf16 [M][ldo] with box {64, 32} (EPI_BF16*, EPI_SWIGLU) or fp32
+// [M][ldo] with box {32, 32} (EPI_RESID_F32, TMA reduce-add), 128-byte swizzle
+void launch_gemm(int epi, const CUtensorMap& tmA, const CUtensorMap& tmB, const CUtensorMap& tmC,
+                 const GemmParams& p, int num_sms, cudaStream_t stream);
 
 // ------------------------------------------------------------------ bipartite attention
 struct AttnParams {
