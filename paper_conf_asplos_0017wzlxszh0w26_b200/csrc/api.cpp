@@ -87,7 +87,9 @@ static CUtensorMap make_tmap(const void* ptr, int64_t rows, int64_t cols, int64_
 struct DevBuf {
   void* p = nullptr;
   size_t cap = 0;
-  void ensure(size_t bytes) {
+  // zero: clear on (re)allocation — q-tiles and suffix pages rely on never-written padding
+  // (head-dim padding columns, rows 126-127 of a q-tile) staying zero
+  void ensure(size_t bytes, bool zero = false) {
     if (bytes <= cap) return;
     if (p) cudaFree(p);
     p = nullptr;
@@ -95,6 +97,7 @@ struct DevBuf {
     size_t want = std::max(bytes, size_t(1) << 16);
     want = (want + (want >> 2) + 255) & ~size_t(255);
     CUDA_OK(cudaMalloc(&p, want));
+    if (zero) CUDA_OK(cudaMemset(p, 0, want));
     cap = want;
   }
   ~DevBuf() {
@@ -258,8 +261,8 @@ static const int32_t* prepare(Pool& pool, Model& m, Plan& plan, cudaStream_t st,
   ws.h.ensure(size_t(M) * H * 4);
   ws.xn.ensure(size_t(M) * std::max(H, nq) * 2);
   ws.qkv.ensure(size_t(M) * m.nqkv() * 2);
-  ws.qp.ensure(size_t(plan.n_qtiles_total) * c.kv_heads * tile_bytes);
-  ws.scratch.ensure(size_t(std::max(plan.n_spages, 1)) * pool.geo.layer_bytes);
+  ws.qp.ensure(size_t(plan.n_qtiles_total) * c.kv_heads * tile_bytes, true);
+  ws.scratch.ensure(size_t(std::max(plan.n_spages, 1)) * pool.geo.layer_bytes, true);
   ws.o.ensure(size_t(M) * nq * 2);
   ws.act.ensure(size_t(M) * F * 2);
   ws.hc.ensure(size_t(B) * H * 4);

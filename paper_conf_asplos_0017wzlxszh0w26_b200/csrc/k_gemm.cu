@@ -168,7 +168,7 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
       ptx::tc_fence_after();
       const uint32_t tbase = tmem + ((sub * 32) << 16) + acc * BN;
       const int row0 = m * BM + sub * 32;
-      if (EPI == EPI_SWIGLU) {
+      if constexpr (EPI == EPI_SWIGLU) {
 #pragma unroll 1
         for (int c = 0; c < BN / 2; c += 64) {  // 64 output columns per staging buffer
           uint8_t* buf = next_buf();
@@ -190,7 +190,7 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
           }
           flush(buf, n * (BN / 2) + c, row0);
         }
-      } else if (EPI == EPI_RESID_F32) {
+      } else if constexpr (EPI == EPI_RESID_F32) {
 #pragma unroll 1
         for (int c = 0; c < BN; c += 32) {  // 32 fp32 columns per staging buffer
           uint8_t* buf = next_buf();
@@ -250,23 +250,22 @@ void launch_gemm(int epi, const CUtensorMap& tmA, const CUtensorMap& tmB, const 
   const int tiles = ((p.M + BM - 1) / BM) * ((p.N + out_bn - 1) / out_bn);
   const int grid = tiles < num_sms ? tiles : num_sms;
   if (grid <= 0) return;
+  auto launch = [&](auto kern) {
+    static const void* attr_done[16] = {nullptr};  // kernels whose smem attribute is set
+    bool found = false;
+    for (const void* f : attr_done) found |= (f == reinterpret_cast<const void*>(kern));
+    if (!found) {
+      cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, static_cast<int>(kGemmSmem));
+      for (auto& f : attr_done)
+        if (!f) { f = reinterpret_cast<const void*>(kern); break; }
+    }
+    kern<<<grid, NUM_THREADS, kGemmSmem, stream>>>(tmA, tmB, tmC, p);
+  };
   switch (epi) {
-#define BAT_GEMM_CASE(E)                                                                        \
-  case E: {                                                                                     \
-    static bool attr = false;                                                                   \
-    if (!attr) {                                                                                \
-      cudaFuncSetAttribute(gemm_tc_kernel<E>, cudaFuncAttributeMaxDynamicSharedMemorySize,     \
-                           static_cast<int>(kGemmSmem));                                        \
-      attr = true;                                                                              \
-    }                                                                                           \
-    gemm_tc_kernel<E><<<grid, NUM_THREADS, kGemmSmem, stream>>>(tmA, tmB, tmC, p);             \
-    break;                                                                                      \
-  }
-    BAT_GEMM_CASE(EPI_BF16)
-    BAT_GEMM_CASE(EPI_BF16_BIAS)
-    BAT_GEMM_CASE(EPI_RESID_F32)
-    BAT_GEMM_CASE(EPI_SWIGLU)
-#undef BAT_GEMM_CASE
+    case EPI_BF16: launch(gemm_tc_kernel<EPI_BF16>); break;
+    case EPI_BF16_BIAS: launch(gemm_tc_kernel<EPI_BF16_BIAS>); break;
+    case EPI_RESID_F32: launch(gemm_tc_kernel<EPI_RESID_F32>); break;
+    case EPI_SWIGLU: launch(gemm_tc_kernel<EPI_SWIGLU>); break;
   }
   count_launch();
 }
