@@ -272,15 +272,17 @@ def main():
     stream = torch.cuda.current_stream(dev)
 
     # ---- item corpus: Zipf hotness, HRCS placement (Alg. 1) for N > 1
+    from paper_conf_asplos_0017wzlxszh0w26_b200 import dist as bdist
     zipf_p = synth.zipf_weights(args.corpus)
-    t_req_est = 0.0015  # s per request; refined below from the measured step time
+    t_req_est = 0.0015  # s per request (prefill time t of Alg. 1 line 4, measured order on B200)
     owner = np.full(args.corpus, -1, np.int32)
     r_rep = 1.0
+    r_max = None
     if world > 1:
-        B_tok = 770e9 / (2 * cfg["kv_heads"] * cfg["head_dim"] * cfg["layers"] * 2)  # NVLink peer GB/s -> tokens/s
-        r_max = bat.bat_hrcs_rmax(B_tok, t_req_est, args.alpha, args.n_items, args.item_len, world)
-        r_rep, owner = bat.bat_hrcs_place(zipf_p, r_max, world)
-    local_items = [i for i in range(args.corpus) if owner[i] < 0 or owner[i] == rank]
+        kv_tok = 2 * cfg["kv_heads"] * cfg["head_dim"] * cfg["layers"] * 2
+        r_max = bdist.rmax_for_nvlink(770.0, t_req_est, args.alpha, args.n_items, args.item_len, world, kv_tok)
+        r_rep, owner = bdist.place_items(zipf_p, r_max, world)
+    local_items = bdist.local_items(owner, rank)
     item_toks = {i: synth.item_tokens(args.seed, i, args.item_len, cfg["vocab"]) for i in local_items}
     t0 = time.perf_counter()
     for s in range(0, len(local_items), 1024):
@@ -290,25 +292,7 @@ def main():
     torch.cuda.synchronize()
     t_corpus = time.perf_counter() - t0
     if world > 1:
-        # exchange IPC handles and the owners' page tables of the cold items
-        h = bat.bat_pool_ipc_handle(pool.handle)
-        handles = [None] * world
-        dist.all_gather_object(handles, h)
-        for r in range(world):
-            if r != rank:
-                bat.bat_pool_attach_peer(pool.handle, r, handles[r])
-        mine = {}
-        for i in local_items:
-            if owner[i] == rank:
-                n_tok, pg = bat.bat_kv_lookup(pool.handle, bat.BAT_ENT_ITEM, i)
-                mine[i] = (n_tok, [int(x) for x in pg])
-        allmaps = [None] * world
-        dist.all_gather_object(allmaps, mine)
-        for r in range(world):
-            if r == rank:
-                continue
-            for i, (n_tok, pg) in allmaps[r].items():
-                bat.bat_kv_register_remote(pool.handle, bat.BAT_ENT_ITEM, i, r, pg, n_tok)
+        bdist.exchange_remote(pool.handle, owner, rank, world)
         dist.barrier()
 
     # ---- batches
@@ -317,20 +301,14 @@ def main():
     batches = [make_queries(args, cfg, rng, 10_000_000 * (rank + 1) + 100_000 * k, args.batch, zipf_p)
                for k in range(n_batches)]
     qarrays = [bat.QueryArray(b) for b in batches]
-    cold_ids = []
-    for b in batches:
-        ids = sorted({int(i) for q in b for i in q.item_ids if owner[int(i)] >= 0 and owner[int(i)] != rank})
-        cold_ids.append(np.asarray(ids, np.int64))
+    cold_ids = [bdist.cold_items(b, owner, rank) for b in batches]
 
     def fetch(k):
-        if world > 1 and len(cold_ids[k]):
-            return bat.bat_kv_fetch(pool.handle, bat.BAT_ENT_ITEM, cold_ids[k], stream=stream)
-        return 0
+        return bdist.fetch_cold(pool.handle, cold_ids[k], stream) if world > 1 else 0
 
     def drop(k):
         if world > 1:
-            for i in cold_ids[k]:
-                bat.bat_kv_evict(pool.handle, bat.BAT_ENT_ITEM, int(i))
+            bdist.drop_fetched(pool.handle, cold_ids[k])
 
     B = args.batch
     n_max = args.n_items
@@ -477,7 +455,9 @@ def main():
             config=dict(workload=WORKLOAD, batch_per_gpu=B, global_batch=B * world, seq_len=args.n_user + args.n_items * args.item_len + args.n_instr,
                         suffix_tokens_per_request=args.n_user + args.n_instr, prefix_tokens_per_request=args.n_items * args.item_len,
                         corpus_items=args.corpus, item_hotness="Zipf s=1.093", parallelism=f"dp{world}",
-                        hrcs=dict(replication_ratio=r_rep, alpha=args.alpha) if world > 1 else None,
+                        hrcs=dict(replication_ratio=r_rep, r_max=r_max, alpha=args.alpha, t_request_s=0.0015,
+                                  link_gbs=770.0, cold_items_per_step=float(np.mean([len(c) for c in cold_ids])))
+                        if world > 1 else None,
                         l2="inputs larger than L2 (2.6 GB of weights streamed every step)"),
             prefill_tokens_per_s=sfx_tokens * world / (ms / 1e3),
             served_tokens_per_s=total_req * (args.n_user + args.n_instr + args.n_items * args.item_len) / (ms / 1e3),

@@ -261,9 +261,15 @@ BAT_API bat_status bat_pool_attach_peer(bat_pool p, int32_t peer_rank, const voi
 BAT_API bat_status bat_kv_register_remote(bat_pool p, int32_t kind, int64_t id, int32_t owner,
                                   const int32_t* owner_pages, int32_t n_pages,
                                   int32_t n_tokens);
+/* Host query of a registered remote entry: owner rank, token count, owner page ids. */
+BAT_API bat_status bat_kv_lookup_remote(bat_pool p, int32_t kind, int64_t id, int32_t* owner,
+                                        int32_t* n_tokens, int32_t* pages_out, int32_t pages_cap,
+                                        int32_t* n_pages);
 /* Pull the listed remote entries (deduplicated, skipping ones already local) from their
- * owners' arenas over NVLink into local pages (one copy kernel on `stream`), making them
- * resolvable by bat_bipartite_prefill.  *n_fetched = entries pulled. */
+ * owners' arenas over NVLink into local pages (one copy kernel on `stream`, asynchronous:
+ * work on `stream` after this call sees the pages), making them resolvable by
+ * bat_bipartite_prefill.  *n_fetched = entries pulled.  The owners must not evict them while
+ * the copy runs. */
 BAT_API bat_status bat_kv_fetch(bat_pool p, int32_t kind, const int64_t* ids, int32_t n,
                         int32_t* n_fetched, bat_stream_t stream);
 

@@ -100,6 +100,8 @@ def lib() -> ctypes.CDLL:
         "bat_pool_ipc_handle": (S, [c_void_p, c_void_p]),
         "bat_pool_attach_peer": (S, [c_void_p, c_int32, c_void_p]),
         "bat_kv_register_remote": (S, [c_void_p, c_int32, c_int64, c_int32, POINTER(c_int32), c_int32, c_int32]),
+        "bat_kv_lookup_remote": (S, [c_void_p, c_int32, c_int64, POINTER(c_int32), POINTER(c_int32),
+                                     POINTER(c_int32), c_int32, POINTER(c_int32)]),
         "bat_kv_fetch": (S, [c_void_p, c_int32, POINTER(c_int64), c_int32, POINTER(c_int32), c_void_p]),
         "bat_plan_build": (S, [c_void_p, c_void_p, POINTER(bat_query), c_int32, c_void_p, POINTER(c_void_p)]),
         "bat_prefill_plan": (S, [c_void_p, c_void_p, c_void_p, c_void_p, c_void_p]),
@@ -127,7 +129,7 @@ EXPORTED = ("bat_last_error", "bat_version", "bat_kernel_launch_count", "bat_mod
             "bat_kv_read", "bat_kv_prefill_entities", "bat_bipartite_prefill", "bat_score",
             "bat_plan_create", "bat_plan_destroy", "bat_plan_query_info", "bat_plan_export",
             "bat_hrcs_rmax", "bat_hrcs_place", "bat_pool_ipc_handle", "bat_pool_attach_peer",
-            "bat_kv_register_remote", "bat_kv_fetch", "bat_debug_gemm", "bat_debug_attention_layer",
+            "bat_kv_register_remote", "bat_kv_lookup_remote", "bat_kv_fetch", "bat_debug_gemm", "bat_debug_attention_layer",
             "bat_plan_build", "bat_prefill_plan", "bat_profile_enable", "bat_profile_read",
             "bat_profile_reset", "bat_debug_attach_peer_pool")
 
@@ -390,6 +392,15 @@ def bat_kv_register_remote(pool: int, kind: int, id_: int, owner: int, pages: Se
                            n_tokens: int) -> None:
     pg = np.ascontiguousarray(pages, dtype=np.int32)
     _check(lib().bat_kv_register_remote(pool, kind, id_, owner, _i32p(pg), len(pg), n_tokens))
+
+
+def bat_kv_lookup_remote(pool: int, kind: int, id_: int):
+    owner, n_tok, n_pg = c_int32(), c_int32(), c_int32()
+    _check(lib().bat_kv_lookup_remote(pool, kind, id_, byref(owner), byref(n_tok), None, 0, byref(n_pg)))
+    pages = np.zeros(max(n_pg.value, 1), dtype=np.int32)
+    _check(lib().bat_kv_lookup_remote(pool, kind, id_, byref(owner), byref(n_tok), _i32p(pages), len(pages),
+                                      byref(n_pg)))
+    return owner.value, n_tok.value, pages[: n_pg.value]
 
 
 def bat_kv_fetch(pool: int, kind: int, ids: Sequence[int], stream=None) -> int:

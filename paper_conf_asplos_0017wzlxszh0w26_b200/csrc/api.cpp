@@ -589,6 +589,8 @@ bat_status bat_kv_pool_destroy(bat_pool p) {
       cudaDeviceSynchronize();
       for (size_t r = 0; r < p->pool.peer_arena.size(); ++r)
         if (p->pool.peer_arena[r] && p->pool.peer_ipc[r]) cudaIpcCloseMemHandle(p->pool.peer_arena[r]);
+      if (p->pool.fetch_host) cudaFreeHost(p->pool.fetch_host);
+      if (p->pool.fetch_done) cudaEventDestroy(static_cast<cudaEvent_t>(p->pool.fetch_done));
       cudaFree(p->pool.arena);
     }
     delete p;
@@ -953,6 +955,23 @@ bat_status bat_kv_register_remote(bat_pool p, int32_t kind, int64_t id, int32_t 
   });
 }
 
+bat_status bat_kv_lookup_remote(bat_pool p, int32_t kind, int64_t id, int32_t* owner, int32_t* n_tokens,
+                                int32_t* pages_out, int32_t pages_cap, int32_t* n_pages) {
+  return guarded([&] {
+    BAT_REQUIRE(p, "null pool");
+    auto it = p->pool.remote.find(EntityKey{kind, id});
+    if (it == p->pool.remote.end()) fail(BAT_E_NOTFOUND, "remote entry not registered");
+    const RemoteEntity& r = it->second;
+    if (owner) *owner = r.owner;
+    if (n_tokens) *n_tokens = r.n_tokens;
+    if (n_pages) *n_pages = int32_t(r.pages.size());
+    if (pages_out) {
+      BAT_REQUIRE(pages_cap >= int32_t(r.pages.size()), "pages_cap too small");
+      std::copy(r.pages.begin(), r.pages.end(), pages_out);
+    }
+  });
+}
+
 bat_status bat_kv_fetch(bat_pool p, int32_t kind, const int64_t* ids, int32_t n, int32_t* n_fetched,
                         bat_stream_t stream) {
   return guarded([&] {
@@ -990,17 +1009,31 @@ bat_status bat_kv_fetch(bat_pool p, int32_t kind, const int64_t* ids, int32_t n,
       }
       if (!src.empty()) {
         cudaStream_t st = static_cast<cudaStream_t>(stream);
-        void* buf = nullptr;
         const size_t bytes = src.size() * 8 + dst.size() * 4;
+        // asynchronous: descriptors go through a pool-owned pinned buffer (reused once the
+        // previous upload has read it), the device copy is freed in stream order
+        if (!P.fetch_done) {
+          cudaEvent_t e;
+          CUDA_OK(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
+          P.fetch_done = e;
+        }
+        CUDA_OK(cudaEventSynchronize(static_cast<cudaEvent_t>(P.fetch_done)));
+        if (P.fetch_host_cap < bytes) {
+          if (P.fetch_host) cudaFreeHost(P.fetch_host);
+          P.fetch_host_cap = bytes * 2;
+          CUDA_OK(cudaMallocHost(&P.fetch_host, P.fetch_host_cap));
+        }
+        std::memcpy(P.fetch_host, src.data(), src.size() * 8);
+        std::memcpy(static_cast<char*>(P.fetch_host) + src.size() * 8, dst.data(), dst.size() * 4);
+        void* buf = nullptr;
         CUDA_OK(cudaMallocAsync(&buf, bytes, st));
-        CUDA_OK(cudaMemcpyAsync(buf, src.data(), src.size() * 8, cudaMemcpyHostToDevice, st));
-        CUDA_OK(cudaMemcpyAsync(static_cast<char*>(buf) + src.size() * 8, dst.data(), dst.size() * 4,
-                                cudaMemcpyHostToDevice, st));
+        CUDA_OK(cudaMemcpyAsync(buf, P.fetch_host, bytes, cudaMemcpyHostToDevice, st));
+        CUDA_OK(cudaEventRecord(static_cast<cudaEvent_t>(P.fetch_done), st));
         launch_page_copy(static_cast<const uint64_t*>(buf),
                          reinterpret_cast<const int32_t*>(static_cast<char*>(buf) + src.size() * 8), P.arena,
                          P.geo.page_bytes, int(src.size()), st);
         CUDA_OK(cudaFreeAsync(buf, st));
-        CUDA_OK(cudaStreamSynchronize(st));  // host vectors above are temporaries
+        CUDA_OK(cudaGetLastError());
       }
     } catch (...) {
       for (auto& k : made) {

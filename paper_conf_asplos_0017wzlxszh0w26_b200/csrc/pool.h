@@ -70,6 +70,10 @@ struct Pool {
   std::vector<char*> peer_arena;  // by rank (IPC-mapped), nullptr for self / unattached
   std::vector<uint8_t> peer_ipc;  // 1 if peer_arena[r] came from cudaIpcOpenMemHandle
   uint64_t ipc_handle[8] = {0};
+  // pinned staging of the fetch descriptors (bat_kv_fetch stays asynchronous on its stream)
+  void* fetch_host = nullptr;
+  size_t fetch_host_cap = 0;
+  void* fetch_done = nullptr;  // cudaEvent_t: last descriptor upload finished reading fetch_host
 
   const Entity* find(int32_t kind, int64_t id) const {
     auto it = index.find(EntityKey{kind, id});
