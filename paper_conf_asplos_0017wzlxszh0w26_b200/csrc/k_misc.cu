@@ -92,36 +92,41 @@ __global__ void rope_table_kernel(float2* tab, int max_pos, int d, double theta)
   }
 }
 
-// rotate 8 consecutive columns [c0, c0+8) of one head vector x (d columns, bf16, rotate-half)
-__device__ __forceinline__ void rope8(const __nv_bfloat16* __restrict__ x, int c0, int d,
-                                      const float2* __restrict__ cs, bool enabled, float (&o)[8]) {
-  const int half = d / 2;
-  uint4 raw = *reinterpret_cast<const uint4*>(x + c0);
-  const __nv_bfloat16* xs = reinterpret_cast<const __nv_bfloat16*>(&raw);
+// rotate-half RoPE of the column pair (c, c + d/2) for 8 consecutive c = c0..c0+7 of one head
+// vector x (bf16): o1 = x1 cos - x2 sin, o2 = x2 cos + x1 sin; cs = the position's (cos, sin)
+// row.  Both 16-byte halves and the 64 bytes of cos/sin are read once.
+__device__ __forceinline__ void rope_pair8(const __nv_bfloat16* __restrict__ x, int c0, int d,
+                                           const float2* __restrict__ cs, bool enabled, uint4& o1, uint4& o2) {
+  const uint4 r1 = *reinterpret_cast<const uint4*>(x + c0);
+  const uint4 r2 = *reinterpret_cast<const uint4*>(x + c0 + d / 2);
   if (!enabled) {
-#pragma unroll
-    for (int i = 0; i < 8; ++i) o[i] = __bfloat162float(xs[i]);
+    o1 = r1;
+    o2 = r2;
     return;
   }
-  const int pc = c0 < half ? c0 + half : c0 - half;
-  uint4 praw = *reinterpret_cast<const uint4*>(x + pc);
-  const __nv_bfloat16* ps = reinterpret_cast<const __nv_bfloat16*>(&praw);
+  const __nv_bfloat162* a = reinterpret_cast<const __nv_bfloat162*>(&r1);
+  const __nv_bfloat162* b = reinterpret_cast<const __nv_bfloat162*>(&r2);
+  const float4* t4 = reinterpret_cast<const float4*>(cs + c0);
+  uint32_t w1[4], w2[4];
 #pragma unroll
-  for (int i = 0; i < 8; ++i) {
-    const int c = c0 + i;
-    const float2 t = cs[c < half ? c : c - half];
-    const float a = __bfloat162float(xs[i]), b = __bfloat162float(ps[i]);
-    o[i] = c < half ? a * t.x - b * t.y : a * t.x + b * t.y;
+  for (int i = 0; i < 4; ++i) {
+    const float4 t = t4[i];  // (cos, sin) of columns c0+2i, c0+2i+1
+    const float2 fa = __bfloat1622float2(a[i]), fb = __bfloat1622float2(b[i]);
+    w1[i] = ptx::pack_bf16x2(fa.x * t.x - fb.x * t.y, fa.y * t.z - fb.y * t.w);
+    w2[i] = ptx::pack_bf16x2(fb.x * t.x + fa.x * t.y, fb.y * t.z + fa.y * t.w);
   }
+  o1 = make_uint4(w1[0], w1[1], w1[2], w1[3]);
+  o2 = make_uint4(w2[0], w2[1], w2[2], w2[3]);
 }
 
 // a4: RoPE(q, k) at the plan's positions; write the q-tiles (GQA-packed rows = token x
-// head-in-group, 128-byte swizzled [Dp/64][128][64]) and the suffix K/V pages.
+// head-in-group, 128-byte swizzled [Dp/64][128][64]) and the suffix K/V pages.  Only real rows
+// and columns are written: the buffers are zeroed at allocation and padding is never written.
 __global__ void stage_kernel(const StageParams p) {
-  const int d = p.head_dim, dp = p.dpad;
+  const int d = p.head_dim;
   const int nqkv = (p.q_heads + 2 * p.kv_heads) * d;
   const int32_t* img = p.img;
-  const int chunks_per_row = dp / 8;
+  const int pairs = d / 16;  // 8-column chunk pairs (c, c + d/2) per head
   int blk = blockIdx.x;
   const int n_q_blocks = p.n_qtiles * p.kv_heads;
   if (blk < n_q_blocks) {
@@ -129,21 +134,18 @@ __global__ void stage_kernel(const StageParams p) {
     const int4 qt = *reinterpret_cast<const int4*>(img + p.off_qtiles + int64_t(gq) * 4);
     const int b = qt.x, t0 = qt.y, ntok = qt.z;
     const int tok_off = img[p.off_qinfo + int64_t(b) * 8];
-    char* tile = reinterpret_cast<char*>(p.qp) + (int64_t(gq) * p.kv_heads + kvh) * (dp / 64) * 16384;
-    for (int e = threadIdx.x; e < 128 * chunks_per_row; e += blockDim.x) {
-      const int r = e / chunks_per_row, cc = e % chunks_per_row;
-      const int c0 = cc * 8;
-      float o[8] = {0, 0, 0, 0, 0, 0, 0, 0};
-      const int tl = r / p.group;
-      if (r < p.qt * p.group && tl < ntok && c0 < d) {
-        const int m = tok_off + t0 + tl;
-        const int head = kvh * p.group + r % p.group;
-        const int pos = min(img[p.off_pos + m], p.max_pos - 1);
-        rope8(p.qkv + int64_t(m) * nqkv + head * d, c0, d, p.rope + int64_t(pos) * (d / 2), p.rope_enabled, o);
-      }
-      uint4 pk = make_uint4(ptx::pack_bf16x2(o[0], o[1]), ptx::pack_bf16x2(o[2], o[3]),
-                            ptx::pack_bf16x2(o[4], o[5]), ptx::pack_bf16x2(o[6], o[7]));
-      *reinterpret_cast<uint4*>(tile + (c0 / 64) * 16384 + ptx::swz128(r, (c0 % 64) / 8)) = pk;
+    char* tile = reinterpret_cast<char*>(p.qp) + (int64_t(gq) * p.kv_heads + kvh) * (p.dpad / 64) * 16384;
+    const int rows = ntok * p.group;
+    for (int e = threadIdx.x; e < rows * pairs; e += blockDim.x) {
+      const int r = e / pairs, pc = e % pairs;
+      const int c0 = pc * 8, c1 = c0 + d / 2;
+      const int m = tok_off + t0 + r / p.group;
+      const int head = kvh * p.group + r % p.group;
+      const int pos = min(img[p.off_pos + m], p.max_pos - 1);
+      uint4 o1, o2;
+      rope_pair8(p.qkv + int64_t(m) * nqkv + head * d, c0, d, p.rope + int64_t(pos) * (d / 2), p.rope_enabled, o1, o2);
+      *reinterpret_cast<uint4*>(tile + (c0 / 64) * 16384 + ptx::swz128(r, (c0 % 64) / 8)) = o1;
+      *reinterpret_cast<uint4*>(tile + (c1 / 64) * 16384 + ptx::swz128(r, (c1 % 64) / 8)) = o2;
     }
     return;
   }
@@ -154,22 +156,19 @@ __global__ void stage_kernel(const StageParams p) {
   const int tok_off = img[p.off_qinfo + int64_t(b) * 8];
   char* page = target >= 0 ? p.pool + int64_t(target) * p.pool_page_bytes + p.pool_layer_off
                            : p.scratch + int64_t(-target - 1) * p.scratch_page_bytes + p.scratch_layer_off;
-  for (int e = threadIdx.x; e < 2 * kPageTokens * chunks_per_row; e += blockDim.x) {
-    const int kv = e / (kPageTokens * chunks_per_row);
-    const int rem = e % (kPageTokens * chunks_per_row);
-    const int j = rem / chunks_per_row, cc = rem % chunks_per_row;
-    const int c0 = cc * 8;
-    float o[8] = {0, 0, 0, 0, 0, 0, 0, 0};
-    if (j < ntok && c0 < d) {
-      const int m = tok_off + t0 + j;
-      const __nv_bfloat16* src = p.qkv + int64_t(m) * nqkv + (p.q_heads + kv * p.kv_heads + kvh) * d;
-      const int pos = min(img[p.off_pos + m], p.max_pos - 1);
-      rope8(src, c0, d, p.rope + int64_t(pos) * (d / 2), kv == 0 && p.rope_enabled, o);
-    }
-    uint4 pk = make_uint4(ptx::pack_bf16x2(o[0], o[1]), ptx::pack_bf16x2(o[2], o[3]),
-                          ptx::pack_bf16x2(o[4], o[5]), ptx::pack_bf16x2(o[6], o[7]));
-    char* blockp = page + (int64_t(kv) * p.kv_heads + kvh) * p.head_bytes + (c0 / 64) * 2048;
-    *reinterpret_cast<uint4*>(blockp + ptx::swz128(j, (c0 % 64) / 8)) = pk;
+  for (int e = threadIdx.x; e < 2 * ntok * pairs; e += blockDim.x) {
+    const int kv = e / (ntok * pairs);
+    const int rem = e % (ntok * pairs);
+    const int j = rem / pairs, pc = rem % pairs;
+    const int c0 = pc * 8, c1 = c0 + d / 2;
+    const int m = tok_off + t0 + j;
+    const __nv_bfloat16* src = p.qkv + int64_t(m) * nqkv + (p.q_heads + kv * p.kv_heads + kvh) * d;
+    const int pos = min(img[p.off_pos + m], p.max_pos - 1);
+    uint4 o1, o2;
+    rope_pair8(src, c0, d, p.rope + int64_t(pos) * (d / 2), kv == 0 && p.rope_enabled, o1, o2);
+    char* blockp = page + (int64_t(kv) * p.kv_heads + kvh) * p.head_bytes;
+    *reinterpret_cast<uint4*>(blockp + (c0 / 64) * 2048 + ptx::swz128(j, (c0 % 64) / 8)) = o1;
+    *reinterpret_cast<uint4*>(blockp + (c1 / 64) * 2048 + ptx::swz128(j, (c1 % 64) / 8)) = o2;
   }
 }
 

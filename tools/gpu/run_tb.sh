@@ -3,7 +3,7 @@
 cd $GRAFT_REPO_ROOT
 mkdir -p gpurun_out
 export PYTHONUNBUFFERED=1
-timeout 400 python -m pytest tests -m gpu -q -x -p no:cacheprovider --timeout 150 --timeout-method=thread > gpurun_out/tb_tests.log 2>&1
+timeout 400 python -m pytest tests -m "gpu and not slow" -q -x -p no:cacheprovider --timeout 150 --timeout-method=thread > gpurun_out/tb_tests.log 2>&1
 echo "tests exit $?"; tail -3 gpurun_out/tb_tests.log
 timeout 600 python bench.py --steps 5 --warmup 3 --no-cpu-baseline ${BENCH_ARGS} > gpurun_out/tb_bench.json 2> gpurun_out/tb_bench.err
 echo "bench exit $?"
