@@ -8,19 +8,22 @@
 // with a state per q-tile: 0 dead (P = 0), 1 full (no element mask), 2 partial (apply
 //   kord <= rord && (kseg == rseg || (kseg|rseg) < 0)  per element).
 //
-// Warp roles (384 threads, one CTA per SM, persistent over work items, FA4-style):
-//   warp 0      loader: lanes 0-7 each bulk-copy one page's K (then V) blocks of a k-tile —
-//               pages are stored in the tensor-core operand layout (128-byte swizzle), so
-//               2 KB blocks drop into shared memory ready for tcgen05.mma; page ids of the
-//               next tile are prefetched into registers while waiting for a free stage.
+// Warp roles (640 threads, one CTA per SM, persistent over work items, FA4-style):
+//   warps 0,2,3 loaders: each moves a third of the pages of every k-tile (2 KB bulk copies of
+//               the page's K, then V chunks) — pages are stored in the tensor-core operand layout
+//               (128-byte swizzle), so they drop into shared memory ready for tcgen05.mma; page
+//               ids are read three tiles ahead and the tile two ahead is prefetched into L2.
 //   warp 1      MMA issuer (one thread): S0 = Q0 K^T, S1 = Q1 K^T (SS, M=128 N=128 K=16) and
 //               O0 += P0 V, O1 += P1 V (TS: P read from TMEM, V MN-major from smem), issued as
-//               S0_0 S1_0 | PV0_j S0_{j+1} PV1_j S1_{j+1} | ... so one softmax warpgroup works
-//               while the tensor core serves the other.
-//   warps 4-7   softmax warpgroup 0 (q-tile 0), warps 8-11 warpgroup 1 (q-tile 1), one row per
-//               thread: max pass over the S row (tcgen05.ld), exp2 pass writing P as bf16 into
-//               the S buffer's TMEM columns (tcgen05.st), lazy rescaling of O (only when the
-//               running max grows by > 2^8), final O / l -> bf16 stores.
+//               S0_0 S1_0 | PV0_j S0_{j+1} PV1_j S1_{j+1} | ... so the softmax of one q-tile
+//               runs while the tensor core serves the other.
+//   warps 4-19  four softmax warpgroups: q-tile q = wg & 1, key half h = wg >> 1.  Thread
+//               (q, h, row) owns the 64 S columns [64h, 64h+64) of one row: exp2 of its half
+//               against the row's reference max, P as bf16 into TMEM columns [64h, 64h+32) of
+//               the S buffer, and the O columns [DP/2 h, DP/2 (h+1)) for rescaling and the
+//               epilogue.  The two halves of a row agree on the reference max through shared
+//               memory and a 64-thread named barrier per warp pair; the reference max only
+//               moves when a row's exponent would exceed 2^8 (lazy rescaling).
 // TMEM (512 columns): S0 [0,128) S1 [128,256) O0 [256,384) O1 [384,512).
 #include <cuda_bf16.h>
 #include <cuda_runtime.h>
@@ -32,7 +35,9 @@
 namespace bat {
 namespace {
 
-constexpr int NUM_THREADS = 384;
+constexpr int NUM_THREADS = 640;
+constexpr int kLoaders = 3;  // loader warps 0, 2, 3: one warp issues cp.async.bulk at ~30 B/clk only
+constexpr int NCH = 2;  // 32-column S chunks per softmax thread (half of a 128-key row)
 constexpr float kRescaleThreshold = 8.0f;  // log2 units: P <= 2^8 between rescales
 #ifndef BAT_POLY_PAIRS
 #define BAT_POLY_PAIRS 4  // of every 16 column pairs, exp2 on the FMA pipe (rest: MUFU)
@@ -46,9 +51,18 @@ struct AttnSmem {
   static constexpr int K_OFF = Q_OFF + 2 * TILE_BYTES;   // 2 stages
   static constexpr int V_OFF = K_OFF + 2 * TILE_BYTES;   // 2 stages
   static constexpr int META_OFF = V_OFF + 2 * TILE_BYTES;  // 2 x 128 x int2 (with V)
-  static constexpr int BAR_OFF = META_OFF + 2 * 1024;
+  static constexpr int XCH_OFF = META_OFF + 2 * 1024;  // row-half exchange (see XchSmem)
+  static constexpr int BAR_OFF = XCH_OFF + 8192;
   static constexpr int TOTAL = BAR_OFF + 256;
 };
+
+// exchange between the two key halves of a row ([parity][q][h]...)
+struct XchSmem {
+  float rmax[2][2][2][128];  // partial raw row maxima (slow path)
+  int ok[2][2][2][4];        // per-warp "all exponents <= threshold" votes (fast path)
+  float lsum[2][2][128];     // partial row sums (epilogue)
+};
+static_assert(sizeof(XchSmem) <= 8192, "exchange area");
 
 struct __align__(8) AttnBars {
   uint64_t q_full, q_empty;
@@ -123,21 +137,21 @@ __device__ __forceinline__ uint64_t exp2_poly2(uint64_t x) {
   } while (0)
 
 struct WorkItem {
-  int b, kvh, q0, q1, kt_off, kt_n;
+  int b, kvh, q0, q1, kt_off, kt_n, tp_off;
 };
 __device__ __forceinline__ WorkItem load_work(const int32_t* work, int w) {
   const int4 a = *reinterpret_cast<const int4*>(work + int64_t(w) * 8);
   const int4 c = *reinterpret_cast<const int4*>(work + int64_t(w) * 8 + 4);
-  return WorkItem{a.x, a.y, a.z, a.w, c.x, c.y};
+  return WorkItem{a.x, a.y, a.z, a.w, c.x, c.y, c.z};
 }
 
 // ---- softmax passes over one 128-column S row held in TMEM (one row per thread) ----------
 // Row max of the raw scores; MASKED applies the visibility bits.
-template <bool MASKED>
-__device__ __forceinline__ float row_max(uint32_t tS, const uint32_t (&vis)[4]) {
+template <bool MASKED, int NC>
+__device__ __forceinline__ float row_max(uint32_t tS, const uint32_t (&vis)[NC]) {
   float mt = -INFINITY;
 #pragma unroll
-  for (int c = 0; c < 4; c += 2) {
+  for (int c = 0; c < NC; c += 2) {
     uint32_t r[32], q[32];
     ptx::tmem_ld32(tS + c * 32, r);
     ptx::tmem_ld32(tS + (c + 1) * 32, q);
@@ -164,17 +178,17 @@ __device__ __forceinline__ float row_max(uint32_t tS, const uint32_t (&vis)[4]) 
 
 // P = exp2(s * scale - mref) written as bf16 pairs into the row's first 64 TMEM columns
 // (columns [16c, 16c+16) after S columns [32c, 32c+32) were read); returns the row sum.
-template <bool MASKED>
-__device__ __forceinline__ float row_exp(uint32_t tS, const uint32_t (&vis)[4], uint64_t sc2, uint64_t nm2) {
+template <bool MASKED, int NC>
+__device__ __forceinline__ float row_exp(uint32_t tS, const uint32_t (&vis)[NC], uint64_t sc2, uint64_t nm2) {
   uint64_t acc0 = pk2(0.0f, 0.0f), acc1 = acc0;
   uint32_t ra[32], rb[32];
   ptx::tmem_ld32(tS, ra);
   ptx::tmem_ld_wait();
 #pragma unroll
-  for (int c = 0; c < 4; ++c) {
+  for (int c = 0; c < NC; ++c) {
     uint32_t (&r)[32] = (c & 1) ? rb : ra;
     uint32_t (&rn)[32] = (c & 1) ? ra : rb;
-    if (c < 3) ptx::tmem_ld32(tS + (c + 1) * 32, rn);  // in flight while chunk c computes
+    if (c + 1 < NC) ptx::tmem_ld32(tS + (c + 1) * 32, rn);  // in flight while chunk c computes
     uint32_t pk[16];
 #pragma unroll
     for (int i = 0; i < 16; ++i) {
@@ -205,7 +219,7 @@ __device__ __forceinline__ float row_exp(uint32_t tS, const uint32_t (&vis)[4], 
         "r"(pk[0]), "r"(pk[1]), "r"(pk[2]), "r"(pk[3]), "r"(pk[4]), "r"(pk[5]), "r"(pk[6]), "r"(pk[7]),
         "r"(pk[8]), "r"(pk[9]), "r"(pk[10]), "r"(pk[11]), "r"(pk[12]), "r"(pk[13]), "r"(pk[14]),
         "r"(pk[15]));
-    if (c < 3) ptx::tmem_ld_wait();
+    if (c + 1 < NC) ptx::tmem_ld_wait();
   }
   float a0, a1, b0, b1;
   up2(acc0, a0, a1);
@@ -217,14 +231,14 @@ __device__ __forceinline__ float row_exp(uint32_t tS, const uint32_t (&vis)[4], 
 // tracks the row's largest exponent; P is written to TMEM only if no visible exponent exceeds
 // `limit` (the lazy-rescale threshold) — the common case once the running max has settled.
 // Returns false (nothing written, S intact) when the caller must take the two-pass path.
-template <bool MASKED>
-__device__ __forceinline__ bool row_exp_opt(uint32_t tS, const uint32_t (&vis)[4], uint64_t sc2, uint64_t nm2,
-                                            float limit, float& lsum) {
+template <bool MASKED, int NC, class Agree>
+__device__ __forceinline__ bool row_exp_opt(uint32_t tS, const uint32_t (&vis)[NC], uint64_t sc2, uint64_t nm2,
+                                            float limit, float& lsum, Agree&& agree) {
   uint64_t acc0 = pk2(0.0f, 0.0f), acc1 = acc0;
-  uint32_t pk[64];
+  uint32_t pk[NC * 16];
   float xm0 = -INFINITY, xm1 = -INFINITY;
 #pragma unroll
-  for (int c = 0; c < 4; ++c) {
+  for (int c = 0; c < NC; ++c) {
     uint32_t r[32];
     ptx::tmem_ld32(tS + c * 32, r);
     ptx::tmem_ld_wait();
@@ -258,10 +272,9 @@ __device__ __forceinline__ bool row_exp_opt(uint32_t tS, const uint32_t (&vis)[4
       pk[c * 16 + i] = ptx::pack_bf16x2(p0, p1);
     }
   }
-  const bool ok = fmaxf(xm0, xm1) <= limit;
-  if (!__all_sync(0xffffffffu, ok)) return false;
+  if (!agree(__all_sync(0xffffffffu, fmaxf(xm0, xm1) <= limit))) return false;
 #pragma unroll
-  for (int c = 0; c < 4; ++c)
+  for (int c = 0; c < NC; ++c)
     asm volatile(
         "tcgen05.st.sync.aligned.32x32b.x16.b32 [%0], "
         "{%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,%16};" ::"r"(tS + c * 16),
@@ -276,9 +289,10 @@ __device__ __forceinline__ bool row_exp_opt(uint32_t tS, const uint32_t (&vis)[4
   return true;
 }
 
+template <int NC>
 __device__ __forceinline__ void row_zero_p(uint32_t tS) {
 #pragma unroll
-  for (int c = 0; c < 4; ++c)
+  for (int c = 0; c < NC; ++c)
     asm volatile(
         "tcgen05.st.sync.aligned.32x32b.x16.b32 [%0], "
         "{%1,%1,%1,%1,%1,%1,%1,%1,%1,%1,%1,%1,%1,%1,%1,%1};" ::"r"(tS + c * 16), "r"(0u));
@@ -298,14 +312,14 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) attn_tc_kernel(const __grid_co
     ptx::mbar_init(&bars->q_full, 1);
     ptx::mbar_init(&bars->q_empty, 1);
     for (int i = 0; i < 2; ++i) {
-      ptx::mbar_init(&bars->k_full[i], 1);
+      ptx::mbar_init(&bars->k_full[i], kLoaders);
       ptx::mbar_init(&bars->k_empty[i], 1);
-      ptx::mbar_init(&bars->v_full[i], 1);
+      ptx::mbar_init(&bars->v_full[i], kLoaders);
       ptx::mbar_init(&bars->v_empty[i], 1);
       ptx::mbar_init(&bars->s_full[i], 1);
-      ptx::mbar_init(&bars->p_full[i], 4);
+      ptx::mbar_init(&bars->p_full[i], 8);
       ptx::mbar_init(&bars->o_full[i], 1);
-      ptx::mbar_init(&bars->o_empty[i], 4);
+      ptx::mbar_init(&bars->o_empty[i], 8);
     }
     ptx::fence_mbar_init();
   }
@@ -318,18 +332,34 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) attn_tc_kernel(const __grid_co
   const int32_t* img = p.img;
   const int32_t* work = img + p.off_work;
 
-  if (warp == 0) {  // --------------------------------------------------------- loader
+  if (warp == 0 || warp == 2 || warp == 3) {  // ------------------------------------ loaders
+    // Loader warp lw (0, 1, 2) moves pages lw, lw+3, ... of each k-tile: lane 0 issues the
+    // 2 KB bulk copies of those pages' K (then V) chunks — three warps because one warp issues
+    // bulk copies at only ~30 B/clk (tools/bulk_rate.cu).  Page ids come from the work item's
+    // tile-page records (8 per listed tile, lanes 0-7) at addresses known in advance, loaded three
+    // tiles ahead; the K and V blocks of the tile two ahead are prefetched into L2.
+    const int lw = warp == 0 ? 0 : int(warp) - 1;
     uint32_t qc = 0, kc = 0;
+    const bool pl = lane < kKtilePages;
+    constexpr int32_t kNone = kZeroPage + 1;  // "no tile": nothing to prefetch
+    auto ids = [&](const WorkItem& a, const WorkItem& n, int t) -> int32_t {
+      if (!pl) return kNone;
+      if (t < a.kt_n) return img[a.tp_off + t * kKtilePages + lane];
+      t -= a.kt_n;
+      if (t < n.kt_n) return img[n.tp_off + t * kKtilePages + lane];
+      return kNone;
+    };
+    const bool mine = pl && (lane % kLoaders) == lw;  // lanes whose page this warp prefetches
+    const WorkItem none{0, 0, -1, -1, 0, 0, 0};
     for (int w = blockIdx.x; w < p.n_work; w += gridDim.x, ++qc) {
       const WorkItem wi = load_work(work, w);
+      const WorkItem nx = (w + int(gridDim.x) < p.n_work) ? load_work(work, w + gridDim.x) : none;
       const int32_t* q_info = img + p.off_qinfo + int64_t(wi.b) * 8;
       const int qtile0 = q_info[2], page_off = q_info[4];
-      const int32_t* pages = img + p.off_pages + page_off;
       const int32_t* ktl = img + wi.kt_off;
-      // prefetch tile 0's page ids (lanes 0-7)
-      int32_t next_page = 0;
-      if (wi.kt_n > 0 && lane < kKtilePages) next_page = pages[(ktl[0] & 0xFFFFFF) * kKtilePages + lane];
-      if (lane == 0) {
+      int32_t pa = ids(wi, nx, 0), pb = ids(wi, nx, 1), pc = ids(wi, nx, 2);
+      int32_t jn = wi.kt_n > 0 ? ktl[0] : 0;
+      if (lw == 0 && lane == 0) {
         ptx::mbar_wait(&bars->q_empty, (qc & 1) ^ 1);
         const int nq = wi.q1 >= 0 ? 2 : 1;
         ptx::mbar_expect_tx(&bars->q_full, nq * L::TILE_BYTES);
@@ -342,44 +372,67 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) attn_tc_kernel(const __grid_co
                         &bars->q_full);
       }
       for (int x = 0; x < wi.kt_n; ++x, ++kc) {
-        const int j = ktl[x] & 0xFFFFFF;
-        const int32_t my_page = next_page;
-        if (x + 1 < wi.kt_n && lane < kKtilePages)
-          next_page = pages[(ktl[x + 1] & 0xFFFFFF) * kKtilePages + lane];
+        const int j = jn & 0xFFFFFF;
+        if (x + 1 < wi.kt_n) jn = ktl[x + 1];
+        const int32_t pd = ids(wi, nx, x + 3);
+        if (mine && pc != kNone && pc != kZeroPage) {  // L2 prefetch of tile x + 2 (maybe the next item's)
+          const char* src = resolve_page(p, pc);
+          const int kvh = (x + 2 < wi.kt_n) ? wi.kvh : nx.kvh;
+          ptx::bulk_prefetch_l2(src + int64_t(kvh) * p.head_bytes, L::CHUNKS * 2048);
+          ptx::bulk_prefetch_l2(src + int64_t(p.kv_heads + kvh) * p.head_bytes, L::CHUNKS * 2048);
+        }
+        const char* src[3];
+#pragma unroll
+        for (int i = 0; i < 3; ++i) {
+          const int pg = lw + kLoaders * i;
+          const int32_t id = __shfl_sync(0xffffffffu, pa, pg < kKtilePages ? pg : 0);
+          src[i] = pg < kKtilePages ? resolve_page(p, id) : nullptr;
+        }
         const int s = kc & 1;
         const uint32_t ph = ((kc >> 1) & 1) ^ 1;
-        const char* src = (lane < kKtilePages) ? resolve_page(p, my_page) : nullptr;
         uint8_t* sk = smem + L::K_OFF + s * L::TILE_BYTES;
         uint8_t* sv = smem + L::V_OFF + s * L::TILE_BYTES;
-        const bool dbg_first = (qc == 0);
+        const bool dbg_first = (qc == 0) && lw == 0;
         if (lane == 0) {
+          const int npg = (kKtilePages - lw + kLoaders - 1) / kLoaders;
           DBG(0, x);
           ptx::mbar_wait(&bars->k_empty[s], ph);
           DBG(1, x);
-          ptx::mbar_expect_tx(&bars->k_full[s], L::TILE_BYTES);
-        }
-        __syncwarp();
-        if (lane < kKtilePages) {
-          const char* kb = src + int64_t(wi.kvh) * p.head_bytes;
+          ptx::mbar_expect_tx(&bars->k_full[s], npg * L::CHUNKS * 2048);
 #pragma unroll
-          for (int c = 0; c < L::CHUNKS; ++c)
-            ptx::bulk_g2s(sk + c * 16384 + lane * 2048, kb + c * 2048, 2048, &bars->k_full[s]);
-        }
-        if (lane == 0) {
-          ptx::mbar_wait(&bars->v_empty[s], ph);
+          for (int i = 0; i < 3; ++i) {
+            const int pg = lw + kLoaders * i;
+            if (pg < kKtilePages) {
+              const char* kb = src[i] + int64_t(wi.kvh) * p.head_bytes;
+#pragma unroll
+              for (int c = 0; c < L::CHUNKS; ++c)
+                ptx::bulk_g2s(sk + c * 16384 + pg * 2048, kb + c * 2048, 2048, &bars->k_full[s]);
+            }
+          }
           DBG(2, x);
-          ptx::mbar_expect_tx(&bars->v_full[s], L::TILE_BYTES + 1024);
-          ptx::bulk_g2s(smem + L::META_OFF + s * 1024,
-                        img + p.off_kmeta + (int64_t(page_off) + int64_t(j) * kKtilePages) * kPageTokens * 2,
-                        1024, &bars->v_full[s]);
+          ptx::mbar_wait(&bars->v_empty[s], ph);
+          DBG(3, x);
+          ptx::mbar_expect_tx(&bars->v_full[s], npg * L::CHUNKS * 2048 + (lw == 0 ? 1024 : 0));
+          if (lw == 0)
+            ptx::bulk_g2s(smem + L::META_OFF + s * 1024,
+                          img + p.off_kmeta + (int64_t(page_off) + int64_t(j) * kKtilePages) * kPageTokens * 2,
+                          1024, &bars->v_full[s]);
+#pragma unroll
+          for (int i = 0; i < 3; ++i) {
+            const int pg = lw + kLoaders * i;
+            if (pg < kKtilePages) {
+              const char* vb = src[i] + int64_t(p.kv_heads + wi.kvh) * p.head_bytes;
+#pragma unroll
+              for (int c = 0; c < L::CHUNKS; ++c)
+                ptx::bulk_g2s(sv + c * 16384 + pg * 2048, vb + c * 2048, 2048, &bars->v_full[s]);
+            }
+          }
+          DBG(4, x);
         }
         __syncwarp();
-        if (lane < kKtilePages) {
-          const char* vb = src + int64_t(p.kv_heads + wi.kvh) * p.head_bytes;
-#pragma unroll
-          for (int c = 0; c < L::CHUNKS; ++c)
-            ptx::bulk_g2s(sv + c * 16384 + lane * 2048, vb + c * 2048, 2048, &bars->v_full[s]);
-        }
+        pa = pb;
+        pb = pc;
+        pc = pd;
       }
     }
   } else if (warp == 1) {  // ---------------------------------------------- MMA issuer
@@ -398,9 +451,9 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) attn_tc_kernel(const __grid_co
       };
       auto issue_pv = [&](uint32_t tS, uint32_t tO, uint32_t sv, bool acc) {
 #pragma unroll
-        for (int kk = 0; kk < 8; ++kk)
-          ptx::mma_ts(tO, tS + kk * 8, ptx::desc_sw128(sv + kk * 2048, 16384, 1024), IDESC_PV,
-                      (acc || kk) ? 1u : 0u);
+        for (int kk = 0; kk < 8; ++kk)  // keys [16kk, 16kk+16): P of half kk/4 at columns 64(kk/4) + 8(kk%4)
+          ptx::mma_ts(tO, tS + (kk >> 2) * 64 + (kk & 3) * 8, ptx::desc_sw128(sv + kk * 2048, 16384, 1024),
+                      IDESC_PV, (acc || kk) ? 1u : 0u);
       };
       for (int w = blockIdx.x; w < p.n_work; w += gridDim.x, ++qc) {
         const WorkItem wi = load_work(work, w);
@@ -428,23 +481,23 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) attn_tc_kernel(const __grid_co
           const uint32_t g = kc + x;
           const int s = g & 1;
           const uint32_t sv = ptx::smem_u32(smem + L::V_OFF + s * L::TILE_BYTES);
-          DBG(3, x);
+          DBG(5, x);
           const bool more = x + 1 < n;
           const uint32_t gn = g + 1;
           const int sn = gn & 1;
           const uint32_t skn = ptx::smem_u32(smem + L::K_OFF + sn * L::TILE_BYTES);
           // ---- q-tile 0: PV0_x, then S0_{x+1}
           ptx::mbar_wait(&bars->p_full[0], pc0 & 1);
-          DBG(4, x);
+          DBG(6, x);
           ++pc0;
           ptx::mbar_wait(&bars->v_full[s], (g >> 1) & 1);
-          DBG(5, x);
+          DBG(7, x);
           if (x == 0) ptx::mbar_wait(&bars->o_empty[0], (oc0 & 1) ^ 1);
           ptx::tc_fence_after();
           issue_pv(tS0, tO0, sv, x > 0);
           if (more) {
             ptx::mbar_wait(&bars->k_full[sn], (gn >> 1) & 1);
-            DBG(6, x);
+            DBG(8, x);
             ptx::tc_fence_after();
             issue_s(sq0, tS0, skn);
             ptx::mma_commit(&bars->s_full[0]);
@@ -452,7 +505,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) attn_tc_kernel(const __grid_co
           // ---- q-tile 1: PV1_x, then S1_{x+1}
           if (has1) {
             ptx::mbar_wait(&bars->p_full[1], pc1 & 1);
-            DBG(7, x);
+            DBG(9, x);
             ++pc1;
             if (x == 0) ptx::mbar_wait(&bars->o_empty[1], (oc1 & 1) ^ 1);
             ptx::tc_fence_after();
@@ -467,6 +520,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) attn_tc_kernel(const __grid_co
             ptx::mma_commit(&bars->k_empty[sn]);
             if (x + 1 == n - 1) ptx::mma_commit(&bars->q_empty);
           }
+          DBG(10, x);
         }
         ptx::mma_commit(&bars->o_full[0]);
         ++oc0;
@@ -480,12 +534,16 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) attn_tc_kernel(const __grid_co
       }
     }
   } else if (warp >= 4) {  // ------------------------------------------ softmax warpgroups
-    const int wg = (warp - 4) >> 2;  // 0 or 1
+    const int wgi = (warp - 4) >> 2;
+    const int wg = wgi & 1, h = wgi >> 1;  // q-tile, key half
     const uint32_t sub = warp & 3;
     const int row = sub * 32 + lane;
     const uint32_t lane_base = (sub * 32) << 16;
-    const uint32_t tS = tmem + wg * 128 + lane_base;
-    const uint32_t tO = tmem + 256 + wg * 128 + lane_base;
+    const uint32_t tS = tmem + wg * 128 + h * 64 + lane_base;       // my S half; P at its first 32 columns
+    constexpr int OCH = DP / 64;                                     // 32-column O chunks per half
+    const uint32_t tO = tmem + 256 + wg * 128 + h * (DP / 2) + lane_base;
+    const uint32_t pair_bar = 1 + wg * 4 + sub;                      // named barrier of the warp pair
+    XchSmem* xch = reinterpret_cast<XchSmem*>(smem + L::XCH_OFF);
     uint32_t kc = 0, sc = 0, oc = 0;
     for (int w = blockIdx.x; w < p.n_work; w += gridDim.x) {
       const WorkItem wi = load_work(work, w);
@@ -506,18 +564,20 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) attn_tc_kernel(const __grid_co
         const uint32_t g = kc + x;
         const int s = g & 1;
         const int state = (ktl[x] >> (24 + 2 * wg)) & 3;
-        const bool dbg_first = (kc == 0) && row == 0;
-        DBG(8 + 4 * wg, x);
+        const bool dbg_first = (kc == 0) && row == 0 && h == 0;
+        
         ptx::mbar_wait(&bars->s_full[wg], sc & 1);
-        DBG(9 + 4 * wg, x);
+        DBG(11 + 3 * wg, x);
         ++sc;
         ptx::tc_fence_after();
-        uint32_t vis[4] = {0xffffffffu, 0xffffffffu, 0xffffffffu, 0xffffffffu};
+        uint32_t vis[NCH];
+#pragma unroll
+        for (int c = 0; c < NCH; ++c) vis[c] = 0xffffffffu;
         if (state == 2) {
           ptx::mbar_wait(&bars->v_full[s], (g >> 1) & 1);  // key metadata travels with V
-          const int4* meta = reinterpret_cast<const int4*>(smem + L::META_OFF + s * 1024);
+          const int4* meta = reinterpret_cast<const int4*>(smem + L::META_OFF + s * 1024) + h * NCH * 16;
 #pragma unroll
-          for (int c = 0; c < 4; ++c) {
+          for (int c = 0; c < NCH; ++c) {
             uint32_t bits = 0;
 #pragma unroll
             for (int i = 0; i < 16; ++i) {
@@ -529,83 +589,91 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) attn_tc_kernel(const __grid_co
             vis[c] = bits;
           }
         }
-        // fast path: one pass against the settled reference max
+        // fast path: one pass against the settled reference max; both halves must agree
         bool done = false;
         float lsum = 0.0f;
         if (state == 0) {
-          row_zero_p(tS);
+          row_zero_p<NCH>(tS);
           done = true;
-        } else if (__all_sync(0xffffffffu, m_ref != -INFINITY)) {  // warp-uniform: .sync.aligned ops
-          const float mref0 = m_ref;
-          const uint64_t sc2 = pk2(p.scale_log2, p.scale_log2), nm2 = pk2(-mref0, -mref0);
-          done = (state == 1) ? row_exp_opt<false>(tS, vis, sc2, nm2, kRescaleThreshold, lsum)
-                              : row_exp_opt<true>(tS, vis, sc2, nm2, kRescaleThreshold, lsum);
+        } else if (__all_sync(0xffffffffu, m_ref != -INFINITY)) {  // same in both halves of the pair
+          const uint64_t sc2 = pk2(p.scale_log2, p.scale_log2), nm2 = pk2(-m_ref, -m_ref);
+          auto agree = [&](bool ok) {
+            if (lane == 0) xch->ok[s][wg][h][sub] = ok;
+            ptx::bar_sync(pair_bar, 64);
+            return ok && xch->ok[s][wg][h ^ 1][sub] != 0;
+          };
+          done = (state == 1) ? row_exp_opt<false>(tS, vis, sc2, nm2, kRescaleThreshold, lsum, agree)
+                              : row_exp_opt<true>(tS, vis, sc2, nm2, kRescaleThreshold, lsum, agree);
         }
-        DBG(10 + 4 * wg, x);
+        if (wg == 0) DBG(12, x);
         if (!done) {
-        // slow path, pass 1: row max of the raw scores
-        float mt = -INFINITY;
-        if (state == 1) mt = row_max<false>(tS, vis);
-        else if (state == 2) mt = row_max<true>(tS, vis);
-        const float m_old = m_ref;
-        const float m_new = fmaxf(m_ref, mt * p.scale_log2);
-        const bool grow = m_new > m_ref + kRescaleThreshold;
-        float alpha = 1.0f;
-        if (grow) {
-          alpha = ex2(m_ref - m_new);  // 0 when m_ref = -inf
-          l_sum *= alpha;
-          m_ref = m_new;
-        }
-        // O rows of this warp are rescaled when a lane's reference max moved.  The previous
-        // P.V of this q-tile is complete: it was issued before this S (in-order tensor pipe).
-        const bool need_o = grow && (m_old != -INFINITY) && (x > 0);
-        if (__any_sync(0xffffffffu, need_o)) {
-          const float a = need_o ? alpha : 1.0f;
-#pragma unroll 1
-          for (int c = 0; c < DP / 32; ++c) {
-            uint32_t r[32];
-            ptx::tmem_ld32(tO + c * 32, r);
-            ptx::tmem_ld_wait();
-#pragma unroll
-            for (int i = 0; i < 32; ++i) r[i] = __float_as_uint(__uint_as_float(r[i]) * a);
-            ptx::tmem_st32(tO + c * 32, r);
+          // slow path, pass 1: row max of the raw scores over both halves
+          float mt = (state == 1) ? row_max<false>(tS, vis) : row_max<true>(tS, vis);
+          xch->rmax[s][wg][h][row] = mt;
+          ptx::bar_sync(pair_bar, 64);
+          mt = fmaxf(mt, xch->rmax[s][wg][h ^ 1][row]);
+          const float m_old = m_ref;
+          const float m_new = fmaxf(m_ref, mt * p.scale_log2);
+          const bool grow = m_new > m_ref + kRescaleThreshold;
+          float alpha = 1.0f;
+          if (grow) {
+            alpha = ex2(m_ref - m_new);  // 0 when m_ref = -inf
+            l_sum *= alpha;
+            m_ref = m_new;
           }
-          ptx::tmem_st_wait();
-        }
-        // pass 2: P = exp2(s * scale - m_ref) -> bf16 into the S buffer's first 64 columns;
-        // BAT_POLY_PAIRS of every 16 column pairs on the FMA pipe (polynomial), rest on MUFU.
-        const float mref = (m_ref == -INFINITY) ? 0.0f : m_ref;
-        const uint64_t sc2 = pk2(p.scale_log2, p.scale_log2), nm2 = pk2(-mref, -mref);
-        if (state == 1) lsum = row_exp<false>(tS, vis, sc2, nm2);
-        else if (state == 2) lsum = row_exp<true>(tS, vis, sc2, nm2);
+          // O rows of this warp are rescaled (my half of the columns) when a lane's reference
+          // max moved.  The previous P.V of this q-tile is complete: it was issued before this
+          // S (in-order tensor pipe).
+          const bool need_o = grow && (m_old != -INFINITY) && (x > 0);
+          if (__any_sync(0xffffffffu, need_o)) {
+            const float a = need_o ? alpha : 1.0f;
+#pragma unroll 1
+            for (int c = 0; c < OCH; ++c) {
+              uint32_t r[32];
+              ptx::tmem_ld32(tO + c * 32, r);
+              ptx::tmem_ld_wait();
+#pragma unroll
+              for (int i = 0; i < 32; ++i) r[i] = __float_as_uint(__uint_as_float(r[i]) * a);
+              ptx::tmem_st32(tO + c * 32, r);
+            }
+            ptx::tmem_st_wait();
+          }
+          // pass 2: P = exp2(s * scale - m_ref) -> bf16 into my half's first 32 columns
+          const float mref = (m_ref == -INFINITY) ? 0.0f : m_ref;
+          const uint64_t sc2 = pk2(p.scale_log2, p.scale_log2), nm2 = pk2(-mref, -mref);
+          lsum = (state == 1) ? row_exp<false>(tS, vis, sc2, nm2) : row_exp<true>(tS, vis, sc2, nm2);
         }
         l_sum += lsum;
         ptx::tmem_st_wait();
         ptx::tc_fence_before();
         __syncwarp();
         if (lane == 0) ptx::mbar_arrive(&bars->p_full[wg]);
-        DBG(11 + 4 * wg, x);
+        DBG(13 + 2 * wg, x);
       }
       kc += wi.kt_n;
-      // ---- epilogue: O / l -> bf16
+      // ---- epilogue: O / l -> bf16, my half of the head's columns
+      xch->lsum[wg][h][row] = l_sum;
       ptx::mbar_wait(&bars->o_full[wg], oc & 1);
       ++oc;
       ptx::tc_fence_after();
-      const float inv = (l_sum > 0.0f) ? 1.0f / l_sum : 0.0f;
+      ptx::bar_sync(pair_bar, 64);
+      const float l_tot = l_sum + xch->lsum[wg][h ^ 1][row];
+      const float inv = (l_tot > 0.0f) ? 1.0f / l_tot : 0.0f;
       const int head = wi.kvh * p.group + row % p.group;
       __nv_bfloat16* dst = p.out + int64_t(tok_off + tok_local) * p.ldo + int64_t(head) * p.head_dim;
 #pragma unroll 1
-      for (int c = 0; c < DP / 32; ++c) {
+      for (int c = 0; c < OCH; ++c) {
+        const int col0 = h * (DP / 2) + c * 32;
         uint32_t r[32];
         ptx::tmem_ld32(tO + c * 32, r);
         ptx::tmem_ld_wait();
-        if (valid_row && c * 32 < p.head_dim) {
+        if (valid_row && col0 < p.head_dim) {
           uint32_t pk[16];
 #pragma unroll
           for (int i = 0; i < 16; ++i)
             pk[i] = ptx::pack_bf16x2(__uint_as_float(r[2 * i]) * inv, __uint_as_float(r[2 * i + 1]) * inv);
-          const int n16 = min(4, (p.head_dim - c * 32) / 8);  // 16-byte stores of real columns
-          uint4* d4 = reinterpret_cast<uint4*>(dst + c * 32);
+          const int n16 = min(4, (p.head_dim - col0) / 8);  // 16-byte stores of real columns
+          uint4* d4 = reinterpret_cast<uint4*>(dst + col0);
           for (int i = 0; i < n16; ++i) d4[i] = make_uint4(pk[4 * i], pk[4 * i + 1], pk[4 * i + 2], pk[4 * i + 3]);
         }
       }

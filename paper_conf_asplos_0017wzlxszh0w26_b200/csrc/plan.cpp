@@ -341,12 +341,22 @@ void build_plan(const Pool& pool, int32_t group, int32_t kv_heads,
     int64_t total_kt = 0;
     for (auto& w : ws) total_kt += w.n;
     int64_t off_kt = reserve_at(total_kt);
+    // the page ids of every listed k-tile, in list order (8 per tile): the attention loader
+    // reads them at addresses known in advance instead of chasing kt list -> page table
+    int64_t off_tp = reserve_at(total_kt * kKtilePages);
     int64_t cur = 0;
     for (int32_t w = 0; w < n_work; ++w) {
       int32_t* e = &v[off_work + int64_t(w) * 8];
       e[0] = ws[w].b; e[1] = ws[w].kvh; e[2] = ws[w].q0; e[3] = ws[w].q1;
-      e[4] = static_cast<int32_t>(off_kt + cur); e[5] = ws[w].n; e[6] = 0; e[7] = 0;
-      for (int32_t x : ws[w].kt) v[off_kt + cur++] = x;
+      e[4] = static_cast<int32_t>(off_kt + cur); e[5] = ws[w].n;
+      e[6] = static_cast<int32_t>(off_tp + cur * kKtilePages); e[7] = 0;
+      const int32_t page_off = plan.q[ws[w].b].page_off;
+      for (int32_t x : ws[w].kt) {
+        const int32_t j = x & 0xFFFFFF;
+        for (int l = 0; l < kKtilePages; ++l)
+          v[off_tp + cur * kKtilePages + l] = v[im.off_pages + page_off + int64_t(j) * kKtilePages + l];
+        v[off_kt + cur++] = x;
+      }
     }
   };
   make_work(false, im.off_work, plan.n_work);

@@ -45,7 +45,7 @@ struct PlanImage {
   int64_t off_kmeta = 0;                            // [16 * n_pages_padded_total][2]
   int64_t off_qtiles = 0;                           // [n_qtiles_total][4] {b, t0, ntok, 0}
   int64_t off_spages = 0;                           // [n_spages][4] {b, t0, ntok, target}
-  int64_t off_work = 0, off_work_last = 0;          // [W][8] {b, kvh, q0, q1|-1, kt_off, kt_n, 0, 0}
+  int64_t off_work = 0, off_work_last = 0;          // [W][8] {b, kvh, q0, q1|-1, kt_off, kt_n, tp_off, 0}
   int64_t off_ktl = 0;                              // kt list: ktile | state0 << 24 | state1 << 26
   int64_t off_disc = 0;                             // [B] global discriminant row
 };

@@ -43,8 +43,8 @@ e1.record(); torch.cuda.synchronize()
 ms = e0.elapsed_time(e1) / 10
 print(f"{order} B={B}: stage+attention {ms:.3f} ms/layer (host sync included); flops {4*128*12*live/1e9:.1f} GF -> {4*128*12*live/ms/1e9:.0f} TFLOP/s lower bound")
 t = np.loadtxt("gpurun_out/attn_timeline.txt").astype(np.int64)
-names = ["ld_k_wait0", "ld_k_go", "ld_v_go", "mma_u", "mma_pv0", "mma_s0", "mma_pv1", "mma_s1",
-         "sm0_wait", "sm0_s", "sm0_fast", "sm0_p", "-", "-", "-", "-"]
+names = ["ld_top", "ld_kfree", "ld_kiss", "ld_vfree", "ld_viss", "mma_top", "mma_p0", "mma_vful",
+         "mma_kful", "mma_p1", "mma_end", "sm0_s", "sm0_fast", "sm0_p", "sm1_s", "sm1_p"]
 t0 = t[t > 0].min()
 n = int((t[3] > 0).sum())
 print("tile " + " ".join(f"{nm:>10}" for nm in names))
