@@ -20,7 +20,7 @@ from typing import List, Optional, Sequence
 import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libbat.so")
+LIB_PATH = os.environ.get("BAT_LIB") or os.path.join(_HERE, "libbat.so")  # BAT_LIB: experiment builds
 
 BAT_OK = 0
 BAT_BF16, BAT_FP32 = 0, 1

@@ -246,6 +246,12 @@ static void check_compat(const Pool& p, const Model& m) {
   BAT_REQUIRE(p.device == m.device, "pool and model are on different devices");
 }
 
+// Device-side part of a plan image: the visibility masks of its partial tiles.
+static void build_masks(const Plan& plan, int32_t* dev_img, cudaStream_t st) {
+  const PlanImage& im = plan.img;
+  launch_masks(dev_img, im.off_mdesc, im.off_qinfo, im.off_kmeta, im.off_rseg, im.off_masks, im.n_masks, plan.qt, st);
+}
+
 // Workspace sizing + plan upload; returns the device image.
 static const int32_t* prepare(Pool& pool, Model& m, Plan& plan, cudaStream_t st,
                               const int32_t* dev_img = nullptr) {
@@ -271,7 +277,7 @@ static const int32_t* prepare(Pool& pool, Model& m, Plan& plan, cudaStream_t st,
   ws.actc.ensure(size_t(B) * F * 2);
   if (dev_img) return dev_img;
   const size_t img_bytes = plan.img.buf.size() * 4;
-  ws.img.ensure(img_bytes);
+  ws.img.ensure(size_t(plan.img.total_ints) * 4);
   if (!ws.img_done) CUDA_OK(cudaEventCreateWithFlags(&ws.img_done, cudaEventDisableTiming));
   CUDA_OK(cudaEventSynchronize(ws.img_done));  // the previous upload finished reading the staging buffer
   if (ws.img_host_cap < img_bytes) {
@@ -282,6 +288,7 @@ static const int32_t* prepare(Pool& pool, Model& m, Plan& plan, cudaStream_t st,
   std::memcpy(ws.img_host, plan.img.buf.data(), img_bytes);
   CUDA_OK(cudaMemcpyAsync(ws.img.p, ws.img_host, img_bytes, cudaMemcpyHostToDevice, st));
   CUDA_OK(cudaEventRecord(ws.img_done, st));
+  build_masks(plan, ws.img.as<int32_t>(), st);
   return ws.img.as<int32_t>();
 }
 
@@ -311,6 +318,7 @@ static AttnParams attn_params(const Pool& pool, const Model& m, const Plan& plan
   ap.qp = m.ws.qp.as<__nv_bfloat16>();
   ap.out = m.ws.o.as<__nv_bfloat16>();
   ap.scale_log2 = float(1.4426950408889634 / std::sqrt(double(c.head_dim)));
+  ap.off_masks = im.off_masks;
   return ap;
 }
 
@@ -408,9 +416,32 @@ static void run_plan(Pool& pool, Model& m, Plan& plan, float* out_hidden, cudaSt
     if (!last) {
       ap.off_work = im.off_work;
       ap.n_work = plan.n_work;
+      // debug (BAT_ATTN_ITEMS=file, BAT_ATTN_LAYER=l): per-work-item clock64 records of one layer
+      static const char* items_file = std::getenv("BAT_ATTN_ITEMS");
+      static const int items_layer = std::getenv("BAT_ATTN_LAYER") ? std::atoi(std::getenv("BAT_ATTN_LAYER")) : 1;
+      long long* dbi = nullptr;
+      if (items_file && l == items_layer) {
+        CUDA_OK(cudaMalloc(&dbi, size_t(ap.n_work) * 6 * sizeof(long long)));
+        CUDA_OK(cudaMemsetAsync(dbi, 0, size_t(ap.n_work) * 6 * sizeof(long long), st));
+      }
+      ap.dbg_items = dbi;
       pf.begin(st);
       launch_attention(dp, ap, m.num_sms, st);
       pf.end(st, BAT_K_ATTN, attn_fl, attn_by);
+      ap.dbg_items = nullptr;
+      if (dbi) {
+        std::vector<long long> h(size_t(ap.n_work) * 6);
+        CUDA_OK(cudaMemcpyAsync(h.data(), dbi, h.size() * sizeof(long long), cudaMemcpyDeviceToHost, st));
+        CUDA_OK(cudaStreamSynchronize(st));
+        if (FILE* f = std::fopen(items_file, "w")) {
+          for (int w = 0; w < ap.n_work; ++w) {
+            for (int e = 0; e < 6; ++e) std::fprintf(f, "%lld ", h[size_t(w) * 6 + e]);
+            std::fprintf(f, "\n");
+          }
+          std::fclose(f);
+        }
+        cudaFree(dbi);
+      }
       GemmParams go{M, H, nq, ws.h.p, H, nullptr, 0};
       auto fo = gemm_fb(M, H, nq, 8);
       pf.begin(st);
@@ -757,7 +788,7 @@ bat_status bat_kv_prefill_entities(bat_pool p, bat_model mdl, int32_t kind, int3
         reqs[e].ent_pages = &pages[e];
       }
       Plan plan;
-      build_plan(P, m.cfg.q_heads / m.cfg.kv_heads, m.cfg.kv_heads, reqs, plan, true);
+      build_plan(P, m.cfg.q_heads / m.cfg.kv_heads, m.cfg.kv_heads, reqs, plan, true, m.num_sms);
       run_plan(P, m, plan, nullptr, static_cast<cudaStream_t>(stream));
       CUDA_OK(cudaStreamSynchronize(static_cast<cudaStream_t>(stream)));
     } catch (...) {
@@ -801,7 +832,7 @@ bat_status bat_bipartite_prefill(bat_pool p, bat_model mdl, const bat_query* que
     for (int b = 0; b < B; ++b) validate_tokens(queries[b], m.cfg.vocab);
     DeviceGuard dg(P.device);
     Plan plan;
-    build_plan(P, m.cfg.q_heads / m.cfg.kv_heads, m.cfg.kv_heads, wrap(queries, B), plan, true);
+    build_plan(P, m.cfg.q_heads / m.cfg.kv_heads, m.cfg.kv_heads, wrap(queries, B), plan, true, m.num_sms);
     run_plan(P, m, plan, out_hidden, static_cast<cudaStream_t>(stream));
   });
 }
@@ -1081,7 +1112,7 @@ bat_status bat_debug_attention_layer(bat_pool p, bat_model mdl, const bat_query*
     DeviceGuard dg(P.device);
     cudaStream_t st = static_cast<cudaStream_t>(stream);
     Plan plan;
-    build_plan(P, m.cfg.q_heads / m.cfg.kv_heads, m.cfg.kv_heads, wrap(queries, B), plan, true);
+    build_plan(P, m.cfg.q_heads / m.cfg.kv_heads, m.cfg.kv_heads, wrap(queries, B), plan, true, m.num_sms);
     const int32_t* I = prepare(P, m, plan, st);
     StageParams sp = stage_params(P, m, plan, I);
     sp.qkv = static_cast<const __nv_bfloat16*>(qkv);
@@ -1094,25 +1125,45 @@ bat_status bat_debug_attention_layer(bat_pool p, bat_model mdl, const bat_query*
     const char* tl = std::getenv("BAT_ATTN_TIMELINE");  // debug: clock64 timeline of CTA 0
     long long* dbg = nullptr;
     if (tl) {
-      CUDA_OK(cudaMalloc(&dbg, 16 * 64 * sizeof(long long)));
-      CUDA_OK(cudaMemsetAsync(dbg, 0, 16 * 64 * sizeof(long long), st));
+      CUDA_OK(cudaMalloc(&dbg, 24 * 64 * sizeof(long long)));
+      CUDA_OK(cudaMemsetAsync(dbg, 0, 24 * 64 * sizeof(long long), st));
       ap.dbg = dbg;
+    }
+    const char* ti = std::getenv("BAT_ATTN_ITEMS");  // debug: per-work-item clock64 records
+    long long* dbi = nullptr;
+    if (ti) {
+      CUDA_OK(cudaMalloc(&dbi, size_t(ap.n_work) * 6 * sizeof(long long)));
+      CUDA_OK(cudaMemsetAsync(dbi, 0, size_t(ap.n_work) * 6 * sizeof(long long), st));
+      ap.dbg_items = dbi;
     }
     launch_attention(m.dpad, ap, m.num_sms, st);
     CUDA_OK(cudaGetLastError());
     CUDA_OK(cudaStreamSynchronize(st));
     if (dbg) {
-      std::vector<long long> h(16 * 64);
+      std::vector<long long> h(24 * 64);
       CUDA_OK(cudaMemcpy(h.data(), dbg, h.size() * sizeof(long long), cudaMemcpyDeviceToHost));
       FILE* f = std::fopen(tl, "w");
       if (f) {
-        for (int e = 0; e < 16; ++e) {
+        for (int e = 0; e < 24; ++e) {
           for (int x = 0; x < 64; ++x) std::fprintf(f, "%lld ", h[e * 64 + x]);
           std::fprintf(f, "\n");
         }
         std::fclose(f);
       }
       cudaFree(dbg);
+    }
+    if (dbi) {
+      std::vector<long long> h(size_t(ap.n_work) * 6);
+      CUDA_OK(cudaMemcpy(h.data(), dbi, h.size() * sizeof(long long), cudaMemcpyDeviceToHost));
+      FILE* f = std::fopen(ti, "w");
+      if (f) {
+        for (int w = 0; w < ap.n_work; ++w) {
+          for (int e = 0; e < 6; ++e) std::fprintf(f, "%lld ", h[size_t(w) * 6 + e]);
+          std::fprintf(f, "\n");
+        }
+        std::fclose(f);
+      }
+      cudaFree(dbi);
     }
   });
 }
@@ -1129,11 +1180,12 @@ bat_status bat_plan_build(bat_pool p, bat_model mdl, const bat_query* queries, i
     for (int b = 0; b < B; ++b) validate_tokens(queries[b], m.cfg.vocab);
     DeviceGuard dg(P.device);
     auto pl = std::make_unique<bat_plan_s>();
-    build_plan(P, m.cfg.q_heads / m.cfg.kv_heads, m.cfg.kv_heads, wrap(queries, B), pl->plan, true);
+    build_plan(P, m.cfg.q_heads / m.cfg.kv_heads, m.cfg.kv_heads, wrap(queries, B), pl->plan, true, m.num_sms);
     const size_t bytes = pl->plan.img.buf.size() * 4;
-    CUDA_OK(cudaMalloc(&pl->dev_img, bytes));
+    CUDA_OK(cudaMalloc(&pl->dev_img, size_t(pl->plan.img.total_ints) * 4));
     CUDA_OK(cudaMemcpyAsync(pl->dev_img, pl->plan.img.buf.data(), bytes, cudaMemcpyHostToDevice,
                             static_cast<cudaStream_t>(stream)));
+    build_masks(pl->plan, static_cast<int32_t*>(pl->dev_img), static_cast<cudaStream_t>(stream));
     CUDA_OK(cudaStreamSynchronize(static_cast<cudaStream_t>(stream)));
     pl->device = P.device;
     *out = pl.release();

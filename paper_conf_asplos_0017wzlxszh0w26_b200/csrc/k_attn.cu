@@ -5,14 +5,18 @@
 // qt suffix tokens x the g query heads sharing the KV head (GQA packing).  Both q-tiles of
 // the pair share every 128-key K/V tile the loader brings in (halving K/V traffic per FLOP).
 // The plan lists the pair's live k-tiles (block-skip: dead tiles never reach the kernel)
-// with a state per q-tile: 0 dead (P = 0), 1 full (no element mask), 2 partial (apply
-//   kord <= rord && (kseg == rseg || (kseg|rseg) < 0)  per element).
+// with a state per q-tile: 0 dead (P = 0), 1 full (no element mask), 2 partial: the element
+// mask  kord <= rord && (kseg == rseg || (kseg|rseg) < 0)  precomputed once per plan by
+// launch_masks (shared by all KV heads and layers); a row reads its 64 bits per tile.
 //
 // Warp roles (640 threads, one CTA per SM, persistent over work items, FA4-style):
-//   warps 0,2,3 loaders: each moves a third of the pages of every k-tile (2 KB bulk copies of
-//               the page's K, then V chunks) — pages are stored in the tensor-core operand layout
-//               (128-byte swizzle), so they drop into shared memory ready for tcgen05.mma; page
-//               ids are read three tiles ahead and the tile two ahead is prefetched into L2.
+//   warps 0,2,3 loaders, three independent streams: warp 0 Q and K (a 3-tile ring), warps 2 / 3
+//               the first / second V half of every tile (a 3-slot ring of 64-key halves; the
+//               tile's key metadata rides with the first half).  One bulk copy per page block:
+//               pages are stored in the tensor-core operand layout (128-byte swizzle,
+//               ptx::page_blk_off), so a block drops into shared memory ready for tcgen05.mma
+//               (8-row-group stride Dp/64 KB).  Page ids are read three tiles ahead and the
+//               blocks of the tile two ahead are prefetched into L2.
 //   warp 1      MMA issuer (one thread): S0 = Q0 K^T, S1 = Q1 K^T (SS, M=128 N=128 K=16) and
 //               O0 += P0 V, O1 += P1 V (TS: P read from TMEM, V MN-major from smem), issued as
 //               S0_0 S1_0 | PV0_j S0_{j+1} PV1_j S1_{j+1} | ... so the softmax of one q-tile
@@ -36,9 +40,11 @@ namespace bat {
 namespace {
 
 constexpr int NUM_THREADS = 640;
-constexpr int kLoaders = 3;  // loader warps 0, 2, 3: one warp issues cp.async.bulk at ~30 B/clk only
 constexpr int NCH = 2;  // 32-column S chunks per softmax thread (half of a 128-key row)
 constexpr float kRescaleThreshold = 8.0f;  // log2 units: P <= 2^8 between rescales
+#ifndef BAT_ATTN_L2PF
+#define BAT_ATTN_L2PF 0  // 1: prefetch the K/V blocks of the tile two ahead into L2 (measured slower)
+#endif
 #ifndef BAT_POLY_PAIRS
 #define BAT_POLY_PAIRS 4  // of every 16 column pairs, exp2 on the FMA pipe (rest: MUFU)
 #endif
@@ -46,15 +52,22 @@ constexpr float kRescaleThreshold = 8.0f;  // log2 units: P <= 2^8 between resca
 template <int DP>
 struct AttnSmem {
   static constexpr int CHUNKS = DP / 64;
-  static constexpr int TILE_BYTES = CHUNKS * 128 * 128;  // [CHUNKS][128 rows][64] bf16
-  static constexpr int Q_OFF = 0;                        // Q0, Q1
-  static constexpr int K_OFF = Q_OFF + 2 * TILE_BYTES;   // 2 stages
-  static constexpr int V_OFF = K_OFF + 2 * TILE_BYTES;   // 2 stages
-  static constexpr int META_OFF = V_OFF + 2 * TILE_BYTES;  // 2 x 128 x int2 (with V)
-  static constexpr int XCH_OFF = META_OFF + 2 * 1024;  // row-half exchange (see XchSmem)
+  static constexpr int TILE_BYTES = CHUNKS * 128 * 128;  // Q: [CHUNKS][128 rows][64] bf16
+  // K / V tiles: 8 page blocks [2 slot groups][CHUNKS][8][64] (ptx::page_blk_off), i.e. 16
+  // 8-row groups at stride GROUP_BYTES, chunk c of a group at +c * 1024
+  static constexpr int PAGE_BYTES = CHUNKS * 2048;
+  static constexpr int GROUP_BYTES = CHUNKS * 1024;
+  static constexpr int HALF_BYTES = TILE_BYTES / 2;        // 4 pages = 64 keys
+  static constexpr int KST = 3;                            // K ring: whole tiles (S needs N = 128 contiguous keys)
+  static constexpr int VST = 3;                            // V ring: half tiles (P.V runs 16 keys per MMA)
+  static constexpr int Q_OFF = 0;                          // Q0, Q1
+  static constexpr int K_OFF = Q_OFF + 2 * TILE_BYTES;
+  static constexpr int V_OFF = K_OFF + KST * TILE_BYTES;
+  static constexpr int XCH_OFF = V_OFF + VST * HALF_BYTES;  // row-half exchange (see XchSmem)
   static constexpr int BAR_OFF = XCH_OFF + 8192;
   static constexpr int TOTAL = BAR_OFF + 256;
 };
+static_assert(AttnSmem<128>::TOTAL + 1024 <= 232448, "attention shared memory");
 
 // exchange between the two key halves of a row ([parity][q][h]...)
 struct XchSmem {
@@ -66,10 +79,15 @@ static_assert(sizeof(XchSmem) <= 8192, "exchange area");
 
 struct __align__(8) AttnBars {
   uint64_t q_full, q_empty;
-  uint64_t k_full[2], k_empty[2], v_full[2], v_empty[2];
+  uint64_t k_full[3], k_empty[3], v_full[3], v_empty[3];
   uint64_t s_full[2], p_full[2], o_full[2], o_empty[2];
   uint32_t tmem_base;
 };
+static_assert(sizeof(AttnBars) <= 256, "barrier area");
+
+// ring positions: K tile g -> slot g % 3; V half h (= 2 g + {0,1}) -> slot h % 3
+__device__ __forceinline__ uint32_t ring_slot(uint32_t i) { return i % 3u; }
+__device__ __forceinline__ uint32_t ring_phase(uint32_t i) { return (i / 3u) & 1u; }
 
 __device__ __forceinline__ const char* resolve_page(const AttnParams& p, int32_t page) {
   if (page == kZeroPage) return p.zero_page;
@@ -137,12 +155,12 @@ __device__ __forceinline__ uint64_t exp2_poly2(uint64_t x) {
   } while (0)
 
 struct WorkItem {
-  int b, kvh, q0, q1, kt_off, kt_n, tp_off;
+  int b, kvh, q0, q1, kt_off, kt_n, tp_off, km_off;
 };
 __device__ __forceinline__ WorkItem load_work(const int32_t* work, int w) {
   const int4 a = *reinterpret_cast<const int4*>(work + int64_t(w) * 8);
   const int4 c = *reinterpret_cast<const int4*>(work + int64_t(w) * 8 + 4);
-  return WorkItem{a.x, a.y, a.z, a.w, c.x, c.y, c.z};
+  return WorkItem{a.x, a.y, a.z, a.w, c.x, c.y, c.z, c.w};
 }
 
 // ---- softmax passes over one 128-column S row held in TMEM (one row per thread) ----------
@@ -302,7 +320,9 @@ template <int DP>
 __global__ void __launch_bounds__(NUM_THREADS, 1) attn_tc_kernel(const __grid_constant__ AttnParams p) {
   using L = AttnSmem<DP>;
   extern __shared__ uint8_t smem_raw[];
-  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  // 1 KB-align by offsetting the __shared__ array itself (keeps the shared address space, so
+  // the compiler emits LDS/STS rather than generic loads and stores)
+  uint8_t* smem = smem_raw + ((1024u - (ptx::smem_u32(smem_raw) & 1023u)) & 1023u);
   AttnBars* bars = reinterpret_cast<AttnBars*>(smem + L::BAR_OFF);
   const uint32_t warp = ptx::warp_id(), lane = ptx::lane_id();
   constexpr uint32_t IDESC_S = ptx::idesc_bf16(128, 128, 0, 0);
@@ -311,11 +331,13 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) attn_tc_kernel(const __grid_co
   if (warp == 0 && lane == 0) {
     ptx::mbar_init(&bars->q_full, 1);
     ptx::mbar_init(&bars->q_empty, 1);
-    for (int i = 0; i < 2; ++i) {
-      ptx::mbar_init(&bars->k_full[i], kLoaders);
+    for (int i = 0; i < 3; ++i) {
+      ptx::mbar_init(&bars->k_full[i], 1);
       ptx::mbar_init(&bars->k_empty[i], 1);
-      ptx::mbar_init(&bars->v_full[i], kLoaders);
+      ptx::mbar_init(&bars->v_full[i], 1);
       ptx::mbar_init(&bars->v_empty[i], 1);
+    }
+    for (int i = 0; i < 2; ++i) {
       ptx::mbar_init(&bars->s_full[i], 1);
       ptx::mbar_init(&bars->p_full[i], 8);
       ptx::mbar_init(&bars->o_full[i], 1);
@@ -333,12 +355,13 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) attn_tc_kernel(const __grid_co
   const int32_t* work = img + p.off_work;
 
   if (warp == 0 || warp == 2 || warp == 3) {  // ------------------------------------ loaders
-    // Loader warp lw (0, 1, 2) moves pages lw, lw+3, ... of each k-tile: lane 0 issues the
-    // 2 KB bulk copies of those pages' K (then V) chunks — three warps because one warp issues
-    // bulk copies at only ~30 B/clk (tools/bulk_rate.cu).  Page ids come from the work item's
-    // tile-page records (8 per listed tile, lanes 0-7) at addresses known in advance, loaded three
-    // tiles ahead; the K and V blocks of the tile two ahead are prefetched into L2.
-    const int lw = warp == 0 ? 0 : int(warp) - 1;
+    // Three independent streams so each runs as far ahead as its ring allows: warp 0 loads Q and
+    // the K tiles (one bulk copy per page: the page block is the operand layout), warp 2 the first
+    // V half of every tile (pages 0-3, plus the tile's key metadata), warp 3 the second half.
+    // Page ids come from the work item's tile-page records (8 per listed tile, lanes 0-7) at
+    // addresses known in advance, loaded three tiles ahead; the blocks of the tile two ahead are
+    // prefetched into L2 by the stream that will load them.
+    const int role = warp == 0 ? 0 : int(warp) - 1;  // 0: Q + K, 1: V half a, 2: V half b
     uint32_t qc = 0, kc = 0;
     const bool pl = lane < kKtilePages;
     constexpr int32_t kNone = kZeroPage + 1;  // "no tile": nothing to prefetch
@@ -349,17 +372,17 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) attn_tc_kernel(const __grid_co
       if (t < n.kt_n) return img[n.tp_off + t * kKtilePages + lane];
       return kNone;
     };
-    const bool mine = pl && (lane % kLoaders) == lw;  // lanes whose page this warp prefetches
-    const WorkItem none{0, 0, -1, -1, 0, 0, 0};
-    for (int w = blockIdx.x; w < p.n_work; w += gridDim.x, ++qc) {
+    const bool mine = pl && (role == 0 || (lane >> 2) == role - 1);  // lanes whose page this stream prefetches
+    const int64_t kv_off = role == 0 ? 0 : int64_t(p.kv_heads) * p.head_bytes;  // K or V block of a page
+    const WorkItem none{0, 0, -1, -1, 0, 0, 0, 0};
+    for (int w = blockIdx.x; w < p.n_work; w += gridDim.x) {
       const WorkItem wi = load_work(work, w);
+      if (wi.kt_n == 0) continue;  // padding of the planner's LPT rounds
       const WorkItem nx = (w + int(gridDim.x) < p.n_work) ? load_work(work, w + gridDim.x) : none;
       const int32_t* q_info = img + p.off_qinfo + int64_t(wi.b) * 8;
-      const int qtile0 = q_info[2], page_off = q_info[4];
-      const int32_t* ktl = img + wi.kt_off;
+      const int qtile0 = q_info[2];
       int32_t pa = ids(wi, nx, 0), pb = ids(wi, nx, 1), pc = ids(wi, nx, 2);
-      int32_t jn = wi.kt_n > 0 ? ktl[0] : 0;
-      if (lw == 0 && lane == 0) {
+      if (role == 0 && lane == 0) {
         ptx::mbar_wait(&bars->q_empty, (qc & 1) ^ 1);
         const int nq = wi.q1 >= 0 ? 2 : 1;
         ptx::mbar_expect_tx(&bars->q_full, nq * L::TILE_BYTES);
@@ -372,134 +395,129 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) attn_tc_kernel(const __grid_co
                         &bars->q_full);
       }
       for (int x = 0; x < wi.kt_n; ++x, ++kc) {
-        const int j = jn & 0xFFFFFF;
-        if (x + 1 < wi.kt_n) jn = ktl[x + 1];
         const int32_t pd = ids(wi, nx, x + 3);
-        if (mine && pc != kNone && pc != kZeroPage) {  // L2 prefetch of tile x + 2 (maybe the next item's)
-          const char* src = resolve_page(p, pc);
+        if (BAT_ATTN_L2PF && mine && pc != kNone && pc != kZeroPage) {  // L2 prefetch of tile x + 2 (maybe the next item's)
           const int kvh = (x + 2 < wi.kt_n) ? wi.kvh : nx.kvh;
-          ptx::bulk_prefetch_l2(src + int64_t(kvh) * p.head_bytes, L::CHUNKS * 2048);
-          ptx::bulk_prefetch_l2(src + int64_t(p.kv_heads + kvh) * p.head_bytes, L::CHUNKS * 2048);
+          ptx::bulk_prefetch_l2(resolve_page(p, pc) + kv_off + int64_t(kvh) * p.head_bytes, L::PAGE_BYTES);
         }
-        const char* src[3];
+        const bool dbg_first = (qc == 0) && role <= 1;
+        if (role == 0) {
+          const char* src[kKtilePages];
 #pragma unroll
-        for (int i = 0; i < 3; ++i) {
-          const int pg = lw + kLoaders * i;
-          const int32_t id = __shfl_sync(0xffffffffu, pa, pg < kKtilePages ? pg : 0);
-          src[i] = pg < kKtilePages ? resolve_page(p, id) : nullptr;
-        }
-        const int s = kc & 1;
-        const uint32_t ph = ((kc >> 1) & 1) ^ 1;
-        uint8_t* sk = smem + L::K_OFF + s * L::TILE_BYTES;
-        uint8_t* sv = smem + L::V_OFF + s * L::TILE_BYTES;
-        const bool dbg_first = (qc == 0) && lw == 0;
-        if (lane == 0) {
-          const int npg = (kKtilePages - lw + kLoaders - 1) / kLoaders;
-          DBG(0, x);
-          ptx::mbar_wait(&bars->k_empty[s], ph);
-          DBG(1, x);
-          ptx::mbar_expect_tx(&bars->k_full[s], npg * L::CHUNKS * 2048);
+          for (int i = 0; i < kKtilePages; ++i) src[i] = resolve_page(p, __shfl_sync(0xffffffffu, pa, i));
+          if (lane == 0) {
+            const uint32_t ks = ring_slot(kc);
+            uint8_t* sk = smem + L::K_OFF + ks * L::TILE_BYTES;
+            DBG(0, x);
+            ptx::mbar_wait(&bars->k_empty[ks], ring_phase(kc) ^ 1);
+            DBG(1, x);
+            ptx::mbar_expect_tx(&bars->k_full[ks], kKtilePages * L::PAGE_BYTES);
 #pragma unroll
-          for (int i = 0; i < 3; ++i) {
-            const int pg = lw + kLoaders * i;
-            if (pg < kKtilePages) {
-              const char* kb = src[i] + int64_t(wi.kvh) * p.head_bytes;
-#pragma unroll
-              for (int c = 0; c < L::CHUNKS; ++c)
-                ptx::bulk_g2s(sk + c * 16384 + pg * 2048, kb + c * 2048, 2048, &bars->k_full[s]);
-            }
+            for (int i = 0; i < kKtilePages; ++i)
+              ptx::bulk_g2s(sk + i * L::PAGE_BYTES, src[i] + int64_t(wi.kvh) * p.head_bytes, L::PAGE_BYTES,
+                            &bars->k_full[ks]);
+            DBG(2, x);
           }
-          DBG(2, x);
-          ptx::mbar_wait(&bars->v_empty[s], ph);
-          DBG(3, x);
-          ptx::mbar_expect_tx(&bars->v_full[s], npg * L::CHUNKS * 2048 + (lw == 0 ? 1024 : 0));
-          if (lw == 0)
-            ptx::bulk_g2s(smem + L::META_OFF + s * 1024,
-                          img + p.off_kmeta + (int64_t(page_off) + int64_t(j) * kKtilePages) * kPageTokens * 2,
-                          1024, &bars->v_full[s]);
+        } else {
+          const int hf = role - 1;
+          const char* src[4];
 #pragma unroll
-          for (int i = 0; i < 3; ++i) {
-            const int pg = lw + kLoaders * i;
-            if (pg < kKtilePages) {
-              const char* vb = src[i] + int64_t(p.kv_heads + wi.kvh) * p.head_bytes;
+          for (int i = 0; i < 4; ++i) src[i] = resolve_page(p, __shfl_sync(0xffffffffu, pa, 4 * hf + i));
+          if (lane == 0) {
+            const uint32_t vi = 2 * kc + hf, vs = ring_slot(vi);
+            uint8_t* sv = smem + L::V_OFF + vs * L::HALF_BYTES;
+            if (hf == 0) DBG(3, x);
+            ptx::mbar_wait(&bars->v_empty[vs], ring_phase(vi) ^ 1);
+            if (hf == 0) DBG(4, x);
+            ptx::mbar_expect_tx(&bars->v_full[vs], 4 * L::PAGE_BYTES);
 #pragma unroll
-              for (int c = 0; c < L::CHUNKS; ++c)
-                ptx::bulk_g2s(sv + c * 16384 + pg * 2048, vb + c * 2048, 2048, &bars->v_full[s]);
-            }
+            for (int i = 0; i < 4; ++i)
+              ptx::bulk_g2s(sv + i * L::PAGE_BYTES, src[i] + kv_off + int64_t(wi.kvh) * p.head_bytes, L::PAGE_BYTES,
+                            &bars->v_full[vs]);
           }
-          DBG(4, x);
         }
         __syncwarp();
         pa = pb;
         pb = pc;
         pc = pd;
       }
+      ++qc;
     }
   } else if (warp == 1) {  // ---------------------------------------------- MMA issuer
     if (lane == 0) {
-      uint32_t qc = 0, kc = 0, sc0 = 0, sc1 = 0, pc0 = 0, pc1 = 0, oc0 = 0, oc1 = 0;
+      uint32_t qc = 0, kc = 0, pc0 = 0, pc1 = 0, oc0 = 0, oc1 = 0;
       const uint32_t sq0 = ptx::smem_u32(smem + L::Q_OFF);
       const uint32_t sq1 = sq0 + L::TILE_BYTES;
       const uint32_t tS0 = tmem, tS1 = tmem + 128, tO0 = tmem + 256, tO1 = tmem + 384;
+      auto sk_of = [&](uint32_t g) { return ptx::smem_u32(smem + L::K_OFF + ring_slot(g) * L::TILE_BYTES); };
+      auto sv_of = [&](uint32_t vi) { return ptx::smem_u32(smem + L::V_OFF + ring_slot(vi) * L::HALF_BYTES); };
+      auto wait_k = [&](uint32_t g) {
+        ptx::mbar_wait(&bars->k_full[ring_slot(g)], ring_phase(g));
+        ptx::tc_fence_after();
+      };
       auto issue_s = [&](uint32_t sq, uint32_t tS, uint32_t sk) {
 #pragma unroll
         for (int kk = 0; kk < DP / 16; ++kk) {
-          const uint32_t off = (kk >> 2) * 16384 + (kk & 3) * 32;
-          ptx::mma_ss(tS, ptx::desc_sw128(sq + off, 16, 1024), ptx::desc_sw128(sk + off, 16, 1024), IDESC_S,
-                      kk ? 1u : 0u);
+          const uint32_t qoff = (kk >> 2) * 16384 + (kk & 3) * 32;  // Q: chunk-major, 8-row groups 1 KB apart
+          const uint32_t koff = (kk >> 2) * 1024 + (kk & 3) * 32;   // K: page blocks, groups GROUP_BYTES apart
+          ptx::mma_ss(tS, ptx::desc_sw128(sq + qoff, 16, 1024), ptx::desc_sw128(sk + koff, 16, L::GROUP_BYTES),
+                      IDESC_S, kk ? 1u : 0u);
         }
       };
-      auto issue_pv = [&](uint32_t tS, uint32_t tO, uint32_t sv, bool acc) {
+      // O += P V for one V half (keys [64 hf, 64 hf + 64) = pages 4 hf .. 4 hf + 3): the P of key half
+      // hf (bf16 pairs) sits at S columns [64 hf, 64 hf + 32), so keys [16 i, 16 i + 16) of the half
+      // are at column 64 hf + 8 i; V page i of the half at sv + i * PAGE_BYTES
+      auto issue_pv = [&](uint32_t tS, uint32_t tO, uint32_t sv, int hf, bool acc) {
 #pragma unroll
-        for (int kk = 0; kk < 8; ++kk)  // keys [16kk, 16kk+16): P of half kk/4 at columns 64(kk/4) + 8(kk%4)
-          ptx::mma_ts(tO, tS + (kk >> 2) * 64 + (kk & 3) * 8, ptx::desc_sw128(sv + kk * 2048, 16384, 1024),
-                      IDESC_PV, (acc || kk) ? 1u : 0u);
+        for (int i = 0; i < 4; ++i)
+          ptx::mma_ts(tO, tS + hf * 64 + i * 8, ptx::desc_sw128(sv + i * L::PAGE_BYTES, 1024, L::GROUP_BYTES),
+                      IDESC_PV, (acc || hf || i) ? 1u : 0u);
       };
-      for (int w = blockIdx.x; w < p.n_work; w += gridDim.x, ++qc) {
+      for (int w = blockIdx.x; w < p.n_work; w += gridDim.x) {
         const WorkItem wi = load_work(work, w);
         const bool has1 = wi.q1 >= 0;
         const int n = wi.kt_n;
-        if (n == 0) continue;
+        if (n == 0) continue;  // padding of the planner's LPT rounds
         ptx::mbar_wait(&bars->q_full, qc & 1);
+        if (p.dbg_items) p.dbg_items[int64_t(w) * 6 + 0] = clock64();
         // S for tile 0
         {
-          const int s = kc & 1;
-          ptx::mbar_wait(&bars->k_full[s], (kc >> 1) & 1);
-          ptx::tc_fence_after();
-          const uint32_t sk = ptx::smem_u32(smem + L::K_OFF + s * L::TILE_BYTES);
+          wait_k(kc);
+          const uint32_t sk = sk_of(kc);
           issue_s(sq0, tS0, sk);
           ptx::mma_commit(&bars->s_full[0]);
           if (has1) {
             issue_s(sq1, tS1, sk);
             ptx::mma_commit(&bars->s_full[1]);
           }
-          ptx::mma_commit(&bars->k_empty[s]);
+          ptx::mma_commit(&bars->k_empty[ring_slot(kc)]);
           if (n == 1) ptx::mma_commit(&bars->q_empty);
+          if (p.dbg_items) p.dbg_items[int64_t(w) * 6 + 1] = clock64();
         }
         const bool dbg_first = (qc == 0);
         for (int x = 0; x < n; ++x) {
           const uint32_t g = kc + x;
-          const int s = g & 1;
-          const uint32_t sv = ptx::smem_u32(smem + L::V_OFF + s * L::TILE_BYTES);
+          const uint32_t va = 2 * g, vb = 2 * g + 1;
+          const uint32_t sva = sv_of(va), svb = sv_of(vb);
           DBG(5, x);
           const bool more = x + 1 < n;
           const uint32_t gn = g + 1;
-          const int sn = gn & 1;
-          const uint32_t skn = ptx::smem_u32(smem + L::K_OFF + sn * L::TILE_BYTES);
           // ---- q-tile 0: PV0_x, then S0_{x+1}
           ptx::mbar_wait(&bars->p_full[0], pc0 & 1);
           DBG(6, x);
           ++pc0;
-          ptx::mbar_wait(&bars->v_full[s], (g >> 1) & 1);
-          DBG(7, x);
           if (x == 0) ptx::mbar_wait(&bars->o_empty[0], (oc0 & 1) ^ 1);
+          ptx::mbar_wait(&bars->v_full[ring_slot(va)], ring_phase(va));
+          DBG(7, x);
           ptx::tc_fence_after();
-          issue_pv(tS0, tO0, sv, x > 0);
+          issue_pv(tS0, tO0, sva, 0, x > 0);
+          ptx::mbar_wait(&bars->v_full[ring_slot(vb)], ring_phase(vb));
+          ptx::tc_fence_after();
+          issue_pv(tS0, tO0, svb, 1, true);
           if (more) {
-            ptx::mbar_wait(&bars->k_full[sn], (gn >> 1) & 1);
+            wait_k(gn);
             DBG(8, x);
-            ptx::tc_fence_after();
-            issue_s(sq0, tS0, skn);
+            issue_s(sq0, tS0, sk_of(gn));
             ptx::mma_commit(&bars->s_full[0]);
           }
           // ---- q-tile 1: PV1_x, then S1_{x+1}
@@ -509,28 +527,34 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) attn_tc_kernel(const __grid_co
             ++pc1;
             if (x == 0) ptx::mbar_wait(&bars->o_empty[1], (oc1 & 1) ^ 1);
             ptx::tc_fence_after();
-            issue_pv(tS1, tO1, sv, x > 0);
+            issue_pv(tS1, tO1, sva, 0, x > 0);
           }
-          ptx::mma_commit(&bars->v_empty[s]);
+          ptx::mma_commit(&bars->v_empty[ring_slot(va)]);
+          if (has1) issue_pv(tS1, tO1, svb, 1, true);
+          ptx::mma_commit(&bars->v_empty[ring_slot(vb)]);
           if (more) {
             if (has1) {
-              issue_s(sq1, tS1, skn);
+              issue_s(sq1, tS1, sk_of(gn));
               ptx::mma_commit(&bars->s_full[1]);
             }
-            ptx::mma_commit(&bars->k_empty[sn]);
+            ptx::mma_commit(&bars->k_empty[ring_slot(gn)]);
             if (x + 1 == n - 1) ptx::mma_commit(&bars->q_empty);
           }
           DBG(10, x);
         }
         ptx::mma_commit(&bars->o_full[0]);
+        if (p.dbg_items) {
+          p.dbg_items[int64_t(w) * 6 + 2] = clock64();
+          p.dbg_items[int64_t(w) * 6 + 4] = n;
+          p.dbg_items[int64_t(w) * 6 + 5] = blockIdx.x;
+        }
         ++oc0;
         if (has1) {
           ptx::mma_commit(&bars->o_full[1]);
           ++oc1;
         }
         kc += n;
-        (void)sc0;
-        (void)sc1;
+        ++qc;
       }
     }
   } else if (warp >= 4) {  // ------------------------------------------ softmax warpgroups
@@ -556,8 +580,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) attn_tc_kernel(const __grid_co
       const int tok_off = q_info[0], S = q_info[1];
       const int tok_local = qi * p.qt + row / p.group;
       const bool valid_row = row < p.qt * p.group && tok_local < S;
-      const int32_t rseg = valid_row ? img[p.off_rseg + tok_off + tok_local] : -1;
-      const int32_t rord = valid_row ? tok_local + 1 : kInvalidOrd - 1;
+      const int mrow = valid_row ? row / p.group : p.qt;  // row of this thread in the masks
       const int32_t* ktl = img + wi.kt_off;
       float m_ref = -INFINITY, l_sum = 0.0f;
       for (int x = 0; x < wi.kt_n; ++x) {
@@ -565,30 +588,18 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) attn_tc_kernel(const __grid_co
         const int s = g & 1;
         const int state = (ktl[x] >> (24 + 2 * wg)) & 3;
         const bool dbg_first = (kc == 0) && row == 0 && h == 0;
-        
+        // partial tile: this row's 64 visibility bits from the plan's precomputed mask (issued
+        // before the S wait so the load latency hides behind the MMA)
+        uint2 mv = make_uint2(0xffffffffu, 0xffffffffu);
+        if (state == 2) {
+          const int mid = img[wi.km_off + 2 * x + wg];
+          mv = __ldg(reinterpret_cast<const uint2*>(img + p.off_masks + (int64_t(mid) * (p.qt + 1) + mrow) * 4) + h);
+        }
         ptx::mbar_wait(&bars->s_full[wg], sc & 1);
         DBG(11 + 3 * wg, x);
         ++sc;
         ptx::tc_fence_after();
-        uint32_t vis[NCH];
-#pragma unroll
-        for (int c = 0; c < NCH; ++c) vis[c] = 0xffffffffu;
-        if (state == 2) {
-          ptx::mbar_wait(&bars->v_full[s], (g >> 1) & 1);  // key metadata travels with V
-          const int4* meta = reinterpret_cast<const int4*>(smem + L::META_OFF + s * 1024) + h * NCH * 16;
-#pragma unroll
-          for (int c = 0; c < NCH; ++c) {
-            uint32_t bits = 0;
-#pragma unroll
-            for (int i = 0; i < 16; ++i) {
-              const int4 km = meta[c * 16 + i];  // (kseg, kord) x 2, broadcast across the warp
-              const bool v0 = (km.y <= rord) && ((km.x == rseg) || ((km.x | rseg) < 0));
-              const bool v1 = (km.w <= rord) && ((km.z == rseg) || ((km.z | rseg) < 0));
-              bits |= (uint32_t(v0) << (2 * i)) | (uint32_t(v1) << (2 * i + 1));
-            }
-            vis[c] = bits;
-          }
-        }
+        const uint32_t vis[NCH] = {mv.x, mv.y};
         // fast path: one pass against the settled reference max; both halves must agree
         bool done = false;
         float lsum = 0.0f;
@@ -598,8 +609,10 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) attn_tc_kernel(const __grid_co
         } else if (__all_sync(0xffffffffu, m_ref != -INFINITY)) {  // same in both halves of the pair
           const uint64_t sc2 = pk2(p.scale_log2, p.scale_log2), nm2 = pk2(-m_ref, -m_ref);
           auto agree = [&](bool ok) {
+            if (wg == 0) DBG(18, x);
             if (lane == 0) xch->ok[s][wg][h][sub] = ok;
             ptx::bar_sync(pair_bar, 64);
+            if (wg == 0) DBG(19, x);
             return ok && xch->ok[s][wg][h ^ 1][sub] != 0;
           };
           done = (state == 1) ? row_exp_opt<false>(tS, vis, sc2, nm2, kRescaleThreshold, lsum, agree)
@@ -680,6 +693,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) attn_tc_kernel(const __grid_co
       ptx::tc_fence_before();
       __syncwarp();
       if (lane == 0) ptx::mbar_arrive(&bars->o_empty[wg]);
+      if (p.dbg_items && wg == 0 && h == 0 && sub == 0 && lane == 0) p.dbg_items[int64_t(w) * 6 + 3] = clock64();
     }
   }
   ptx::tc_fence_before();

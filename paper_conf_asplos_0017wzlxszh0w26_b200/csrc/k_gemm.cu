@@ -53,7 +53,9 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
 gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
                const __grid_constant__ CUtensorMap tmC, GemmParams p) {
   extern __shared__ uint8_t smem_raw[];
-  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  // 1 KB-align by offsetting the __shared__ array itself (keeps the shared address space, so
+  // the compiler emits LDS/STS rather than generic loads and stores)
+  uint8_t* smem = smem_raw + ((1024u - (ptx::smem_u32(smem_raw) & 1023u)) & 1023u);
   GemmSmemBars* bars = reinterpret_cast<GemmSmemBars*>(smem + STG_OFF + 4 * 2 * STG_BYTES);
   const uint32_t warp = ptx::warp_id(), lane = ptx::lane_id();
 

@@ -167,8 +167,9 @@ __global__ void stage_kernel(const StageParams p) {
     uint4 o1, o2;
     rope_pair8(src, c0, d, p.rope + int64_t(pos) * (d / 2), kv == 0 && p.rope_enabled, o1, o2);
     char* blockp = page + (int64_t(kv) * p.kv_heads + kvh) * p.head_bytes;
-    *reinterpret_cast<uint4*>(blockp + (c0 / 64) * 2048 + ptx::swz128(j, (c0 % 64) / 8)) = o1;
-    *reinterpret_cast<uint4*>(blockp + (c1 / 64) * 2048 + ptx::swz128(j, (c1 % 64) / 8)) = o2;
+    const uint32_t ch = uint32_t(p.dpad / 64);
+    *reinterpret_cast<uint4*>(blockp + ptx::page_blk_off(j, c0, ch)) = o1;
+    *reinterpret_cast<uint4*>(blockp + ptx::page_blk_off(j, c1, ch)) = o2;
   }
 }
 
@@ -289,9 +290,39 @@ __global__ void kv_pages_kernel(PageIO io, __nv_bfloat16* k, __nv_bfloat16* v,
     const int h = rem / cpr, cc = rem % cpr;
     const int c0 = cc * 8;
     __nv_bfloat16* plain = (kv == 0 ? k : v) + ((int64_t(l) * n_total + t) * io.kv_heads + h) * d + c0;
-    char* pg = page + (int64_t(kv) * io.kv_heads + h) * io.head_bytes + (c0 / 64) * 2048 + ptx::swz128(j, (c0 % 64) / 8);
+    char* pg = page + (int64_t(kv) * io.kv_heads + h) * io.head_bytes +
+               ptx::page_blk_off(j, c0, uint32_t(io.head_bytes / 2048));
     if (TO_PAGES) *reinterpret_cast<uint4*>(pg) = *reinterpret_cast<const uint4*>(plain);
     else *reinterpret_cast<uint4*>(plain) = *reinterpret_cast<const uint4*>(pg);
+  }
+}
+
+__global__ void __launch_bounds__(128) mask_kernel(int32_t* img, int64_t off_mdesc, int64_t off_qinfo,
+                                                  int64_t off_kmeta, int64_t off_rseg, int64_t off_masks, int32_t qt) {
+  const int m = blockIdx.x;
+  const int4 d = reinterpret_cast<const int4*>(img + off_mdesc)[m];  // {b, q-tile, k-tile, 0}
+  const int32_t* qinfo = img + off_qinfo + int64_t(d.x) * 8;
+  const int tok_off = qinfo[0], S = qinfo[1], page_off = qinfo[4];
+  __shared__ int2 keys[kKtile];  // (kseg, kord) of the k-tile's slots
+  const int2* km = reinterpret_cast<const int2*>(img + off_kmeta) + (int64_t(page_off) + int64_t(d.z) * kKtilePages) * kPageTokens;
+  for (int k = threadIdx.x; k < kKtile; k += blockDim.x) keys[k] = km[k];
+  __syncthreads();
+  for (int r = threadIdx.x; r <= qt; r += blockDim.x) {
+    const int t = d.y * qt + r;
+    const bool real = r < qt && t < S;
+    const int32_t rseg = real ? img[off_rseg + tok_off + t] : -1;
+    const int32_t rord = real ? t + 1 : kInvalidOrd - 1;
+    uint32_t w[4];
+#pragma unroll
+    for (int c = 0; c < 4; ++c) {
+      uint32_t bits = 0;
+      for (int i = 0; i < 32; ++i) {
+        const int2 k = keys[32 * c + i];
+        bits |= uint32_t((k.y <= rord) && ((k.x == rseg) || ((k.x | rseg) < 0))) << i;
+      }
+      w[c] = bits;
+    }
+    reinterpret_cast<int4*>(img + off_masks)[int64_t(m) * (qt + 1) + r] = make_int4(int(w[0]), int(w[1]), int(w[2]), int(w[3]));
   }
 }
 
@@ -304,6 +335,13 @@ __global__ void page_copy_kernel(const uint64_t* __restrict__ src, const int32_t
 }
 
 }  // namespace
+
+void launch_masks(int32_t* img, int64_t off_mdesc, int64_t off_qinfo, int64_t off_kmeta, int64_t off_rseg,
+                  int64_t off_masks, int32_t n_masks, int32_t qt, cudaStream_t s) {
+  if (n_masks <= 0) return;
+  mask_kernel<<<n_masks, 128, 0, s>>>(img, off_mdesc, off_qinfo, off_kmeta, off_rseg, off_masks, qt);
+  count_launch();
+}
 
 void launch_embed(const __nv_bfloat16* E, const int32_t* tok, float* h, int M, int H, cudaStream_t s) {
   if (M <= 0) return;

@@ -43,8 +43,17 @@ struct AttnParams {
   __nv_bfloat16* out;       // O [M][q_heads*head_dim]
   float scale_log2;         // log2(e) / sqrt(head_dim)
   long long* dbg;           // optional timeline (clock64) of CTA 0's first work item
+  long long* dbg_items;     // optional per-work-item record [n_work][6] (see k_attn.cu)
+  int64_t off_masks;        // visibility masks of the partial tiles (launch_masks)
 };
 size_t attn_smem_bytes(int dpad);
+
+// Visibility masks of the plan's partial (q-tile, k-tile) pairs (PlanImage::off_mdesc): one block
+// per mask, bit (32 c + i) of row r's word c = key slot 32 c + i of the k-tile visible to token
+// r of the q-tile, by kord <= rord && (kseg == rseg || (kseg | rseg) < 0); row qt (and rows past
+// the request's suffix) = the padding rows' mask (every valid key).
+void launch_masks(int32_t* img, int64_t off_mdesc, int64_t off_qinfo, int64_t off_kmeta, int64_t off_rseg,
+                  int64_t off_masks, int32_t n_masks, int32_t qt, cudaStream_t s);
 void launch_attention(int dpad, const AttnParams& p, int num_sms, cudaStream_t stream);
 
 // --------------------------------------------------------------------- small kernels

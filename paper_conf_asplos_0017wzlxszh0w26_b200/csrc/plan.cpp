@@ -212,7 +212,7 @@ void classify_tiles(QueryPlan& qp, int32_t qt) {
 }  // namespace
 
 void build_plan(const Pool& pool, int32_t group, int32_t kv_heads,
-                const std::vector<PlanRequest>& reqs, Plan& plan, bool build_image) {
+                const std::vector<PlanRequest>& reqs, Plan& plan, bool build_image, int32_t grid) {
   BAT_REQUIRE(group >= 1 && group <= kQtileRows, "group in [1,128]");
   plan.group = group;
   plan.kv_heads = kv_heads;
@@ -314,6 +314,17 @@ void build_plan(const Pool& pool, int32_t group, int32_t kv_heads,
   // work items: (b, kvh, q-tile pair) sharing every K/V tile, with the union of the two
   // q-tiles' live k-tiles and a state per q-tile; longest first (LPT over the SMs)
   struct W { int32_t b, kvh, q0, q1, n; std::vector<int32_t> kt; };
+  std::unordered_map<int64_t, int32_t> mask_id;  // (b, q-tile, k-tile) -> mask
+  std::vector<int32_t> mdesc;
+  auto mask_of = [&](int32_t b, int32_t qi, int32_t j) {
+    const int64_t key = (int64_t(b) << 40) | (int64_t(qi) << 20) | int64_t(j);
+    auto it = mask_id.find(key);
+    if (it != mask_id.end()) return it->second;
+    const int32_t id = static_cast<int32_t>(mdesc.size() / 4);
+    mask_id.emplace(key, id);
+    mdesc.insert(mdesc.end(), {b, qi, j, 0});
+    return id;
+  };
   auto make_work = [&](bool last_only, int64_t& off_work, int32_t& n_work) {
     std::vector<W> ws;
     for (int32_t b = 0; b < B; ++b) {
@@ -333,9 +344,32 @@ void build_plan(const Pool& pool, int32_t group, int32_t kv_heads,
         for (int32_t h = 0; h < kv_heads; ++h) ws.push_back(W{b, h, pr.first, pr.second, int32_t(kt.size()), kt});
       }
     }
-    std::stable_sort(ws.begin(), ws.end(), [](const W& a, const W& c) {
-      return a.n * (a.q1 >= 0 ? 2 : 1) > c.n * (c.q1 >= 0 ? 2 : 1);
-    });
+    // cost of an item in k-tile-pair units: its tiles, with a fixed prologue / epilogue share
+    auto cost = [](const W& a) { return int64_t(a.n) * (a.q1 >= 0 ? 4 : 3) + 8; };
+    std::stable_sort(ws.begin(), ws.end(), [&](const W& a, const W& c) { return cost(a) > cost(c); });
+    if (grid > 0 && static_cast<int32_t>(ws.size()) > grid) {
+      // LPT over the persistent grid: CTA c runs items c, c + grid, c + 2 grid, ... of the list,
+      // so place every CTA's greedily balanced share at those positions (empty items pad)
+      std::vector<std::vector<int32_t>> per(grid);
+      std::vector<std::pair<int64_t, int32_t>> heap;  // (load, cta), min-heap
+      for (int32_t c = 0; c < grid; ++c) heap.push_back({0, c});
+      auto gt = [](const std::pair<int64_t, int32_t>& a, const std::pair<int64_t, int32_t>& b) { return a > b; };
+      std::make_heap(heap.begin(), heap.end(), gt);
+      for (int32_t i = 0; i < static_cast<int32_t>(ws.size()); ++i) {
+        std::pop_heap(heap.begin(), heap.end(), gt);
+        heap.back().first += cost(ws[i]);
+        per[heap.back().second].push_back(i);
+        std::push_heap(heap.begin(), heap.end(), gt);
+      }
+      size_t rounds = 0;
+      for (auto& l : per) rounds = std::max(rounds, l.size());
+      std::vector<W> out;
+      out.reserve(rounds * grid);
+      for (size_t r = 0; r < rounds; ++r)
+        for (int32_t c = 0; c < grid; ++c)
+          out.push_back(r < per[c].size() ? ws[per[c][r]] : W{0, 0, -1, -1, 0, {}});
+      ws.swap(out);
+    }
     n_work = static_cast<int32_t>(ws.size());
     off_work = reserve_at(int64_t(n_work) * 8);
     int64_t total_kt = 0;
@@ -344,15 +378,18 @@ void build_plan(const Pool& pool, int32_t group, int32_t kv_heads,
     // the page ids of every listed k-tile, in list order (8 per tile): the attention loader
     // reads them at addresses known in advance instead of chasing kt list -> page table
     int64_t off_tp = reserve_at(total_kt * kKtilePages);
+    int64_t off_km = reserve_at(total_kt * 2);
     int64_t cur = 0;
     for (int32_t w = 0; w < n_work; ++w) {
       int32_t* e = &v[off_work + int64_t(w) * 8];
       e[0] = ws[w].b; e[1] = ws[w].kvh; e[2] = ws[w].q0; e[3] = ws[w].q1;
       e[4] = static_cast<int32_t>(off_kt + cur); e[5] = ws[w].n;
-      e[6] = static_cast<int32_t>(off_tp + cur * kKtilePages); e[7] = 0;
+      e[6] = static_cast<int32_t>(off_tp + cur * kKtilePages); e[7] = static_cast<int32_t>(off_km + cur * 2);
       const int32_t page_off = plan.q[ws[w].b].page_off;
       for (int32_t x : ws[w].kt) {
         const int32_t j = x & 0xFFFFFF;
+        v[off_km + cur * 2] = ((x >> 24) & 3) == 2 ? mask_of(ws[w].b, ws[w].q0, j) : -1;
+        v[off_km + cur * 2 + 1] = ((x >> 26) & 3) == 2 ? mask_of(ws[w].b, ws[w].q1, j) : -1;
         for (int l = 0; l < kKtilePages; ++l)
           v[off_tp + cur * kKtilePages + l] = v[im.off_pages + page_off + int64_t(j) * kKtilePages + l];
         v[off_kt + cur++] = x;
@@ -361,6 +398,12 @@ void build_plan(const Pool& pool, int32_t group, int32_t kv_heads,
   };
   make_work(false, im.off_work, plan.n_work);
   make_work(true, im.off_work_last, plan.n_work_last);
+  im.n_masks = static_cast<int32_t>(mdesc.size() / 4);
+  im.off_mdesc = reserve_at(std::max<int64_t>(1, int64_t(mdesc.size())));
+  std::copy(mdesc.begin(), mdesc.end(), v.begin() + im.off_mdesc);
+  reserve_at(0);  // align the end of the host part
+  im.off_masks = static_cast<int64_t>(v.size());
+  im.total_ints = im.off_masks + int64_t(im.n_masks) * (plan.qt + 1) * 4;
 }
 
 }  // namespace bat

@@ -45,9 +45,16 @@ struct PlanImage {
   int64_t off_kmeta = 0;                            // [16 * n_pages_padded_total][2]
   int64_t off_qtiles = 0;                           // [n_qtiles_total][4] {b, t0, ntok, 0}
   int64_t off_spages = 0;                           // [n_spages][4] {b, t0, ntok, target}
-  int64_t off_work = 0, off_work_last = 0;          // [W][8] {b, kvh, q0, q1|-1, kt_off, kt_n, tp_off, 0}
+  int64_t off_work = 0, off_work_last = 0;          // [W][8] {b, kvh, q0, q1|-1, kt_off, kt_n, tp_off, km_off}
   int64_t off_ktl = 0;                              // kt list: ktile | state0 << 24 | state1 << 26
   int64_t off_disc = 0;                             // [B] global discriminant row
+  // Visibility masks of the partial (state 2) (q-tile, k-tile) pairs, shared by all KV heads and
+  // layers: mask m = (b, q-tile, k-tile) from off_mdesc [n_masks][4]; per listed tile of a work
+  // item, km_off + 2 x + q holds q-tile q's mask id (-1: not partial).  The masks themselves,
+  // [n_masks][qt + 1 rows][4 x 32 bits] (row qt: the padding rows' mask), are computed on the
+  // device into [off_masks, total_ints) beyond the uploaded host part (launch_masks).
+  int64_t off_mdesc = 0, off_masks = 0, total_ints = 0;
+  int32_t n_masks = 0;
 };
 
 struct Plan {
@@ -60,7 +67,9 @@ struct Plan {
 };
 
 // Build the plan of a batch.  Pool supplies the entry -> pages index.  Throws bat::Error.
+// grid > 0: order the attention work lists for a persistent grid of that many CTAs (LPT
+// balance; empty items pad the rounds).
 void build_plan(const Pool& pool, int32_t group, int32_t kv_heads,
-                const std::vector<PlanRequest>& reqs, Plan& plan, bool build_image);
+                const std::vector<PlanRequest>& reqs, Plan& plan, bool build_image, int32_t grid = 0);
 
 }  // namespace bat

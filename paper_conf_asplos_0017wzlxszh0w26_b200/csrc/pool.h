@@ -35,11 +35,12 @@ struct RemoteEntity {
   std::vector<int32_t> pages;  // page ids in the owner's arena
 };
 
-// Page layout (bf16): page = [layers][2 (K,V)][kv_heads][Dp/64][16 slots][64] with the
-// 128-byte swizzle of the tensor-core operand layout applied inside each 2 KB block
-// ([16][64] bf16): element (slot r, col c) sits at r*128 + (((c/8) ^ (r%8)) * 16) + (c%8)*2.
-// A page's K (or V) rows for one head and one layer are therefore (Dp/64) contiguous 2 KB
-// blocks that a bulk copy drops into shared memory ready for tcgen05.mma.
+// Page layout (bf16): page = [layers][2 (K,V)][kv_heads][block], block = one head's 16 K (or
+// V) rows of one layer = [2 slot groups][Dp/64 chunks][8 slots][64] with the 128-byte swizzle of
+// the tensor-core operand layout inside each 1 KB atom: element (slot r, col c) sits at
+// (r/8)*(Dp/64)*1024 + (c/64)*1024 + (r%8)*128 + ((((c%64)/8) ^ (r%8)) * 16) + (c%8)*2
+// (ptx::page_blk_off).  A block is ONE contiguous bulk copy that lands in shared memory ready
+// for tcgen05.mma (8-row-group stride (Dp/64) KB).
 struct PageGeometry {
   int32_t layers = 0, kv_heads = 0, head_dim = 0, dpad = 0;
   int64_t block_bytes = 2048;  // [16][64] bf16

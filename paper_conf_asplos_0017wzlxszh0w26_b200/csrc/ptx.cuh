@@ -213,6 +213,24 @@ __device__ __forceinline__ void tmem_st32(uint32_t taddr, const uint32_t (&r)[32
       "r"(r[22]), "r"(r[23]), "r"(r[24]), "r"(r[25]), "r"(r[26]), "r"(r[27]), "r"(r[28]),
       "r"(r[29]), "r"(r[30]), "r"(r[31]));
 }
+// 32 lanes x 16 consecutive 32-bit columns
+__device__ __forceinline__ void tmem_ld16(uint32_t taddr, uint32_t* r) {
+  asm volatile(
+      "tcgen05.ld.sync.aligned.32x32b.x16.b32 "
+      "{%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15}, [%16];"
+      : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]),
+        "=r"(r[7]), "=r"(r[8]), "=r"(r[9]), "=r"(r[10]), "=r"(r[11]), "=r"(r[12]),
+        "=r"(r[13]), "=r"(r[14]), "=r"(r[15])
+      : "r"(taddr));
+}
+__device__ __forceinline__ void tmem_st16(uint32_t taddr, const uint32_t* r) {
+  asm volatile(
+      "tcgen05.st.sync.aligned.32x32b.x16.b32 [%0], "
+      "{%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,%16};" ::"r"(taddr),
+      "r"(r[0]), "r"(r[1]), "r"(r[2]), "r"(r[3]), "r"(r[4]), "r"(r[5]), "r"(r[6]), "r"(r[7]),
+      "r"(r[8]), "r"(r[9]), "r"(r[10]), "r"(r[11]), "r"(r[12]), "r"(r[13]), "r"(r[14]),
+      "r"(r[15]));
+}
 __device__ __forceinline__ void tmem_ld_wait() {
   asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
 }
@@ -306,6 +324,14 @@ __device__ __forceinline__ uint32_t pack_bf16x2(float lo, float hi) {
 // 16-byte chunk index of column chunk c (of 8 bf16) in row r under the 128-byte swizzle
 __host__ __device__ __forceinline__ uint32_t swz128(uint32_t row, uint32_t chunk16) {
   return row * 128u + ((chunk16 ^ (row & 7u)) << 4);
+}
+
+// Byte offset of (slot j in [0,16), column c0 (multiple of 8)) inside one page block of a head's
+// K (or V) rows: [2 slot groups][chunks = Dp/64][8 slots][64] bf16, 128-byte swizzled per
+// 1024-byte atom.  A whole block (chunks * 2 KB) is one bulk copy, and 8 consecutive blocks in
+// shared memory form a 128-row tcgen05 operand with 8-row-group stride chunks * 1024 bytes.
+__host__ __device__ __forceinline__ uint32_t page_blk_off(uint32_t j, uint32_t c0, uint32_t chunks) {
+  return (j >> 3) * (chunks * 1024u) + (c0 >> 6) * 1024u + swz128(j & 7u, (c0 & 63u) >> 3);
 }
 
 }  // namespace ptx

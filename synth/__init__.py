@@ -39,6 +39,9 @@ MODEL_CONFIGS: Dict[str, dict] = {
     # a Qwen-like (g=6, d=128) small model used for multi-tile GPU parity at oracle speed
     "small": dict(layers=2, hidden=768, q_heads=6, kv_heads=1, head_dim=128, ffn=1024,
                   vocab=4096, rope_theta=1e6, rms_eps=1e-6, tied=False, mlp_std=0.01),
+    # the same at GQA group 7 (Qwen2-7B's 28 Q / 4 KV heads: 18 tokens x 7 heads per q-tile)
+    "small7": dict(layers=2, hidden=896, q_heads=7, kv_heads=1, head_dim=128, ffn=1024,
+                   vocab=4096, rope_theta=1e6, rms_eps=1e-6, tied=False, mlp_std=0.01),
     # Qwen2-1.5B shape (Table 2 P:396-403 + public config for F / vocab / theta / eps)
     "qwen2-1.5b": dict(layers=28, hidden=1536, q_heads=12, kv_heads=2, head_dim=128,
                        ffn=8960, vocab=151936, rope_theta=1e6, rms_eps=1e-6, tied=True),

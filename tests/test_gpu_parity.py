@@ -118,6 +118,15 @@ def test_small_gqa6_multi_tile(B, order):
     _check(cfg, W, qs, out)
 
 
+@pytest.mark.parametrize("order", ["IP", "UP"])
+def test_small_gqa7_multi_tile(B, order):
+    """GQA group 7 (Qwen2-7B's head ratio): 18 tokens x 7 heads per q-tile, 2 idle rows."""
+    cfg = synth.model_config("small7")
+    qs = [synth.make_query(5, cfg, 7, 150, list(range(300, 330)), (16, 16), 8, order)]
+    cfg, W, out = _run(B, "small7", qs)
+    _check(cfg, W, qs, out)
+
+
 def test_small_mixed_batch(B):
     """configs[2]-style mixed batch: UP, IP and RE requests in one call, shared items."""
     cfg = synth.model_config("small")

@@ -44,9 +44,32 @@ ms = e0.elapsed_time(e1) / 10
 print(f"{order} B={B}: stage+attention {ms:.3f} ms/layer (host sync included); flops {4*128*12*live/1e9:.1f} GF -> {4*128*12*live/ms/1e9:.0f} TFLOP/s lower bound")
 t = np.loadtxt("gpurun_out/attn_timeline.txt").astype(np.int64)
 names = ["ld_top", "ld_kfree", "ld_kiss", "ld_vfree", "ld_viss", "mma_top", "mma_p0", "mma_vful",
-         "mma_kful", "mma_p1", "mma_end", "sm0_s", "sm0_fast", "sm0_p", "sm1_s", "sm1_p"]
+         "mma_kful", "mma_p1", "mma_end", "sm0_s", "sm0_fast", "sm0_p", "sm1_s", "sm1_p",
+         "sm0_meta", "sm0_vis", "sm0_cmp", "sm0_agr"]
 t0 = t[t > 0].min()
 n = int((t[3] > 0).sum())
 print("tile " + " ".join(f"{nm:>10}" for nm in names))
 for x in range(min(n, 24)):
-    print(f"{x:4d} " + " ".join(f"{(t[e, x] - t0) if t[e, x] else -1:10d}" for e in range(16)))
+    print(f"{x:4d} " + " ".join(f"{(t[e, x] - t0) if t[e, x] else -1:10d}" for e in range(20)))
+
+# ---- per-work-item records (BAT_ATTN_ITEMS): where the time per item goes, per CTA
+os.environ["BAT_ATTN_ITEMS"] = "gpurun_out/attn_items.txt"
+bat.bat_debug_attention_layer(pool.handle, model.handle, QA, 1, qkv, out)
+del os.environ["BAT_ATTN_ITEMS"]
+it = np.loadtxt("gpurun_out/attn_items.txt").astype(np.int64)  # t_q t_s0 t_lastpv t_end kt_n cta
+cta = it[:, 5]
+print(f"work items {len(it)}  k-tiles mean {it[:,4].mean():.2f} min {it[:,4].min()} max {it[:,4].max()}")
+tot_span, tot_busy = [], []
+per_tile, gaps, epi, head = [], [], [], []
+for c in np.unique(cta):
+    r = it[cta == c]
+    r = r[np.argsort(r[:, 0])]
+    tot_span.append(r[-1, 3] - r[0, 0])
+    per_tile += list((r[:, 2] - r[:, 1]) / np.maximum(1, r[:, 4] - 1))
+    epi += list(r[:, 3] - r[:, 2])
+    head += list(r[:, 1] - r[:, 0])
+    gaps += list(r[1:, 0] - r[:-1, 2])
+span = np.array(tot_span)
+print(f"CTA span (clk): mean {span.mean():.0f} min {span.min()} max {span.max()}  items/CTA {len(it)/len(span):.2f}")
+print(f"per item: q->S0 issued {np.mean(head):.0f}  S0..lastPV per k-tile {np.mean(per_tile):.0f}  "
+      f"lastPV->epilogue done {np.mean(epi):.0f}  lastPV(i)->q_full(i+1) {np.mean(gaps):.0f}")
