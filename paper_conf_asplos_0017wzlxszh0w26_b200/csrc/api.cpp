@@ -558,10 +558,10 @@ bat_status bat_model_create(const bat_model_cfg* cfg, const void* const* weights
       L.ln2 = w(BAT_WL_LN2);
       L.wgu = w(BAT_WL_WGU);
       L.wd = w(BAT_WL_WD);
-      L.t_qkv = make_tmap(L.wqkv, m.nqkv(), H, H, 256);
-      L.t_o = make_tmap(L.wo, H, nq, nq, 256);
+      L.t_qkv = make_tmap(L.wqkv, m.nqkv(), H, H, 128);
+      L.t_o = make_tmap(L.wo, H, nq, nq, 128);
       L.t_gu = make_tmap(L.wgu, 2 * int64_t(F), H, H, 128);
-      L.t_d = make_tmap(L.wd, H, F, F, 256);
+      L.t_d = make_tmap(L.wd, H, F, F, 128);
       m.layers.push_back(L);
     }
     ensure_rope(m, 32768, 0);
@@ -1092,7 +1092,7 @@ bat_status bat_debug_gemm(int32_t epi, int32_t M, int32_t N, int32_t K, const vo
     int sms = 148;
     CUDA_OK(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, device));
     const CUtensorMap ta = make_tmap(A, M, K, K, 128);
-    const CUtensorMap tb = make_tmap(Bw, b_rows, K, K, epi == EPI_SWIGLU ? 128 : 256);
+    const CUtensorMap tb = make_tmap(Bw, b_rows, K, K, 128);  // B is loaded in 128-row boxes
     const CUtensorMap tc = make_tmap(out, M, N, ldo, 32, epi == EPI_RESID_F32);
     GemmParams gp{M, N, K, out, ldo, static_cast<const __nv_bfloat16*>(bias), up_row0};
     launch_gemm(epi, ta, tb, tc, gp, sms, static_cast<cudaStream_t>(stream));
