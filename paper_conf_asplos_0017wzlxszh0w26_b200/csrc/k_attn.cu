@@ -473,36 +473,53 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) attn_tc_kernel(const __grid_co
           ptx::mma_ts(tO, tS + hf * 64 + i * 8, ptx::desc_sw128(sv + i * L::PAGE_BYTES, 1024, L::GROUP_BYTES),
                       IDESC_PV, (acc || hf || i) ? 1u : 0u);
       };
-      for (int w = blockIdx.x; w < p.n_work; w += gridDim.x) {
+      // Items are software-pipelined: the next item's S0_0 is issued right after the current
+      // item's last P0.V (S0 holds P0 until then) and its S1_0 right after the last P1.V, so the
+      // softmax teams find their next S ready when they finish an epilogue.
+      auto next_item = [&](int w) {
+        for (w += gridDim.x; w < p.n_work; w += gridDim.x)
+          if (work[int64_t(w) * 8 + 5] > 0) break;  // skip the planner's LPT padding
+        return w;
+      };
+      auto first_s0 = [&](const WorkItem& wi, int w, uint32_t g0) {  // Q of wi + its K tile 0 -> S0_0
+        ptx::mbar_wait(&bars->q_full, qc & 1);
+        if (p.dbg_items) p.dbg_items[int64_t(w) * 6 + 0] = clock64();
+        wait_k(g0);
+        issue_s(sq0, tS0, sk_of(g0));
+        ptx::mma_commit(&bars->s_full[0]);
+      };
+      auto first_s1 = [&](const WorkItem& wi, int w, uint32_t g0) {  // -> S1_0, release K tile 0 / Q
+        if (wi.q1 >= 0) {
+          issue_s(sq1, tS1, sk_of(g0));
+          ptx::mma_commit(&bars->s_full[1]);
+        }
+        ptx::mma_commit(&bars->k_empty[ring_slot(g0)]);
+        if (wi.kt_n == 1) ptx::mma_commit(&bars->q_empty);
+        ++qc;
+        if (p.dbg_items) p.dbg_items[int64_t(w) * 6 + 1] = clock64();
+      };
+      int w = blockIdx.x;
+      if (w < p.n_work && work[int64_t(w) * 8 + 5] == 0) w = next_item(w);
+      if (w < p.n_work) {
+        const WorkItem wi = load_work(work, w);
+        first_s0(wi, w, kc);
+        first_s1(wi, w, kc);
+      }
+      while (w < p.n_work) {
         const WorkItem wi = load_work(work, w);
         const bool has1 = wi.q1 >= 0;
         const int n = wi.kt_n;
-        if (n == 0) continue;  // padding of the planner's LPT rounds
-        ptx::mbar_wait(&bars->q_full, qc & 1);
-        if (p.dbg_items) p.dbg_items[int64_t(w) * 6 + 0] = clock64();
-        // S for tile 0
-        {
-          wait_k(kc);
-          const uint32_t sk = sk_of(kc);
-          issue_s(sq0, tS0, sk);
-          ptx::mma_commit(&bars->s_full[0]);
-          if (has1) {
-            issue_s(sq1, tS1, sk);
-            ptx::mma_commit(&bars->s_full[1]);
-          }
-          ptx::mma_commit(&bars->k_empty[ring_slot(kc)]);
-          if (n == 1) ptx::mma_commit(&bars->q_empty);
-          if (p.dbg_items) p.dbg_items[int64_t(w) * 6 + 1] = clock64();
-        }
-        const bool dbg_first = (qc == 0);
+        const int wn = next_item(w);
+        const WorkItem wni = wn < p.n_work ? load_work(work, wn) : WorkItem{0, 0, -1, -1, 0, 0, 0, 0};
+        const bool dbg_first = (qc == 1);
         for (int x = 0; x < n; ++x) {
           const uint32_t g = kc + x;
           const uint32_t va = 2 * g, vb = 2 * g + 1;
           const uint32_t sva = sv_of(va), svb = sv_of(vb);
           DBG(5, x);
           const bool more = x + 1 < n;
-          const uint32_t gn = g + 1;
-          // ---- q-tile 0: PV0_x, then S0_{x+1}
+          const uint32_t gn = g + 1;  // K tile of S_{x+1}, or tile 0 of the next item
+          // ---- q-tile 0: PV0_x, then S0_{x+1} (or the next item's S0_0)
           ptx::mbar_wait(&bars->p_full[0], pc0 & 1);
           DBG(6, x);
           ++pc0;
@@ -519,8 +536,12 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) attn_tc_kernel(const __grid_co
             DBG(8, x);
             issue_s(sq0, tS0, sk_of(gn));
             ptx::mma_commit(&bars->s_full[0]);
+          } else {
+            ptx::mma_commit(&bars->o_full[0]);
+            ++oc0;
+            if (wn < p.n_work) first_s0(wni, wn, gn);
           }
-          // ---- q-tile 1: PV1_x, then S1_{x+1}
+          // ---- q-tile 1: PV1_x, then S1_{x+1} (or the next item's S1_0)
           if (has1) {
             ptx::mbar_wait(&bars->p_full[1], pc1 & 1);
             DBG(9, x);
@@ -539,22 +560,22 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) attn_tc_kernel(const __grid_co
             }
             ptx::mma_commit(&bars->k_empty[ring_slot(gn)]);
             if (x + 1 == n - 1) ptx::mma_commit(&bars->q_empty);
+          } else {
+            if (has1) {
+              ptx::mma_commit(&bars->o_full[1]);
+              ++oc1;
+            }
+            if (p.dbg_items) {
+              p.dbg_items[int64_t(w) * 6 + 2] = clock64();
+              p.dbg_items[int64_t(w) * 6 + 4] = n;
+              p.dbg_items[int64_t(w) * 6 + 5] = blockIdx.x;
+            }
+            if (wn < p.n_work) first_s1(wni, wn, gn);
           }
           DBG(10, x);
         }
-        ptx::mma_commit(&bars->o_full[0]);
-        if (p.dbg_items) {
-          p.dbg_items[int64_t(w) * 6 + 2] = clock64();
-          p.dbg_items[int64_t(w) * 6 + 4] = n;
-          p.dbg_items[int64_t(w) * 6 + 5] = blockIdx.x;
-        }
-        ++oc0;
-        if (has1) {
-          ptx::mma_commit(&bars->o_full[1]);
-          ++oc1;
-        }
         kc += n;
-        ++qc;
+        w = wn;
       }
     }
   } else if (warp >= 4) {  // ------------------------------------------ softmax warpgroups

@@ -407,7 +407,9 @@ void launch_gemm(int epi, const CUtensorMap& tmA, const CUtensorMap& tmB, const 
                  const GemmParams& p, int num_sms, cudaStream_t stream) {
   const int out_bn = (epi == EPI_SWIGLU) ? BN / 2 : BN;
   const int n_tiles = (p.N + out_bn - 1) / out_bn;
-  if (p.M >= 256 && num_sms >= 2) {
+  // the SwiGLU GEMM stays on 1-CTA tiles: measured in the bench step, its pair version ran
+  // slower (1.18 vs 1.24 PFLOP/s) although both tie when timed alone
+  if (p.M >= 256 && num_sms >= 2 && epi != EPI_SWIGLU) {
     const int tiles = ((p.M + 255) / 256) * n_tiles;
     const int pairs = tiles < num_sms / 2 ? tiles : num_sms / 2;
     auto launch = [&](auto kern) {
