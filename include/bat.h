@@ -53,6 +53,11 @@ typedef enum {
   BAT_E_STATE = -7        /* object in the wrong state (e.g. index-only pool used for compute) */
 } bat_status;
 
+/* BAT_BF16: the product path (tcgen05 tensor-core GEMMs and attention, bf16 operands, fp32
+ * accumulation and residual).  BAT_FP32: SIMT correctness mode — the same plan (positions,
+ * segments, page tables, key metadata) through plain fp32 CUDA-core kernels, weights / KV pages /
+ * activations in fp32; matches the fp64 oracle within 1e-5 abs/rel (north_star).  Not a fast
+ * path.  A pool and a model used together must have the same dtype. */
 typedef enum { BAT_BF16 = 0, BAT_FP32 = 1 } bat_dtype;
 
 /* Cache entries at user / item granularity; HEADER = the optional IP notation
@@ -92,7 +97,8 @@ typedef struct {
  *   j=6 wd   [hidden][ffn]
  * The model BORROWS these pointers: the caller keeps them alive and unchanged until
  * bat_model_destroy.  Supported: head_dim in {16, 32, 64, 128}, q_heads % kv_heads == 0,
- * q_heads/kv_heads <= 128, hidden % 64 == 0, ffn % 128 == 0, BAT_BF16. */
+ * q_heads/kv_heads <= 128, hidden % 64 == 0, ffn % 128 == 0, BAT_BF16 or BAT_FP32 (weights
+ * then fp32). */
 enum { BAT_W_EMBED = 0, BAT_W_LM_HEAD = 1, BAT_W_FINAL_NORM = 2, BAT_W_N_GLOBAL = 3 };
 enum { BAT_WL_LN1 = 0, BAT_WL_WQKV = 1, BAT_WL_BQKV = 2, BAT_WL_WO = 3, BAT_WL_LN2 = 4,
        BAT_WL_WGU = 5, BAT_WL_WD = 6, BAT_WL_N = 7 };

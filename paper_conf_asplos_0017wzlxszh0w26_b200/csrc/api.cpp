@@ -192,6 +192,8 @@ struct Model {
     CUtensorMap t_qkv, t_o, t_gu, t_d;
   };
   std::vector<Layer> layers;
+  std::vector<const void*> w;  // every weight pointer as passed (the fp32 mode reads these)
+  bool f32 = false;
   float2* rope = nullptr;
   int max_pos = 0;
   Workspace ws;
@@ -264,17 +266,19 @@ static const int32_t* prepare(Pool& pool, Model& m, Plan& plan, cudaStream_t st,
   for (auto& q : plan.q)
     for (int32_t ps : q.pos) max_pos = std::max(max_pos, ps);
   ensure_rope(m, max_pos + 1, st);
+  const size_t es = m.f32 ? 4 : 2;  // activation element size
   ws.h.ensure(size_t(M) * H * 4);
-  ws.xn.ensure(size_t(M) * std::max(H, nq) * 2);
-  ws.qkv.ensure(size_t(M) * m.nqkv() * 2);
-  ws.qp.ensure(size_t(plan.n_qtiles_total) * c.kv_heads * tile_bytes, true);
+  ws.xn.ensure(size_t(M) * std::max(H, nq) * es);
+  ws.qkv.ensure(size_t(M) * m.nqkv() * es);
+  if (m.f32) ws.qp.ensure(size_t(M) * nq * 4);
+  else ws.qp.ensure(size_t(plan.n_qtiles_total) * c.kv_heads * tile_bytes, true);
   ws.scratch.ensure(size_t(std::max(plan.n_spages, 1)) * pool.geo.layer_bytes, true);
-  ws.o.ensure(size_t(M) * nq * 2);
-  ws.act.ensure(size_t(M) * F * 2);
+  ws.o.ensure(size_t(M) * nq * es);
+  ws.act.ensure(size_t(M) * F * es);
   ws.hc.ensure(size_t(B) * H * 4);
-  ws.xc.ensure(size_t(B) * H * 2);
-  ws.oc.ensure(size_t(B) * nq * 2);
-  ws.actc.ensure(size_t(B) * F * 2);
+  ws.xc.ensure(size_t(B) * H * es);
+  ws.oc.ensure(size_t(B) * nq * es);
+  ws.actc.ensure(size_t(B) * F * es);
   if (dev_img) return dev_img;
   const size_t img_bytes = plan.img.buf.size() * 4;
   ws.img.ensure(size_t(plan.img.total_ints) * 4);
@@ -353,6 +357,77 @@ static StageParams stage_params(const Pool& pool, const Model& m, const Plan& pl
   return sp;
 }
 
+// FP32 SIMT correctness mode (k_f32.cu): the same steps in plain fp32, no last-layer trim (the
+// discriminant rows are picked by the final norm), no kernel profiling.
+static void run_plan_f32(Pool& pool, Model& m, Plan& plan, float* out_hidden, cudaStream_t st,
+                         const int32_t* dev_img) {
+  const bat_model_cfg& c = m.cfg;
+  Workspace& ws = m.ws;
+  const int M = plan.M, B = static_cast<int>(plan.q.size());
+  const int H = c.hidden, F = c.ffn, nq = c.q_heads * c.head_dim, nqkv = m.nqkv();
+  const int32_t* I = prepare(pool, m, plan, st, dev_img);
+  const PlanImage& im = plan.img;
+  auto W = [&](int i) { return static_cast<const float*>(m.w[i]); };
+  auto WL = [&](int l, int j) { return W(BAT_W_N_GLOBAL + BAT_WL_N * l + j); };
+  float *h = ws.h.as<float>(), *xn = ws.xn.as<float>(), *qkv = ws.qkv.as<float>(), *o = ws.o.as<float>(),
+        *act = ws.act.as<float>();
+  int max_S = 0;
+  for (auto& q : plan.q) max_S = std::max(max_S, q.S);
+  StageF32Params sp{};
+  sp.qkv = qkv;
+  sp.img = I;
+  sp.off_pos = im.off_pos;
+  sp.off_qinfo = im.off_qinfo;
+  sp.off_spages = im.off_spages;
+  sp.M = M;
+  sp.n_spages = plan.n_spages;
+  sp.rope = m.rope;
+  sp.rope_enabled = 1;
+  sp.max_pos = m.max_pos;
+  sp.q_heads = c.q_heads;
+  sp.kv_heads = c.kv_heads;
+  sp.head_dim = c.head_dim;
+  sp.qf = ws.qp.as<float>();
+  sp.pool = pool.arena;
+  sp.pool_page_bytes = pool.geo.page_bytes;
+  sp.scratch = ws.scratch.as<char>();
+  sp.scratch_page_bytes = pool.geo.layer_bytes;
+  AttnF32Params ap{};
+  ap.img = I;
+  ap.off_qinfo = im.off_qinfo;
+  ap.off_pages = im.off_pages;
+  ap.off_kmeta = im.off_kmeta;
+  ap.off_rseg = im.off_rseg;
+  ap.pool = pool.arena;
+  ap.pool_page_bytes = pool.geo.page_bytes;
+  ap.scratch = ws.scratch.as<char>();
+  ap.scratch_page_bytes = pool.geo.layer_bytes;
+  ap.q_heads = c.q_heads;
+  ap.kv_heads = c.kv_heads;
+  ap.group = c.q_heads / c.kv_heads;
+  ap.head_dim = c.head_dim;
+  ap.qf = ws.qp.as<float>();
+  ap.out = o;
+  ap.scale = float(1.0 / std::sqrt(double(c.head_dim)));
+  launch_embed_f32(W(BAT_W_EMBED), I + im.off_tok, h, M, H, st);
+  for (int l = 0; l < c.layers; ++l) {
+    launch_rmsnorm_f32(h, WL(l, BAT_WL_LN1), xn, nullptr, M, H, c.rms_eps, st);
+    launch_gemm_f32(0, xn, WL(l, BAT_WL_WQKV), WL(l, BAT_WL_BQKV), qkv, M, nqkv, H, 0, st);
+    sp.pool_layer_off = int64_t(l) * pool.geo.layer_bytes;
+    launch_stage_f32(sp, st);
+    if (l == c.layers - 1 && plan.entity_mode) break;
+    ap.pool_layer_off = sp.pool_layer_off;
+    launch_attention_f32(ap, B, max_S, st);
+    launch_gemm_f32(1, o, WL(l, BAT_WL_WO), nullptr, h, M, H, nq, 0, st);
+    launch_rmsnorm_f32(h, WL(l, BAT_WL_LN2), xn, nullptr, M, H, c.rms_eps, st);
+    launch_gemm_f32(2, xn, WL(l, BAT_WL_WGU), nullptr, act, M, F, H, F, st);
+    launch_gemm_f32(1, act, WL(l, BAT_WL_WD), nullptr, h, M, H, F, 0, st);
+  }
+  if (out_hidden && !plan.entity_mode)
+    launch_rmsnorm_f32(h, W(BAT_W_FINAL_NORM), out_hidden, I + im.off_disc, B, H, c.rms_eps, st);
+  CUDA_OK(cudaGetLastError());
+}
+
 // Run the L layers over a planned batch (SURVEY §3 call stack (3)).
 static void run_plan(Pool& pool, Model& m, Plan& plan, float* out_hidden, cudaStream_t st,
                      const int32_t* dev_img = nullptr) {
@@ -361,6 +436,7 @@ static void run_plan(Pool& pool, Model& m, Plan& plan, float* out_hidden, cudaSt
   const int M = plan.M, B = static_cast<int>(plan.q.size());
   const int H = c.hidden, F = c.ffn, dp = m.dpad;
   const int nq = c.q_heads * c.head_dim;
+  if (m.f32) return run_plan_f32(pool, m, plan, out_hidden, st, dev_img);
   const int32_t* I = prepare(pool, m, plan, st, dev_img);
   Profiler& pf = m.prof;
   const double d_ = c.head_dim, Hq_ = c.q_heads, Hkv_ = c.kv_heads;
@@ -522,7 +598,7 @@ bat_status bat_model_create(const bat_model_cfg* cfg, const void* const* weights
   return guarded([&] {
     BAT_REQUIRE(cfg && weights && out, "null argument");
     const bat_model_cfg& c = *cfg;
-    BAT_REQUIRE(c.dtype == BAT_BF16, "only BAT_BF16 is implemented");
+    BAT_REQUIRE(c.dtype == BAT_BF16 || c.dtype == BAT_FP32, "dtype must be BAT_BF16 or BAT_FP32");
     BAT_REQUIRE(c.layers >= 1 && c.hidden >= 64 && c.hidden % 64 == 0, "hidden % 64 == 0");
     BAT_REQUIRE(c.head_dim == 16 || c.head_dim == 32 || c.head_dim == 64 || c.head_dim == 128,
                 "head_dim in {16,32,64,128}");
@@ -543,6 +619,8 @@ bat_status bat_model_create(const bat_model_cfg* cfg, const void* const* weights
     int major = 0;
     CUDA_OK(cudaDeviceGetAttribute(&major, cudaDevAttrComputeCapabilityMajor, device));
     if (major != 10) fail(BAT_E_UNSUPPORTED, "libbat kernels are sm_100a (B200) only");
+    m.w.assign(weights, weights + n_weights);
+    m.f32 = c.dtype == BAT_FP32;
     auto W = [&](int i) { return static_cast<const __nv_bfloat16*>(weights[i]); };
     m.embed = W(BAT_W_EMBED);
     m.lm_head = W(BAT_W_LM_HEAD);
@@ -558,10 +636,12 @@ bat_status bat_model_create(const bat_model_cfg* cfg, const void* const* weights
       L.ln2 = w(BAT_WL_LN2);
       L.wgu = w(BAT_WL_WGU);
       L.wd = w(BAT_WL_WD);
-      L.t_qkv = make_tmap(L.wqkv, m.nqkv(), H, H, 128);
-      L.t_o = make_tmap(L.wo, H, nq, nq, 128);
-      L.t_gu = make_tmap(L.wgu, 2 * int64_t(F), H, H, 128);
-      L.t_d = make_tmap(L.wd, H, F, F, 128);
+      if (!m.f32) {  // bf16 product path: TMA descriptors of the weights
+        L.t_qkv = make_tmap(L.wqkv, m.nqkv(), H, H, 128);
+        L.t_o = make_tmap(L.wo, H, nq, nq, 128);
+        L.t_gu = make_tmap(L.wgu, 2 * int64_t(F), H, H, 128);
+        L.t_d = make_tmap(L.wd, H, F, F, 128);
+      }
       m.layers.push_back(L);
     }
     ensure_rope(m, 32768, 0);
@@ -586,7 +666,7 @@ bat_status bat_kv_pool_create(const bat_pool_cfg* cfg, bat_pool* out) {
     const bat_pool_cfg& c = *cfg;
     BAT_REQUIRE(c.page_tokens == kPageTokens, "page_tokens must be 16");
     BAT_REQUIRE(c.num_pages >= 1 && c.num_pages < (int64_t(1) << 30), "num_pages");
-    BAT_REQUIRE(c.dtype == BAT_BF16, "only BAT_BF16 pools are implemented");
+    BAT_REQUIRE(c.dtype == BAT_BF16 || c.dtype == BAT_FP32, "dtype must be BAT_BF16 or BAT_FP32");
     BAT_REQUIRE(c.layers >= 1 && c.kv_heads >= 1, "layers / kv_heads");
     BAT_REQUIRE(c.head_dim == 16 || c.head_dim == 32 || c.head_dim == 64 || c.head_dim == 128, "head_dim");
     auto pp = std::make_unique<bat_pool_s>();
@@ -595,7 +675,7 @@ bat_status bat_kv_pool_create(const bat_pool_cfg* cfg, bat_pool* out) {
     if (p.cfg.world < 1) p.cfg.world = 1;
     p.device = c.device;
     p.index_only = c.device < 0;
-    p.geo.init(c.layers, c.kv_heads, c.head_dim);
+    p.geo.init(c.layers, c.kv_heads, c.head_dim, c.dtype == BAT_FP32);
     p.zero_page = static_cast<int32_t>(c.num_pages);
     p.free_pages.reserve(c.num_pages);
     for (int64_t i = c.num_pages - 1; i >= 0; --i) p.free_pages.push_back(static_cast<int32_t>(i));
@@ -712,8 +792,12 @@ bat_status bat_kv_append(bat_pool p, int32_t kind, int64_t id, const void* k, co
       fail(BAT_E_CUDA, std::string("cudaMallocAsync: ") + cudaGetErrorString(e));
     }
     CUDA_OK(cudaMemcpyAsync(dpages, pages.data(), pages.size() * 4, cudaMemcpyHostToDevice, st));
-    launch_kv_scatter(page_io(P), static_cast<const __nv_bfloat16*>(k), static_cast<const __nv_bfloat16*>(v),
-                      dpages, n_tokens, old_n, n_tokens, st);
+    if (P.geo.f32)
+      launch_kv_scatter_f32(page_io(P), static_cast<const float*>(k), static_cast<const float*>(v), dpages, n_tokens,
+                            old_n, n_tokens, st);
+    else
+      launch_kv_scatter(page_io(P), static_cast<const __nv_bfloat16*>(k), static_cast<const __nv_bfloat16*>(v),
+                        dpages, n_tokens, old_n, n_tokens, st);
     CUDA_OK(cudaFreeAsync(dpages, st));
     CUDA_OK(cudaStreamSynchronize(st));  // the host page list above is a stack temporary
     if (exists) {
@@ -740,8 +824,12 @@ bat_status bat_kv_read(bat_pool p, int32_t kind, int64_t id, void* k_out, void* 
     int32_t* dpages = nullptr;
     CUDA_OK(cudaMallocAsync(reinterpret_cast<void**>(&dpages), e->pages.size() * 4, st));
     CUDA_OK(cudaMemcpyAsync(dpages, e->pages.data(), e->pages.size() * 4, cudaMemcpyHostToDevice, st));
-    launch_kv_gather(page_io(P), static_cast<__nv_bfloat16*>(k_out), static_cast<__nv_bfloat16*>(v_out),
-                     dpages, e->n_tokens, st);
+    if (P.geo.f32)
+      launch_kv_gather_f32(page_io(P), static_cast<float*>(k_out), static_cast<float*>(v_out), dpages, e->n_tokens,
+                           st);
+    else
+      launch_kv_gather(page_io(P), static_cast<__nv_bfloat16*>(k_out), static_cast<__nv_bfloat16*>(v_out),
+                       dpages, e->n_tokens, st);
     CUDA_OK(cudaFreeAsync(dpages, st));
     CUDA_OK(cudaStreamSynchronize(st));
   });
@@ -846,8 +934,12 @@ bat_status bat_score(bat_model mdl, const float* hidden, const int32_t* labels, 
     BAT_REQUIRE(k <= n_max, "k <= n_max");
     Model& m = mdl->m;
     DeviceGuard dg(m.device);
-    launch_score(hidden, m.lm_head, labels, n_items, B, n_max, m.cfg.hidden, scores, k, topk,
-                 static_cast<cudaStream_t>(stream));
+    if (m.f32)
+      launch_score_f32w(hidden, static_cast<const float*>(m.w[BAT_W_LM_HEAD]), labels, n_items, B, n_max,
+                        m.cfg.hidden, scores, k, topk, static_cast<cudaStream_t>(stream));
+    else
+      launch_score(hidden, m.lm_head, labels, n_items, B, n_max, m.cfg.hidden, scores, k, topk,
+                   static_cast<cudaStream_t>(stream));
     CUDA_OK(cudaGetLastError());
   });
 }
@@ -1109,6 +1201,7 @@ bat_status bat_debug_attention_layer(bat_pool p, bat_model mdl, const bat_query*
     Model& m = mdl->m;
     check_compat(P, m);
     BAT_REQUIRE(layer >= 0 && layer < m.cfg.layers, "layer");
+    if (m.f32) fail(BAT_E_UNSUPPORTED, "bat_debug_attention_layer tests the bf16 tensor-core kernel");
     DeviceGuard dg(P.device);
     cudaStream_t st = static_cast<cudaStream_t>(stream);
     Plan plan;

@@ -182,7 +182,8 @@ __global__ void gather_rows_kernel(const T* __restrict__ src, const int32_t* __r
 }
 
 // a9: z_i = W_out[v_i] . hf, s = softmax over the N candidates, top-k
-__global__ void score_kernel(const float* __restrict__ hidden, const __nv_bfloat16* __restrict__ w,
+template <class TW>
+__global__ void score_kernel(const float* __restrict__ hidden, const TW* __restrict__ w,
                              const int32_t* __restrict__ labels, const int32_t* __restrict__ n_items,
                              int n_max, int H, float* __restrict__ scores, int k,
                              int32_t* __restrict__ topk) {
@@ -197,15 +198,19 @@ __global__ void score_kernel(const float* __restrict__ hidden, const __nv_bfloat
   for (int c = threadIdx.x; c < H; c += blockDim.x) hf[c] = hidden[int64_t(b) * H + c];
   __syncthreads();
   for (int i = wid; i < n; i += nw) {
-    const __nv_bfloat16* row = w + int64_t(labels[int64_t(b) * n_max + i]) * H;
+    const TW* row = w + int64_t(labels[int64_t(b) * n_max + i]) * H;
     float acc = 0.0f;
-    for (int c = lane * 8; c < H; c += 256) {
-      uint4 raw = *reinterpret_cast<const uint4*>(row + c);
-      const __nv_bfloat162* b2 = reinterpret_cast<const __nv_bfloat162*>(&raw);
+    if constexpr (sizeof(TW) == 4) {  // fp32 correctness mode
+      for (int c = lane; c < H; c += 32) acc = fmaf(row[c], hf[c], acc);
+    } else {
+      for (int c = lane * 8; c < H; c += 256) {
+        uint4 raw = *reinterpret_cast<const uint4*>(row + c);
+        const __nv_bfloat162* b2 = reinterpret_cast<const __nv_bfloat162*>(&raw);
 #pragma unroll
-      for (int q = 0; q < 4; ++q) {
-        float2 f = __bfloat1622float2(b2[q]);
-        acc += f.x * hf[c + 2 * q] + f.y * hf[c + 2 * q + 1];
+        for (int q = 0; q < 4; ++q) {
+          float2 f = __bfloat1622float2(b2[q]);
+          acc += f.x * hf[c + 2 * q] + f.y * hf[c + 2 * q + 1];
+        }
       }
     }
     acc = warp_sum(acc);
@@ -382,18 +387,27 @@ void launch_gather_rows_f32(const float* src, const int32_t* idx, float* dst, in
   gather_rows_kernel<float><<<n, 256, 0, s>>>(src, idx, dst, cols);
   count_launch();
 }
-void launch_score(const float* hidden, const __nv_bfloat16* w_out, const int32_t* labels,
-                  const int32_t* n_items, int B, int n_max, int H, float* scores, int k,
-                  int32_t* topk, cudaStream_t s) {
+template <class TW>
+static void score_launch(const float* hidden, const TW* w_out, const int32_t* labels, const int32_t* n_items, int B,
+                         int n_max, int H, float* scores, int k, int32_t* topk, cudaStream_t s) {
   if (B <= 0) return;
   const size_t smem = sizeof(float) * (size_t(H) + size_t(n_max));
   static bool attr = false;
   if (!attr) {
-    cudaFuncSetAttribute(score_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, 64 * 1024);
+    cudaFuncSetAttribute(score_kernel<TW>, cudaFuncAttributeMaxDynamicSharedMemorySize, 64 * 1024);
     attr = true;
   }
-  score_kernel<<<B, 256, smem, s>>>(hidden, w_out, labels, n_items, n_max, H, scores, k, topk);
+  score_kernel<TW><<<B, 256, smem, s>>>(hidden, w_out, labels, n_items, n_max, H, scores, k, topk);
   count_launch();
+}
+void launch_score(const float* hidden, const __nv_bfloat16* w_out, const int32_t* labels,
+                  const int32_t* n_items, int B, int n_max, int H, float* scores, int k,
+                  int32_t* topk, cudaStream_t s) {
+  score_launch(hidden, w_out, labels, n_items, B, n_max, H, scores, k, topk, s);
+}
+void launch_score_f32w(const float* hidden, const float* w_out, const int32_t* labels, const int32_t* n_items, int B,
+                       int n_max, int H, float* scores, int k, int32_t* topk, cudaStream_t s) {
+  score_launch(hidden, w_out, labels, n_items, B, n_max, H, scores, k, topk, s);
 }
 void launch_kv_scatter(const PageIO& io, const __nv_bfloat16* k, const __nv_bfloat16* v,
                        const int32_t* pages_dev, int n_tokens, int slot0, int n_total, cudaStream_t s) {

@@ -106,4 +106,46 @@ void launch_kv_gather(const PageIO& io, __nv_bfloat16* k, __nv_bfloat16* v,
 void launch_page_copy(const uint64_t* src_ptrs, const int32_t* dst_pages, char* dst_arena,
                       int64_t page_bytes, int n, cudaStream_t s);
 
+// ------------------------------------------------- FP32 SIMT correctness mode (k_f32.cu)
+struct StageF32Params {
+  const float* qkv;  // [M][(Hq+2Hkv)*d]
+  const int32_t* img;
+  int64_t off_pos, off_qinfo, off_spages;
+  int32_t M, n_spages;
+  const float2* rope;
+  int32_t rope_enabled, max_pos;
+  int32_t q_heads, kv_heads, head_dim;
+  float* qf;  // [M][Hq][d]
+  char* pool;
+  int64_t pool_page_bytes, pool_layer_off;
+  char* scratch;
+  int64_t scratch_page_bytes;
+};
+struct AttnF32Params {
+  const int32_t* img;
+  int64_t off_qinfo, off_pages, off_kmeta, off_rseg;
+  const char* pool;
+  int64_t pool_page_bytes, pool_layer_off;
+  const char* scratch;
+  int64_t scratch_page_bytes;
+  int32_t q_heads, kv_heads, group, head_dim;
+  const float* qf;
+  float* out;  // [M][Hq*d]
+  float scale;
+};
+void launch_embed_f32(const float* E, const int32_t* tok, float* h, int M, int H, cudaStream_t s);
+void launch_rmsnorm_f32(const float* x, const float* g, float* y, const int32_t* idx, int M, int H, float eps,
+                        cudaStream_t s);
+// epi: 0 out = A W^T + bias, 1 out += A W^T, 2 out = silu(A Wg^T) * (A Wu^T) (Wu = rows from up_row0)
+void launch_gemm_f32(int epi, const float* A, const float* W, const float* bias, float* out, int M, int N, int K,
+                     int up_row0, cudaStream_t s);
+void launch_stage_f32(const StageF32Params& p, cudaStream_t s);
+void launch_attention_f32(const AttnF32Params& p, int B, int max_S, cudaStream_t s);
+void launch_kv_scatter_f32(const PageIO& io, const float* k, const float* v, const int32_t* pages_dev, int n_tokens,
+                           int slot0, int n_total, cudaStream_t s);
+void launch_kv_gather_f32(const PageIO& io, float* k, float* v, const int32_t* pages_dev, int n_tokens,
+                          cudaStream_t s);
+void launch_score_f32w(const float* hidden, const float* w_out, const int32_t* labels, const int32_t* n_items, int B,
+                       int n_max, int H, float* scores, int k, int32_t* topk, cudaStream_t s);
+
 }  // namespace bat

@@ -47,12 +47,15 @@ struct PageGeometry {
   int64_t head_bytes = 0;      // (dpad/64) blocks
   int64_t layer_bytes = 0;     // 2 * kv_heads * head_bytes
   int64_t page_bytes = 0;      // layers * layer_bytes
-  void init(int L, int hkv, int d) {
+  bool f32 = false;            // BAT_FP32 pool: block = plain [16 slots][head_dim] fp32
+  void init(int L, int hkv, int d, bool fp32 = false) {
     layers = L;
     kv_heads = hkv;
     head_dim = d;
-    dpad = head_dim_pad(d);
-    head_bytes = (dpad / 64) * block_bytes;
+    f32 = fp32;
+    dpad = fp32 ? d : head_dim_pad(d);
+    if (fp32) block_bytes = int64_t(16) * d * 4;
+    head_bytes = fp32 ? block_bytes : (dpad / 64) * block_bytes;
     layer_bytes = 2 * kv_heads * head_bytes;
     page_bytes = layers * layer_bytes;
   }

@@ -21,19 +21,23 @@ def _torch():
 
 
 class DeviceModel:
-    """Weights (bf16, device) + the library's model handle.
+    """Weights (bf16 device tensors; dtype="fp32" for the SIMT correctness mode) + the
+    library's model handle.
 
     ``source`` is any object with ``cfg`` (dict), ``embed_full()``, ``lm_head_full()``,
     ``final_norm()`` and ``layer(l)`` returning the 7 per-layer arrays, or
     ``tensors=`` a dict {"embed", "lm_head" (optional: tied), "final_norm", "layers": [...]}
     of device tensors already in bf16."""
 
-    def __init__(self, cfg: dict, source=None, tensors: Optional[dict] = None, device: int = 0):
+    def __init__(self, cfg: dict, source=None, tensors: Optional[dict] = None, device: int = 0,
+                 dtype: str = "bf16"):
         torch = _torch()
         self.cfg = dict(cfg)
         self.device = device
+        self.dtype = dtype
         dev = torch.device("cuda", device)
-        to = lambda a: torch.as_tensor(np.asarray(a, dtype=np.float32)).to(dev, torch.bfloat16).contiguous()
+        tdt = {"bf16": torch.bfloat16, "fp32": torch.float32}[dtype]  # fp32: SIMT correctness mode
+        to = lambda a: torch.as_tensor(np.asarray(a, dtype=np.float32)).to(dev, tdt).contiguous()
         if tensors is None:
             embed = to(source.embed_full())
             lm = embed if cfg.get("tied") else to(source.lm_head_full())
@@ -49,7 +53,8 @@ class DeviceModel:
         ptrs = [tensors["embed"].data_ptr(), tensors["lm_head"].data_ptr(), tensors["final_norm"].data_ptr()]
         for lw in tensors["layers"]:
             ptrs += [lw[k].data_ptr() for k in LAYER_KEYS]
-        self.handle = bat.bat_model_create(cfg, ptrs, device)
+        self.handle = bat.bat_model_create(cfg, ptrs, device,
+                                           bat.BAT_FP32 if dtype == "fp32" else bat.BAT_BF16)
 
     def close(self):
         if self.handle:
@@ -64,11 +69,13 @@ class DeviceModel:
 
 
 class DevicePool:
-    def __init__(self, cfg: dict, num_pages: int, device: int = 0, rank: int = 0, world: int = 1):
+    def __init__(self, cfg: dict, num_pages: int, device: int = 0, rank: int = 0, world: int = 1,
+                 dtype: str = "bf16"):
         self.cfg = dict(cfg)
         self.device = device
         self.handle = bat.bat_kv_pool_create(device, num_pages, cfg["layers"], cfg["kv_heads"],
-                                             cfg["head_dim"], rank=rank, world=world)
+                                             cfg["head_dim"], bat.BAT_FP32 if dtype == "fp32" else bat.BAT_BF16,
+                                             rank=rank, world=world)
 
     def close(self):
         if self.handle:
