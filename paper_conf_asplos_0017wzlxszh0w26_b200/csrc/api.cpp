@@ -83,6 +83,21 @@ static CUtensorMap make_tmap(const void* ptr, int64_t rows, int64_t cols, int64_
   return m;
 }
 
+// a byte buffer viewed as rows of 128 bytes (64 bf16), box = box_rows rows, no swizzle: TMA
+// copies page blocks that are already in the tensor-core operand layout verbatim
+static CUtensorMap make_tmap_rows(const void* ptr, int64_t bytes, int box_rows) {
+  CUtensorMap m;
+  cuuint64_t dims[2] = {64, cuuint64_t(bytes / 128)};
+  cuuint64_t strides[1] = {128};
+  cuuint32_t box[2] = {64, cuuint32_t(box_rows)};
+  cuuint32_t estr[2] = {1, 1};
+  CUresult r = encode_fn()(&m, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 2, const_cast<void*>(ptr), dims, strides, box, estr,
+                           CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE,
+                           CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  if (r != CUDA_SUCCESS) fail(BAT_E_CUDA, "cuTensorMapEncodeTiled (rows) failed (" + std::to_string(int(r)) + ")");
+  return m;
+}
+
 // ------------------------------------------------------------------------ device buffer
 struct DevBuf {
   void* p = nullptr;
@@ -326,6 +341,25 @@ static AttnParams attn_params(const Pool& pool, const Model& m, const Plan& plan
   return ap;
 }
 
+// a5 launch: the CTA-pair kernel (head_dim 128) or the 1-CTA kernel
+static void run_attention(const Pool& pool, const Model& m, const Plan& plan, const AttnParams& ap, cudaStream_t st) {
+  if (!attn_pair_supported(m.dpad)) {
+    launch_attention(m.dpad, ap, m.num_sms, st);
+    return;
+  }
+  AttnPairParams pp{};
+  const int64_t arena_bytes = int64_t(pool.cfg.num_pages + 1) * pool.geo.page_bytes;
+  pp.tm_pool_k = make_tmap_rows(pool.arena, arena_bytes, 32);
+  pp.tm_pool_v = pp.tm_pool_k;  // whole 4 KB page blocks for V too
+  const int64_t scr_bytes = int64_t(std::max(plan.n_spages, 1)) * pool.geo.layer_bytes;
+  pp.tm_scr_k = make_tmap_rows(m.ws.scratch.p, scr_bytes, 32);
+  pp.tm_scr_v = pp.tm_scr_k;
+  pp.tm_q = make_tmap_rows(m.ws.qp.p, int64_t(plan.n_qtiles_total) * plan.kv_heads * 32768, 256);
+  pp.a = ap;
+  pp.zero_row = int64_t(pool.zero_page) * pool.geo.page_bytes / 128;
+  launch_attention_pair(pp, m.num_sms, st);
+}
+
 static StageParams stage_params(const Pool& pool, const Model& m, const Plan& plan, const int32_t* I) {
   const bat_model_cfg& c = m.cfg;
   const PlanImage& im = plan.img;
@@ -434,7 +468,7 @@ static void run_plan(Pool& pool, Model& m, Plan& plan, float* out_hidden, cudaSt
   const bat_model_cfg& c = m.cfg;
   Workspace& ws = m.ws;
   const int M = plan.M, B = static_cast<int>(plan.q.size());
-  const int H = c.hidden, F = c.ffn, dp = m.dpad;
+  const int H = c.hidden, F = c.ffn;
   const int nq = c.q_heads * c.head_dim;
   if (m.f32) return run_plan_f32(pool, m, plan, out_hidden, st, dev_img);
   const int32_t* I = prepare(pool, m, plan, st, dev_img);
@@ -502,7 +536,7 @@ static void run_plan(Pool& pool, Model& m, Plan& plan, float* out_hidden, cudaSt
       }
       ap.dbg_items = dbi;
       pf.begin(st);
-      launch_attention(dp, ap, m.num_sms, st);
+      run_attention(pool, m, plan, ap, st);
       pf.end(st, BAT_K_ATTN, attn_fl, attn_by);
       ap.dbg_items = nullptr;
       if (dbi) {
@@ -541,7 +575,7 @@ static void run_plan(Pool& pool, Model& m, Plan& plan, float* out_hidden, cudaSt
       ap.off_work = im.off_work_last;
       ap.n_work = plan.n_work_last;
       pf.begin(st);
-      launch_attention(dp, ap, m.num_sms, st);
+      run_attention(pool, m, plan, ap, st);
       pf.end(st, BAT_K_ATTN, attn_fl_last, attn_by);
       const int32_t* disc = I + im.off_disc;
       pf.begin(st);
@@ -876,7 +910,7 @@ bat_status bat_kv_prefill_entities(bat_pool p, bat_model mdl, int32_t kind, int3
         reqs[e].ent_pages = &pages[e];
       }
       Plan plan;
-      build_plan(P, m.cfg.q_heads / m.cfg.kv_heads, m.cfg.kv_heads, reqs, plan, true, m.num_sms);
+      build_plan(P, m.cfg.q_heads / m.cfg.kv_heads, m.cfg.kv_heads, reqs, plan, true, attn_grid_slots(m.dpad, m.num_sms));
       run_plan(P, m, plan, nullptr, static_cast<cudaStream_t>(stream));
       CUDA_OK(cudaStreamSynchronize(static_cast<cudaStream_t>(stream)));
     } catch (...) {
@@ -920,7 +954,7 @@ bat_status bat_bipartite_prefill(bat_pool p, bat_model mdl, const bat_query* que
     for (int b = 0; b < B; ++b) validate_tokens(queries[b], m.cfg.vocab);
     DeviceGuard dg(P.device);
     Plan plan;
-    build_plan(P, m.cfg.q_heads / m.cfg.kv_heads, m.cfg.kv_heads, wrap(queries, B), plan, true, m.num_sms);
+    build_plan(P, m.cfg.q_heads / m.cfg.kv_heads, m.cfg.kv_heads, wrap(queries, B), plan, true, attn_grid_slots(m.dpad, m.num_sms));
     run_plan(P, m, plan, out_hidden, static_cast<cudaStream_t>(stream));
   });
 }
@@ -1205,7 +1239,7 @@ bat_status bat_debug_attention_layer(bat_pool p, bat_model mdl, const bat_query*
     DeviceGuard dg(P.device);
     cudaStream_t st = static_cast<cudaStream_t>(stream);
     Plan plan;
-    build_plan(P, m.cfg.q_heads / m.cfg.kv_heads, m.cfg.kv_heads, wrap(queries, B), plan, true, m.num_sms);
+    build_plan(P, m.cfg.q_heads / m.cfg.kv_heads, m.cfg.kv_heads, wrap(queries, B), plan, true, attn_grid_slots(m.dpad, m.num_sms));
     const int32_t* I = prepare(P, m, plan, st);
     StageParams sp = stage_params(P, m, plan, I);
     sp.qkv = static_cast<const __nv_bfloat16*>(qkv);
@@ -1229,7 +1263,7 @@ bat_status bat_debug_attention_layer(bat_pool p, bat_model mdl, const bat_query*
       CUDA_OK(cudaMemsetAsync(dbi, 0, size_t(ap.n_work) * 6 * sizeof(long long), st));
       ap.dbg_items = dbi;
     }
-    launch_attention(m.dpad, ap, m.num_sms, st);
+    run_attention(P, m, plan, ap, st);
     CUDA_OK(cudaGetLastError());
     CUDA_OK(cudaStreamSynchronize(st));
     if (dbg) {
@@ -1273,7 +1307,7 @@ bat_status bat_plan_build(bat_pool p, bat_model mdl, const bat_query* queries, i
     for (int b = 0; b < B; ++b) validate_tokens(queries[b], m.cfg.vocab);
     DeviceGuard dg(P.device);
     auto pl = std::make_unique<bat_plan_s>();
-    build_plan(P, m.cfg.q_heads / m.cfg.kv_heads, m.cfg.kv_heads, wrap(queries, B), pl->plan, true, m.num_sms);
+    build_plan(P, m.cfg.q_heads / m.cfg.kv_heads, m.cfg.kv_heads, wrap(queries, B), pl->plan, true, attn_grid_slots(m.dpad, m.num_sms));
     const size_t bytes = pl->plan.img.buf.size() * 4;
     CUDA_OK(cudaMalloc(&pl->dev_img, size_t(pl->plan.img.total_ints) * 4));
     CUDA_OK(cudaMemcpyAsync(pl->dev_img, pl->plan.img.buf.data(), bytes, cudaMemcpyHostToDevice,

@@ -48,6 +48,24 @@ struct AttnParams {
 };
 size_t attn_smem_bytes(int dpad);
 
+// CTA-pair bipartite attention (k_attn_pair.cu, head_dim 128): the K / V page blocks and the
+// q-tiles are fetched by 2-D TMA through byte-row views (128-byte rows, no swizzle: the pages
+// are already in the operand layout) so the peer CTA's loads signal the pair leader's barriers.
+struct AttnPairParams {
+  CUtensorMap tm_pool_k;   // pool arena, box 32 rows (one 4 KB page block)
+  CUtensorMap tm_pool_v;   // pool arena, box 8 rows (one 1 KB 8-key x 64-column atom)
+  CUtensorMap tm_scr_k;    // suffix scratch pages, box 32 rows
+  CUtensorMap tm_scr_v;    // suffix scratch pages, box 8 rows
+  CUtensorMap tm_q;        // q-tiles, box 256 rows (one 32 KB tile)
+  AttnParams a;
+  int64_t zero_row;        // first 128-byte row of the all-zero page in the pool view
+  int32_t total_tiles_hint;
+};
+bool attn_pair_supported(int dpad);
+// number of persistent work slots the planner should balance over (CTA pairs or CTAs)
+int attn_grid_slots(int dpad, int num_sms);
+void launch_attention_pair(const AttnPairParams& p, int num_sms, cudaStream_t stream);
+
 // Visibility masks of the plan's partial (q-tile, k-tile) pairs (PlanImage::off_mdesc): one block
 // per mask, bit (32 c + i) of row r's word c = key slot 32 c + i of the k-tile visible to token
 // r of the q-tile, by kord <= rord && (kseg == rseg || (kseg | rseg) < 0); row qt (and rows past
