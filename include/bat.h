@@ -260,6 +260,49 @@ BAT_API bat_status bat_hrcs_rmax(double B, double t, double alpha, int32_t c, do
 BAT_API bat_status bat_hrcs_place(const double* freq, int64_t n_items, double r_max, int32_t world,
                           int32_t* owner_out, double* r_out);
 
+/* ------------------------------------------------------------------------------------------
+ * Prompt scheduler + cache meta service for user prefixes (P:288-294
+ * scheduler / meta service, P:366-381 prefix selection, P:405 hotness upkeep, P:441 hit rate).
+ * Host-only bookkeeping: it decides each request's prefix side and the user-cache actions; the
+ * caller applies them to a pool (bat_kv_evict the evicted users, bat_kv_prefill_entities the
+ * admitted user, then bat_bipartite_prefill with the decided order).
+ *   policy BAT_SCHED_HOTNESS: UP iff tau_u >= tau_i and (u is cached, or its pages fit
+ *     in free space, or evicting cached users of lower sliding-window frequency f_p < f_u in
+ *     ascending (f_p, last access, id) order frees enough pages); else IP.
+ *   BAT_SCHED_GREEDY: UP iff tau_u >= tau_i, admitting with LRU replacement.
+ *   BAT_SCHED_UP / BAT_SCHED_IP / BAT_SCHED_RE: the fixed baselines of P:441 (UP admits with LRU).
+ * f_u(t) = the user's requests in (t - window, t], this one included.  A user entry
+ * occupies ceil(tau_u / 16) pages.  Requests must arrive with non-decreasing t
+ * (BAT_E_INVAL otherwise).  Readings: DESIGN.md R15-R19.
+ * ---------------------------------------------------------------------------------------- */
+typedef enum { BAT_SCHED_HOTNESS = 0, BAT_SCHED_GREEDY = 1, BAT_SCHED_UP = 2, BAT_SCHED_IP = 3,
+               BAT_SCHED_RE = 4 } bat_sched_policy;
+typedef struct {
+  int32_t policy;         /* bat_sched_policy */
+  int64_t capacity_pages; /* pages of the pool set aside for user prefixes */
+  double window;          /* sliding-window length W (same unit as the request times) */
+} bat_sched_cfg;
+typedef struct {
+  int32_t order;    /* BAT_ORDER_UP, BAT_ORDER_IP, or -1 (RE: full recompute, no cache) */
+  int32_t user_hit; /* UP served from the cached user prefix */
+  int32_t admit;    /* UP miss: the user's prefix must be computed and cached (after evictions) */
+  int32_t n_evict;  /* users to evict first, written to evict_ids */
+  int32_t freq;     /* f_u(t) of the request's user */
+} bat_sched_decision;
+typedef struct bat_sched_s* bat_sched;
+BAT_API bat_status bat_sched_create(const bat_sched_cfg* cfg, bat_sched* out);
+BAT_API bat_status bat_sched_destroy(bat_sched s);
+/* Decide one request (user_id, tau_u user tokens, tau_i item tokens) arriving at time t and
+ * update the user-cache index.  evict_ids: host array of evict_cap entries (BAT_E_INVAL if the
+ * evictions do not fit; the state is then unchanged). */
+BAT_API bat_status bat_sched_decide(bat_sched s, double t, int64_t user_id, int32_t tau_u, int32_t tau_i,
+                                    bat_sched_decision* out, int64_t* evict_ids, int32_t evict_cap);
+/* Totals so far: [0] prompt tokens, [1] reused prefix tokens (P:441 hit rate = [1]/[0]),
+ * [2] UP hits, [3] UP requests, [4] IP requests, [5] cached users, [6] used pages. */
+BAT_API bat_status bat_sched_stats(bat_sched s, int64_t out[7]);
+/* Whether user_id's prefix is cached. */
+BAT_API int32_t bat_sched_is_cached(bat_sched s, int64_t user_id);
+
 /* CUDA-IPC export of the pool arena (64-byte handle) and import of a peer's arena. */
 BAT_API bat_status bat_pool_ipc_handle(bat_pool p, void* handle_out64);
 BAT_API bat_status bat_pool_attach_peer(bat_pool p, int32_t peer_rank, const void* handle64);

@@ -63,6 +63,20 @@ class bat_query(Structure):
 _lib = None
 
 
+class bat_sched_cfg(Structure):
+    _fields_ = [("policy", c_int32), ("capacity_pages", c_int64), ("window", c_double)]
+
+
+class bat_sched_decision(Structure):
+    _fields_ = [("order", c_int32), ("user_hit", c_int32), ("admit", c_int32), ("n_evict", c_int32),
+                ("freq", c_int32)]
+
+
+BAT_SCHED_HOTNESS, BAT_SCHED_GREEDY, BAT_SCHED_UP, BAT_SCHED_IP, BAT_SCHED_RE = range(5)
+SCHED_POLICY = {"hotness": BAT_SCHED_HOTNESS, "greedy": BAT_SCHED_GREEDY, "up": BAT_SCHED_UP,
+                "ip": BAT_SCHED_IP, "re": BAT_SCHED_RE}
+
+
 def lib() -> ctypes.CDLL:
     """Load libbat.so (fails loudly when the extension has not been built)."""
     global _lib
@@ -114,6 +128,12 @@ def lib() -> ctypes.CDLL:
                                c_int32, c_void_p, c_int32, c_int32, c_void_p]),
         "bat_debug_attention_layer": (S, [c_void_p, c_void_p, POINTER(bat_query), c_int32, c_int32, c_void_p,
                                           c_void_p, c_int32, c_void_p]),
+        "bat_sched_create": (S, [POINTER(bat_sched_cfg), POINTER(c_void_p)]),
+        "bat_sched_destroy": (S, [c_void_p]),
+        "bat_sched_decide": (S, [c_void_p, c_double, c_int64, c_int32, c_int32, POINTER(bat_sched_decision),
+                                 POINTER(c_int64), c_int32]),
+        "bat_sched_stats": (S, [c_void_p, POINTER(c_int64)]),
+        "bat_sched_is_cached": (c_int32, [c_void_p, c_int64]),
     }
     for name, (res, args) in sig.items():
         f = getattr(L, name)
@@ -131,7 +151,8 @@ EXPORTED = ("bat_last_error", "bat_version", "bat_kernel_launch_count", "bat_mod
             "bat_hrcs_rmax", "bat_hrcs_place", "bat_pool_ipc_handle", "bat_pool_attach_peer",
             "bat_kv_register_remote", "bat_kv_lookup_remote", "bat_kv_fetch", "bat_debug_gemm", "bat_debug_attention_layer",
             "bat_plan_build", "bat_prefill_plan", "bat_profile_enable", "bat_profile_read",
-            "bat_profile_reset", "bat_debug_attach_peer_pool")
+            "bat_profile_reset", "bat_debug_attach_peer_pool", "bat_sched_create", "bat_sched_destroy",
+            "bat_sched_decide", "bat_sched_stats", "bat_sched_is_cached")
 
 
 def _check(status: int) -> None:
@@ -425,3 +446,34 @@ def bat_debug_attention_layer(pool: int, model: int, queries: QueryArray, layer:
 
 def bat_debug_attach_peer_pool(pool: int, peer: int, other: int) -> None:
     _check(lib().bat_debug_attach_peer_pool(pool, peer, other))
+
+
+# ------------------------------------------------------------------ prompt scheduler (NEXT-2)
+def bat_sched_create(policy: str, capacity_pages: int, window: float) -> int:
+    h = c_void_p()
+    _check(lib().bat_sched_create(byref(bat_sched_cfg(SCHED_POLICY[policy], capacity_pages, window)), byref(h)))
+    return h.value
+
+
+def bat_sched_destroy(s: int) -> None:
+    _check(lib().bat_sched_destroy(s))
+
+
+def bat_sched_decide(s: int, t: float, user_id: int, tau_u: int, tau_i: int, evict_cap: int = 4096):
+    """-> (order: "UP" | "IP" | "RE", user_hit, admit, evicted user ids, f_u)"""
+    d = bat_sched_decision()
+    ev = (c_int64 * max(1, evict_cap))()
+    _check(lib().bat_sched_decide(s, t, user_id, tau_u, tau_i, byref(d), ev, evict_cap))
+    order = {BAT_ORDER_UP: "UP", BAT_ORDER_IP: "IP"}.get(d.order, "RE")
+    return order, bool(d.user_hit), bool(d.admit), [int(ev[i]) for i in range(d.n_evict)], d.freq
+
+
+def bat_sched_stats(s: int) -> dict:
+    out = (c_int64 * 7)()
+    _check(lib().bat_sched_stats(s, out))
+    return dict(tokens=out[0], reused=out[1], hits=out[2], up=out[3], ip=out[4], cached_users=out[5],
+                used_pages=out[6])
+
+
+def bat_sched_is_cached(s: int, user_id: int) -> bool:
+    return bool(lib().bat_sched_is_cached(s, user_id))

@@ -147,3 +147,78 @@ def prefill_missing_entities(pool: DevicePool, model: DeviceModel, queries, stre
                                                 [t for _, t in chunk], 0, stream=stream)
                 n += len(chunk)
     return n
+
+
+class TraceServer:
+    """The serving loop of P:288-294 on one GPU: the prompt scheduler
+    (bat_sched_*: P:366 / P:377 prefix selection over the user-prefix cache index) decides each
+    request's prefix side in arrival order; its cache actions are applied to the pool (evicted
+    users -> bat_kv_evict, admitted users -> their prefix KV computed by the prefix-miss path);
+    batches run through bat_bipartite_prefill + bat_score.  Bookkeeping only — every step of the
+    method runs in libbat."""
+
+    def __init__(self, pool: DevicePool, model: DeviceModel, policy: str, user_capacity_pages: int,
+                 window: float, seed: int = 0, n_instr: int = 8, item_len=(16, 16)):
+        self.pool, self.model, self.cfg = pool, model, model.cfg
+        self.sched = bat.bat_sched_create(policy, user_capacity_pages, window)
+        self.seed, self.n_instr, self.item_len = seed, n_instr, item_len
+        self.decisions = []
+
+    def close(self):
+        if self.sched:
+            bat.bat_sched_destroy(self.sched)
+            self.sched = None
+
+    def _run(self, pending, k, out):
+        if not pending:
+            return
+        torch = _torch()
+        prefill_missing_entities(self.pool, self.model, pending)
+        dev = torch.device("cuda", self.model.device)
+        Bn = len(pending)
+        n_max = max(q.n_items for q in pending)
+        hidden = torch.empty(Bn, self.cfg["hidden"], device=dev)
+        bat.bat_bipartite_prefill(self.pool.handle, self.model.handle, bat.QueryArray(pending), hidden)
+        labels = np.zeros((Bn, n_max), np.int32)
+        for b, q in enumerate(pending):
+            labels[b, : q.n_items] = q.labels
+        scores = torch.empty(Bn, n_max, device=dev)
+        topk = torch.empty(Bn, max(k, 1), dtype=torch.int32, device=dev)
+        bat.bat_score(self.model.handle, hidden, torch.tensor(labels, device=dev),
+                      torch.tensor([q.n_items for q in pending], dtype=torch.int32, device=dev), Bn, n_max,
+                      scores, k, topk if k else None)
+        out.append((list(pending), hidden, scores))
+        pending.clear()
+
+    def serve(self, requests, batch: int = 16, k: int = 0):
+        """requests: iterable of (time, user_id, n_user_tokens, item_ids).  Returns a list of
+        (queries, hidden [B][H], scores [B][n_max]) per executed batch, in order."""
+        import synth
+        out, pending, pinned = [], [], set()
+        for (t, uid, n_user, item_ids) in requests:
+            tau_i = sum(synth.item_length(int(i), *self.item_len, self.seed) for i in item_ids)
+            order, hit, admit, evicted, f = bat.bat_sched_decide(self.sched, t, uid, n_user, tau_i)
+            if any(e in pinned for e in evicted):  # a queued UP request still needs that user
+                self._run(pending, k, out)
+                pinned.clear()
+            for e in evicted:
+                try:
+                    bat.bat_kv_evict(self.pool.handle, bat.BAT_ENT_USER, e)
+                except bat.BatError:
+                    pass  # admitted but never materialised (its batch had not run)
+            q = synth.make_query(self.seed, self.cfg, uid, n_user, item_ids, self.item_len, self.n_instr,
+                                 "UP" if order == "UP" else "IP", use_cache=(order != "RE"))
+            if order == "UP" and not admit and not hit:
+                q.use_cache = False  # UP-only baseline with a user larger than the cache
+            if order == "UP" and q.use_cache:
+                pinned.add(uid)
+            self.decisions.append((order, hit, admit, evicted))
+            pending.append(q)
+            if len(pending) == batch:
+                self._run(pending, k, out)
+                pinned.clear()
+        self._run(pending, k, out)
+        return out
+
+    def stats(self) -> dict:
+        return bat.bat_sched_stats(self.sched)

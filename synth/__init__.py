@@ -52,7 +52,7 @@ MODEL_CONFIGS: Dict[str, dict] = {
 
 _TAG = dict(embed=1, lm_head=2, final_norm=3, ln1=10, wqkv=11, bqkv=12, wo=13, ln2=14,
             wgu=15, wd=16, user_tok=40, item_tok=41, item_label=42, instr_tok=43,
-            header_tok=44, user_len=45, query=46, kv=47)
+            header_tok=44, user_len=45, query=46, kv=47, trace=48)
 
 ROW_BLOCK = 1024
 
@@ -293,3 +293,20 @@ def random_kv(seed: int, entity_key: int, layers: int, n: int, kv_heads: int, he
     r = _rng(seed, _TAG["kv"], entity_key)
     x = r.standard_normal((layers, 2, n, kv_heads, head_dim), dtype=np.float32) * np.float32(std)
     return bf16_round(x)
+
+
+def request_trace(seed: int, n_requests: int, n_users: int, activity_s: float = 1.2,
+                  rate: float = 50.0, tau_i: int = 1600, median: float = 1500.0,
+                  sigma: float = 0.8):
+    """Synthetic ranking-request trace for the prompt scheduler (the real
+    traces are out of scope): user activity Zipf(activity_s) over n_users (a long tail of
+    inactive users, P:284 / Fig. 2(c)), user profile lengths lognormal (Table 1),
+    Poisson arrivals at `rate` requests per time unit, tau_i item tokens per request
+    (100 candidates x 16 tokens).  Returns [(time, user_id, tau_u, tau_i)], times increasing."""
+    r = _rng(seed, _TAG["trace"])
+    p = np.arange(1, n_users + 1, dtype=np.float64) ** (-activity_s)
+    p /= p.sum()
+    users = r.choice(n_users, size=n_requests, p=p)
+    lens = user_lengths(seed, n_users, median=median, sigma=sigma)
+    times = np.cumsum(r.exponential(1.0 / rate, size=n_requests))
+    return [(float(t), int(u), int(lens[u]), int(tau_i)) for t, u in zip(times, users)]

@@ -95,3 +95,33 @@ def test_hotness_aware_rule():
 def test_window_similarity():
     assert scheduler.window_similarity(3, 3) == 1.0
     assert scheduler.window_similarity(3, 1) == 0.5
+
+
+# ------------------------------------------------- scheduler simulation (NEXT-2)
+def test_simulation_hand_trace():
+    """Pinned by hand (see tests/test_sched.py::test_scheduler_hand_trace for the arithmetic)."""
+    tr = [(0.0, 1, 4000, 1600), (1.0, 2, 5000, 1600), (2.0, 1, 4000, 1600), (3.0, 3, 6000, 1600),
+          (3.5, 4, 500, 1600), (4.0, 3, 6000, 1600)]
+    d, tot = scheduler.simulate(tr, "hotness", 700, 10.0)
+    assert [x[0] for x in d] == ["UP", "UP", "UP", "IP", "IP", "UP"]
+    assert d[5][2] == [2] and d[2][1] is True
+    d, tot = scheduler.simulate(tr, "greedy", 700, 10.0)  # LRU evicts u2 (last access 1.0) for u3
+    assert [x[0] for x in d] == ["UP", "UP", "UP", "UP", "IP", "UP"] and d[3][2] == [2]
+    assert tot["hits"] == 2 and tot["reused"] == 4000 + 1600 + 6000
+
+
+def test_simulation_degenerate_policies_are_closed_forms():
+    import synth
+    tr = synth.request_trace(3, 500, 50)
+    tokens = sum(a + b for _, _, a, b in tr)
+    _, t_re = scheduler.simulate(tr, "re", 1000, 5.0)
+    assert t_re["reused"] == 0 and t_re["tokens"] == tokens
+    _, t_ip = scheduler.simulate(tr, "ip", 1000, 5.0)
+    assert t_ip["reused"] == sum(b for *_, b in tr) and t_ip["ip"] == len(tr)
+    # unbounded cache: UP-only hits every repeat visit of a user, misses each first visit
+    _, t_up = scheduler.simulate(tr, "up", 10 ** 9, 5.0)
+    first = len({u for _, u, _, _ in tr})
+    assert t_up["hits"] == len(tr) - first
+    # zero capacity: hotness never admits, so it is IP for every request
+    _, t_h = scheduler.simulate(tr, "hotness", 0, 5.0)
+    assert t_h["ip"] == len(tr) and t_h["hits"] == 0
