@@ -9,9 +9,10 @@
 //   O += P V    (M=256 N=128 K=16 x 8): A = P from each CTA's TMEM, B = the V tile split along
 //               N = head_dim — rank r supplies columns [64 r, 64 r + 64) of all 128 keys.
 // Per SM this halves the MMA instructions and the K/V shared-memory traffic against the 1-CTA
-// kernel, and frees TMEM for a DOUBLE-BUFFERED S: TMEM = O [0,128) S0 [128,256) S1 [256,384), so
-// S_{t+2} is issued right after P_t.V and the S -> softmax -> P.V chain of a q-tile is off the
-// tensor pipe's critical path (tools/attn_timeline*.py measured it there in the 1-CTA kernel).
+// kernel, and frees TMEM for DOUBLE-BUFFERED S and P: TMEM = O [0,128) S0 [128,256) S1 [256,384)
+// P0 [384,448) P1 [448,512).  S_{t+2} is issued as soon as the softmax of tile t holds S_t in
+// registers, P.V_t reads P from its own buffer, so the S -> softmax -> P.V chain of a tile no
+// longer gates the next S (tools/attn_timeline*.py measured it on the critical path).
 //
 // Softmax: four warpgroups (tile parity, key half): warpgroup (w, h) handles the tiles t with
 // t % 2 == w (S buffer w), 64 key columns [64 h, 64 h + 64) per row in registers; the two halves
@@ -79,8 +80,8 @@ static_assert(sizeof(PairX) <= 12288, "exchange area");
 struct __align__(8) PairBars {
   uint64_t q_full[2], q_empty[2];
   uint64_t k_full[NST], k_empty[NST], v_full[NST], v_empty[NST];
-  uint64_t s_full[2], p_full[2];
-  uint64_t o_full, o_empty, pv_done;
+  uint64_t s_full[2], s_free[2], p_full[2], pv_done[2];
+  uint64_t o_full, o_empty;
   uint32_t tmem_base;
 };
 static_assert(sizeof(PairBars) <= 256, "barrier area");
@@ -115,6 +116,8 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(PT, 1)
       ptx::mbar_init(&bars->q_empty[i], 1);
       ptx::mbar_init(&bars->s_full[i], 1);
       ptx::mbar_init(&bars->p_full[i], 16);  // 8 softmax warps (both key halves) of each CTA
+      ptx::mbar_init(&bars->s_free[i], 16);  // the same warps, once they hold S in registers
+      ptx::mbar_init(&bars->pv_done[i], 1);  // pair commit: P.V of the P buffer done
     }
     for (int i = 0; i < NST; ++i) {
       ptx::mbar_init(&bars->k_full[i], 1);
@@ -124,7 +127,6 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(PT, 1)
     }
     ptx::mbar_init(&bars->o_full, 1);
     ptx::mbar_init(&bars->o_empty, 32);  // 16 softmax warps of each CTA
-    ptx::mbar_init(&bars->pv_done, 1);
     ptx::fence_mbar_init();
     ptx::prefetch_tmap(&P.tm_pool_k);
     ptx::prefetch_tmap(&P.tm_pool_v);
@@ -212,79 +214,91 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(PT, 1)
     if (rank == 0) {
       const uint32_t sq0 = ptx::smem_u32(smem + Q_OFF);
       const uint32_t tO = tmem;
-      uint32_t oc = 0;
-      // S of global tile t (item tile x of an item whose q-tile buffer is qb) into S buffer t & 1
-      auto issue_s = [&](const WorkItem& wi, int x, uint32_t qb, uint32_t t) {
-        const uint32_t st = t % NST;
-        ptx::mbar_wait(&bars->k_full[st], (t / NST) & 1);
-        PDBG(12, t);
-        ptx::tc_fence_after();
-        const uint32_t sq = sq0 + qb * Q_BYTES;
-        const uint32_t sk = ptx::smem_u32(smem + K_OFF + st * KH_BYTES);
-        const uint32_t tS = tmem + 128 + (t & 1) * 128;
-#pragma unroll
-        for (int kk = 0; kk < 8; ++kk)
-          ptx::mma2_ss_elect(tS, ptx::desc_sw128(sq + (kk >> 2) * 16384 + (kk & 3) * 32, 16, 1024),
-                             ptx::desc_sw128(sk + (kk >> 2) * 1024 + (kk & 3) * 32, 16, 2048), IDESC_S, kk ? 1u : 0u);
-        ptx::mma2_commit_elect(&bars->s_full[t & 1], 3);
-        PDBG(0, t);
-        ptx::mma2_commit_elect(&bars->k_empty[st], 3);
-        if (x == wi.kt_n - 1) ptx::mma2_commit_elect(&bars->q_empty[qb], 3);
+      // Event loop over two cursors walking the pair's tiles: S(g) is issued as soon as the
+      // softmax of tile g-2 released S buffer g & 1 (s_free), its item's q-tile and K tile are
+      // resident and P.V(g-4) has been issued (so when tile g's softmax runs, P.V(g-4) is
+      // complete: every pv_done wait below is unambiguous); P.V(g) as soon as P(g) and V(g) are
+      // ready.  Neither stream blocks the other.
+      struct Cur {
+        int w;
+        WorkItem wi;
+        uint32_t it, g;
+        int x;
       };
-      int w = first_item();
-      uint32_t it = 0, tb = 0;  // item counter, global index of the item's first tile
-      int pre = 0;              // S of the current item already issued during the previous one
-      bool q_ready = false;
-      while (w < p.n_work) {
-        const WorkItem wi = load_work(work, w);
-        const int n = wi.kt_n;
-        const uint32_t qb = it & 1;
-        if (!q_ready) ptx::mbar_wait(&bars->q_full[qb], (it >> 1) & 1);
-        for (int x = pre; x < 2 && x < n; ++x) issue_s(wi, x, qb, tb + x);
-        const int wn = next_item(w);
-        const WorkItem wni = wn < p.n_work ? load_work(work, wn) : WorkItem{0, 0, -1, -1, 0, 0, 0, 0};
-        int npre = 0;
-        bool nq = false;
-        for (int x = 0; x < n; ++x) {
-          const uint32_t t = tb + x, b = t & 1, st = t % NST;
-          PDBG(1, t);
-          ptx::mbar_wait(&bars->p_full[b], (t >> 1) & 1);
-          PDBG(2, t);
-          if (x == 0) ptx::mbar_wait(&bars->o_empty, (oc & 1) ^ 1);
-          ptx::mbar_wait(&bars->v_full[st], (t / NST) & 1);
-          PDBG(3, t);
-          ptx::tc_fence_after();
-          const uint32_t sv = ptx::smem_u32(smem + V_OFF + st * V_STRIDE);
-          const uint32_t tP = tmem + 128 + b * 128;
+      auto start = [&](Cur& c) {
+        c.w = first_item();
+        c.wi = c.w < p.n_work ? load_work(work, c.w) : WorkItem{0, 0, -1, -1, 0, 0, 0, 0};
+        c.it = 0;
+        c.g = 0;
+        c.x = 0;
+      };
+      auto advance = [&](Cur& c) {  // returns true when it moved to the next item
+        ++c.g;
+        if (++c.x < c.wi.kt_n) return false;
+        c.w = next_item(c.w);
+        c.wi = c.w < p.n_work ? load_work(work, c.w) : WorkItem{0, 0, -1, -1, 0, 0, 0, 0};
+        ++c.it;
+        c.x = 0;
+        return true;
+      };
+      auto ready = [&](uint64_t* bar, uint32_t parity) {
+        return __shfl_sync(0xffffffffu, int(ptx::mbar_test(bar, parity)), 0) != 0;
+      };
+      uint32_t total = 0;
+      for (int w = first_item(); w < p.n_work; w = next_item(w)) total += uint32_t(work[int64_t(w) * 8 + 5]);
+      Cur sc, pc;
+      start(sc);
+      start(pc);
+      bool sq_ok = false;
+      while (pc.g < total) {
+        bool prog = false;
+        if (sc.g < total) {
+          const uint32_t g = sc.g, st = g % NST, qb = sc.it & 1;
+          bool ok = g < 2 || ready(&bars->s_free[g & 1], ((g - 2) >> 1) & 1);
+          if (ok && g >= 4) ok = pc.g > g - 4;
+          if (ok && !sq_ok) ok = sq_ok = ready(&bars->q_full[qb], (sc.it >> 1) & 1);
+          if (ok) ok = ready(&bars->k_full[st], (g / NST) & 1);
+          if (ok) {
+            PDBG(12, g);
+            ptx::tc_fence_after();
+            const uint32_t sq = sq0 + qb * Q_BYTES;
+            const uint32_t sk = ptx::smem_u32(smem + K_OFF + st * KH_BYTES);
+            const uint32_t tS = tmem + 128 + (g & 1) * 128;
 #pragma unroll
-          for (int i = 0; i < 8; ++i)
-            ptx::mma2_ts_elect(tO, tP + (i >> 2) * 64 + (i & 3) * 8, ptx::desc_sw128(sv + i * 4096, 1024, 2048), IDESC_PV,
-                               (x > 0 || i > 0) ? 1u : 0u);
-          ptx::mma2_commit_elect(&bars->pv_done, 3);
-          PDBG(4, t);
-          ptx::mma2_commit_elect(&bars->v_empty[st], 3);
-          if (x == n - 1) {
-            ptx::mma2_commit_elect(&bars->o_full, 3);
-            ++oc;
-          }
-          // the S that reuses buffer b: tile x + 2 of this item, or tile x + 2 - n of the next
-          // (only as an in-order prefix and only once its q-tile is resident)
-          if (x + 2 < n) {
-            issue_s(wi, x + 2, qb, t + 2);
-          } else if (wn < p.n_work) {
-            const int xn = x + 2 - n;
-            if (xn == 0) nq = __shfl_sync(0xffffffffu, int(ptx::mbar_test(&bars->q_full[qb ^ 1], ((it + 1) >> 1) & 1)), 0) != 0;
-            if (nq && npre == xn && xn < wni.kt_n) {
-              issue_s(wni, xn, qb ^ 1, t + 2);
-              ++npre;
-            }
+            for (int kk = 0; kk < 8; ++kk)
+              ptx::mma2_ss_elect(tS, ptx::desc_sw128(sq + (kk >> 2) * 16384 + (kk & 3) * 32, 16, 1024),
+                                 ptx::desc_sw128(sk + (kk >> 2) * 1024 + (kk & 3) * 32, 16, 2048), IDESC_S, kk ? 1u : 0u);
+            ptx::mma2_commit_elect(&bars->s_full[g & 1], 3);
+            PDBG(0, g);
+            ptx::mma2_commit_elect(&bars->k_empty[st], 3);
+            if (sc.x == sc.wi.kt_n - 1) ptx::mma2_commit_elect(&bars->q_empty[qb], 3);
+            if (advance(sc)) sq_ok = false;
+            prog = true;
           }
         }
-        ++it;
-        tb += n;
-        pre = npre;
-        q_ready = nq;
-        w = wn;
+        if (pc.g < sc.g) {
+          const uint32_t g = pc.g, st = g % NST, b = g & 1;
+          bool ok = ready(&bars->p_full[b], (g >> 1) & 1);
+          if (ok && pc.x == 0) ok = ready(&bars->o_empty, (pc.it & 1) ^ 1);
+          if (ok) ok = ready(&bars->v_full[st], (g / NST) & 1);
+          if (ok) {
+            PDBG(2, g);
+            ptx::tc_fence_after();
+            const uint32_t sv = ptx::smem_u32(smem + V_OFF + st * V_STRIDE);
+            const uint32_t tP = tmem + 384 + b * 64;
+#pragma unroll
+            for (int i = 0; i < 8; ++i)
+              ptx::mma2_ts_elect(tO, tP + (i >> 2) * 32 + (i & 3) * 8, ptx::desc_sw128(sv + i * 4096, 1024, 2048),
+                                 IDESC_PV, (pc.x > 0 || i > 0) ? 1u : 0u);
+            ptx::mma2_commit_elect(&bars->pv_done[b], 3);
+            PDBG(4, g);
+            ptx::mma2_commit_elect(&bars->v_empty[st], 3);
+            if (pc.x == pc.wi.kt_n - 1) ptx::mma2_commit_elect(&bars->o_full, 3);
+            advance(pc);
+            prog = true;
+          }
+        }
+        if (!prog) __nanosleep(20);
       }
     }
   } else if (warp >= 3) {  // -------------------------------------------- softmax warpgroups
@@ -295,13 +309,15 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(PT, 1)
     const uint32_t sub = warp & 3;
     const int row = sub * 32 + lane;
     const uint32_t lane_base = (sub * 32) << 16;
-    const uint32_t tS = tmem + 128 + par * 128 + h * 64 + lane_base;  // my S half; P at its first 32 columns
+    const uint32_t tS = tmem + 128 + par * 128 + h * 64 + lane_base;  // my S half
     const uint32_t tO = tmem + lane_base;
     // named barriers: 1-4 / 5-8 the reference chain into parity 0 / 1 (per sub; 128 threads:
     // both key halves of both parities — it also publishes the halves' row maxima to each
     // other), 9 the item-end rendezvous, 10-13 the halves' max exchange of tile 0 (no chain yet)
     const uint32_t id_in = 1 + par * 4 + sub, id_out = 1 + (par ^ 1) * 4 + sub;
     const uint32_t p_full_leader = ptx::mapa(ptx::smem_u32(&bars->p_full[par]), 0);
+    const uint32_t s_free_leader = ptx::mapa(ptx::smem_u32(&bars->s_free[par]), 0);
+    const uint32_t tP = tmem + 384 + par * 64 + h * 32 + lane_base;  // my P half (bf16 pairs)
     const uint32_t o_empty_leader = ptx::mapa(ptx::smem_u32(&bars->o_empty), 0);
     const uint64_t sc2 = pk2(p.scale_log2, p.scale_log2);
     uint32_t total = 0;  // tiles of this pair (the last one publishes no reference)
@@ -389,7 +405,11 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(PT, 1)
         // O holds this item's earlier tiles relative to m_prev: rescale my 64 O columns
         const bool need_o = x > 0 && m_prev != -INFINITY && m_new != m_prev;
         if (__any_sync(0xffffffffu, need_o)) {
-          ptx::mbar_wait(&bars->pv_done, (t - 1) & 1);  // P.V of tile t-1 (and all before) done
+          // P.V of tile t-1 (and all before) done.  Its P buffer's barrier completes for t-3 and
+          // then t-1; P.V(t-4), hence t-5, is complete (S_t was issued after P.V(t-4)), so waiting
+          // for t-3 and then t-1 is unambiguous.
+          if (t >= 3) ptx::mbar_wait(&bars->pv_done[(t - 1) & 1], ((t - 3) >> 1) & 1);
+          ptx::mbar_wait(&bars->pv_done[(t - 1) & 1], ((t - 1) >> 1) & 1);
           ptx::tc_fence_after();
           const float a = need_o ? ex2(m_prev - m_new) : 1.0f;
 #pragma unroll 1
@@ -402,15 +422,12 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(PT, 1)
             ptx::tmem_st32(tO + h * 64 + c * 32, o);
           }
         }
-        // ---- P = 2^(s * scale - m_new) as bf16 into my S half's first 32 columns
+        // ---- P = 2^(s * scale - m_new) as bf16 into my half of P buffer par.  S_t is read into
+        // registers first and released (s_free) so the next S can overwrite it while the
+        // exponentials run; P buffer par is free once P.V of tile t-2 completed.
         float lsum = 0.0f;
-        if (state == 0) {
-#pragma unroll
-          for (int c = 0; c < 2; ++c)
-            asm volatile(
-                "tcgen05.st.sync.aligned.32x32b.x16.b32 [%0], "
-                "{%1,%1,%1,%1,%1,%1,%1,%1,%1,%1,%1,%1,%1,%1,%1,%1};" ::"r"(tS + c * 16), "r"(0u));
-        } else {
+        uint32_t pk[2][16];
+        if (state != 0) {
           const float mu = (m_new == -INFINITY) ? 0.0f : m_new;
           const uint64_t nm2 = pk2(-mu, -mu);
           uint64_t acc0 = pk2(0.0f, 0.0f), acc1 = acc0;
@@ -419,12 +436,16 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(PT, 1)
             uint32_t r[32];
             ptx::tmem_ld32(tS + c * 32, r);
             ptx::tmem_ld_wait();
+            if (c == 1) {  // all of S_t is in registers: release the buffer
+              ptx::tc_fence_before();
+              __syncwarp();
+              if (lane == 0) ptx::mbar_arrive_remote(s_free_leader);
+            }
             if (state == 2) {
               const uint32_t vw = c ? mv.y : mv.x;
 #pragma unroll
               for (int i = 0; i < 32; ++i) r[i] = ((vw >> i) & 1u) ? r[i] : 0xff800000u;
             }
-            uint32_t pk[16];
 #pragma unroll
             for (int i = 0; i < 16; ++i) {
               const uint32_t ra = r[2 * i], rb = r[2 * i + 1];
@@ -446,20 +467,30 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(PT, 1)
               else acc0 = fadd2(acc0, e);
               float p0, p1;
               up2(e, p0, p1);
-              pk[i] = ptx::pack_bf16x2(p0, p1);
+              pk[c][i] = ptx::pack_bf16x2(p0, p1);
             }
-            asm volatile(
-                "tcgen05.st.sync.aligned.32x32b.x16.b32 [%0], "
-                "{%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,%16};" ::"r"(tS + c * 16),
-                "r"(pk[0]), "r"(pk[1]), "r"(pk[2]), "r"(pk[3]), "r"(pk[4]), "r"(pk[5]), "r"(pk[6]), "r"(pk[7]),
-                "r"(pk[8]), "r"(pk[9]), "r"(pk[10]), "r"(pk[11]), "r"(pk[12]), "r"(pk[13]), "r"(pk[14]),
-                "r"(pk[15]));
           }
           float a0, a1, b0, b1;
           up2(acc0, a0, a1);
           up2(acc1, b0, b1);
           lsum = (a0 + a1) + (b0 + b1);
+        } else {
+          ptx::tc_fence_before();
+          __syncwarp();
+          if (lane == 0) ptx::mbar_arrive_remote(s_free_leader);
+#pragma unroll
+          for (int i = 0; i < 16; ++i) pk[0][i] = pk[1][i] = 0u;
         }
+        if (t >= 2) ptx::mbar_wait(&bars->pv_done[par], ((t >> 1) + 1) & 1);  // P.V of tile t-2 read P buffer par
+        ptx::tc_fence_after();
+#pragma unroll
+        for (int c = 0; c < 2; ++c)
+          asm volatile(
+              "tcgen05.st.sync.aligned.32x32b.x16.b32 [%0], "
+              "{%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,%16};" ::"r"(tP + c * 16),
+              "r"(pk[c][0]), "r"(pk[c][1]), "r"(pk[c][2]), "r"(pk[c][3]), "r"(pk[c][4]), "r"(pk[c][5]), "r"(pk[c][6]),
+              "r"(pk[c][7]), "r"(pk[c][8]), "r"(pk[c][9]), "r"(pk[c][10]), "r"(pk[c][11]), "r"(pk[c][12]),
+              "r"(pk[c][13]), "r"(pk[c][14]), "r"(pk[c][15]));
         if (l_own > 0.0f && m_own != m_new) l_own *= ex2(m_own - m_new);
         l_own += lsum;
         m_own = m_new;
