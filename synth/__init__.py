@@ -42,6 +42,14 @@ MODEL_CONFIGS: Dict[str, dict] = {
     # the same at GQA group 7 (Qwen2-7B's 28 Q / 4 KV heads: 18 tokens x 7 heads per q-tile)
     "small7": dict(layers=2, hidden=896, q_heads=7, kv_heads=1, head_dim=128, ffn=1024,
                    vocab=4096, rope_theta=1e6, rms_eps=1e-6, tied=False, mlp_std=0.01),
+    # the head_dim-64 GQA-4 shape of Llama3-1B (Table 2: 8 KV heads, d = 64) at parity size
+    "small64": dict(layers=2, hidden=512, q_heads=8, kv_heads=2, head_dim=64, ffn=1024,
+                    vocab=4096, rope_theta=5e5, rms_eps=1e-5, tied=False, mlp_std=0.01),
+    # Llama3-1B shape (Table 2: 16 layers, 8 KV heads, d 64; hidden / F / vocab /
+    # theta / eps / tying from the public Llama-3.2-1B config; weights random, shapes only; the
+    # Qwen2-style qkv bias is kept (drawn, not zero) since the shapes are what matter)
+    "llama3-1b": dict(layers=16, hidden=2048, q_heads=32, kv_heads=8, head_dim=64, ffn=8192,
+                      vocab=128256, rope_theta=5e5, rms_eps=1e-5, tied=True),
     # Qwen2-1.5B shape (Table 2 P:396-403 + public config for F / vocab / theta / eps)
     "qwen2-1.5b": dict(layers=28, hidden=1536, q_heads=12, kv_heads=2, head_dim=128,
                        ffn=8960, vocab=151936, rope_theta=1e6, rms_eps=1e-6, tied=True),

@@ -144,3 +144,10 @@ def test_fp32_pool_and_bf16_model_are_rejected(B):
     with pytest.raises(B.BatError):
         B.bat_bipartite_prefill(pool.handle, model.handle, B.QueryArray([q]), hidden)
     pool.close()
+
+
+@pytest.mark.parametrize("order", ["IP", "UP"])
+def test_fp32_small64_llama_head_shape(B, order):
+    cfg = synth.model_config("small64")
+    qs = [synth.make_query(8, cfg, 9, 120, list(range(400, 424)), (16, 16), 8, order)]
+    _run_check(B, "small64", qs)

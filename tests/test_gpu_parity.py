@@ -135,3 +135,14 @@ def test_small_mixed_batch(B):
           for i, (n_u, order) in enumerate([(40, "IP"), (250, "UP"), (8, "IP"), (60, "IP"), (130, "UP")])]
     cfg, W, out = _run(B, "small", qs)
     _check(cfg, W, qs, out)
+
+
+@pytest.mark.parametrize("order", ["IP", "UP", "RE"])
+def test_small64_llama_head_shape(B, order):
+    """head_dim 64, GQA group 4 (Llama3-1B's attention shape, Table 2; SURVEY §8(f)
+    NEXT-3): 32 tokens x 4 heads per q-tile, the Dp = 64 kernel instantiations."""
+    cfg = synth.model_config("small64")
+    qs = [synth.make_query(8, cfg, 9, 120, list(range(400, 424)), (16, 16), 8,
+                           "UP" if order == "UP" else "IP", use_cache=(order != "RE"))]
+    cfg, W, out = _run(B, "small64", qs)
+    _check(cfg, W, qs, out)

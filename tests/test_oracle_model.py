@@ -237,3 +237,14 @@ def test_rope_rotation_properties():
     a, b = rng.normal(size=(1, 1, 8)), rng.normal(size=(1, 1, 8))
     dot = lambda p1, p2: float(np.sum(om.rope(a, np.array([p1]), 1e4) * om.rope(b, np.array([p2]), 1e4)))
     assert abs(dot(5, 2) - dot(13, 10)) < 1e-12
+
+
+@pytest.mark.parametrize("order", ["UP", "IP"])
+def test_mask_sensitivity_guard_small64(order):
+    """Guard at the head_dim-64 GQA-4 parity config (Llama3-1B's head shape, Table 2)."""
+    cfg = synth.model_config("small64")
+    Ws = synth.Weights(cfg, seed=1)
+    q = synth.make_query(8, cfg, 9, 120, list(range(400, 424)), (16, 16), 8, order)
+    good = om.run_query(cfg, Ws, q, "full")
+    bad = om.run_query(cfg, Ws, q, "full", mask_fn=lambda seg: causal_mask(len(seg)))
+    assert np.max(np.abs(good["z"] - bad["z"])) > 10 * 2e-2

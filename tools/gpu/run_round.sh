@@ -15,5 +15,5 @@ echo "bench exit $?"; head -c 4000 gpurun_out/bench_$TAG.json; tail -3 gpurun_ou
 ARGS="--steps 2 --warmup 1 --no-cpu-baseline --plans 1 --corpus 2048"
 BAT_PROFILE_RANGE=1 timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none --profile-from-start off --csv --log-file gpurun_out/launches_$TAG.csv python bench.py $ARGS > gpurun_out/ncu_list_$TAG.out 2>&1
 echo "list exit $?"
-BAT_PROFILE_RANGE=1 timeout 900 ncu --set full --import-source on --clock-control none --profile-from-start off -k regex:"attn_tc|gemm_tc" -c 6 -o gpurun_out/full_$TAG python bench.py $ARGS > gpurun_out/ncu_full_$TAG.out 2>&1
+BAT_PROFILE_RANGE=1 timeout 900 ncu --set full --import-source on --clock-control none --profile-from-start off -k regex:"attn|gemm" -c 8 -o gpurun_out/full_$TAG python bench.py $ARGS > gpurun_out/ncu_full_$TAG.out 2>&1
 echo "full exit $?"
