@@ -54,6 +54,8 @@ def parse():
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="bat", choices=["bat", "reference"])
     ap.add_argument("--batch", type=int, default=64, help="requests per step per GPU")
+    ap.add_argument("--model", default="qwen2-1.5b", choices=["qwen2-1.5b", "qwen2-7b", "llama3-1b"],
+                    help="model shape (the driver's line is qwen2-1.5b = configs[1])")
     ap.add_argument("--n-user", type=int, default=512)
     ap.add_argument("--n-items", type=int, default=100)
     ap.add_argument("--item-len", type=int, default=16)
@@ -173,7 +175,7 @@ def oracle_time_per_request(args, budget_s, max_layers=None):
     sample description, threads)."""
     from oracle import model as om
     from oracle.sequence import bipartite_mask, build_sequence
-    cfg = synth.model_config("qwen2-1.5b")
+    cfg = synth.model_config(args.model)
     W = synth.Weights(cfg, seed=args.seed)
     q = synth.make_query(args.seed, cfg, 0, args.n_user, list(range(args.n_items)),
                          (args.item_len, args.item_len), args.n_instr, "IP")
@@ -206,7 +208,7 @@ def _blas_threads():
 
 
 def run_reference(args):
-    cfg = synth.model_config("qwen2-1.5b")
+    cfg = synth.model_config(args.model)
     S = args.n_user + args.n_instr
     from oracle import model as om
     from oracle.sequence import bipartite_mask, build_sequence
@@ -260,7 +262,7 @@ def main():
     dev = torch.device("cuda", local)
     if world > 1:
         dist.init_process_group("nccl", device_id=dev)
-    cfg = synth.model_config("qwen2-1.5b")
+    cfg = synth.model_config(args.model)
     pk = peaks()
 
     # ---- model + pool
@@ -452,7 +454,9 @@ def main():
             metric=METRIC, value=value, unit="requests/s", n_gpus=world, steps=args.steps, warmup=args.warmup,
             ms_per_step=ms_step, higher_is_better=True, scaling="weak", vs_baseline=None, dtype="bf16",
             data="synthetic (random-init weights, seeded synthetic requests; item KV computed by the model)",
-            config=dict(workload=WORKLOAD, batch_per_gpu=B, global_batch=B * world, seq_len=args.n_user + args.n_items * args.item_len + args.n_instr,
+            config=dict(workload=WORKLOAD if args.model == "qwen2-1.5b" else
+                        f"{args.model}-shaped, 1 user of {args.n_user} tokens + {args.n_items} items of "
+                        f"{args.item_len} tokens, bf16, item-as-prefix", batch_per_gpu=B, global_batch=B * world, seq_len=args.n_user + args.n_items * args.item_len + args.n_instr,
                         suffix_tokens_per_request=args.n_user + args.n_instr, prefix_tokens_per_request=args.n_items * args.item_len,
                         corpus_items=args.corpus, item_hotness="Zipf s=1.093", parallelism=f"dp{world}",
                         hrcs=dict(replication_ratio=r_rep, r_max=r_max, alpha=args.alpha, t_request_s=0.0015,

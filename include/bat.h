@@ -176,13 +176,20 @@ typedef struct {
   const int32_t* instr_tok; int32_t n_instr;        /* host; n_instr >= 1 (discriminant) */
   int64_t header_id;                                /* IP notation tokens, may be 0-length */
   const int32_t* header_tok; int32_t n_header;      /* host */
+  int32_t multi_disc; /* 1: one discriminant token per item — the last token of every
+                         item, whose hidden state has attended to U and its own item; requires
+                         order UP (the items must be computed) and the same value for the whole
+                         batch.  0: the last sequence token is the discriminant. */
 } bat_query;
 
 /* Run the L layers for B requests (data-parallel batch): every request's suffix
  * tokens are computed and attend to its cached prefix entries (BAT_E_NOTFOUND if one is
  * missing and use_cache = 1).  Writes the final-RMSNormed discriminant hidden state of every
  * request to out_hidden (device fp32 [B][hidden]).  Positions follow P:257 with the readings
- * of DESIGN.md §2 (tokens after the item set continue from the longest item). */
+ * of DESIGN.md §2 (tokens after the item set continue from the longest item).  With
+ * multi_disc out_hidden is device fp32 [B][n_max][hidden], n_max = the batch's largest
+ * n_items: row (b, i) is the final-RMSNormed hidden state of item i's last token (rows
+ * i >= n_items[b] repeat the request's last token); the last layer then runs on every row. */
 BAT_API bat_status bat_bipartite_prefill(bat_pool p, bat_model m, const bat_query* queries, int32_t B,
                                  float* out_hidden, bat_stream_t stream);
 
@@ -195,6 +202,12 @@ BAT_API bat_status bat_bipartite_prefill(bat_pool p, bat_model m, const bat_quer
 BAT_API bat_status bat_score(bat_model m, const float* hidden, const int32_t* labels,
                      const int32_t* n_items, int32_t B, int32_t n_max, float* scores,
                      int32_t k, int32_t* topk, bat_stream_t stream);
+/* Multi-discriminant scoring: s[b][i] = softmax_i(W_out[labels[b][i]] . hidden[b][i])
+ * with hidden device fp32 [B][n_max][hidden] (bat_bipartite_prefill with multi_disc); the
+ * other arguments as bat_score. */
+BAT_API bat_status bat_score_multi(bat_model m, const float* hidden, const int32_t* labels,
+                                   const int32_t* n_items, int32_t B, int32_t n_max, float* scores,
+                                   int32_t k, int32_t* topk, bat_stream_t stream);
 
 /* ------------------------------------------------------------------------------------------
  * Planned execution: build (host) + upload (device, async on `stream`) the plan of a batch

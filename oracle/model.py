@@ -162,6 +162,33 @@ def run_query(cfg: dict, W, q, mode: str = "full", rope_on: bool = True, k: int 
     return dict(hf=hf, z=z, s=s, topk=top, h_last=h[-1])
 
 
+def run_query_multi(cfg: dict, W, q, mode: str = "full", rope_on: bool = True, k: int = 0):
+    """Multi-discriminant variant (reading R20): in User-as-prefix order the last token of
+    every item I_i is item i's discriminant; z_i = W_out[v_i] . RMSNorm(h_last(I_i)) (P:175 per
+    item), s = softmax_i z_i, top-k.  Returns dict(hf [N][H], z, s, topk)."""
+    assert q.order == "UP", "one discriminant per item needs the items computed (User-as-prefix)"
+    tokens, seg, pos = build_sequence(q.order, q.user_tok, q.item_toks, q.instr_tok, ())
+    mask = bipartite_mask(seg)
+    if mode == "full" or not q.use_cache:
+        h, _ = forward_full(cfg, W, tokens, pos, mask, rope_on)
+        off = 0
+    elif mode == "cached":
+        P = _prefix_len(q)
+        h, _ = forward_cached(cfg, W, tokens[P:], pos[P:], _prefix_kv(cfg, W, q, rope_on), mask[P:, :], rope_on)
+        off = P
+    else:
+        raise ValueError(mode)
+    seg = np.asarray(seg)
+    rows = [int(np.nonzero(seg == i)[0].max()) - off for i in range(len(q.item_toks))]
+    hf = np.stack([final_hidden(cfg, W, h[r]) for r in rows])
+    Wl = np.asarray(W.lm_head_rows(q.labels), np.float64)
+    z = np.einsum("ij,ij->i", Wl, hf)
+    s = np.exp(z - z.max())
+    s = s / s.sum()
+    order = sorted(range(len(s)), key=lambda i: (-s[i], i))[:k]
+    return dict(hf=hf, z=z, s=s, topk=np.asarray(order, np.int64))
+
+
 def _prefix_len(q) -> int:
     if q.order == "UP":
         return len(q.user_tok)

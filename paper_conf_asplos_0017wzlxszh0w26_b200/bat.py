@@ -57,7 +57,7 @@ class bat_query(Structure):
                 ("item_id", POINTER(c_int64)), ("item_off", POINTER(c_int32)),
                 ("item_tok", POINTER(c_int32)), ("instr_tok", POINTER(c_int32)),
                 ("n_instr", c_int32), ("header_id", c_int64), ("header_tok", POINTER(c_int32)),
-                ("n_header", c_int32)]
+                ("n_header", c_int32), ("multi_disc", c_int32)]
 
 
 _lib = None
@@ -128,6 +128,8 @@ def lib() -> ctypes.CDLL:
                                c_int32, c_void_p, c_int32, c_int32, c_void_p]),
         "bat_debug_attention_layer": (S, [c_void_p, c_void_p, POINTER(bat_query), c_int32, c_int32, c_void_p,
                                           c_void_p, c_int32, c_void_p]),
+        "bat_score_multi": (S, [c_void_p, c_void_p, c_void_p, c_void_p, c_int32, c_int32, c_void_p, c_int32, c_void_p,
+                                c_void_p]),
         "bat_sched_create": (S, [POINTER(bat_sched_cfg), POINTER(c_void_p)]),
         "bat_sched_destroy": (S, [c_void_p]),
         "bat_sched_decide": (S, [c_void_p, c_double, c_int64, c_int32, c_int32, POINTER(bat_sched_decision),
@@ -152,7 +154,7 @@ EXPORTED = ("bat_last_error", "bat_version", "bat_kernel_launch_count", "bat_mod
             "bat_kv_register_remote", "bat_kv_lookup_remote", "bat_kv_fetch", "bat_debug_gemm", "bat_debug_attention_layer",
             "bat_plan_build", "bat_prefill_plan", "bat_profile_enable", "bat_profile_read",
             "bat_profile_reset", "bat_debug_attach_peer_pool", "bat_sched_create", "bat_sched_destroy",
-            "bat_sched_decide", "bat_sched_stats", "bat_sched_is_cached")
+            "bat_sched_decide", "bat_sched_stats", "bat_sched_is_cached", "bat_score_multi")
 
 
 def _check(status: int) -> None:
@@ -305,6 +307,7 @@ class QueryArray:
             s.header_id = int(getattr(q, "header_id", 0))
             s.header_tok = _i32p(ht)
             s.n_header = len(q.header_tok)
+            s.multi_disc = 1 if getattr(q, "multi_disc", False) else 0
 
     def __len__(self):
         return len(self.arr)
@@ -317,6 +320,12 @@ def bat_bipartite_prefill(pool: int, model: int, queries: QueryArray, out_hidden
 def bat_score(model: int, hidden, labels, n_items, B: int, n_max: int, scores, k: int = 0,
               topk=None, stream=None) -> None:
     _check(lib().bat_score(model, _vp(hidden), _vp(labels), _vp(n_items), B, n_max, _vp(scores),
+                           k, _vp(topk), _vp(stream)))
+
+
+def bat_score_multi(model: int, hidden, labels, n_items, B: int, n_max: int, scores, k: int = 0,
+              topk=None, stream=None) -> None:
+    _check(lib().bat_score_multi(model, _vp(hidden), _vp(labels), _vp(n_items), B, n_max, _vp(scores),
                            k, _vp(topk), _vp(stream)))
 
 

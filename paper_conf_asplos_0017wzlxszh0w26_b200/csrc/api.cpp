@@ -290,10 +290,11 @@ static const int32_t* prepare(Pool& pool, Model& m, Plan& plan, cudaStream_t st,
   ws.scratch.ensure(size_t(std::max(plan.n_spages, 1)) * pool.geo.layer_bytes, true);
   ws.o.ensure(size_t(M) * nq * es);
   ws.act.ensure(size_t(M) * F * es);
-  ws.hc.ensure(size_t(B) * H * 4);
-  ws.xc.ensure(size_t(B) * H * es);
-  ws.oc.ensure(size_t(B) * nq * es);
-  ws.actc.ensure(size_t(B) * F * es);
+  const size_t D = size_t(B) * plan.n_disc;  // discriminant rows
+  ws.hc.ensure(D * H * 4);
+  ws.xc.ensure(D * H * es);
+  ws.oc.ensure(D * nq * es);
+  ws.actc.ensure(D * F * es);
   if (dev_img) return dev_img;
   const size_t img_bytes = plan.img.buf.size() * 4;
   ws.img.ensure(size_t(plan.img.total_ints) * 4);
@@ -458,7 +459,7 @@ static void run_plan_f32(Pool& pool, Model& m, Plan& plan, float* out_hidden, cu
     launch_gemm_f32(1, act, WL(l, BAT_WL_WD), nullptr, h, M, H, F, 0, st);
   }
   if (out_hidden && !plan.entity_mode)
-    launch_rmsnorm_f32(h, W(BAT_W_FINAL_NORM), out_hidden, I + im.off_disc, B, H, c.rms_eps, st);
+    launch_rmsnorm_f32(h, W(BAT_W_FINAL_NORM), out_hidden, I + im.off_disc, B * plan.n_disc, H, c.rms_eps, st);
   CUDA_OK(cudaGetLastError());
 }
 
@@ -491,15 +492,16 @@ static void run_plan(Pool& pool, Model& m, Plan& plan, float* out_hidden, cudaSt
   const CUtensorMap tA_xn = make_tmap(ws.xn.p, M, H, H, 128);
   const CUtensorMap tA_o = make_tmap(ws.o.p, M, nq, nq, 128);
   const CUtensorMap tA_act = make_tmap(ws.act.p, M, F, F, 128);
-  const CUtensorMap tA_xc = make_tmap(ws.xc.p, B, H, H, 128);
-  const CUtensorMap tA_oc = make_tmap(ws.oc.p, B, nq, nq, 128);
-  const CUtensorMap tA_actc = make_tmap(ws.actc.p, B, F, F, 128);
+  const int Dr = B * plan.n_disc;  // discriminant rows (multi_disc: n_disc per request)
+  const CUtensorMap tA_xc = make_tmap(ws.xc.p, Dr, H, H, 128);
+  const CUtensorMap tA_oc = make_tmap(ws.oc.p, Dr, nq, nq, 128);
+  const CUtensorMap tA_actc = make_tmap(ws.actc.p, Dr, F, F, 128);
   // outputs (epilogue TMA store / reduce-add, 32-row boxes)
   const CUtensorMap tC_qkv = make_tmap(ws.qkv.p, M, m.nqkv(), m.nqkv(), 32);
   const CUtensorMap tC_h = make_tmap(ws.h.p, M, H, H, 32, true);
   const CUtensorMap tC_act = make_tmap(ws.act.p, M, F, F, 32);
-  const CUtensorMap tC_hc = make_tmap(ws.hc.p, B, H, H, 32, true);
-  const CUtensorMap tC_actc = make_tmap(ws.actc.p, B, F, F, 32);
+  const CUtensorMap tC_hc = make_tmap(ws.hc.p, Dr, H, H, 32, true);
+  const CUtensorMap tC_actc = make_tmap(ws.actc.p, Dr, F, F, 32);
   AttnParams ap = attn_params(pool, m, plan, I);
   StageParams sp = stage_params(pool, m, plan, I);
 
@@ -571,38 +573,39 @@ static void run_plan(Pool& pool, Model& m, Plan& plan, float* out_hidden, cudaSt
       launch_gemm(EPI_RESID_F32, tA_act, Lw.t_d, tC_h, gd, m.num_sms, st);
       pf.end(st, BAT_K_GEMM_DOWN, fd.first, fd.second);
     } else {
-      // a8: after the last layer's K/V only the discriminant rows matter
-      ap.off_work = im.off_work_last;
-      ap.n_work = plan.n_work_last;
+      // a8: after the last layer's K/V only the discriminant rows matter; with one
+      // discriminant per item they are spread over the suffix: attend for every row
+      ap.off_work = plan.multi_disc ? im.off_work : im.off_work_last;
+      ap.n_work = plan.multi_disc ? plan.n_work : plan.n_work_last;
       pf.begin(st);
       run_attention(pool, m, plan, ap, st);
-      pf.end(st, BAT_K_ATTN, attn_fl_last, attn_by);
+      pf.end(st, BAT_K_ATTN, plan.multi_disc ? attn_fl : attn_fl_last, attn_by);
       const int32_t* disc = I + im.off_disc;
       pf.begin(st);
-      launch_gather_rows_bf16(ws.o.as<__nv_bfloat16>(), disc, ws.oc.as<__nv_bfloat16>(), B, nq, st);
-      launch_gather_rows_f32(ws.h.as<float>(), disc, ws.hc.as<float>(), B, H, st);
-      pf.end(st, BAT_K_OTHER, 0, 2.0 * B * (2.0 * nq + 4.0 * H));
-      GemmParams go{B, H, nq, ws.hc.p, H, nullptr, 0};
-      auto fo = gemm_fb(B, H, nq, 8);
+      launch_gather_rows_bf16(ws.o.as<__nv_bfloat16>(), disc, ws.oc.as<__nv_bfloat16>(), Dr, nq, st);
+      launch_gather_rows_f32(ws.h.as<float>(), disc, ws.hc.as<float>(), Dr, H, st);
+      pf.end(st, BAT_K_OTHER, 0, 2.0 * Dr * (2.0 * nq + 4.0 * H));
+      GemmParams go{Dr, H, nq, ws.hc.p, H, nullptr, 0};
+      auto fo = gemm_fb(Dr, H, nq, 8);
       pf.begin(st);
       launch_gemm(EPI_RESID_F32, tA_oc, Lw.t_o, tC_hc, go, m.num_sms, st);
       pf.end(st, BAT_K_GEMM_O, fo.first, fo.second);
       pf.begin(st);
-      launch_rmsnorm_bf16(ws.hc.as<float>(), Lw.ln2, ws.xc.as<__nv_bfloat16>(), B, H, c.rms_eps, st);
-      pf.end(st, BAT_K_RMSNORM, 0, 6.0 * B * H);
-      GemmParams gg{B, F, H, ws.actc.p, F, nullptr, F};
-      auto fg = gemm_fb(B, 2 * F, H, 1);
+      launch_rmsnorm_bf16(ws.hc.as<float>(), Lw.ln2, ws.xc.as<__nv_bfloat16>(), Dr, H, c.rms_eps, st);
+      pf.end(st, BAT_K_RMSNORM, 0, 6.0 * Dr * H);
+      GemmParams gg{Dr, F, H, ws.actc.p, F, nullptr, F};
+      auto fg = gemm_fb(Dr, 2 * F, H, 1);
       pf.begin(st);
       launch_gemm(EPI_SWIGLU, tA_xc, Lw.t_gu, tC_actc, gg, m.num_sms, st);
       pf.end(st, BAT_K_GEMM_GU, fg.first, fg.second);
-      GemmParams gd{B, H, F, ws.hc.p, H, nullptr, 0};
-      auto fd = gemm_fb(B, H, F, 8);
+      GemmParams gd{Dr, H, F, ws.hc.p, H, nullptr, 0};
+      auto fd = gemm_fb(Dr, H, F, 8);
       pf.begin(st);
       launch_gemm(EPI_RESID_F32, tA_actc, Lw.t_d, tC_hc, gd, m.num_sms, st);
       pf.end(st, BAT_K_GEMM_DOWN, fd.first, fd.second);
       pf.begin(st);
-      launch_rmsnorm_f32out(ws.hc.as<float>(), m.final_norm, out_hidden, B, H, c.rms_eps, st);
-      pf.end(st, BAT_K_OTHER, 0, 8.0 * B * H);
+      launch_rmsnorm_f32out(ws.hc.as<float>(), m.final_norm, out_hidden, Dr, H, c.rms_eps, st);
+      pf.end(st, BAT_K_OTHER, 0, 8.0 * Dr * H);
     }
   }
   CUDA_OK(cudaGetLastError());
@@ -956,6 +959,20 @@ bat_status bat_bipartite_prefill(bat_pool p, bat_model mdl, const bat_query* que
     Plan plan;
     build_plan(P, m.cfg.q_heads / m.cfg.kv_heads, m.cfg.kv_heads, wrap(queries, B), plan, true, attn_grid_slots(m.dpad, m.num_sms));
     run_plan(P, m, plan, out_hidden, static_cast<cudaStream_t>(stream));
+  });
+}
+
+bat_status bat_score_multi(bat_model mdl, const float* hidden, const int32_t* labels, const int32_t* n_items,
+                           int32_t B, int32_t n_max, float* scores, int32_t k, int32_t* topk, bat_stream_t stream) {
+  return guarded([&] {
+    BAT_REQUIRE(mdl && hidden && labels && n_items && scores, "null argument");
+    BAT_REQUIRE(B >= 1 && n_max >= 1 && n_max <= 4096, "B >= 1, 1 <= n_max <= 4096");
+    BAT_REQUIRE(k >= 0 && (k == 0 || topk) && k <= n_max, "k / topk");
+    Model& m = mdl->m;
+    DeviceGuard dg(m.device);
+    launch_score_multi(hidden, m.f32 ? nullptr : m.lm_head, m.f32 ? static_cast<const float*>(m.w[BAT_W_LM_HEAD]) : nullptr,
+                       labels, n_items, B, n_max, m.cfg.hidden, scores, k, topk, static_cast<cudaStream_t>(stream));
+    CUDA_OK(cudaGetLastError());
   });
 }
 

@@ -182,7 +182,7 @@ __global__ void gather_rows_kernel(const T* __restrict__ src, const int32_t* __r
 }
 
 // a9: z_i = W_out[v_i] . hf, s = softmax over the N candidates, top-k
-template <class TW>
+template <class TW, bool MULTI>
 __global__ void score_kernel(const float* __restrict__ hidden, const TW* __restrict__ w,
                              const int32_t* __restrict__ labels, const int32_t* __restrict__ n_items,
                              int n_max, int H, float* __restrict__ scores, int k,
@@ -195,12 +195,16 @@ __global__ void score_kernel(const float* __restrict__ hidden, const TW* __restr
   const int b = blockIdx.x;
   const int n = n_items[b];
   const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5, nw = blockDim.x >> 5;
-  for (int c = threadIdx.x; c < H; c += blockDim.x) hf[c] = hidden[int64_t(b) * H + c];
+  if (!MULTI)
+    for (int c = threadIdx.x; c < H; c += blockDim.x) hf[c] = hidden[int64_t(b) * H + c];
   __syncthreads();
   for (int i = wid; i < n; i += nw) {
     const TW* row = w + int64_t(labels[int64_t(b) * n_max + i]) * H;
     float acc = 0.0f;
-    if constexpr (sizeof(TW) == 4) {  // fp32 correctness mode
+    if constexpr (MULTI) {  // one discriminant hidden state per item
+      const float* hi = hidden + (int64_t(b) * n_max + i) * H;
+      for (int c = lane; c < H; c += 32) acc = fmaf(float(row[c]), hi[c], acc);
+    } else if constexpr (sizeof(TW) == 4) {  // fp32 correctness mode
       for (int c = lane; c < H; c += 32) acc = fmaf(row[c], hf[c], acc);
     } else {
       for (int c = lane * 8; c < H; c += 256) {
@@ -387,18 +391,24 @@ void launch_gather_rows_f32(const float* src, const int32_t* idx, float* dst, in
   gather_rows_kernel<float><<<n, 256, 0, s>>>(src, idx, dst, cols);
   count_launch();
 }
-template <class TW>
+template <class TW, bool MULTI = false>
 static void score_launch(const float* hidden, const TW* w_out, const int32_t* labels, const int32_t* n_items, int B,
                          int n_max, int H, float* scores, int k, int32_t* topk, cudaStream_t s) {
   if (B <= 0) return;
   const size_t smem = sizeof(float) * (size_t(H) + size_t(n_max));
   static bool attr = false;
   if (!attr) {
-    cudaFuncSetAttribute(score_kernel<TW>, cudaFuncAttributeMaxDynamicSharedMemorySize, 64 * 1024);
+    cudaFuncSetAttribute(score_kernel<TW, MULTI>, cudaFuncAttributeMaxDynamicSharedMemorySize, 64 * 1024);
     attr = true;
   }
-  score_kernel<TW><<<B, 256, smem, s>>>(hidden, w_out, labels, n_items, n_max, H, scores, k, topk);
+  score_kernel<TW, MULTI><<<B, 256, smem, s>>>(hidden, w_out, labels, n_items, n_max, H, scores, k, topk);
   count_launch();
+}
+void launch_score_multi(const float* hidden, const __nv_bfloat16* w_bf16, const float* w_f32, const int32_t* labels,
+                        const int32_t* n_items, int B, int n_max, int H, float* scores, int k, int32_t* topk,
+                        cudaStream_t s) {
+  if (w_f32) score_launch<float, true>(hidden, w_f32, labels, n_items, B, n_max, H, scores, k, topk, s);
+  else score_launch<__nv_bfloat16, true>(hidden, w_bf16, labels, n_items, B, n_max, H, scores, k, topk, s);
 }
 void launch_score(const float* hidden, const __nv_bfloat16* w_out, const int32_t* labels,
                   const int32_t* n_items, int B, int n_max, int H, float* scores, int k,

@@ -163,6 +163,10 @@ void launch_kv_scatter_f32(const PageIO& io, const float* k, const float* v, con
                            int slot0, int n_total, cudaStream_t s);
 void launch_kv_gather_f32(const PageIO& io, float* k, float* v, const int32_t* pages_dev, int n_tokens,
                           cudaStream_t s);
+// one discriminant hidden row per item: hidden [B][n_max][H] (exactly one of w_bf16 / w_f32)
+void launch_score_multi(const float* hidden, const __nv_bfloat16* w_bf16, const float* w_f32, const int32_t* labels,
+                        const int32_t* n_items, int B, int n_max, int H, float* scores, int k, int32_t* topk,
+                        cudaStream_t s);
 void launch_score_f32w(const float* hidden, const float* w_out, const int32_t* labels, const int32_t* n_items, int B,
                        int n_max, int H, float* scores, int k, int32_t* topk, cudaStream_t s);
 

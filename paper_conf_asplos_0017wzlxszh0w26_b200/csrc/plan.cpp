@@ -218,6 +218,15 @@ void build_plan(const Pool& pool, int32_t group, int32_t kv_heads,
   plan.kv_heads = kv_heads;
   plan.qt = kQtileRows / group;
   plan.q.assign(reqs.size(), QueryPlan{});
+  plan.multi_disc = !reqs.empty() && reqs[0].q && reqs[0].q->multi_disc;
+  plan.n_disc = 1;
+  for (const PlanRequest& r : reqs) {
+    BAT_REQUIRE(bool(r.q && r.q->multi_disc) == plan.multi_disc, "multi_disc must be the same for the whole batch");
+    if (plan.multi_disc) {
+      BAT_REQUIRE(r.q->order == BAT_ORDER_UP, "multi_disc requires User-as-prefix (the items must be computed, P:259)");
+      plan.n_disc = std::max(plan.n_disc, r.q->n_items);
+    }
+  }
   int32_t tok = 0, sp = 0, qt0 = 0, pg = 0;
   for (size_t b = 0; b < reqs.size(); ++b) {
     QueryPlan& qp = plan.q[b];
@@ -229,6 +238,14 @@ void build_plan(const Pool& pool, int32_t group, int32_t kv_heads,
       plan.entity_mode = true;
     }
     BAT_REQUIRE(qp.S >= 1, "request with no suffix tokens");
+    if (plan.multi_disc) {  // the last suffix token of every item
+      qp.disc.assign(r.q->n_items, -1);
+      for (int32_t t = 0; t < qp.S; ++t)
+        if (qp.seg[t] >= 0) qp.disc[qp.seg[t]] = t;
+      for (int32_t d : qp.disc) BAT_REQUIRE(d >= 0, "multi_disc: an item is not in the suffix");
+    } else {
+      qp.disc.assign(1, qp.S - 1);
+    }
     // the suffix's own pages follow the prefix pages (reading: virtual key order)
     const int32_t n_sfx = static_cast<int32_t>(ceil_div(qp.S, kPageTokens));
     if (r.ent_pages) BAT_REQUIRE(static_cast<int32_t>(r.ent_pages->size()) == n_sfx, "entity pages");
@@ -278,7 +295,7 @@ void build_plan(const Pool& pool, int32_t group, int32_t kv_heads,
   im.off_kmeta = reserve_at(int64_t(plan.n_pages_padded) * kPageTokens * 2);
   im.off_qtiles = reserve_at(int64_t(plan.n_qtiles_total) * 4);
   im.off_spages = reserve_at(int64_t(plan.n_spages) * 4);
-  im.off_disc = reserve_at(B);
+  im.off_disc = reserve_at(int64_t(B) * plan.n_disc);
   for (int32_t b = 0; b < B; ++b) {
     const QueryPlan& qp = plan.q[b];
     for (int32_t t = 0; t < qp.S; ++t) {
@@ -309,7 +326,8 @@ void build_plan(const Pool& pool, int32_t group, int32_t kv_heads,
       e[0] = b; e[1] = s * kPageTokens; e[2] = std::min(kPageTokens, qp.S - s * kPageTokens);
       e[3] = qp.pages[qp.n_prefix_pages + s];
     }
-    v[im.off_disc + b] = qp.token_off + qp.S - 1;
+    for (int32_t i = 0; i < plan.n_disc; ++i)  // padding rows repeat the last token
+      v[im.off_disc + int64_t(b) * plan.n_disc + i] = qp.token_off + (i < int32_t(qp.disc.size()) ? qp.disc[i] : qp.S - 1);
   }
   // work items: (b, kvh, q-tile pair) sharing every K/V tile, with the union of the two
   // q-tiles' live k-tiles and a state per q-tile; longest first (LPT over the SMs)

@@ -22,6 +22,7 @@ struct QueryPlan {
   std::vector<int32_t> pages, valid;      // [n_pages]
   std::vector<int32_t> kseg, kord;        // [16 * n_pages]
   std::vector<uint8_t> tiles;             // [n_qtiles * n_ktiles]: 0 skip, 1 full, 2 partial
+  std::vector<int32_t> disc;              // suffix rows of the discriminant(s): [1] or, multi, [n_items]
 };
 
 // One request description, independent of the C struct (entity prefill builds these too).
@@ -47,7 +48,7 @@ struct PlanImage {
   int64_t off_spages = 0;                           // [n_spages][4] {b, t0, ntok, target}
   int64_t off_work = 0, off_work_last = 0;          // [W][8] {b, kvh, q0, q1|-1, kt_off, kt_n, tp_off, km_off}
   int64_t off_ktl = 0;                              // kt list: ktile | state0 << 24 | state1 << 26
-  int64_t off_disc = 0;                             // [B] global discriminant row
+  int64_t off_disc = 0;                             // [B][n_disc] global discriminant rows
   // Visibility masks of the partial (state 2) (q-tile, k-tile) pairs, shared by all KV heads and
   // layers: mask m = (b, q-tile, k-tile) from off_mdesc [n_masks][4]; per listed tile of a work
   // item, km_off + 2 x + q holds q-tile q's mask id (-1: not partial).  The masks themselves,
@@ -63,6 +64,8 @@ struct Plan {
   int32_t M = 0, n_qtiles_total = 0, n_spages = 0, n_pages_padded = 0;
   int32_t n_work = 0, n_work_last = 0;
   bool entity_mode = false;
+  bool multi_disc = false;  // one discriminant per item: off_disc holds [B][n_disc]
+  int32_t n_disc = 1;       // discriminant rows per request in the image (multi: max n_items)
   PlanImage img;
 };
 

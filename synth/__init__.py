@@ -234,6 +234,7 @@ class Query:
     use_cache: bool = True
     header_id: int = -1
     header_tok: np.ndarray = field(default_factory=lambda: np.zeros(0, np.int32))
+    multi_disc: bool = False  # one discriminant token per item (UP only)
 
     @property
     def n_items(self) -> int:

@@ -248,3 +248,40 @@ def test_mask_sensitivity_guard_small64(order):
     good = om.run_query(cfg, Ws, q, "full")
     bad = om.run_query(cfg, Ws, q, "full", mask_fn=lambda seg: causal_mask(len(seg)))
     assert np.max(np.abs(good["z"] - bad["z"])) > 10 * 2e-2
+
+
+# ---------------------------------------------- multi-discriminant variant (R20)
+def _mq(seed=0, items=(11, 22, 33, 44), n_user=16):
+    q = synth.make_query(seed, CFG, 3, n_user, list(items), (8, 8), 2, "UP")
+    q.multi_disc = True
+    return q
+
+
+def test_multi_disc_cached_equals_full(W):
+    """I1 for the per-item discriminants: serving U from its cached KV changes nothing."""
+    q = _mq()
+    a = om.run_query_multi(CFG, W, q, "full")
+    b = om.run_query_multi(CFG, W, q, "cached")
+    np.testing.assert_allclose(a["hf"], b["hf"], rtol=1e-10, atol=1e-10)
+    np.testing.assert_allclose(a["s"], b["s"], rtol=1e-10, atol=1e-12)
+
+
+def test_multi_disc_item_independence(W):
+    """I2: item i's discriminant sees U and its own item only — changing another item's
+    tokens leaves hf_i (and z_i) unchanged, while hf_j of the changed item moves."""
+    q = _mq()
+    a = om.run_query_multi(CFG, W, q, "full")
+    q2 = _mq()
+    q2.item_toks = list(q2.item_toks)
+    q2.item_toks[2] = (np.asarray(q2.item_toks[2]) + 7) % CFG["vocab"]
+    b = om.run_query_multi(CFG, W, q2, "full")
+    for i in (0, 1, 3):
+        np.testing.assert_allclose(a["hf"][i], b["hf"][i], rtol=1e-12, atol=1e-12)
+    assert np.max(np.abs(a["hf"][2] - b["hf"][2])) > 1e-3
+
+
+def test_multi_disc_permutation_equivariance(W):
+    """I3: permuting the candidates permutes the scores."""
+    a = om.run_query_multi(CFG, W, _mq(items=(11, 22, 33, 44)), "full")
+    b = om.run_query_multi(CFG, W, _mq(items=(33, 11, 44, 22)), "full")
+    np.testing.assert_allclose(b["s"], a["s"][[2, 0, 3, 1]], rtol=1e-10, atol=1e-12)
