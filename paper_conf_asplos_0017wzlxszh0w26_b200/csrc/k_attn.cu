@@ -83,9 +83,13 @@ struct __align__(8) AttnBars {
   uint64_t q_full, q_empty;
   uint64_t k_full[3], k_empty[3], v_full[3], v_empty[3];
   uint64_t s_full[2], p_full[2], o_full[2], o_empty[2];
+  uint64_t seq[2];  // softmax turn token: seq[q] completes when it is q-tile team q's turn
   uint32_t tmem_base;
 };
 static_assert(sizeof(AttnBars) <= 256, "barrier area");
+#ifndef BAT_ATTN_SEQ
+#define BAT_ATTN_SEQ 0  // 1: the two q-tile softmax teams take turns (FA4-style); measured 543 vs 600 TFLOP/s
+#endif
 
 // ring positions: K tile g -> slot g % 3; V half h (= 2 g + {0,1}) -> slot h % 3
 __device__ __forceinline__ uint32_t ring_slot(uint32_t i) { return i % 3u; }
@@ -281,6 +285,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) attn_tc_kernel(const __grid_co
       ptx::mbar_init(&bars->p_full[i], 8);
       ptx::mbar_init(&bars->o_full[i], 1);
       ptx::mbar_init(&bars->o_empty[i], 8);
+      ptx::mbar_init(&bars->seq[i], 8);
     }
     ptx::fence_mbar_init();
   }
@@ -531,10 +536,34 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) attn_tc_kernel(const __grid_co
     const uint32_t pair_bar = 1 + wg * 4 + sub;                      // named barrier of the warp pair
     XchSmem* xch = reinterpret_cast<XchSmem*>(smem + L::XCH_OFF);
     uint32_t kc = 0, sc = 0, oc = 0;
+    // Turn-taking (FA4-style softmax sequencing): team 0 runs the softmax of its tile x, then
+    // team 1 of its tile x, then team 0 of tile x + 1, ... — each softmax runs alone on the
+    // MUFU/FMA pipes while the tensor pipe serves the other q-tile's P.V and next S, instead of
+    // both overlapping at half speed with both q-tiles' MMAs bunched together.  A team without a
+    // q-tile in an item passes the token through for each of its tiles.
+    uint32_t turn = 0;
+    auto seq_wait = [&]() {
+      if (!BAT_ATTN_SEQ) return;
+      if (wg == 0) {
+        if (turn > 0) ptx::mbar_wait(&bars->seq[0], (turn - 1) & 1);
+      } else {
+        ptx::mbar_wait(&bars->seq[1], turn & 1);
+      }
+    };
+    auto seq_pass = [&]() {
+      if (!BAT_ATTN_SEQ) return;
+      __syncwarp();
+      if (lane == 0) ptx::mbar_arrive(&bars->seq[wg ^ 1]);
+      ++turn;
+    };
     for (int w = blockIdx.x; w < p.n_work; w += gridDim.x) {
       const WorkItem wi = load_work(work, w);
       const int qi = wg == 0 ? wi.q0 : wi.q1;
       if (qi < 0 || wi.kt_n == 0) {
+        for (int x = 0; x < wi.kt_n; ++x) {
+          seq_wait();
+          seq_pass();
+        }
         kc += wi.kt_n;
         continue;
       }
@@ -560,6 +589,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) attn_tc_kernel(const __grid_co
         ptx::mbar_wait(&bars->s_full[wg], sc & 1);
         DBG(11 + 3 * wg, x);
         ++sc;
+        seq_wait();
         ptx::tc_fence_after();
         const uint32_t vis[NCH] = {mv.x, mv.y};
         // fast path: one pass against the settled reference max; both halves must agree
@@ -623,6 +653,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) attn_tc_kernel(const __grid_co
         ptx::tc_fence_before();
         __syncwarp();
         if (lane == 0) ptx::mbar_arrive(&bars->p_full[wg]);
+        seq_pass();
         DBG(13 + 2 * wg, x);
       }
       kc += wi.kt_n;
