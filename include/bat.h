@@ -254,7 +254,8 @@ enum {
   BAT_PF_VALID = 4,   /* int32 [n_pages] valid slots per page */
   BAT_PF_KSEG = 5,    /* int32 [16*n_pages] key segment (-1 for empty slots) */
   BAT_PF_KORD = 6,    /* int32 [16*n_pages] 0 prefix key, suffix index+1, INT32_MAX empty */
-  BAT_PF_TILES = 7    /* int32 [n_qtiles][n_ktiles] 0 skip / 1 full / 2 partial */
+  BAT_PF_TILES = 7,   /* int32 [n_qtiles][n_ktiles] 0 skip / 1 full / 2 partial */
+  BAT_PF_DISC = 8     /* int32 [1] or, multi_disc, [n_items]: suffix rows of the discriminants */
 };
 /* Copy field `field` of request b into out (cap elements); *count = its length. */
 BAT_API bat_status bat_plan_export(bat_plan plan, int32_t b, int32_t field, int32_t* out, int64_t cap,

@@ -103,7 +103,13 @@ def plan_query(q, entity_pages: Dict[Tuple[int, int], Tuple[Sequence[int], int]]
             n_live = int(blk.sum())
             full_pairs = (r1 - r0) * KTILE  # slots past the last page are empty (invalid)
             state[i, j] = 0 if n_live == 0 else (1 if n_live == full_pairs else 2)
-    return dict(tokens=tokens[P:].astype(np.int64), pos=pos[P:].astype(np.int64),
+    # discriminant suffix rows: the last token or, with one discriminant per item
+    # (reading R20), the last token of every item, in candidate order
+    if getattr(q, "multi_disc", False):
+        disc = np.array([int(np.nonzero(rseg == i)[0].max()) for i in range(len(q.item_toks))], dtype=np.int64)
+    else:
+        disc = np.array([S - 1], dtype=np.int64)
+    return dict(tokens=tokens[P:].astype(np.int64), pos=pos[P:].astype(np.int64), disc=disc,
                 seg=rseg, P=P, S=S, pages=np.array(pages, dtype=np.int64),
                 valid=np.array(valid, dtype=np.int64), n_prefix_pages=n_pre,
                 kseg=kseg_a, kord=kord_a, rord=rord, tile_state=state,

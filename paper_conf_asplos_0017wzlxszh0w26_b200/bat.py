@@ -26,7 +26,7 @@ BAT_OK = 0
 BAT_BF16, BAT_FP32 = 0, 1
 BAT_ENT_USER, BAT_ENT_ITEM, BAT_ENT_HEADER = 0, 1, 2
 BAT_ORDER_UP, BAT_ORDER_IP = 0, 1
-BAT_PF_TOKENS, BAT_PF_POS, BAT_PF_SEG, BAT_PF_PAGES, BAT_PF_VALID, BAT_PF_KSEG, BAT_PF_KORD, BAT_PF_TILES = range(8)
+BAT_PF_TOKENS, BAT_PF_POS, BAT_PF_SEG, BAT_PF_PAGES, BAT_PF_VALID, BAT_PF_KSEG, BAT_PF_KORD, BAT_PF_TILES, BAT_PF_DISC = range(9)
 STATUS_NAMES = {0: "BAT_OK", -1: "BAT_E_INVAL", -2: "BAT_E_OOM", -3: "BAT_E_CUDA",
                 -4: "BAT_E_NOTFOUND", -5: "BAT_E_POOLFULL", -6: "BAT_E_UNSUPPORTED",
                 -7: "BAT_E_STATE"}

@@ -1037,6 +1037,7 @@ bat_status bat_plan_export(bat_plan plan, int32_t b, int32_t field, int32_t* out
         tiles.assign(q.tiles.begin(), q.tiles.end());
         src = &tiles;
         break;
+      case BAT_PF_DISC: src = &q.disc; break;
       default: BAT_REQUIRE(false, "unknown field");
     }
     if (count) *count = int64_t(src->size());

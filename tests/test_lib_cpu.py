@@ -65,7 +65,7 @@ def _compare_plan(B, plan, b, ref):
     assert info["scratch0"] == ref["scratch_page0"] and info["token_off"] == ref["token_off"]
     for field, key in [(B.BAT_PF_TOKENS, "tokens"), (B.BAT_PF_POS, "pos"), (B.BAT_PF_SEG, "seg"),
                        (B.BAT_PF_PAGES, "pages"), (B.BAT_PF_VALID, "valid"), (B.BAT_PF_KSEG, "kseg"),
-                       (B.BAT_PF_KORD, "kord")]:
+                       (B.BAT_PF_KORD, "kord"), (B.BAT_PF_DISC, "disc")]:
         np.testing.assert_array_equal(B.bat_plan_export(plan, b, field), ref[key].astype(np.int32), err_msg=key)
     tiles = B.bat_plan_export(plan, b, B.BAT_PF_TILES).reshape(info["n_qtiles"], info["n_ktiles"])
     np.testing.assert_array_equal(tiles, ref["tile_state"])
@@ -123,6 +123,39 @@ def test_plan_qwen_shaped_single_query(B):
             assert B.bat_plan_query_info(plan, 0)["n_live_pairs"] * 12 == 967460 * 12
         finally:
             B.bat_plan_destroy(plan)
+    finally:
+        B.bat_kv_pool_destroy(pool)
+
+
+@pytest.mark.parametrize("seed", range(3))
+def test_plan_multi_discriminant_rows_bit_exact(B, seed):
+    """One discriminant per item: the planner's discriminant rows (the last suffix token
+    of every item) equal the oracle plan's, for UP requests with cached or recomputed users and
+    ragged items; IP is rejected."""
+    cfg = synth.model_config("tiny")
+    rng = np.random.default_rng(300 + seed)
+    qs = []
+    for k in range(3):
+        q = synth.make_query(seed, cfg, user_id=k, n_user=int(rng.integers(1, 60)),
+                             item_ids=rng.choice(40, size=int(rng.integers(1, 9)), replace=False),
+                             item_len=(3, 21), n_instr=int(rng.integers(1, 5)), order="UP", use_cache=(k != 1))
+        q.multi_disc = True
+        qs.append(q)
+    pool = _index_pool(B, cfg)
+    try:
+        ep = _reserve_for(B, pool, qs)
+        refs = oplan.plan_batch(qs, ep, 2)
+        plan = B.bat_plan_create(pool, 2, B.QueryArray(qs))
+        try:
+            for b, ref in enumerate(refs):
+                _compare_plan(B, plan, b, ref)
+                assert len(ref["disc"]) == qs[b].n_items
+        finally:
+            B.bat_plan_destroy(plan)
+        bad = synth.make_query(seed, cfg, 0, qs[0].user_tok.size, qs[0].item_ids, (3, 21), 2, "IP")
+        bad.multi_disc = True
+        with pytest.raises(B.BatError):
+            B.bat_plan_create(pool, 2, B.QueryArray([bad]))
     finally:
         B.bat_kv_pool_destroy(pool)
 
