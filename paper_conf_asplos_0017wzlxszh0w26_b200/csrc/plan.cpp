@@ -6,6 +6,7 @@
 #include "plan.h"
 
 #include <algorithm>
+#include <cstdlib>
 #include <numeric>
 #include <unordered_map>
 
@@ -363,7 +364,14 @@ void build_plan(const Pool& pool, int32_t group, int32_t kv_heads,
       }
     }
     // cost of an item in k-tile-pair units: its tiles, with a fixed prologue / epilogue share
-    auto cost = [](const W& a) { return int64_t(a.n) * (a.q1 >= 0 ? 4 : 3) + 8; };
+    // (BAT_LPT_SINGLE, BAT_LPT_ITEM: experiment knobs for the per-tile weight of single-q-tile
+    // items and the fixed per-item cost, in quarter k-tile-pair units.  A single-q-tile item
+    // costs about as much per tile as a pair — the attention kernel is bound by each q-tile's
+    // S -> softmax -> P.V chain, not by tensor work — so both weigh 4; measured in-step
+    // 593.5 (3/8) vs 597.4 (4/8) vs 598.0 (4/4) vs 593.0 (4/16) TFLOP/s)
+    static const int64_t w1 = std::getenv("BAT_LPT_SINGLE") ? std::atoi(std::getenv("BAT_LPT_SINGLE")) : 4;
+    static const int64_t wi = std::getenv("BAT_LPT_ITEM") ? std::atoi(std::getenv("BAT_LPT_ITEM")) : 8;
+    auto cost = [](const W& a) { return int64_t(a.n) * (a.q1 >= 0 ? 4 : w1) + wi; };
     std::stable_sort(ws.begin(), ws.end(), [&](const W& a, const W& c) { return cost(a) > cost(c); });
     if (grid > 0 && static_cast<int32_t>(ws.size()) > grid) {
       // LPT over the persistent grid: CTA c runs items c, c + grid, c + 2 grid, ... of the list,
