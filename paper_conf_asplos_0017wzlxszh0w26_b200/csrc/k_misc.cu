@@ -79,6 +79,36 @@ __global__ void rmsnorm_kernel(const float* __restrict__ x, const __nv_bfloat16*
   }
 }
 
+// Register-resident variant for H = 128 NV: the row is read from HBM once (NV float4 per lane
+// kept in registers across the reduction), normalised and written as bf16.
+template <int NV>
+__global__ void __launch_bounds__(256) rmsnorm_reg_kernel(const float* __restrict__ x, const __nv_bfloat16* __restrict__ g,
+                                                          __nv_bfloat16* __restrict__ y, int M, float eps) {
+  constexpr int H = NV * 128;
+  const int row = blockIdx.x * 8 + (threadIdx.x >> 5);
+  const int lane = threadIdx.x & 31;
+  if (row >= M) return;
+  const float4* xr = reinterpret_cast<const float4*>(x + int64_t(row) * H);
+  float4 v[NV];
+#pragma unroll
+  for (int i = 0; i < NV; ++i) v[i] = __ldcs(xr + lane + 32 * i);  // streamed: read once
+  float ss = 0.0f;
+#pragma unroll
+  for (int i = 0; i < NV; ++i) ss += v[i].x * v[i].x + v[i].y * v[i].y + v[i].z * v[i].z + v[i].w * v[i].w;
+  ss = warp_sum(ss);
+  const float r = rsqrtf(ss / float(H) + eps);
+  uint2* yr = reinterpret_cast<uint2*>(y + int64_t(row) * H);
+  const uint2* g2 = reinterpret_cast<const uint2*>(g);
+#pragma unroll
+  for (int i = 0; i < NV; ++i) {
+    const uint2 gg = g2[lane + 32 * i];
+    const float2 ga = __bfloat1622float2(*reinterpret_cast<const __nv_bfloat162*>(&gg.x));
+    const float2 gb = __bfloat1622float2(*reinterpret_cast<const __nv_bfloat162*>(&gg.y));
+    yr[lane + 32 * i] = make_uint2(ptx::pack_bf16x2(v[i].x * r * ga.x, v[i].y * r * ga.y),
+                                   ptx::pack_bf16x2(v[i].z * r * gb.x, v[i].w * r * gb.y));
+  }
+}
+
 // cos/sin table in double precision, rounded once to fp32: tab[pos][i] = (cos, sin)(pos * theta^(-2i/d))
 __global__ void rope_table_kernel(float2* tab, int max_pos, int d, double theta) {
   const int half = d / 2;
@@ -360,7 +390,16 @@ void launch_embed(const __nv_bfloat16* E, const int32_t* tok, float* h, int M, i
 void launch_rmsnorm_bf16(const float* x, const __nv_bfloat16* g, __nv_bfloat16* y, int M, int H,
                          float eps, cudaStream_t s) {
   if (M <= 0) return;
-  rmsnorm_kernel<false><<<(M + 7) / 8, 256, 0, s>>>(x, g, y, M, H, eps);
+  const int grid = (M + 7) / 8;
+  switch (H) {  // register-resident rows for the model widths in use
+    case 512: rmsnorm_reg_kernel<4><<<grid, 256, 0, s>>>(x, g, y, M, eps); break;
+    case 768: rmsnorm_reg_kernel<6><<<grid, 256, 0, s>>>(x, g, y, M, eps); break;
+    case 896: rmsnorm_reg_kernel<7><<<grid, 256, 0, s>>>(x, g, y, M, eps); break;
+    case 1536: rmsnorm_reg_kernel<12><<<grid, 256, 0, s>>>(x, g, y, M, eps); break;
+    case 2048: rmsnorm_reg_kernel<16><<<grid, 256, 0, s>>>(x, g, y, M, eps); break;
+    case 3584: rmsnorm_reg_kernel<28><<<grid, 256, 0, s>>>(x, g, y, M, eps); break;
+    default: rmsnorm_kernel<false><<<grid, 256, 0, s>>>(x, g, y, M, H, eps);
+  }
   count_launch();
 }
 void launch_rmsnorm_f32out(const float* x, const __nv_bfloat16* g, float* y, int M, int H, float eps,
