@@ -584,18 +584,30 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) attn_tc_kernel(const __grid_co
       const int mrow = valid_row ? row / p.group : p.qt;  // row of this thread in the masks
       const int32_t* ktl = img + wi.kt_off;
       float m_ref = -INFINITY, l_sum = 0.0f;
+      // tile state and partial-tile visibility bits, loaded ONE TILE AHEAD: the state / mask-id
+      // loads (independent, plan image in L2) are issued at the top of the previous tile and
+      // the mask bits once they land, so none of the ~1k clk L2 round trips sits between S
+      // landing and the softmax (tools/chain_rate.cu: the bare chain runs at 2.75k clk per
+      // k-tile pair, the kernel at ~3.9k before this)
+      auto mask_of = [&](int mid) {
+        return __ldg(reinterpret_cast<const uint2*>(img + p.off_masks + (int64_t(mid) * (p.qt + 1) + mrow) * 4) + h);
+      };
+      int n_state = (ktl[0] >> (24 + 2 * wg)) & 3;
+      int n_mid = img[wi.km_off + wg];
+      uint2 n_mv = make_uint2(0xffffffffu, 0xffffffffu);
+      if (n_state == 2) n_mv = mask_of(n_mid);
       for (int x = 0; x < wi.kt_n; ++x) {
         const uint32_t g = kc + x;
         const int s = g & 1;
-        const int state = (ktl[x] >> (24 + 2 * wg)) & 3;
-        const bool dbg_first = (kc == 0) && row == 0 && h == 0;
-        // partial tile: this row's 64 visibility bits from the plan's precomputed mask (issued
-        // before the S wait so the load latency hides behind the MMA)
-        uint2 mv = make_uint2(0xffffffffu, 0xffffffffu);
-        if (state == 2) {
-          const int mid = img[wi.km_off + 2 * x + wg];
-          mv = __ldg(reinterpret_cast<const uint2*>(img + p.off_masks + (int64_t(mid) * (p.qt + 1) + mrow) * 4) + h);
+        const int state = n_state;
+        const uint2 mv = n_mv;
+        if (x + 1 < wi.kt_n) {
+          n_state = (ktl[x + 1] >> (24 + 2 * wg)) & 3;
+          n_mid = img[wi.km_off + 2 * (x + 1) + wg];
+        } else {
+          n_state = 0;
         }
+        const bool dbg_first = (kc == 0) && row == 0 && h == 0;
         ptx::mbar_wait(&bars->s_full[wg], sc & 1);
         DBG(11 + 3 * wg, x);
         ++sc;
@@ -665,6 +677,8 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) attn_tc_kernel(const __grid_co
         if (lane == 0) ptx::mbar_arrive(&bars->p_full[wg]);
         seq_pass();
         DBG(13 + 2 * wg, x);
+        n_mv = make_uint2(0xffffffffu, 0xffffffffu);
+        if (n_state == 2) n_mv = mask_of(n_mid);
       }
       kc += wi.kt_n;
       // ---- epilogue: O / l -> bf16, my half of the head's columns

@@ -1,0 +1,126 @@
+// Microbenchmark: the attention kernel's per-q-tile dependency chain in isolation —
+//   S = Q K^T (8 SS MMAs, M = N = 128) -> softmax of the 128 x 128 tile (row_exp_opt of k_attn.cu,
+//   key halves agreeing through a named barrier, P written back over S) -> O += P V (8 TS MMAs)
+//   -> the next S into the same TMEM columns
+// with no loaders, masks or work items.  One CTA per SM (all SMs busy); clk per chain step.
+//   mode 0: one q-tile chain (8 softmax warps)
+//   mode 1: one chain, softmax replaced by an immediate hand-off (MMA + barrier round trips only)
+//   mode 2: two independent q-tile chains (16 softmax warps), the default kernel's structure
+// build: nvcc -gencode arch=compute_100a,code=sm_100a -O3 -std=c++17 --expt-relaxed-constexpr
+//        -I paper_conf_asplos_0017wzlxszh0w26_b200/csrc -I include tools/chain_rate.cu -o tools/chain_rate -lcuda
+#include "../paper_conf_asplos_0017wzlxszh0w26_b200/csrc/k_attn.cu"
+
+namespace bat {
+void count_launch(int) {}
+namespace {
+
+template <int MODE>
+__global__ void __launch_bounds__(640, 1) chain(long long* out, int iters) {
+  extern __shared__ __align__(1024) uint8_t smem[];
+  __shared__ uint64_t s_full[2], p_full[2];
+  __shared__ uint32_t tbase;
+  __shared__ int okx[2][2][4];
+  const uint32_t warp = ptx::warp_id(), lane = ptx::lane_id();
+  constexpr int NQ = MODE == 2 ? 2 : 1;
+  if (threadIdx.x == 0) {
+    for (int q = 0; q < 2; ++q) {
+      ptx::mbar_init(&s_full[q], 1);
+      ptx::mbar_init(&p_full[q], 8);
+    }
+    ptx::fence_mbar_init();
+  }
+  for (int i = threadIdx.x; i < 131072 / 16; i += blockDim.x) reinterpret_cast<uint4*>(smem)[i] = make_uint4(0, 0, 0, 0);
+  ptx::fence_proxy_async_smem();
+  if (warp == 1) ptx::tmem_alloc(&tbase, 512);
+  ptx::tc_fence_before();
+  __syncthreads();
+  ptx::tc_fence_after();
+  const uint32_t tmem = tbase;
+  if (warp == 1) {  // converged MMA issuer, as in attn_tc_kernel
+    const uint32_t sq = ptx::smem_u32(smem), sk = sq + 65536, sv = sq + 98304;
+    constexpr uint32_t IS = ptx::idesc_bf16(128, 128, 0, 0), IP = ptx::idesc_bf16(128, 128, 0, 1);
+    auto issue_s = [&](int q) {
+#pragma unroll
+      for (int kk = 0; kk < 8; ++kk)
+        ptx::mma_ss_elect(tmem + q * 128, ptx::desc_sw128(sq + q * 32768 + (kk >> 2) * 16384 + (kk & 3) * 32, 16, 1024),
+                          ptx::desc_sw128(sk + (kk >> 2) * 1024 + (kk & 3) * 32, 16, 2048), IS, kk ? 1u : 0u);
+      ptx::mma_commit_elect(&s_full[q]);
+    };
+    auto issue_pv = [&](int q) {
+#pragma unroll
+      for (int hf = 0; hf < 2; ++hf)
+#pragma unroll
+        for (int i = 0; i < 4; ++i)
+          ptx::mma_ts_elect(tmem + 256 + q * 128, tmem + q * 128 + hf * 64 + i * 8,
+                            ptx::desc_sw128(sv + hf * 16384 + i * 4096, 1024, 2048), IP, 1u);
+    };
+    const long long t0 = clock64();
+    for (int q = 0; q < NQ; ++q) issue_s(q);
+    for (int i = 0; i < iters; ++i)
+      for (int q = 0; q < NQ; ++q) {
+        ptx::mbar_wait(&p_full[q], i & 1);
+        ptx::tc_fence_after();
+        issue_pv(q);
+        if (i + 1 < iters) issue_s(q);
+      }
+    ptx::mma_commit_elect(&s_full[0]);
+    ptx::mbar_wait(&s_full[0], (iters + (NQ == 1 ? 0 : 0)) & 1);
+    const long long t1 = clock64();
+    if (lane == 0 && blockIdx.x == 0) out[0] = t1 - t0;
+  } else if (warp >= 4 && warp < 4 + 8 * NQ) {
+    const int wgi = (warp - 4) >> 2;
+    const int q = NQ == 2 ? (wgi & 1) : 0, h = NQ == 2 ? (wgi >> 1) : wgi;
+    const uint32_t sub = warp & 3;
+    const uint32_t tS = tmem + q * 128 + h * 64 + ((sub * 32) << 16);
+    const uint64_t sc2 = pk2(0.01f, 0.01f), nm2 = pk2(-1.0f, -1.0f);
+    float acc = 0.0f;
+    for (int i = 0; i < iters; ++i) {
+      ptx::mbar_wait(&s_full[q], i & 1);
+      ptx::tc_fence_after();
+      if (MODE != 1) {
+        uint32_t vis[2] = {~0u, ~0u};
+        float lsum = 0.0f;
+        auto agree = [&](bool ok) {
+          if (lane == 0) okx[q][h][sub] = ok;
+          ptx::bar_sync(1 + q * 4 + sub, 64);
+          return ok && okx[q][h ^ 1][sub] != 0;
+        };
+        row_exp_opt<false>(tS, vis, sc2, nm2, INFINITY, lsum, agree);
+        acc += lsum;
+        ptx::tmem_st_wait();
+      }
+      ptx::tc_fence_before();
+      __syncwarp();
+      if (lane == 0) ptx::mbar_arrive(&p_full[q]);
+    }
+    if (acc == 12345.0f) out[1] = 1;
+  }
+  ptx::tc_fence_before();
+  __syncthreads();
+  if (warp == 1) ptx::tmem_dealloc(tmem, 512);
+}
+
+}  // namespace
+}  // namespace bat
+
+int main() {
+  using namespace bat;
+  long long* d;
+  cudaMalloc(&d, 8 * sizeof(long long));
+  const int iters = 400;
+  const size_t smem = 131072;
+  auto run = [&](auto kern, const char* name, int nq) {
+    cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, int(smem));
+    cudaMemset(d, 0, 8 * sizeof(long long));
+    kern<<<148, 640, smem>>>(d, iters);
+    cudaError_t e = cudaDeviceSynchronize();
+    long long h[8];
+    cudaMemcpy(h, d, sizeof(h), cudaMemcpyDeviceToHost);
+    printf("%-46s %s  clk per chain step %.0f  (tensor work per step %d clk)\n", name, cudaGetErrorString(e),
+           double(h[0]) / iters, 1024 * nq);
+  };
+  run(chain<0>, "1 q-tile: S -> softmax -> P.V -> S", 1);
+  run(chain<1>, "1 q-tile, softmax skipped (MMA + hand-offs)", 1);
+  run(chain<2>, "2 q-tiles (default kernel structure)", 2);
+  return 0;
+}
