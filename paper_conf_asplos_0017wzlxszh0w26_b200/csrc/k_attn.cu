@@ -47,6 +47,9 @@ constexpr float kRescaleThreshold = 8.0f;  // log2 units: P <= 2^8 between resca
 #ifndef BAT_ATTN_L2PF
 #define BAT_ATTN_L2PF 0  // 1: prefetch the K/V blocks of the tile two ahead into L2 (measured slower)
 #endif
+#ifndef BAT_ATTN_NOLOAD
+#define BAT_ATTN_NOLOAD 0  // timing experiment: skip the K / V copies (wrong results)
+#endif
 #ifndef BAT_SUMCHECK
 #define BAT_SUMCHECK 0  // 1: fast-path bound from the row-half sum instead of a per-element max (measured equal: 598.7 vs 601.0 TFLOP/s)
 #endif
@@ -365,11 +368,15 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) attn_tc_kernel(const __grid_co
             DBG(0, x);
             ptx::mbar_wait(&bars->k_empty[ks], ring_phase(kc) ^ 1);
             DBG(1, x);
+            if (BAT_ATTN_NOLOAD) {  // timing experiment only: K never loaded (results are garbage)
+              ptx::mbar_arrive(&bars->k_full[ks]);
+            } else {
             ptx::mbar_expect_tx(&bars->k_full[ks], kKtilePages * L::PAGE_BYTES);
 #pragma unroll
             for (int i = 0; i < kKtilePages; ++i)
               ptx::bulk_g2s(sk + i * L::PAGE_BYTES, src[i] + int64_t(wi.kvh) * p.head_bytes, L::PAGE_BYTES,
                             &bars->k_full[ks]);
+            }
             DBG(2, x);
           }
         } else {
@@ -383,11 +390,15 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) attn_tc_kernel(const __grid_co
             if (hf == 0) DBG(3, x);
             ptx::mbar_wait(&bars->v_empty[vs], ring_phase(vi) ^ 1);
             if (hf == 0) DBG(4, x);
+            if (BAT_ATTN_NOLOAD) {
+              ptx::mbar_arrive(&bars->v_full[vs]);
+            } else {
             ptx::mbar_expect_tx(&bars->v_full[vs], 4 * L::PAGE_BYTES);
 #pragma unroll
             for (int i = 0; i < 4; ++i)
               ptx::bulk_g2s(sv + i * L::PAGE_BYTES, src[i] + kv_off + int64_t(wi.kvh) * p.head_bytes, L::PAGE_BYTES,
                             &bars->v_full[vs]);
+            }
           }
         }
         __syncwarp();
