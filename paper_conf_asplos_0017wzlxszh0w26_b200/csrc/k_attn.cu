@@ -47,6 +47,9 @@ constexpr float kRescaleThreshold = 8.0f;  // log2 units: P <= 2^8 between resca
 #ifndef BAT_ATTN_L2PF
 #define BAT_ATTN_L2PF 0  // 1: prefetch the K/V blocks of the tile two ahead into L2 (measured slower)
 #endif
+#ifndef BAT_ATTN_NOMASK
+#define BAT_ATTN_NOMASK 0  // timing experiment: partial tiles take the unmasked path (wrong results)
+#endif
 #ifndef BAT_ATTN_NOLOAD
 #define BAT_ATTN_NOLOAD 0  // timing experiment: skip the K / V copies (wrong results)
 #endif
@@ -610,7 +613,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) attn_tc_kernel(const __grid_co
       for (int x = 0; x < wi.kt_n; ++x) {
         const uint32_t g = kc + x;
         const int s = g & 1;
-        const int state = n_state;
+        const int state = (BAT_ATTN_NOMASK && n_state == 2) ? 1 : n_state;  // NOMASK: timing experiment only
         const uint2 mv = n_mv;
         if (x + 1 < wi.kt_n) {
           n_state = (ktl[x + 1] >> (24 + 2 * wg)) & 3;

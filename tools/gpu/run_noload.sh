@@ -1,7 +1,7 @@
 #!/bin/bash
 cd $GRAFT_REPO_ROOT
-for v in normal noload; do
-  if [ $v = normal ]; then L=libbat.so; else L=libbat_noload.so; fi
+for v in normal nomask; do
+  if [ $v = normal ]; then L=libbat.so; else L=libbat_nomask.so; fi
   BAT_LIB=$PWD/paper_conf_asplos_0017wzlxszh0w26_b200/$L timeout 300 python bench.py --steps 4 --warmup 3 --no-cpu-baseline > gpurun_out/nl_$v.json 2>/dev/null
   python -c "import json;d=json.loads(open('gpurun_out/nl_$v.json').read().strip().splitlines()[-1]);print('$v attn', round(d['attention']['tflops'],1), 'clk', d['clocks']['sm_mhz'])"
 done
