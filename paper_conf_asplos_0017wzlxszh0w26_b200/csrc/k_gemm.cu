@@ -21,6 +21,7 @@
 // Tiles are rasterised in groups of 8 M-tiles so concurrently running CTAs share weight tiles
 // in L2.
 #include <cuda.h>
+#include <cstdlib>
 #include <cuda_bf16.h>
 #include <cuda_runtime.h>
 
@@ -32,7 +33,7 @@ namespace {
 
 constexpr int BN = 256, BK = 64, BROWS = 128;  // B is loaded in 128-row boxes
 constexpr int A_BYTES = 128 * BK * 2;           // 16 KB: 128 rows of A per CTA
-constexpr int GROUP_M = 8;
+constexpr int GROUP_M = 8;  // default rasterisation group (M-tiles); BAT_GEMM_GROUP_M / _SWIGLU override
 constexpr int NUM_THREADS = 192;
 constexpr int STG_BYTES = 4096;  // per-warp epilogue staging buffer: [32 rows][128 B], 128B-swizzled
 
@@ -53,12 +54,12 @@ constexpr size_t kGemmSmem1 = 1024 /*align slack*/ + STG1_OFF + 4 * 2 * STG_BYTE
 constexpr size_t kGemmSmem2 = 1024 /*align slack*/ + STG2_OFF + 4 * 2 * STG_BYTES + sizeof(GemmSmemBars);
 static_assert(kGemmSmem1 <= 232448 && kGemmSmem2 <= 232448, "GEMM shared memory");
 
-__device__ __forceinline__ void tile_coords(int t, int num_m, int num_n, int& m, int& n) {
-  const int per_group = GROUP_M * num_n;
+__device__ __forceinline__ void tile_coords(int t, int num_m, int num_n, int group_m, int& m, int& n) {
+  const int per_group = group_m * num_n;
   const int g = t / per_group;
   const int r = t - g * per_group;
-  const int rows = min(GROUP_M, num_m - g * GROUP_M);
-  m = g * GROUP_M + r % rows;
+  const int rows = min(group_m, num_m - g * group_m);
+  m = g * group_m + r % rows;
   n = r / rows;
 }
 
@@ -89,6 +90,7 @@ struct Epilogue {
     __syncwarp();
     if (lane == 0) {
       if (EPI == EPI_RESID_F32) ptx::tma_reduce_add_2d(tmC, buf, col, row);
+      else if (p->hints & 2) ptx::tma_store_2d_hint(tmC, buf, col, row, ptx::policy_evict_first());
       else ptx::tma_store_2d(tmC, buf, col, row);
       ptx::bulk_commit();
     }
@@ -205,19 +207,25 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
 
   if (warp == 0) {
     if (lane == 0) {  // ---------------- TMA producer
+      const uint64_t pol_b = ptx::policy_evict_last();
       int stage = 0;
       uint32_t phase = 0;
       for (int t = blockIdx.x; t < num_tiles; t += gridDim.x) {
         int m, n;
-        tile_coords(t, num_m, num_n, m, n);
+        tile_coords(t, num_m, num_n, p.group_m, m, n);
         for (int kb = 0; kb < num_kb; ++kb) {
           ptx::mbar_wait(&bars->empty[stage], phase ^ 1);
           uint8_t* sa = smem + stage * STAGE1_BYTES;
           uint8_t* sb = sa + A_BYTES;
           ptx::mbar_expect_tx(&bars->full[stage], STAGE1_BYTES);
           ptx::tma_load_2d(sa, &tmA, kb * BK, m * 128, &bars->full[stage]);
-          ptx::tma_load_2d(sb, &tmB, kb * BK, b_row<EPI>(p, n, 0), &bars->full[stage]);
-          ptx::tma_load_2d(sb + BROWS * BK * 2, &tmB, kb * BK, b_row<EPI>(p, n, 1), &bars->full[stage]);
+          if (p.hints & 1) {
+            ptx::tma_load_2d_hint(sb, &tmB, kb * BK, b_row<EPI>(p, n, 0), &bars->full[stage], pol_b);
+            ptx::tma_load_2d_hint(sb + BROWS * BK * 2, &tmB, kb * BK, b_row<EPI>(p, n, 1), &bars->full[stage], pol_b);
+          } else {
+            ptx::tma_load_2d(sb, &tmB, kb * BK, b_row<EPI>(p, n, 0), &bars->full[stage]);
+            ptx::tma_load_2d(sb + BROWS * BK * 2, &tmB, kb * BK, b_row<EPI>(p, n, 1), &bars->full[stage]);
+          }
           if (++stage == STAGES1) { stage = 0; phase ^= 1; }
         }
       }
@@ -257,7 +265,7 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
     uint32_t acc_phase = 0;
     for (int t = blockIdx.x; t < num_tiles; t += gridDim.x) {
       int m, n;
-      tile_coords(t, num_m, num_n, m, n);
+      tile_coords(t, num_m, num_n, p.group_m, m, n);
       ptx::mbar_wait(&bars->tfull[acc], acc_phase);
       ptx::tc_fence_after();
       epi.run(tmem + ((sub * 32) << 16) + acc * BN, n, m * 128 + sub * 32);
@@ -320,7 +328,7 @@ gemm2_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__
       uint32_t phase = 0;
       for (int t = pair; t < num_tiles; t += n_pairs) {
         int m, n;
-        tile_coords(t, num_m, num_n, m, n);
+        tile_coords(t, num_m, num_n, p.group_m, m, n);
         for (int kb = 0; kb < num_kb; ++kb) {
           ptx::mbar_wait(&bars->empty[stage], phase ^ 1);
           uint8_t* sa = smem + stage * STAGE2_BYTES;
@@ -368,7 +376,7 @@ gemm2_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__
     uint32_t acc_phase = 0;
     for (int t = pair; t < num_tiles; t += n_pairs) {
       int m, n;
-      tile_coords(t, num_m, num_n, m, n);
+      tile_coords(t, num_m, num_n, p.group_m, m, n);
       ptx::mbar_wait(&bars->tfull[acc], acc_phase);
       ptx::tc_fence_after();
       epi.run(tmem + ((sub * 32) << 16) + acc * BN, n, m * 256 + int(rank) * 128 + sub * 32);
@@ -403,8 +411,18 @@ void set_smem_once(K kern, size_t bytes) {
 
 size_t gemm_smem_bytes() { return kGemmSmem2 > kGemmSmem1 ? kGemmSmem2 : kGemmSmem1; }
 
+static int env_group(const char* name) {
+  const char* v = std::getenv(name);
+  return v && std::atoi(v) > 0 ? std::atoi(v) : 0;
+}
+
 void launch_gemm(int epi, const CUtensorMap& tmA, const CUtensorMap& tmB, const CUtensorMap& tmC,
-                 const GemmParams& p, int num_sms, cudaStream_t stream) {
+                 const GemmParams& p_in, int num_sms, cudaStream_t stream) {
+  static const int g_all = env_group("BAT_GEMM_GROUP_M"), g_swiglu = env_group("BAT_GEMM_GROUP_SWIGLU");
+  static const int hints = env_group("BAT_GEMM_HINTS");
+  GemmParams p = p_in;
+  if (!p.hints) p.hints = hints;
+  if (p.group_m <= 0) p.group_m = (epi == EPI_SWIGLU && g_swiglu) ? g_swiglu : (g_all ? g_all : GROUP_M);
   const int out_bn = (epi == EPI_SWIGLU) ? BN / 2 : BN;
   const int n_tiles = (p.N + out_bn - 1) / out_bn;
   // the SwiGLU GEMM stays on 1-CTA tiles: measured in the bench step, its pair version ran

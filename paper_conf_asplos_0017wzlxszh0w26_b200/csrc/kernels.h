@@ -20,6 +20,8 @@ struct GemmParams {
   int ldo;
   const __nv_bfloat16* bias;  // EPI_BF16_BIAS
   int up_row0;        // EPI_SWIGLU: first "up" row of B (= F)
+  int group_m = 0;    // M-tiles per rasterisation group (0: launch_gemm's default)
+  int hints = 0;      // 1-CTA kernel L2 hints: bit 0 B loads evict_last, bit 1 bf16 C stores evict_first
 };
 size_t gemm_smem_bytes();
 // tmC: output tensor map — bf16 [M][ldo] with box {64, 32} (EPI_BF16*, EPI_SWIGLU) or fp32
