@@ -18,8 +18,8 @@
 //    tile, M=128 N=256 K=16 MMAs, 4-stage ring.
 // In both, warp 0 issues TMA (2-D tensor maps, 128-byte swizzle), warp 1 issues the MMAs, and
 // warps 2-5 drain TMEM with tcgen05.ld and run the epilogue while the next tile accumulates.
-// Tiles are rasterised in groups of 8 M-tiles so concurrently running CTAs share weight tiles
-// in L2.
+// Tiles are rasterised in groups of 8 M-tiles (32 for SwiGLU) so concurrently running CTAs share
+// weight tiles in L2.
 #include <cuda.h>
 #include <cstdlib>
 #include <cuda_bf16.h>
@@ -34,6 +34,7 @@ namespace {
 constexpr int BN = 256, BK = 64, BROWS = 128;  // B is loaded in 128-row boxes
 constexpr int A_BYTES = 128 * BK * 2;           // 16 KB: 128 rows of A per CTA
 constexpr int GROUP_M = 8;  // default rasterisation group (M-tiles); BAT_GEMM_GROUP_M / _SWIGLU override
+constexpr int GROUP_M_SWIGLU = 32;
 constexpr int NUM_THREADS = 192;
 constexpr int STG_BYTES = 4096;  // per-warp epilogue staging buffer: [32 rows][128 B], 128B-swizzled
 
@@ -422,7 +423,13 @@ void launch_gemm(int epi, const CUtensorMap& tmA, const CUtensorMap& tmB, const 
   static const int hints = env_group("BAT_GEMM_HINTS");
   GemmParams p = p_in;
   if (!p.hints) p.hints = hints;
-  if (p.group_m <= 0) p.group_m = (epi == EPI_SWIGLU && g_swiglu) ? g_swiglu : (g_all ? g_all : GROUP_M);
+  // SwiGLU (1-CTA, 128-row tiles, 55 MB of gate/up weights re-streamed once per group): groups of
+  // 32 M-tiles with evict_last weight loads read 574 MB of DRAM per launch instead of 705 MB at
+  // equal speed (profiles/r1_gemm_raster.txt); the pair kernels keep 8 (O GEMM already at its
+  // algorithmic bytes)
+  if (p.group_m <= 0)
+    p.group_m = epi == EPI_SWIGLU ? (g_swiglu ? g_swiglu : GROUP_M_SWIGLU) : (g_all ? g_all : GROUP_M);
+  if (epi == EPI_SWIGLU && !std::getenv("BAT_GEMM_HINTS")) p.hints |= 1;
   const int out_bn = (epi == EPI_SWIGLU) ? BN / 2 : BN;
   const int n_tiles = (p.N + out_bn - 1) / out_bn;
   // the SwiGLU GEMM stays on 1-CTA tiles: measured in the bench step, its pair version ran
