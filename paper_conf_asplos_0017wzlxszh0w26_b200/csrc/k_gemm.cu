@@ -18,8 +18,8 @@
 //    tile, M=128 N=256 K=16 MMAs, 4-stage ring.
 // In both, warp 0 issues TMA (2-D tensor maps, 128-byte swizzle), warp 1 issues the MMAs, and
 // warps 2-5 drain TMEM with tcgen05.ld and run the epilogue while the next tile accumulates.
-// Tiles are rasterised in groups of 8 M-tiles (32 for SwiGLU) so concurrently running CTAs share
-// weight tiles in L2.
+// Tiles are rasterised in groups of M-tiles (GROUP_M; 32 for SwiGLU) so concurrently running CTAs
+// share operand tiles in L2.
 #include <cuda.h>
 #include <cstdlib>
 #include <cuda_bf16.h>
@@ -33,7 +33,10 @@ namespace {
 
 constexpr int BN = 256, BK = 64, BROWS = 128;  // B is loaded in 128-row boxes
 constexpr int A_BYTES = 128 * BK * 2;           // 16 KB: 128 rows of A per CTA
-constexpr int GROUP_M = 8;  // default rasterisation group (M-tiles); BAT_GEMM_GROUP_M / _SWIGLU override
+// default rasterisation group (M-tiles) of the QKV / O / down GEMMs: 1 = the N-tiles of one M-tile
+// run back to back (down GEMM DRAM reads 1.43 GB at 8, 1.27 at 4, 1.12 at 1, 2.26 at 32 per launch,
+// profiles/r1_gemm_raster.txt); BAT_GEMM_GROUP_M / _SWIGLU override
+constexpr int GROUP_M = 1;
 constexpr int GROUP_M_SWIGLU = 32;
 constexpr int NUM_THREADS = 192;
 constexpr int STG_BYTES = 4096;  // per-warp epilogue staging buffer: [32 rows][128 B], 128B-swizzled
@@ -425,8 +428,7 @@ void launch_gemm(int epi, const CUtensorMap& tmA, const CUtensorMap& tmB, const 
   if (!p.hints) p.hints = hints;
   // SwiGLU (1-CTA, 128-row tiles, 55 MB of gate/up weights re-streamed once per group): groups of
   // 32 M-tiles with evict_last weight loads read 574 MB of DRAM per launch instead of 705 MB at
-  // equal speed (profiles/r1_gemm_raster.txt); the pair kernels keep 8 (O GEMM already at its
-  // algorithmic bytes)
+  // equal speed (profiles/r1_gemm_raster.txt)
   if (p.group_m <= 0)
     p.group_m = epi == EPI_SWIGLU ? (g_swiglu ? g_swiglu : GROUP_M_SWIGLU) : (g_all ? g_all : GROUP_M);
   if (epi == EPI_SWIGLU && !std::getenv("BAT_GEMM_HINTS")) p.hints |= 1;
