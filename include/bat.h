@@ -141,7 +141,8 @@ BAT_API bat_status bat_kv_append(bat_pool p, int32_t kind, int64_t id, const voi
 /* Reserve pages for a new entry without writing data (index-only pools, and the entity
  * prefill below).  BAT_E_INVAL if the entry exists. */
 BAT_API bat_status bat_kv_reserve(bat_pool p, int32_t kind, int64_t id, int32_t n_tokens);
-/* Drop an entry and free its pages. */
+/* Drop an entry and free its pages (BAT_E_STATE if a live bat_plan_build plan references it).
+ * The caller must not evict an entry that queued device work still reads. */
 BAT_API bat_status bat_kv_evict(bat_pool p, int32_t kind, int64_t id);
 /* Host query of an entry: its token count and page ids (pages_out may be NULL). */
 BAT_API bat_status bat_kv_lookup(bat_pool p, int32_t kind, int64_t id, int32_t* n_tokens,
@@ -193,27 +194,31 @@ typedef struct {
 BAT_API bat_status bat_bipartite_prefill(bat_pool p, bat_model m, const bat_query* queries, int32_t B,
                                  float* out_hidden, bat_stream_t stream);
 
-/* s[b][i] = softmax_i(W_out[labels[b][i]] . hidden[b]) over i < n_items[b];
- * topk[b][0..k) = candidate indices by descending s (ties -> lower index).
+/* z[b][i] = W_out[labels[b][i]] . hidden[b] (the logit of item i's identifier token),
+ * s[b][i] = softmax_i z[b][i] over i < n_items[b]; topk[b][0..k) = candidate indices by
+ * descending s (ties -> lower index).
  * hidden: device fp32 [B][hidden]; labels: device int32 [B][n_max] (identifier token v_i,
- * P:177); n_items: device int32 [B]; scores: device fp32 [B][n_max] (entries >= n_items[b]
- * set to 0); topk: device int32 [B][k] or NULL when k = 0.  Requires n_max <= 4096,
- * k <= n_items. */
+ * P:177); n_items: device int32 [B] (values are clamped to [0, n_max]); scores: device fp32
+ * [B][n_max] (entries >= n_items[b] set to 0); topk: device int32 [B][k] or NULL when k = 0
+ * (ranks >= n_items[b] are -1); logits: device fp32 [B][n_max] receiving z (entries >= n_items[b]
+ * set to 0) or NULL.  Requires 1 <= n_max <= 4096 and k <= n_max. */
 BAT_API bat_status bat_score(bat_model m, const float* hidden, const int32_t* labels,
                      const int32_t* n_items, int32_t B, int32_t n_max, float* scores,
-                     int32_t k, int32_t* topk, bat_stream_t stream);
-/* Multi-discriminant scoring: s[b][i] = softmax_i(W_out[labels[b][i]] . hidden[b][i])
- * with hidden device fp32 [B][n_max][hidden] (bat_bipartite_prefill with multi_disc); the
- * other arguments as bat_score. */
+                     int32_t k, int32_t* topk, float* logits, bat_stream_t stream);
+/* Multi-discriminant scoring: z[b][i] = W_out[labels[b][i]] . hidden[b][i],
+ * s[b][i] = softmax_i z[b][i], with hidden device fp32 [B][n_max][hidden]
+ * (bat_bipartite_prefill with multi_disc); the other arguments as bat_score. */
 BAT_API bat_status bat_score_multi(bat_model m, const float* hidden, const int32_t* labels,
                                    const int32_t* n_items, int32_t B, int32_t n_max, float* scores,
-                                   int32_t k, int32_t* topk, bat_stream_t stream);
+                                   int32_t k, int32_t* topk, float* logits, bat_stream_t stream);
 
 /* ------------------------------------------------------------------------------------------
  * Planned execution: build (host) + upload (device, async on `stream`) the plan of a batch
  * once, then run it any number of times — the same computation as bat_bipartite_prefill
- * without the per-call planning and H2D upload.  The plan must be destroyed with
- * bat_plan_destroy; it is invalidated when a referenced pool entry is evicted.
+ * without the per-call planning and H2D upload.  The plan PINS every pool entry it reads:
+ * bat_kv_evict / bat_kv_release of a pinned entry fail with BAT_E_STATE until bat_plan_destroy,
+ * and bat_kv_pool_destroy fails while the pool has live plans.  bat_prefill_plan returns
+ * BAT_E_STATE for a plan built on another pool.
  * ---------------------------------------------------------------------------------------- */
 typedef struct bat_plan_s* bat_plan;
 BAT_API bat_status bat_plan_build(bat_pool p, bat_model m, const bat_query* queries, int32_t B,
@@ -260,6 +265,24 @@ enum {
 /* Copy field `field` of request b into out (cap elements); *count = its length. */
 BAT_API bat_status bat_plan_export(bat_plan plan, int32_t b, int32_t field, int32_t* out, int64_t cap,
                            int64_t* count);
+
+/* The DEVICE side of a bat_plan_build plan, read back and decoded exactly as the attention kernel
+ * consumes it (block-skip work list, per-q-tile tile states, the loader's page ids and the
+ * partial-tile visibility bits computed on the device), for bit-exact checks of the indexing the
+ * kernel sees (north_star "page-table and indexing results must match bit-exact").  Fields:
+ *   BAT_PFD_VIS       uint8 [S][n_ktiles*128]: 1 iff suffix row t attends key slot k in the
+ *                     all-row work list (state 1 = every slot, state 2 = the mask bits, unlisted
+ *                     or state-0 tiles = 0); layers 1..L-1 use it
+ *   BAT_PFD_VIS_LAST  the same for the last layer's list (only the last q-tile, P:173 trim)
+ *   BAT_PFD_KPAGES    int32 [n_ktiles*8]: page id each k-tile's loader copies (pool page >= 0,
+ *                     -(s+1) suffix scratch page s, INT32_MIN the all-zero pad page), or
+ *                     BAT_PFD_NOT_LOADED for a tile no work item lists (skipped)
+ * BAT_E_STATE if the device image is inconsistent: KV heads with different lists, a (q-tile,
+ * k-tile) pair listed twice, a partial tile without a mask, out-of-range indices. */
+enum { BAT_PFD_VIS = 0, BAT_PFD_VIS_LAST = 1, BAT_PFD_KPAGES = 2 };
+#define BAT_PFD_NOT_LOADED (-2147483647)
+BAT_API bat_status bat_plan_export_device(bat_plan plan, int32_t b, int32_t field, void* out, int64_t cap,
+                                          int64_t* count);
 
 /* ------------------------------------------------------------------------------------------
  * Multi-GPU: hot-replicated / cold-sharded item placement (Algorithm 1)

@@ -112,7 +112,7 @@ def plan_query(q, entity_pages: Dict[Tuple[int, int], Tuple[Sequence[int], int]]
     return dict(tokens=tokens[P:].astype(np.int64), pos=pos[P:].astype(np.int64), disc=disc,
                 seg=rseg, P=P, S=S, pages=np.array(pages, dtype=np.int64),
                 valid=np.array(valid, dtype=np.int64), n_prefix_pages=n_pre,
-                kseg=kseg_a, kord=kord_a, rord=rord, tile_state=state,
+                kseg=kseg_a, kord=kord_a, rord=rord, tile_state=state, vis=vis,
                 n_live_pairs=int(vis.sum()))
 
 

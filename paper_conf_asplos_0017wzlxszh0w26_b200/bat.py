@@ -104,7 +104,8 @@ def lib() -> ctypes.CDLL:
         "bat_kv_prefill_entities": (S, [c_void_p, c_void_p, c_int32, c_int32, POINTER(c_int64), POINTER(c_int32),
                                         POINTER(c_int32), c_int32, c_int32, c_int64, c_void_p]),
         "bat_bipartite_prefill": (S, [c_void_p, c_void_p, POINTER(bat_query), c_int32, c_void_p, c_void_p]),
-        "bat_score": (S, [c_void_p, c_void_p, c_void_p, c_void_p, c_int32, c_int32, c_void_p, c_int32, c_void_p, c_void_p]),
+        "bat_score": (S, [c_void_p, c_void_p, c_void_p, c_void_p, c_int32, c_int32, c_void_p, c_int32, c_void_p,
+                          c_void_p, c_void_p]),
         "bat_plan_create": (S, [c_void_p, c_int32, POINTER(bat_query), c_int32, POINTER(c_void_p)]),
         "bat_plan_destroy": (S, [c_void_p]),
         "bat_plan_query_info": (S, [c_void_p, c_int32, POINTER(c_int64)]),
@@ -129,7 +130,8 @@ def lib() -> ctypes.CDLL:
         "bat_debug_attention_layer": (S, [c_void_p, c_void_p, POINTER(bat_query), c_int32, c_int32, c_void_p,
                                           c_void_p, c_int32, c_void_p]),
         "bat_score_multi": (S, [c_void_p, c_void_p, c_void_p, c_void_p, c_int32, c_int32, c_void_p, c_int32, c_void_p,
-                                c_void_p]),
+                                c_void_p, c_void_p]),
+        "bat_plan_export_device": (S, [c_void_p, c_int32, c_int32, c_void_p, c_int64, POINTER(c_int64)]),
         "bat_sched_create": (S, [POINTER(bat_sched_cfg), POINTER(c_void_p)]),
         "bat_sched_destroy": (S, [c_void_p]),
         "bat_sched_decide": (S, [c_void_p, c_double, c_int64, c_int32, c_int32, POINTER(bat_sched_decision),
@@ -154,7 +156,8 @@ EXPORTED = ("bat_last_error", "bat_version", "bat_kernel_launch_count", "bat_mod
             "bat_kv_register_remote", "bat_kv_lookup_remote", "bat_kv_fetch", "bat_debug_gemm", "bat_debug_attention_layer",
             "bat_plan_build", "bat_prefill_plan", "bat_profile_enable", "bat_profile_read",
             "bat_profile_reset", "bat_debug_attach_peer_pool", "bat_sched_create", "bat_sched_destroy",
-            "bat_sched_decide", "bat_sched_stats", "bat_sched_is_cached", "bat_score_multi")
+            "bat_sched_decide", "bat_sched_stats", "bat_sched_is_cached", "bat_score_multi",
+            "bat_plan_export_device")
 
 
 def _check(status: int) -> None:
@@ -318,15 +321,15 @@ def bat_bipartite_prefill(pool: int, model: int, queries: QueryArray, out_hidden
 
 
 def bat_score(model: int, hidden, labels, n_items, B: int, n_max: int, scores, k: int = 0,
-              topk=None, stream=None) -> None:
+              topk=None, stream=None, logits=None) -> None:
     _check(lib().bat_score(model, _vp(hidden), _vp(labels), _vp(n_items), B, n_max, _vp(scores),
-                           k, _vp(topk), _vp(stream)))
+                           k, _vp(topk), _vp(logits), _vp(stream)))
 
 
 def bat_score_multi(model: int, hidden, labels, n_items, B: int, n_max: int, scores, k: int = 0,
-              topk=None, stream=None) -> None:
+                    topk=None, stream=None, logits=None) -> None:
     _check(lib().bat_score_multi(model, _vp(hidden), _vp(labels), _vp(n_items), B, n_max, _vp(scores),
-                           k, _vp(topk), _vp(stream)))
+                                 k, _vp(topk), _vp(logits), _vp(stream)))
 
 
 # ----------------------------------------------------------------------------- plan
@@ -355,6 +358,20 @@ def bat_plan_export(plan: int, b: int, field: int) -> np.ndarray:
     _check(lib().bat_plan_export(plan, b, field, None, 0, byref(n)))
     out = np.zeros(max(n.value, 1), dtype=np.int32)
     _check(lib().bat_plan_export(plan, b, field, _i32p(out), len(out), byref(n)))
+    return out[: n.value]
+
+
+BAT_PFD_VIS, BAT_PFD_VIS_LAST, BAT_PFD_KPAGES = range(3)
+BAT_PFD_NOT_LOADED = -2147483647
+
+
+def bat_plan_export_device(plan: int, b: int, field: int) -> np.ndarray:
+    """The device image of a bat_plan_build plan decoded as the attention kernel reads it:
+    VIS / VIS_LAST uint8 [S][n_ktiles*128]; KPAGES int32 [n_ktiles*8]."""
+    n = c_int64()
+    _check(lib().bat_plan_export_device(plan, b, field, None, 0, byref(n)))
+    out = np.zeros(max(n.value, 1), dtype=np.int32 if field == BAT_PFD_KPAGES else np.uint8)
+    _check(lib().bat_plan_export_device(plan, b, field, out.ctypes.data_as(c_void_p), len(out), byref(n)))
     return out[: n.value]
 
 

@@ -27,6 +27,9 @@ struct bat_plan_s {
   bat::Plan plan;
   void* dev_img = nullptr;  // device copy of plan.img (bat_plan_build)
   int device = -1;
+  bat_pool_s* pool = nullptr;              // the pool whose page ids the device image holds
+  std::vector<bat::EntityKey> pinned;      // entries pinned (not evictable) while the plan lives
+  std::vector<int32_t> dev_copy;           // host copy of the device image (bat_plan_export_device)
   ~bat_plan_s() {
     if (dev_img) cudaFree(dev_img);
   }
@@ -83,20 +86,6 @@ static CUtensorMap make_tmap(const void* ptr, int64_t rows, int64_t cols, int64_
   return m;
 }
 
-// a byte buffer viewed as rows of 128 bytes (64 bf16), box = box_rows rows, no swizzle: TMA
-// copies page blocks that are already in the tensor-core operand layout verbatim
-static CUtensorMap make_tmap_rows(const void* ptr, int64_t bytes, int box_rows) {
-  CUtensorMap m;
-  cuuint64_t dims[2] = {64, cuuint64_t(bytes / 128)};
-  cuuint64_t strides[1] = {128};
-  cuuint32_t box[2] = {64, cuuint32_t(box_rows)};
-  cuuint32_t estr[2] = {1, 1};
-  CUresult r = encode_fn()(&m, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 2, const_cast<void*>(ptr), dims, strides, box, estr,
-                           CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE,
-                           CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
-  if (r != CUDA_SUCCESS) fail(BAT_E_CUDA, "cuTensorMapEncodeTiled (rows) failed (" + std::to_string(int(r)) + ")");
-  return m;
-}
 
 // ------------------------------------------------------------------------ device buffer
 struct DevBuf {
@@ -104,15 +93,20 @@ struct DevBuf {
   size_t cap = 0;
   // zero: clear on (re)allocation — q-tiles and suffix pages rely on never-written padding
   // (head-dim padding columns, rows 126-127 of a q-tile) staying zero
-  void ensure(size_t bytes, bool zero = false) {
+  // (on `st`, the stream of the work that then writes into the buffer: ordered with it for any
+  // stream kind — a legacy-default-stream memset would not be with a non-blocking stream)
+  void ensure(size_t bytes, cudaStream_t st, bool zero = false) {
     if (bytes <= cap) return;
-    if (p) cudaFree(p);
+    if (p) {
+      CUDA_OK(cudaStreamSynchronize(st));  // the old buffer may still be read by queued work
+      cudaFree(p);
+    }
     p = nullptr;
     cap = 0;
     size_t want = std::max(bytes, size_t(1) << 16);
     want = (want + (want >> 2) + 255) & ~size_t(255);
     CUDA_OK(cudaMalloc(&p, want));
-    if (zero) CUDA_OK(cudaMemset(p, 0, want));
+    if (zero) CUDA_OK(cudaMemsetAsync(p, 0, want, st));
     cap = want;
   }
   ~DevBuf() {
@@ -282,22 +276,22 @@ static const int32_t* prepare(Pool& pool, Model& m, Plan& plan, cudaStream_t st,
     for (int32_t ps : q.pos) max_pos = std::max(max_pos, ps);
   ensure_rope(m, max_pos + 1, st);
   const size_t es = m.f32 ? 4 : 2;  // activation element size
-  ws.h.ensure(size_t(M) * H * 4);
-  ws.xn.ensure(size_t(M) * std::max(H, nq) * es);
-  ws.qkv.ensure(size_t(M) * m.nqkv() * es);
-  if (m.f32) ws.qp.ensure(size_t(M) * nq * 4);
-  else ws.qp.ensure(size_t(plan.n_qtiles_total) * c.kv_heads * tile_bytes, true);
-  ws.scratch.ensure(size_t(std::max(plan.n_spages, 1)) * pool.geo.layer_bytes, true);
-  ws.o.ensure(size_t(M) * nq * es);
-  ws.act.ensure(size_t(M) * F * es);
+  ws.h.ensure(size_t(M) * H * 4, st);
+  ws.xn.ensure(size_t(M) * std::max(H, nq) * es, st);
+  ws.qkv.ensure(size_t(M) * m.nqkv() * es, st);
+  if (m.f32) ws.qp.ensure(size_t(M) * nq * 4, st);
+  else ws.qp.ensure(size_t(plan.n_qtiles_total) * c.kv_heads * tile_bytes, st, true);
+  ws.scratch.ensure(size_t(std::max(plan.n_spages, 1)) * pool.geo.layer_bytes, st, true);
+  ws.o.ensure(size_t(M) * nq * es, st);
+  ws.act.ensure(size_t(M) * F * es, st);
   const size_t D = size_t(B) * plan.n_disc;  // discriminant rows
-  ws.hc.ensure(D * H * 4);
-  ws.xc.ensure(D * H * es);
-  ws.oc.ensure(D * nq * es);
-  ws.actc.ensure(D * F * es);
+  ws.hc.ensure(D * H * 4, st);
+  ws.xc.ensure(D * H * es, st);
+  ws.oc.ensure(D * nq * es, st);
+  ws.actc.ensure(D * F * es, st);
   if (dev_img) return dev_img;
   const size_t img_bytes = plan.img.buf.size() * 4;
-  ws.img.ensure(size_t(plan.img.total_ints) * 4);
+  ws.img.ensure(size_t(plan.img.total_ints) * 4, st);
   if (!ws.img_done) CUDA_OK(cudaEventCreateWithFlags(&ws.img_done, cudaEventDisableTiming));
   CUDA_OK(cudaEventSynchronize(ws.img_done));  // the previous upload finished reading the staging buffer
   if (ws.img_host_cap < img_bytes) {
@@ -342,23 +336,9 @@ static AttnParams attn_params(const Pool& pool, const Model& m, const Plan& plan
   return ap;
 }
 
-// a5 launch: the CTA-pair kernel (head_dim 128) or the 1-CTA kernel
-static void run_attention(const Pool& pool, const Model& m, const Plan& plan, const AttnParams& ap, cudaStream_t st) {
-  if (!attn_pair_supported(m.dpad)) {
-    launch_attention(m.dpad, ap, m.num_sms, st);
-    return;
-  }
-  AttnPairParams pp{};
-  const int64_t arena_bytes = int64_t(pool.cfg.num_pages + 1) * pool.geo.page_bytes;
-  pp.tm_pool_k = make_tmap_rows(pool.arena, arena_bytes, 32);
-  pp.tm_pool_v = pp.tm_pool_k;  // whole 4 KB page blocks for V too
-  const int64_t scr_bytes = int64_t(std::max(plan.n_spages, 1)) * pool.geo.layer_bytes;
-  pp.tm_scr_k = make_tmap_rows(m.ws.scratch.p, scr_bytes, 32);
-  pp.tm_scr_v = pp.tm_scr_k;
-  pp.tm_q = make_tmap_rows(m.ws.qp.p, int64_t(plan.n_qtiles_total) * plan.kv_heads * 32768, 256);
-  pp.a = ap;
-  pp.zero_row = int64_t(pool.zero_page) * pool.geo.page_bytes / 128;
-  launch_attention_pair(pp, m.num_sms, st);
+// a5 launch (persistent tcgen05 kernel, one CTA per SM)
+static void run_attention(const Pool&, const Model& m, const Plan&, const AttnParams& ap, cudaStream_t st) {
+  launch_attention(m.dpad, ap, m.num_sms, st);
 }
 
 static StageParams stage_params(const Pool& pool, const Model& m, const Plan& plan, const int32_t* I) {
@@ -732,6 +712,7 @@ bat_status bat_kv_pool_create(const bat_pool_cfg* cfg, bat_pool* out) {
 bat_status bat_kv_pool_destroy(bat_pool p) {
   return guarded([&] {
     if (!p) return;
+    if (p->pool.live_plans > 0) fail(BAT_E_STATE, "destroy the pool's plans (bat_plan_destroy) first");
     if (p->pool.arena) {
       DeviceGuard dg(p->pool.device);
       cudaDeviceSynchronize();
@@ -780,6 +761,7 @@ bat_status bat_kv_evict(bat_pool p, int32_t kind, int64_t id) {
     Pool& P = p->pool;
     auto it = P.index.find(EntityKey{kind, id});
     if (it == P.index.end()) fail(BAT_E_NOTFOUND, "entry not found");
+    if (it->second.pins > 0) fail(BAT_E_STATE, "entry is referenced by a live plan (bat_plan_build)");
     P.release_pages(it->second.pages);
     P.index.erase(it);
   });
@@ -963,7 +945,8 @@ bat_status bat_bipartite_prefill(bat_pool p, bat_model mdl, const bat_query* que
 }
 
 bat_status bat_score_multi(bat_model mdl, const float* hidden, const int32_t* labels, const int32_t* n_items,
-                           int32_t B, int32_t n_max, float* scores, int32_t k, int32_t* topk, bat_stream_t stream) {
+                           int32_t B, int32_t n_max, float* scores, int32_t k, int32_t* topk, float* logits,
+                           bat_stream_t stream) {
   return guarded([&] {
     BAT_REQUIRE(mdl && hidden && labels && n_items && scores, "null argument");
     BAT_REQUIRE(B >= 1 && n_max >= 1 && n_max <= 4096, "B >= 1, 1 <= n_max <= 4096");
@@ -971,13 +954,15 @@ bat_status bat_score_multi(bat_model mdl, const float* hidden, const int32_t* la
     Model& m = mdl->m;
     DeviceGuard dg(m.device);
     launch_score_multi(hidden, m.f32 ? nullptr : m.lm_head, m.f32 ? static_cast<const float*>(m.w[BAT_W_LM_HEAD]) : nullptr,
-                       labels, n_items, B, n_max, m.cfg.hidden, scores, k, topk, static_cast<cudaStream_t>(stream));
+                       labels, n_items, B, n_max, m.cfg.hidden, scores, k, topk, logits,
+                       static_cast<cudaStream_t>(stream));
     CUDA_OK(cudaGetLastError());
   });
 }
 
 bat_status bat_score(bat_model mdl, const float* hidden, const int32_t* labels, const int32_t* n_items,
-                     int32_t B, int32_t n_max, float* scores, int32_t k, int32_t* topk, bat_stream_t stream) {
+                     int32_t B, int32_t n_max, float* scores, int32_t k, int32_t* topk, float* logits,
+                     bat_stream_t stream) {
   return guarded([&] {
     BAT_REQUIRE(mdl && hidden && labels && n_items && scores, "null argument");
     BAT_REQUIRE(B >= 1 && n_max >= 1 && n_max <= 4096, "B >= 1, 1 <= n_max <= 4096");
@@ -987,9 +972,9 @@ bat_status bat_score(bat_model mdl, const float* hidden, const int32_t* labels, 
     DeviceGuard dg(m.device);
     if (m.f32)
       launch_score_f32w(hidden, static_cast<const float*>(m.w[BAT_W_LM_HEAD]), labels, n_items, B, n_max,
-                        m.cfg.hidden, scores, k, topk, static_cast<cudaStream_t>(stream));
+                        m.cfg.hidden, scores, k, topk, logits, static_cast<cudaStream_t>(stream));
     else
-      launch_score(hidden, m.lm_head, labels, n_items, B, n_max, m.cfg.hidden, scores, k, topk,
+      launch_score(hidden, m.lm_head, labels, n_items, B, n_max, m.cfg.hidden, scores, k, topk, logits,
                    static_cast<cudaStream_t>(stream));
     CUDA_OK(cudaGetLastError());
   });
@@ -1006,7 +991,18 @@ bat_status bat_plan_create(bat_pool p, int32_t group, const bat_query* queries, 
 }
 
 bat_status bat_plan_destroy(bat_plan plan) {
-  return guarded([&] { delete plan; });
+  return guarded([&] {
+    if (!plan) return;
+    if (plan->pool) {
+      Pool& P = plan->pool->pool;
+      for (const EntityKey& k : plan->pinned) {
+        auto it = P.index.find(k);
+        if (it != P.index.end() && it->second.pins > 0) --it->second.pins;
+      }
+      --P.live_plans;
+    }
+    delete plan;
+  });
 }
 
 bat_status bat_plan_query_info(bat_plan plan, int32_t b, int64_t info[13]) {
@@ -1044,6 +1040,84 @@ bat_status bat_plan_export(bat_plan plan, int32_t b, int32_t field, int32_t* out
     if (out) {
       BAT_REQUIRE(cap >= int64_t(src->size()), "cap too small");
       std::copy(src->begin(), src->end(), out);
+    }
+  });
+}
+
+// Decode the DEVICE copy of a bat_plan_build plan the way the attention kernel reads it: the
+// work list (per KV head: q-tile pair, listed k-tiles, their per-q-tile state and the page ids
+// the loader copies) and the partial-tile visibility masks mask_kernel wrote on the device.
+bat_status bat_plan_export_device(bat_plan plan, int32_t b, int32_t field, void* out, int64_t cap, int64_t* count) {
+  return guarded([&] {
+    BAT_REQUIRE(plan && plan->dev_img, "plan built with bat_plan_build");
+    const Plan& pl = plan->plan;
+    BAT_REQUIRE(b >= 0 && b < int32_t(pl.q.size()), "request index");
+    BAT_REQUIRE(field >= BAT_PFD_VIS && field <= BAT_PFD_KPAGES, "field");
+    const PlanImage& im = pl.img;
+    if (plan->dev_copy.empty()) {
+      DeviceGuard dg(plan->device);
+      plan->dev_copy.resize(size_t(im.total_ints));
+      CUDA_OK(cudaMemcpy(plan->dev_copy.data(), plan->dev_img, size_t(im.total_ints) * 4, cudaMemcpyDeviceToHost));
+    }
+    const std::vector<int32_t>& I = plan->dev_copy;
+    const QueryPlan& q = pl.q[b];
+    const int64_t n_cols = int64_t(q.n_ktiles) * kKtile;
+    const bool last = field == BAT_PFD_VIS_LAST;
+    const int64_t off_work = last ? im.off_work_last : im.off_work;
+    const int32_t n_work = last ? pl.n_work_last : pl.n_work;
+    // per KV head: decoded visibility [S][n_cols] and the loaded page ids [n_ktiles * 8]
+    std::vector<std::vector<uint8_t>> vis(pl.kv_heads, std::vector<uint8_t>(size_t(q.S) * n_cols, 0));
+    std::vector<std::vector<int32_t>> kp(pl.kv_heads, std::vector<int32_t>(size_t(q.n_ktiles) * kKtilePages, BAT_PFD_NOT_LOADED));
+    std::vector<std::vector<uint8_t>> seen(pl.kv_heads, std::vector<uint8_t>(size_t(q.n_qtiles) * q.n_ktiles, 0));
+    for (int32_t w = 0; w < n_work; ++w) {
+      const int32_t* e = &I[size_t(off_work + int64_t(w) * 8)];
+      if (e[5] == 0 || e[0] != b) continue;  // LPT padding / another request
+      const int kvh = e[1];
+      if (kvh < 0 || kvh >= pl.kv_heads) fail(BAT_E_STATE, "work item KV head out of range");
+      for (int x = 0; x < e[5]; ++x) {
+        const int32_t ktl = I[size_t(e[4] + x)];
+        const int32_t j = ktl & 0xFFFFFF;
+        if (j < 0 || j >= q.n_ktiles) fail(BAT_E_STATE, "listed k-tile out of range");
+        for (int l = 0; l < kKtilePages; ++l) {
+          const int32_t pg = I[size_t(e[6] + int64_t(x) * kKtilePages + l)];
+          int32_t& slot = kp[kvh][size_t(j) * kKtilePages + l];
+          if (slot != BAT_PFD_NOT_LOADED && slot != pg) fail(BAT_E_STATE, "k-tile loaded with two page lists");
+          slot = pg;
+        }
+        for (int h = 0; h < 2; ++h) {
+          const int qi = h == 0 ? e[2] : e[3];
+          if (qi < 0) continue;
+          const int st = (ktl >> (24 + 2 * h)) & 3;
+          if (st == 0) continue;
+          if (qi >= q.n_qtiles) fail(BAT_E_STATE, "q-tile out of range");
+          uint8_t& sn = seen[kvh][size_t(qi) * q.n_ktiles + j];
+          if (sn) fail(BAT_E_STATE, "(q-tile, k-tile) pair listed twice");
+          sn = 1;
+          const int32_t mid = I[size_t(e[7] + 2 * x + h)];
+          if (st == 2 && (mid < 0 || mid >= im.n_masks)) fail(BAT_E_STATE, "partial tile without a mask");
+          for (int r = 0; r < pl.qt; ++r) {
+            const int t = qi * pl.qt + r;
+            if (t >= q.S) break;
+            uint8_t* row = &vis[kvh][size_t(t) * n_cols + int64_t(j) * kKtile];
+            if (st == 1) {
+              std::fill(row, row + kKtile, uint8_t(1));
+            } else {
+              const int32_t* mw = &I[size_t(im.off_masks + (int64_t(mid) * (pl.qt + 1) + r) * 4)];
+              for (int k = 0; k < kKtile; ++k) row[k] = uint8_t((uint32_t(mw[k >> 5]) >> (k & 31)) & 1u);
+            }
+          }
+        }
+      }
+    }
+    for (int h = 1; h < pl.kv_heads; ++h)
+      if (vis[h] != vis[0] || kp[h] != kp[0]) fail(BAT_E_STATE, "KV heads see different tile lists");
+    const bool pages = field == BAT_PFD_KPAGES;
+    const int64_t n = pages ? int64_t(kp[0].size()) : int64_t(vis[0].size());
+    if (count) *count = n;
+    if (out) {
+      BAT_REQUIRE(cap >= n, "cap too small");
+      if (pages) std::copy(kp[0].begin(), kp[0].end(), static_cast<int32_t*>(out));
+      else std::copy(vis[0].begin(), vis[0].end(), static_cast<uint8_t*>(out));
     }
   });
 }
@@ -1326,6 +1400,17 @@ bat_status bat_plan_build(bat_pool p, bat_model mdl, const bat_query* queries, i
     DeviceGuard dg(P.device);
     auto pl = std::make_unique<bat_plan_s>();
     build_plan(P, m.cfg.q_heads / m.cfg.kv_heads, m.cfg.kv_heads, wrap(queries, B), pl->plan, true, attn_grid_slots(m.dpad, m.num_sms));
+    // the device image bakes in page ids: pin every referenced entry until bat_plan_destroy
+    for (const QueryPlan& q : pl->plan.q)
+      for (const EntityKey& k : q.refs) {
+        auto it = P.index.find(k);
+        if (it != P.index.end()) {
+          ++it->second.pins;
+          pl->pinned.push_back(k);
+        }
+      }
+    pl->pool = p;
+    ++P.live_plans;
     const size_t bytes = pl->plan.img.buf.size() * 4;
     CUDA_OK(cudaMalloc(&pl->dev_img, size_t(pl->plan.img.total_ints) * 4));
     CUDA_OK(cudaMemcpyAsync(pl->dev_img, pl->plan.img.buf.data(), bytes, cudaMemcpyHostToDevice,
@@ -1345,6 +1430,7 @@ bat_status bat_prefill_plan(bat_pool p, bat_model mdl, bat_plan plan, float* out
     Model& m = mdl->m;
     check_compat(P, m);
     BAT_REQUIRE(!plan->plan.entity_mode && plan->plan.kv_heads == m.cfg.kv_heads, "plan / model mismatch");
+    if (plan->pool != p) fail(BAT_E_STATE, "plan was built for another pool");
     DeviceGuard dg(P.device);
     run_plan(P, m, plan->plan, out_hidden, static_cast<cudaStream_t>(stream),
              static_cast<const int32_t*>(plan->dev_img));

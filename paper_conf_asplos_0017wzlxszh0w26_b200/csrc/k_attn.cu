@@ -732,376 +732,9 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) attn_tc_kernel(const __grid_co
   if (warp == 1) ptx::tmem_dealloc(tmem, 512);
 }
 
-// ==========================================================================================
-// Double-buffered variant (BAT_ATTN=db; measured slower, see launch_attention): every 128-key k-tile is processed as two 64-key
-// sub-tiles, and each q-tile owns TWO 64-column S buffers, so S_{u+2} = Q K_{u+2}^T is issued
-// as soon as P_u has been consumed by its P.V and is ready long before the softmax of sub-tile
-// u+1 ends — the S -> softmax -> P.V chain of a q-tile is no longer exposed on the tensor pipe.
-// One softmax warpgroup per q-tile, one thread per row owning all 64 columns of a sub-tile
-// (no cross-thread max agreement).  TMEM: O0 [0,128) O1 [128,256) S(q,b) at 256 + 128 q + 64 b.
-// Warps: 0 Q+K loader, 1 MMA issuer, 2/3 V-half loaders, 4-7 softmax q-tile 0, 8-11 q-tile 1.
-constexpr int DB_THREADS = 384;
-// debug timeline (bat_debug_attention_layer + BAT_ATTN_TIMELINE): event ev of the i-th sub-tile of CTA 0
-#define DBT(ev, i)                                                                     \
-  do {                                                                                 \
-    if (p.dbg && blockIdx.x == 0 && (i) < 64) p.dbg[(ev) * 64 + (i)] = clock64();      \
-  } while (0)
-
-struct __align__(8) DbBars {
-  uint64_t q_full, q_empty;
-  uint64_t k_full[3], k_empty[3], v_full[3], v_empty[3];
-  uint64_t s_full[2][2], p_full[2][2];
-  uint64_t o_full[2], o_empty[2], pv_done[2];
-  uint32_t tmem_base;
-};
-static_assert(sizeof(DbBars) <= 256, "barrier area");
-
-template <int DP>
-__global__ void __launch_bounds__(DB_THREADS, 1) attn_db_kernel(const __grid_constant__ AttnParams p) {
-  using L = AttnSmem<DP>;
-  extern __shared__ uint8_t smem_raw[];
-  uint8_t* smem = smem_raw + ((1024u - (ptx::smem_u32(smem_raw) & 1023u)) & 1023u);
-  DbBars* bars = reinterpret_cast<DbBars*>(smem + L::BAR_OFF);
-  const uint32_t warp = ptx::warp_id(), lane = ptx::lane_id();
-  constexpr uint32_t IDESC_S = ptx::idesc_bf16(128, 64, 0, 0);
-  constexpr uint32_t IDESC_PV = ptx::idesc_bf16(128, DP, 0, 1);
-
-  if (warp == 0 && lane == 0) {
-    ptx::mbar_init(&bars->q_full, 1);
-    ptx::mbar_init(&bars->q_empty, 1);
-    for (int i = 0; i < 3; ++i) {
-      ptx::mbar_init(&bars->k_full[i], 1);
-      ptx::mbar_init(&bars->k_empty[i], 1);
-      ptx::mbar_init(&bars->v_full[i], 1);
-      ptx::mbar_init(&bars->v_empty[i], 1);
-    }
-    for (int q = 0; q < 2; ++q) {
-      for (int b = 0; b < 2; ++b) {
-        ptx::mbar_init(&bars->s_full[q][b], 1);
-        ptx::mbar_init(&bars->p_full[q][b], 4);
-      }
-      ptx::mbar_init(&bars->o_full[q], 1);
-      ptx::mbar_init(&bars->o_empty[q], 4);
-      ptx::mbar_init(&bars->pv_done[q], 1);
-    }
-    ptx::fence_mbar_init();
-  }
-  if (warp == 1) ptx::tmem_alloc(&bars->tmem_base, 512);
-  ptx::tc_fence_before();
-  __syncthreads();
-  ptx::tc_fence_after();
-  const uint32_t tmem = bars->tmem_base;
-
-  const int32_t* img = p.img;
-  const int32_t* work = img + p.off_work;
-
-  if (warp == 0 || warp == 2 || warp == 3) {  // ------------------------------------ loaders
-    // identical streams to attn_tc_kernel: warp 0 Q + K tiles, warps 2 / 3 the V halves
-    const int role = warp == 0 ? 0 : int(warp) - 1;
-    uint32_t qc = 0, kc = 0;
-    const bool pl = lane < kKtilePages;
-    constexpr int32_t kNone = kZeroPage + 1;
-    auto ids = [&](const WorkItem& a, const WorkItem& n, int t) -> int32_t {
-      if (!pl) return kNone;
-      if (t < a.kt_n) return img[a.tp_off + t * kKtilePages + lane];
-      t -= a.kt_n;
-      if (t < n.kt_n) return img[n.tp_off + t * kKtilePages + lane];
-      return kNone;
-    };
-    const int64_t kv_off = role == 0 ? 0 : int64_t(p.kv_heads) * p.head_bytes;
-    const WorkItem none{0, 0, -1, -1, 0, 0, 0, 0};
-    for (int w = blockIdx.x; w < p.n_work; w += gridDim.x) {
-      const WorkItem wi = load_work(work, w);
-      if (wi.kt_n == 0) continue;
-      const WorkItem nx = (w + int(gridDim.x) < p.n_work) ? load_work(work, w + gridDim.x) : none;
-      const int32_t* q_info = img + p.off_qinfo + int64_t(wi.b) * 8;
-      const int qtile0 = q_info[2];
-      int32_t pa = ids(wi, nx, 0), pb = ids(wi, nx, 1), pc = ids(wi, nx, 2);
-      if (role == 0 && lane == 0) {
-        ptx::mbar_wait(&bars->q_empty, (qc & 1) ^ 1);
-        const int nq = wi.q1 >= 0 ? 2 : 1;
-        ptx::mbar_expect_tx(&bars->q_full, nq * L::TILE_BYTES);
-        const char* qbase = reinterpret_cast<const char*>(p.qp);
-        ptx::bulk_g2s(smem + L::Q_OFF, qbase + (int64_t(qtile0 + wi.q0) * p.kv_heads + wi.kvh) * L::TILE_BYTES,
-                      L::TILE_BYTES, &bars->q_full);
-        if (wi.q1 >= 0)
-          ptx::bulk_g2s(smem + L::Q_OFF + L::TILE_BYTES,
-                        qbase + (int64_t(qtile0 + wi.q1) * p.kv_heads + wi.kvh) * L::TILE_BYTES, L::TILE_BYTES,
-                        &bars->q_full);
-      }
-      for (int x = 0; x < wi.kt_n; ++x, ++kc) {
-        const int32_t pd = ids(wi, nx, x + 3);
-        if (role == 0) {
-          const char* src[kKtilePages];
-#pragma unroll
-          for (int i = 0; i < kKtilePages; ++i) src[i] = resolve_page(p, __shfl_sync(0xffffffffu, pa, i));
-          if (lane == 0) {
-            const uint32_t ks = ring_slot(kc);
-            uint8_t* sk = smem + L::K_OFF + ks * L::TILE_BYTES;
-            ptx::mbar_wait(&bars->k_empty[ks], ring_phase(kc) ^ 1);
-            ptx::mbar_expect_tx(&bars->k_full[ks], kKtilePages * L::PAGE_BYTES);
-#pragma unroll
-            for (int i = 0; i < kKtilePages; ++i)
-              ptx::bulk_g2s(sk + i * L::PAGE_BYTES, src[i] + int64_t(wi.kvh) * p.head_bytes, L::PAGE_BYTES,
-                            &bars->k_full[ks]);
-          }
-        } else {
-          const int hf = role - 1;
-          const char* src[4];
-#pragma unroll
-          for (int i = 0; i < 4; ++i) src[i] = resolve_page(p, __shfl_sync(0xffffffffu, pa, 4 * hf + i));
-          if (lane == 0) {
-            const uint32_t vi = 2 * kc + hf, vs = ring_slot(vi);
-            uint8_t* sv = smem + L::V_OFF + vs * L::HALF_BYTES;
-            ptx::mbar_wait(&bars->v_empty[vs], ring_phase(vi) ^ 1);
-            ptx::mbar_expect_tx(&bars->v_full[vs], 4 * L::PAGE_BYTES);
-#pragma unroll
-            for (int i = 0; i < 4; ++i)
-              ptx::bulk_g2s(sv + i * L::PAGE_BYTES, src[i] + kv_off + int64_t(wi.kvh) * p.head_bytes, L::PAGE_BYTES,
-                            &bars->v_full[vs]);
-          }
-        }
-        __syncwarp();
-        pa = pb;
-        pb = pc;
-        pc = pd;
-      }
-      ++qc;
-    }
-  } else if (warp == 1) {  // ---------------------------------------------- MMA issuer
-    // the whole warp runs the issuer (converged: uniform-register descriptor math); every
-    // tcgen05.mma / commit is issued by one elected lane
-    {
-      const uint32_t sq_base = ptx::smem_u32(smem + L::Q_OFF);
-      uint32_t qc = 0;                    // Q tiles consumed (q_full phase)
-      uint32_t scnt[2] = {0, 0};          // S issued per q-tile (buffer = scnt & 1)
-      uint32_t pcnt[2] = {0, 0};          // P.V issued per q-tile
-      uint32_t oc[2] = {0, 0};            // items finished per q-tile (o_empty phase)
-      auto sk_of = [&](uint32_t g) { return ptx::smem_u32(smem + L::K_OFF + ring_slot(g) * L::TILE_BYTES); };
-      auto sv_of = [&](uint32_t vi) { return ptx::smem_u32(smem + L::V_OFF + ring_slot(vi) * L::HALF_BYTES); };
-      auto tS_of = [&](int q, uint32_t b) { return tmem + 256 + q * 128 + b * 64; };
-      // S(q, u) of item `it` whose first K tile is global tile kb: 64 keys [64 (u&1), +64) of tile kb + u/2
-      auto issue_s = [&](const WorkItem& it, int q, int u, uint32_t kb) {
-        const uint32_t g = kb + (u >> 1);
-        ptx::mbar_wait(&bars->k_full[ring_slot(g)], ring_phase(g));
-        DBT(16 + 2 * q, scnt[q]);
-        ptx::tc_fence_after();
-        const uint32_t sq = sq_base + q * L::TILE_BYTES;
-        const uint32_t sk = sk_of(g) + (u & 1) * 4 * L::PAGE_BYTES;
-        const uint32_t tS = tS_of(q, scnt[q] & 1);
-#pragma unroll
-        for (int kk = 0; kk < DP / 16; ++kk) {
-          const uint32_t qoff = (kk >> 2) * 16384 + (kk & 3) * 32;
-          const uint32_t koff = (kk >> 2) * 1024 + (kk & 3) * 32;
-          ptx::mma_ss_elect(tS, ptx::desc_sw128(sq + qoff, 16, 1024), ptx::desc_sw128(sk + koff, 16, L::GROUP_BYTES),
-                      IDESC_S, kk ? 1u : 0u);
-        }
-        DBT(17 + 2 * q, scnt[q]);
-        ptx::mma_commit_elect(&bars->s_full[q][scnt[q] & 1]);
-        DBT(q ? 1 : 0, scnt[q]);
-        ++scnt[q];
-        const bool lastq = (q == 1) || it.q1 < 0;
-        if ((u & 1) && lastq) ptx::mma_commit_elect(&bars->k_empty[ring_slot(g)]);
-        if (u == 2 * it.kt_n - 1 && lastq) ptx::mma_commit_elect(&bars->q_empty);
-      };
-      auto next_item = [&](int w) {
-        for (w += gridDim.x; w < p.n_work; w += gridDim.x)
-          if (work[int64_t(w) * 8 + 5] > 0) break;
-        return w;
-      };
-      int w = blockIdx.x;
-      if (w < p.n_work && work[int64_t(w) * 8 + 5] == 0) w = next_item(w);
-      uint32_t kb = 0;
-      int pre[2] = {0, 0};        // S of the current item already issued during the previous one
-      bool q_waited = false;      // q_full of the current item already consumed
-      while (w < p.n_work) {
-        const WorkItem wi = load_work(work, w);
-        const bool has1 = wi.q1 >= 0;
-        const int n2 = 2 * wi.kt_n;
-        if (!q_waited) {
-          ptx::mbar_wait(&bars->q_full, qc & 1);
-          ++qc;
-        }
-        // S of sub-tiles 0 and 1 not issued ahead
-        for (int u = 0; u < 2; ++u)
-          for (int q = 0; q < 2; ++q)
-            if ((q == 0 || has1) && pre[q] <= u) issue_s(wi, q, u, kb);
-        const int wn = next_item(w);
-        const WorkItem wni = wn < p.n_work ? load_work(work, wn) : WorkItem{0, 0, -1, -1, 0, 0, 0, 0};
-        int npre[2] = {0, 0};
-        bool nq_waited = false;
-        for (int u = 0; u < n2; ++u) {
-          const uint32_t vh = 2 * (kb + (u >> 1)) + (u & 1);
-          for (int q = 0; q < 2; ++q) {
-            if (q == 1 && !has1) continue;
-            const uint32_t b = pcnt[q] & 1;
-            DBT(2 + q, pcnt[q]);
-            ptx::mbar_wait(&bars->p_full[q][b], (pcnt[q] >> 1) & 1);
-            DBT(4 + q, pcnt[q]);
-            if (u == 0) ptx::mbar_wait(&bars->o_empty[q], (oc[q] & 1) ^ 1);
-            if (q == 0) ptx::mbar_wait(&bars->v_full[ring_slot(vh)], ring_phase(vh));
-            DBT(6 + q, pcnt[q]);
-            ptx::tc_fence_after();
-            const uint32_t tO = tmem + q * 128, tP = tS_of(q, b), sv = sv_of(vh);
-#pragma unroll
-            for (int i = 0; i < 4; ++i)
-              ptx::mma_ts_elect(tO, tP + i * 8, ptx::desc_sw128(sv + i * L::PAGE_BYTES, 1024, L::GROUP_BYTES), IDESC_PV,
-                          (u || i) ? 1u : 0u);
-            ptx::mma_commit_elect(&bars->pv_done[q]);
-            ++pcnt[q];
-            if (u == n2 - 1) {
-              ptx::mma_commit_elect(&bars->o_full[q]);
-              ++oc[q];
-            }
-            if (q == 1 || !has1) ptx::mma_commit_elect(&bars->v_empty[ring_slot(vh)]);
-            // the S two sub-tiles ahead in this q-tile's stream (maybe the next item's)
-            if (u + 2 < n2) {
-              issue_s(wi, q, u + 2, kb);
-            } else if (wn < p.n_work && (q == 0 || wni.q1 >= 0)) {
-              // The next item's S are issued ahead only as an in-order prefix of S(0,0) S(1,0)
-              // S(0,1) S(1,1) (the K-tile / Q releases ride on the last of them), and only if
-              // its Q is already resident (never stall the P.V stream on it).
-              const int un = u + 2 - n2;
-              if (q == 0 && un == 0 && __shfl_sync(0xffffffffu, int(ptx::mbar_test(&bars->q_full, qc & 1)), 0)) {
-                nq_waited = true;
-                ++qc;
-              }
-              if (nq_waited && npre[q] == un && (q == 0 || npre[0] > un)) {
-                issue_s(wni, q, un, kb + wi.kt_n);
-                ++npre[q];
-              }
-            }
-          }
-        }
-        kb += wi.kt_n;
-        pre[0] = npre[0];
-        pre[1] = npre[1];
-        q_waited = nq_waited;
-        w = wn;
-      }
-    }
-  } else {  // ------------------------------------------------------- softmax warpgroups
-    const int q = (warp - 4) >> 2;
-    const uint32_t sub = warp & 3;
-    const int row = sub * 32 + lane;
-    const uint32_t lane_base = (sub * 32) << 16;
-    const uint32_t tO = tmem + q * 128 + lane_base;
-    constexpr int OCH = DP / 32;
-    uint32_t cnt = 0, oc = 0;
-    for (int w = blockIdx.x; w < p.n_work; w += gridDim.x) {
-      const WorkItem wi = load_work(work, w);
-      const int qi = q == 0 ? wi.q0 : wi.q1;
-      if (qi < 0 || wi.kt_n == 0) continue;
-      const int32_t* q_info = img + p.off_qinfo + int64_t(wi.b) * 8;
-      const int tok_off = q_info[0], S = q_info[1];
-      const int tok_local = qi * p.qt + row / p.group;
-      const bool valid_row = row < p.qt * p.group && tok_local < S;
-      const int mrow = valid_row ? row / p.group : p.qt;
-      const int32_t* ktl = img + wi.kt_off;
-      float m_ref = -INFINITY, l_sum = 0.0f;
-      for (int x = 0; x < wi.kt_n; ++x) {
-        const int state = (ktl[x] >> (24 + 2 * q)) & 3;
-        uint4 mv = make_uint4(~0u, ~0u, ~0u, ~0u);
-        if (state == 2) {
-          const int mid = img[wi.km_off + 2 * x + q];
-          mv = __ldg(reinterpret_cast<const uint4*>(img + p.off_masks + (int64_t(mid) * (p.qt + 1) + mrow) * 4));
-        }
-#pragma unroll
-        for (int hf = 0; hf < 2; ++hf) {
-          const uint32_t b = cnt & 1;
-          const uint32_t tS = tmem + 256 + q * 128 + b * 64 + lane_base;
-          const uint32_t vis[NCH] = {hf ? mv.z : mv.x, hf ? mv.w : mv.y};
-          if (sub == 0 && lane == 0) DBT(8 + q, cnt);
-          ptx::mbar_wait(&bars->s_full[q][b], (cnt >> 1) & 1);
-          if (sub == 0 && lane == 0) DBT(10 + q, cnt);
-          ptx::tc_fence_after();
-          bool done = false;
-          float lsum = 0.0f;
-          if (state == 0) {
-            row_zero_p<NCH>(tS);
-            done = true;
-          } else if (__all_sync(0xffffffffu, m_ref != -INFINITY)) {
-            const uint64_t sc2 = pk2(p.scale_log2, p.scale_log2), nm2 = pk2(-m_ref, -m_ref);
-            auto agree = [](bool ok) { return ok; };
-            done = (state == 1) ? row_exp_opt<false>(tS, vis, sc2, nm2, kRescaleThreshold, lsum, agree)
-                                : row_exp_opt<true>(tS, vis, sc2, nm2, kRescaleThreshold, lsum, agree);
-          }
-          if (!done) {
-            const float mt = (state == 1) ? row_max<false>(tS, vis) : row_max<true>(tS, vis);
-            const float m_old = m_ref;
-            const float m_new = fmaxf(m_ref, mt * p.scale_log2);
-            const bool grow = m_new > m_ref + kRescaleThreshold;
-            float alpha = 1.0f;
-            if (grow) {
-              alpha = ex2(m_ref - m_new);
-              l_sum *= alpha;
-              m_ref = m_new;
-            }
-            const bool need_o = grow && (m_old != -INFINITY);
-            if (__any_sync(0xffffffffu, need_o)) {
-              // O must hold every earlier P.V of this item: wait for the previous one (at most
-              // one is outstanding: S of this sub-tile was issued after the one before it)
-              ptx::mbar_wait(&bars->pv_done[q], (cnt - 1) & 1);
-              ptx::tc_fence_after();
-              const float a = need_o ? alpha : 1.0f;
-#pragma unroll 1
-              for (int c = 0; c < OCH; ++c) {
-                uint32_t r[32];
-                ptx::tmem_ld32(tO + c * 32, r);
-                ptx::tmem_ld_wait();
-#pragma unroll
-                for (int i = 0; i < 32; ++i) r[i] = __float_as_uint(__uint_as_float(r[i]) * a);
-                ptx::tmem_st32(tO + c * 32, r);
-              }
-            }
-            const float mref = (m_ref == -INFINITY) ? 0.0f : m_ref;
-            const uint64_t sc2 = pk2(p.scale_log2, p.scale_log2), nm2 = pk2(-mref, -mref);
-            lsum = (state == 1) ? row_exp<false>(tS, vis, sc2, nm2) : row_exp<true>(tS, vis, sc2, nm2);
-          }
-          l_sum += lsum;
-          ptx::tmem_st_wait();
-          ptx::tc_fence_before();
-          __syncwarp();
-          if (lane == 0) ptx::mbar_arrive(&bars->p_full[q][b]);
-          if (sub == 0 && lane == 0) DBT(12 + q, cnt);
-          if (sub == 0 && lane == 0 && !done) DBT(14 + q, cnt);
-          ++cnt;
-        }
-      }
-      // ---- epilogue: O / l -> bf16
-      ptx::mbar_wait(&bars->o_full[q], oc & 1);
-      ++oc;
-      ptx::tc_fence_after();
-      const float inv = (l_sum > 0.0f) ? 1.0f / l_sum : 0.0f;
-      const int head = wi.kvh * p.group + row % p.group;
-      __nv_bfloat16* dst = p.out + int64_t(tok_off + tok_local) * p.ldo + int64_t(head) * p.head_dim;
-#pragma unroll 1
-      for (int c = 0; c < OCH; ++c) {
-        const int col0 = c * 32;
-        uint32_t r[32];
-        ptx::tmem_ld32(tO + c * 32, r);
-        ptx::tmem_ld_wait();
-        if (valid_row && col0 < p.head_dim) {
-          uint32_t pk[16];
-#pragma unroll
-          for (int i = 0; i < 16; ++i)
-            pk[i] = ptx::pack_bf16x2(__uint_as_float(r[2 * i]) * inv, __uint_as_float(r[2 * i + 1]) * inv);
-          const int n16 = min(4, (p.head_dim - col0) / 8);
-          uint4* d4 = reinterpret_cast<uint4*>(dst + col0);
-          for (int i = 0; i < n16; ++i) d4[i] = make_uint4(pk[4 * i], pk[4 * i + 1], pk[4 * i + 2], pk[4 * i + 3]);
-        }
-      }
-      ptx::tc_fence_before();
-      __syncwarp();
-      if (lane == 0) ptx::mbar_arrive(&bars->o_empty[q]);
-    }
-  }
-  ptx::tc_fence_before();
-  __syncthreads();
-  if (warp == 1) ptx::tmem_dealloc(tmem, 512);
-}
-
 }  // namespace
+
+int attn_grid_slots(int, int num_sms) { return num_sms; }
 
 size_t attn_smem_bytes(int dpad) {
   return 1024 + (dpad == 128 ? AttnSmem<128>::TOTAL : AttnSmem<64>::TOTAL);
@@ -1111,26 +744,12 @@ void launch_attention(int dpad, const AttnParams& p, int num_sms, cudaStream_t s
   const int grid = p.n_work < num_sms ? p.n_work : num_sms;
   if (grid <= 0) return;
   const size_t smem = attn_smem_bytes(dpad);
-  // BAT_ATTN=db selects the double-buffered 64-key-sub-tile kernel (kept for A/B measurements:
-  // N = 64 S MMAs run at 48 clk instead of 32 and it issues 1.5x the MMAs; 555 vs 604 TFLOP/s)
-  static const bool use_tc = [] {
-    const char* e = getenv("BAT_ATTN");
-    return !(e && e[0] == 'd');
-  }();
-  static bool attr[4] = {false, false, false, false};
-  auto run = [&](void (*kern)(AttnParams), int threads, int id) {
-    if (!attr[id]) {
-      cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, int(smem));
-      attr[id] = true;
-    }
-    kern<<<grid, threads, smem, stream>>>(p);
-  };
   if (dpad == 128) {
-    if (use_tc) run(attn_tc_kernel<128>, NUM_THREADS, 0);
-    else run(attn_db_kernel<128>, DB_THREADS, 1);
+    set_smem_attr(attn_tc_kernel<128>, smem);
+    attn_tc_kernel<128><<<grid, NUM_THREADS, smem, stream>>>(p);
   } else {
-    if (use_tc) run(attn_tc_kernel<64>, NUM_THREADS, 2);
-    else run(attn_db_kernel<64>, DB_THREADS, 3);
+    set_smem_attr(attn_tc_kernel<64>, smem);
+    attn_tc_kernel<64><<<grid, NUM_THREADS, smem, stream>>>(p);
   }
   count_launch();
 }

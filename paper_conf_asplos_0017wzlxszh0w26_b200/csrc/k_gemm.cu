@@ -398,19 +398,6 @@ gemm2_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__
   if (warp == 1) ptx::tmem_dealloc2(tmem, 512);
 }
 
-template <class K>
-void set_smem_once(K kern, size_t bytes) {
-  static const void* done[16] = {nullptr};  // kernels whose smem attribute is set
-  for (const void* f : done)
-    if (f == reinterpret_cast<const void*>(kern)) return;
-  cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, static_cast<int>(bytes));
-  for (auto& f : done)
-    if (!f) {
-      f = reinterpret_cast<const void*>(kern);
-      break;
-    }
-}
-
 }  // namespace
 
 size_t gemm_smem_bytes() { return kGemmSmem2 > kGemmSmem1 ? kGemmSmem2 : kGemmSmem1; }
@@ -440,7 +427,7 @@ void launch_gemm(int epi, const CUtensorMap& tmA, const CUtensorMap& tmB, const 
     const int tiles = ((p.M + 255) / 256) * n_tiles;
     const int pairs = tiles < num_sms / 2 ? tiles : num_sms / 2;
     auto launch = [&](auto kern) {
-      set_smem_once(kern, kGemmSmem2);
+      set_smem_attr(kern, kGemmSmem2);
       kern<<<2 * pairs, NUM_THREADS, kGemmSmem2, stream>>>(tmA, tmB, tmC, p);
     };
     switch (epi) {
@@ -454,7 +441,7 @@ void launch_gemm(int epi, const CUtensorMap& tmA, const CUtensorMap& tmB, const 
     const int grid = tiles < num_sms ? tiles : num_sms;
     if (grid <= 0) return;
     auto launch = [&](auto kern) {
-      set_smem_once(kern, kGemmSmem1);
+      set_smem_attr(kern, kGemmSmem1);
       kern<<<grid, NUM_THREADS, kGemmSmem1, stream>>>(tmA, tmB, tmC, p);
     };
     switch (epi) {

@@ -6,6 +6,9 @@
 #include <cuda_runtime.h>
 
 #include <atomic>
+#include <map>
+#include <mutex>
+#include <string>
 
 #include "common.h"
 #include "kernels.h"
@@ -16,6 +19,21 @@ namespace bat {
 static std::atomic<int64_t> g_launches{0};
 void count_launch(int n) { g_launches.fetch_add(n, std::memory_order_relaxed); }
 int64_t launch_count() { return g_launches.load(std::memory_order_relaxed); }
+
+void set_smem_attr_raw(const void* func, int bytes) {
+  static std::mutex mu;
+  static std::map<std::pair<const void*, int>, int> done;  // (kernel, device) -> bytes set
+  int dev = 0;
+  if (cudaGetDevice(&dev) != cudaSuccess) fail(BAT_E_CUDA, "cudaGetDevice failed");
+  std::lock_guard<std::mutex> lk(mu);
+  auto key = std::make_pair(func, dev);
+  auto it = done.find(key);
+  if (it != done.end() && it->second >= bytes) return;
+  const cudaError_t e = cudaFuncSetAttribute(func, cudaFuncAttributeMaxDynamicSharedMemorySize, bytes);
+  if (e != cudaSuccess)
+    fail(BAT_E_CUDA, std::string("cudaFuncSetAttribute(MaxDynamicSharedMemorySize): ") + cudaGetErrorString(e));
+  done[key] = bytes;
+}
 
 namespace {
 
@@ -216,14 +234,15 @@ template <class TW, bool MULTI>
 __global__ void score_kernel(const float* __restrict__ hidden, const TW* __restrict__ w,
                              const int32_t* __restrict__ labels, const int32_t* __restrict__ n_items,
                              int n_max, int H, float* __restrict__ scores, int k,
-                             int32_t* __restrict__ topk) {
+                             int32_t* __restrict__ topk, float* __restrict__ logits) {
   extern __shared__ float sh[];
   float* hf = sh;            // [H]
   float* z = sh + H;         // [n_max]
   __shared__ float red[32];
   __shared__ int redi[32];
   const int b = blockIdx.x;
-  const int n = n_items[b];
+  // n_items is device data: clamp to the row width so a bad count can never overrun z[n_max]
+  const int n = max(0, min(n_items[b], n_max));
   const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5, nw = blockDim.x >> 5;
   if (!MULTI)
     for (int c = threadIdx.x; c < H; c += blockDim.x) hf[c] = hidden[int64_t(b) * H + c];
@@ -251,6 +270,8 @@ __global__ void score_kernel(const float* __restrict__ hidden, const TW* __restr
     if (lane == 0) z[i] = acc;
   }
   __syncthreads();
+  if (logits)  // z_i as computed here, for parity checks of the GEMV itself
+    for (int i = threadIdx.x; i < n_max; i += blockDim.x) logits[int64_t(b) * n_max + i] = i < n ? z[i] : 0.0f;
   // max
   float mx = -INFINITY;
   for (int i = threadIdx.x; i < n; i += blockDim.x) mx = fmaxf(mx, z[i]);
@@ -276,7 +297,7 @@ __global__ void score_kernel(const float* __restrict__ hidden, const TW* __restr
     if (lane == 0) red[0] = v;
   }
   __syncthreads();
-  const float inv = 1.0f / red[0];
+  const float inv = n > 0 ? 1.0f / red[0] : 0.0f;
   __syncthreads();
   for (int i = threadIdx.x; i < n_max; i += blockDim.x) {
     const float s = i < n ? __expf(z[i] - mx) * inv : 0.0f;
@@ -286,6 +307,10 @@ __global__ void score_kernel(const float* __restrict__ hidden, const TW* __restr
   __syncthreads();
   // top-k by repeated arg-max (ties -> lower index); taken entries set to -1
   for (int t = 0; t < k; ++t) {
+    if (t >= n) {  // fewer candidates than k: the remaining ranks are empty (-1)
+      if (threadIdx.x == 0) topk[int64_t(b) * k + t] = -1;
+      continue;
+    }
     float best = -2.0f;
     int bi = 0x7fffffff;
     for (int i = threadIdx.x; i < n; i += blockDim.x) {
@@ -306,7 +331,7 @@ __global__ void score_kernel(const float* __restrict__ hidden, const TW* __restr
       for (int q = 1; q < nw; ++q)
         if (red[q] > bb || (red[q] == bb && redi[q] < bbi)) { bb = red[q]; bbi = redi[q]; }
       topk[int64_t(b) * k + t] = bbi;
-      z[bbi] = -1.0f;
+      if (bbi < n) z[bbi] = -1.0f;
     }
     __syncthreads();
   }
@@ -432,31 +457,27 @@ void launch_gather_rows_f32(const float* src, const int32_t* idx, float* dst, in
 }
 template <class TW, bool MULTI = false>
 static void score_launch(const float* hidden, const TW* w_out, const int32_t* labels, const int32_t* n_items, int B,
-                         int n_max, int H, float* scores, int k, int32_t* topk, cudaStream_t s) {
+                         int n_max, int H, float* scores, int k, int32_t* topk, float* logits, cudaStream_t s) {
   if (B <= 0) return;
   const size_t smem = sizeof(float) * (size_t(H) + size_t(n_max));
-  static bool attr = false;
-  if (!attr) {
-    cudaFuncSetAttribute(score_kernel<TW, MULTI>, cudaFuncAttributeMaxDynamicSharedMemorySize, 64 * 1024);
-    attr = true;
-  }
-  score_kernel<TW, MULTI><<<B, 256, smem, s>>>(hidden, w_out, labels, n_items, n_max, H, scores, k, topk);
+  set_smem_attr(score_kernel<TW, MULTI>, 64 * 1024);
+  score_kernel<TW, MULTI><<<B, 256, smem, s>>>(hidden, w_out, labels, n_items, n_max, H, scores, k, topk, logits);
   count_launch();
 }
 void launch_score_multi(const float* hidden, const __nv_bfloat16* w_bf16, const float* w_f32, const int32_t* labels,
                         const int32_t* n_items, int B, int n_max, int H, float* scores, int k, int32_t* topk,
-                        cudaStream_t s) {
-  if (w_f32) score_launch<float, true>(hidden, w_f32, labels, n_items, B, n_max, H, scores, k, topk, s);
-  else score_launch<__nv_bfloat16, true>(hidden, w_bf16, labels, n_items, B, n_max, H, scores, k, topk, s);
+                        float* logits, cudaStream_t s) {
+  if (w_f32) score_launch<float, true>(hidden, w_f32, labels, n_items, B, n_max, H, scores, k, topk, logits, s);
+  else score_launch<__nv_bfloat16, true>(hidden, w_bf16, labels, n_items, B, n_max, H, scores, k, topk, logits, s);
 }
 void launch_score(const float* hidden, const __nv_bfloat16* w_out, const int32_t* labels,
                   const int32_t* n_items, int B, int n_max, int H, float* scores, int k,
-                  int32_t* topk, cudaStream_t s) {
-  score_launch(hidden, w_out, labels, n_items, B, n_max, H, scores, k, topk, s);
+                  int32_t* topk, float* logits, cudaStream_t s) {
+  score_launch(hidden, w_out, labels, n_items, B, n_max, H, scores, k, topk, logits, s);
 }
 void launch_score_f32w(const float* hidden, const float* w_out, const int32_t* labels, const int32_t* n_items, int B,
-                       int n_max, int H, float* scores, int k, int32_t* topk, cudaStream_t s) {
-  score_launch(hidden, w_out, labels, n_items, B, n_max, H, scores, k, topk, s);
+                       int n_max, int H, float* scores, int k, int32_t* topk, float* logits, cudaStream_t s) {
+  score_launch(hidden, w_out, labels, n_items, B, n_max, H, scores, k, topk, logits, s);
 }
 void launch_kv_scatter(const PageIO& io, const __nv_bfloat16* k, const __nv_bfloat16* v,
                        const int32_t* pages_dev, int n_tokens, int slot0, int n_total, cudaStream_t s) {

@@ -12,6 +12,14 @@ namespace bat {
 void count_launch(int n = 1);
 int64_t launch_count();
 
+// Opt a kernel into `bytes` of dynamic shared memory on the CURRENT device (the attribute is
+// per device context); cached per (kernel, device), thread-safe, fails with BAT_E_CUDA.
+void set_smem_attr_raw(const void* func, int bytes);
+template <class K>
+inline void set_smem_attr(K* kern, size_t bytes) {
+  set_smem_attr_raw(reinterpret_cast<const void*>(kern), static_cast<int>(bytes));
+}
+
 // ------------------------------------------------------------------------ tcgen05 GEMM
 enum GemmEpi { EPI_BF16 = 0, EPI_BF16_BIAS = 1, EPI_RESID_F32 = 2, EPI_SWIGLU = 3 };
 struct GemmParams {
@@ -50,23 +58,8 @@ struct AttnParams {
 };
 size_t attn_smem_bytes(int dpad);
 
-// CTA-pair bipartite attention (k_attn_pair.cu, head_dim 128): the K / V page blocks and the
-// q-tiles are fetched by 2-D TMA through byte-row views (128-byte rows, no swizzle: the pages
-// are already in the operand layout) so the peer CTA's loads signal the pair leader's barriers.
-struct AttnPairParams {
-  CUtensorMap tm_pool_k;   // pool arena, box 32 rows (one 4 KB page block)
-  CUtensorMap tm_pool_v;   // pool arena, box 8 rows (one 1 KB 8-key x 64-column atom)
-  CUtensorMap tm_scr_k;    // suffix scratch pages, box 32 rows
-  CUtensorMap tm_scr_v;    // suffix scratch pages, box 8 rows
-  CUtensorMap tm_q;        // q-tiles, box 256 rows (one 32 KB tile)
-  AttnParams a;
-  int64_t zero_row;        // first 128-byte row of the all-zero page in the pool view
-  int32_t total_tiles_hint;
-};
-bool attn_pair_supported(int dpad);
-// number of persistent work slots the planner should balance over (CTA pairs or CTAs)
+// number of persistent work slots the planner balances the attention work list over
 int attn_grid_slots(int dpad, int num_sms);
-void launch_attention_pair(const AttnPairParams& p, int num_sms, cudaStream_t stream);
 
 // Visibility masks of the plan's partial (q-tile, k-tile) pairs (PlanImage::off_mdesc): one block
 // per mask, bit (32 c + i) of row r's word c = key slot 32 c + i of the k-tile visible to token
@@ -109,7 +102,7 @@ void launch_gather_rows_f32(const float* src, const int32_t* idx, float* dst, in
                             cudaStream_t s);
 void launch_score(const float* hidden, const __nv_bfloat16* w_out, const int32_t* labels,
                   const int32_t* n_items, int B, int n_max, int H, float* scores, int k,
-                  int32_t* topk, cudaStream_t s);
+                  int32_t* topk, float* logits, cudaStream_t s);
 
 // KV pool page scatter / gather in the swizzled page layout (bf16)
 struct PageIO {
@@ -168,8 +161,8 @@ void launch_kv_gather_f32(const PageIO& io, float* k, float* v, const int32_t* p
 // one discriminant hidden row per item: hidden [B][n_max][H] (exactly one of w_bf16 / w_f32)
 void launch_score_multi(const float* hidden, const __nv_bfloat16* w_bf16, const float* w_f32, const int32_t* labels,
                         const int32_t* n_items, int B, int n_max, int H, float* scores, int k, int32_t* topk,
-                        cudaStream_t s);
+                        float* logits, cudaStream_t s);
 void launch_score_f32w(const float* hidden, const float* w_out, const int32_t* labels, const int32_t* n_items, int B,
-                       int n_max, int H, float* scores, int k, int32_t* topk, cudaStream_t s);
+                       int n_max, int H, float* scores, int k, int32_t* topk, float* logits, cudaStream_t s);
 
 }  // namespace bat

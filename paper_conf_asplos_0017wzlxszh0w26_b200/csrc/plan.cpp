@@ -31,6 +31,7 @@ void add_prefix_pages(const Pool& pool, const PrefixEnt& e, QueryPlan& qp) {
                           std::to_string(e.id) + ") holds " + std::to_string(ent->n_tokens) +
                           " tokens but the request has " + std::to_string(e.expect_n));
   }
+  qp.refs.push_back(EntityKey{e.kind, e.id});
   for (size_t pi = 0; pi < ent->pages.size(); ++pi) {
     int32_t nv = std::min<int32_t>(kPageTokens, ent->n_tokens - static_cast<int32_t>(pi) * kPageTokens);
     qp.pages.push_back(ent->pages[pi]);

@@ -23,6 +23,7 @@ struct QueryPlan {
   std::vector<int32_t> kseg, kord;        // [16 * n_pages]
   std::vector<uint8_t> tiles;             // [n_qtiles * n_ktiles]: 0 skip, 1 full, 2 partial
   std::vector<int32_t> disc;              // suffix rows of the discriminant(s): [1] or, multi, [n_items]
+  std::vector<EntityKey> refs;            // prefix entries whose pages the plan reads
 };
 
 // One request description, independent of the C struct (entity prefill builds these too).

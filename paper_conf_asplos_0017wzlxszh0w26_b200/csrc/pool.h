@@ -27,6 +27,8 @@ struct Entity {
   int32_t n_tokens = 0;
   std::vector<int32_t> pages;
   bool fetched = false;  // a local copy of a remote (cold-sharded) entry
+  int32_t pins = 0;      // live device plans referencing the pages (bat_plan_build)
+  int32_t refs = 0;      // fetched copies: batches holding it (bat_kv_fetch / bat_kv_release)
 };
 
 struct RemoteEntity {
@@ -78,6 +80,7 @@ struct Pool {
   void* fetch_host = nullptr;
   size_t fetch_host_cap = 0;
   void* fetch_done = nullptr;  // cudaEvent_t: last descriptor upload finished reading fetch_host
+  int64_t live_plans = 0;      // bat_plan_build plans not yet destroyed
 
   const Entity* find(int32_t kind, int64_t id) const {
     auto it = index.find(EntityKey{kind, id});

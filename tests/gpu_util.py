@@ -20,6 +20,21 @@ def max_excess(got, ref, atol=2e-2, rtol=2e-2):
     return float(np.max(np.abs(got - ref) - (atol + rtol * np.abs(ref))))
 
 
+def score_excess(z_gpu, s_gpu, z_ref, s_ref, atol=2e-2, rtol=2e-2):
+    """Parity of the score kernel's own outputs (a9): the logits z elementwise at the north_star
+    tolerance, and the scores s on a RELATIVE scale — |log s_gpu - log s_ref| within twice the
+    largest logit tolerance (the bound an in-tolerance z implies for log-softmax), so that s ~ 1/N
+    cannot hide behind the absolute tolerance.  Returns the worst excess of each (<= 0 passes)."""
+    z_gpu, s_gpu = np.asarray(z_gpu, np.float64), np.asarray(s_gpu, np.float64)
+    z_ref, s_ref = np.asarray(z_ref, np.float64), np.asarray(s_ref, np.float64)
+    ez = max_excess(z_gpu, z_ref, atol, rtol)
+    bound = 2.0 * float(np.max(atol + rtol * np.abs(z_ref)))
+    with np.errstate(divide="ignore"):
+        dl = np.abs(np.log(np.maximum(s_gpu, 1e-300)) - np.log(s_ref))
+    els = float(np.max(dl) - bound)
+    return ez, els
+
+
 def prefix_entities_in_order(q):
     """(kind, id, tokens) of the prefix entries of a cached request, in prompt order."""
     from paper_conf_asplos_0017wzlxszh0w26_b200 import bat

@@ -1,0 +1,132 @@
+"""Layer-level parity of the bipartite attention kernel on
+the EXACT batches bench.py times, every row of every request (configs[1]) or of sampled requests
+(configs[2]), against the fp64 oracle's masked attention (tests/gpu_util.oracle_attention_layer:
+explicit T x T bipartite mask, naive softmax per head).
+
+bat_debug_attention_layer plans the batch like bat_bipartite_prefill, RoPEs and stages the given
+qkv rows, and runs attn_tc_kernel over the pool's pages of one layer in the production launch
+configuration (persistent grid, LPT work list, device masks).  Prefix KV is random bf16 appended
+with bat_kv_append (values do not change the indexing; the kernel reads them from the pool), q and
+k are scaled so the attention is peaked (|O| ~ 1) and the 2e-2 abs/rel tolerance is not loose
+against the outputs.  A guard asserts that a wrong mask (every key visible) would fail."""
+import numpy as np
+import pytest
+
+import synth
+from oracle import model as om
+from oracle.sequence import build_sequence
+from tests.gpu_util import max_excess, oracle_attention_layer, prefix_entities_in_order
+
+pytestmark = pytest.mark.gpu
+torch = pytest.importorskip("torch")
+
+LAYER = 5
+
+
+@pytest.fixture(scope="module")
+def B():
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    from paper_conf_asplos_0017wzlxszh0w26_b200 import bat
+    bat.lib()
+    return bat
+
+
+def _dummy_model(cfg):
+    from paper_conf_asplos_0017wzlxszh0w26_b200.runtime import DeviceModel
+    H, F, d, Hq, Hkv, V = cfg["hidden"], cfg["ffn"], cfg["head_dim"], cfg["q_heads"], cfg["kv_heads"], cfg["vocab"]
+    e = lambda *s: torch.zeros(*s, dtype=torch.bfloat16, device="cuda")
+    layers = [dict(ln1=e(H), wqkv=e((Hq + 2 * Hkv) * d, H), bqkv=e((Hq + 2 * Hkv) * d), wo=e(H, Hq * d),
+                   ln2=e(H), wgu=e(2 * F, H), wd=e(H, F)) for _ in range(cfg["layers"])]
+    emb = e(V, H)
+    return DeviceModel(cfg, tensors=dict(embed=emb, lm_head=emb, final_norm=e(H), layers=layers))
+
+
+def _run(B, cfg, queries, sample, n_pages, kscale=2.0):
+    from paper_conf_asplos_0017wzlxszh0w26_b200.runtime import DevicePool
+    L, Hkv, d, Hq = cfg["layers"], cfg["kv_heads"], cfg["head_dim"], cfg["q_heads"]
+    model = _dummy_model(cfg)
+    pool = DevicePool(cfg, n_pages)
+    g = torch.Generator(device="cuda").manual_seed(3)
+    ekv = {}
+    for q in queries:
+        for kind, eid, toks in prefix_entities_in_order(q):
+            if (kind, eid) in ekv:
+                continue
+            n = len(toks)
+            k = (torch.randn(L, n, Hkv, d, generator=g, device="cuda") * kscale).to(torch.bfloat16)
+            v = torch.randn(L, n, Hkv, d, generator=g, device="cuda").to(torch.bfloat16)
+            B.bat_kv_append(pool.handle, kind, eid, k, v, n)
+            ekv[(kind, eid)] = ({LAYER: k[LAYER].double().cpu().numpy()}, {LAYER: v[LAYER].double().cpu().numpy()})
+    QA = B.QueryArray(queries)
+    plan = B.bat_plan_create(pool.handle, Hq // Hkv, QA)
+    S = [B.bat_plan_query_info(plan, b)["S"] for b in range(len(queries))]
+    B.bat_plan_destroy(plan)
+    M = sum(S)
+    qkv = torch.randn(M, (Hq + 2 * Hkv) * d, generator=g, device="cuda")
+    qkv[:, : (Hq + Hkv) * d] *= kscale  # q and k: peaked attention
+    qkv = qkv.to(torch.bfloat16)
+    out = torch.zeros(M, Hq * d, dtype=torch.bfloat16, device="cuda")
+    B.bat_debug_attention_layer(pool.handle, model.handle, QA, LAYER, qkv, out, True)
+    torch.cuda.synchronize()
+    qkv_np, out_np = qkv.double().cpu().numpy(), out.double().cpu().numpy()
+    offs = np.concatenate([[0], np.cumsum(S)])
+    worst, guard, rows = -1.0, -1.0, 0
+    for b in sample:
+        q = queries[b]
+        x = qkv_np[offs[b]:offs[b + 1]]
+        ref = oracle_attention_layer(cfg, q, ekv, x, LAYER)
+        got = out_np[offs[b]:offs[b + 1]].reshape(ref.shape)
+        worst = max(worst, max_excess(got, ref))
+        rows += ref.shape[0]
+        if b == sample[0]:  # wrong-mask guard: every key visible
+            guard = max_excess(got, _all_visible_attention(cfg, q, ekv, x))
+    pool.close()
+    model.close()
+    print(f"{len(sample)} requests, {rows} suffix rows x {Hq} heads: worst excess {worst:.4g}, "
+          f"wrong-mask excess {guard:.4g}")
+    return worst, guard
+
+
+def _all_visible_attention(cfg, q, ekv, x):
+    d, Hq, Hkv = cfg["head_dim"], cfg["q_heads"], cfg["kv_heads"]
+    toks, seg, pos = build_sequence(q.order, q.user_tok, q.item_toks, q.instr_tok)
+    ents = prefix_entities_in_order(q)
+    P = sum(len(t) for _, _, t in ents)
+    S = x.shape[0]
+    qq = om.rope(x[:, : Hq * d].reshape(S, Hq, d), pos[P:], cfg["rope_theta"])
+    kk = om.rope(x[:, Hq * d:(Hq + Hkv) * d].reshape(S, Hkv, d), pos[P:], cfg["rope_theta"])
+    vv = x[:, (Hq + Hkv) * d:].reshape(S, Hkv, d)
+    K = np.concatenate([ekv[(k, i)][0][LAYER] for k, i, _ in ents] + [kk]) if ents else kk
+    V = np.concatenate([ekv[(k, i)][1][LAYER] for k, i, _ in ents] + [vv]) if ents else vv
+    return om.attention(qq, K, V, np.ones((S, K.shape[0]), bool), Hq // Hkv)
+
+
+def test_attention_layer_config1_bench_batch_every_row(B):
+    """configs[1] as bench.py serves it: 64 IP requests, |U| = 512, 100 Zipf items of 16 tokens."""
+    cfg = synth.model_config("qwen2-1.5b")
+    rng = np.random.default_rng(7)
+    zp = synth.zipf_weights(8192)
+    qs = [synth.make_query(0, cfg, 1000 + b, 512, synth.distinct_label_items(0, cfg, 100, rng, 8192, zp),
+                           (16, 16), 8, "IP") for b in range(64)]
+    worst, guard = _run(B, cfg, qs, list(range(64)), 8192 + 64)
+    assert worst <= 0
+    assert guard > 0
+
+
+def test_attention_layer_config2_mixed_batch_sampled(B):
+    """configs[2]: 64 requests, 200 Zipf items, lognormal |U|, larger-side rule."""
+    cfg = synth.model_config("qwen2-1.5b")
+    rng = np.random.default_rng(11)
+    zp = synth.zipf_weights(8192)
+    n_user = synth.user_lengths(5, 64)
+    qs = [synth.make_query(0, cfg, 5000 + b, int(n_user[b]),
+                           synth.distinct_label_items(0, cfg, 200, rng, 8192, zp), (16, 16), 8,
+                           "UP" if n_user[b] >= 200 * 16 else "IP") for b in range(64)]
+    up = sorted([b for b, q in enumerate(qs) if q.order == "UP"], key=lambda b: len(qs[b].user_tok))
+    ip = sorted([b for b, q in enumerate(qs) if q.order == "IP"], key=lambda b: len(qs[b].user_tok))
+    sample = [ip[len(ip) // 2], ip[0], ip[-1], up[0], up[len(up) // 2]]
+    pages = 8192 + sum((len(q.user_tok) + 15) // 16 for q in qs) + 64
+    worst, guard = _run(B, cfg, qs, sample, pages)
+    assert worst <= 0
+    assert guard > 0

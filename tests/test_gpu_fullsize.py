@@ -21,7 +21,7 @@ import pytest
 import synth
 from oracle import model as om
 from oracle.sequence import causal_mask
-from tests.gpu_util import max_excess
+from tests.gpu_util import max_excess, score_excess
 
 pytestmark = pytest.mark.gpu
 torch = pytest.importorskip("torch")
@@ -69,17 +69,18 @@ def _serve_batch(B, cfg, W, queries, n_pages, k=10):
     lab = torch.tensor(labels, device="cuda")
     nit = torch.tensor([q.n_items for q in queries], dtype=torch.int32, device="cuda")
     scores = torch.empty(Bn, n_max, device="cuda")
+    logits = torch.empty(Bn, n_max, device="cuda")
     topk = torch.empty(Bn, k, dtype=torch.int32, device="cuda")
     # twice: the second pass must reproduce the first bit for bit (no state leaks between steps)
     outs = []
     for _ in range(2):
         B.bat_prefill_plan(pool.handle, model.handle, plan, hidden, stream)
-        B.bat_score(model.handle, hidden, lab, nit, Bn, n_max, scores, k, topk, stream)
+        B.bat_score(model.handle, hidden, lab, nit, Bn, n_max, scores, k, topk, stream, logits=logits)
         torch.cuda.synchronize()
         outs.append((hidden.clone(), scores.clone(), topk.clone()))
     assert torch.equal(outs[0][0], outs[1][0]) and torch.equal(outs[0][2], outs[1][2])
     out = dict(hf=hidden.double().cpu().numpy(), s=scores.double().cpu().numpy(),
-               topk=topk.cpu().numpy())
+               z=logits.double().cpu().numpy(), topk=topk.cpu().numpy())
     B.bat_plan_destroy(plan)
     pool.close()
     model.close()
@@ -92,10 +93,11 @@ def _check_sampled(cfg, W, queries, out, sample, k=10):
         q = queries[b]
         ref = om.run_query(cfg, W, q, "full", k=k)
         hf = out["hf"][b]
-        z = np.asarray(W.lm_head_rows(q.labels), np.float64) @ hf
+        z = out["z"][b, : q.n_items]  # the score kernel's own logits
         s = out["s"][b, : q.n_items]
         for name, got, want in (("hf", hf, ref["hf"]), ("z", z, ref["z"]), ("s", s, ref["s"])):
             worst[name] = max(worst.get(name, -1.0), max_excess(got, want))
+        worst["log_s"] = max(worst.get("log_s", -1.0), score_excess(z, s, ref["z"], ref["s"])[1])
         srt = np.sort(ref["s"])[::-1]
         for r in range(k):  # top-k agrees wherever the oracle's rank margin exceeds the tolerance
             if r + 1 < len(srt) and srt[r] - srt[r + 1] > 2 * (2e-2 + 2e-2 * srt[r]):

@@ -285,3 +285,21 @@ def test_multi_disc_permutation_equivariance(W):
     a = om.run_query_multi(CFG, W, _mq(items=(11, 22, 33, 44)), "full")
     b = om.run_query_multi(CFG, W, _mq(items=(33, 11, 44, 22)), "full")
     np.testing.assert_allclose(b["s"], a["s"][[2, 0, 3, 1]], rtol=1e-10, atol=1e-12)
+
+
+def test_multi_disc_rows_are_plain_causal_forwards_vs_transformers(W):
+    """Pins WHICH row is item i's discriminant and what it sees (R20): in
+    User-as-prefix order item i's tokens attend to U and to their own item only, at positions
+    |U| + j — exactly an ordinary causal forward of the sequence [U, I_i] — so its discriminant
+    (item i's LAST token) must equal HuggingFace Qwen2's final-normed last hidden state of [U, I_i],
+    and z_i = W_out[v_i] . that state.  Ragged items: the first token, an off-by-one inside the item
+    or another item's row would each fail."""
+    q = synth.make_query(2, CFG, 9, 11, [5, 6, 7], (3, 9), 2, "UP")
+    assert len({len(t) for t in q.item_toks}) > 1
+    q.multi_disc = True
+    a = om.run_query_multi(CFG, W, q, "full")
+    for i, t in enumerate(q.item_toks):
+        ref = _hf_forward(CFG, W, np.concatenate([q.user_tok, t]))[-1]
+        np.testing.assert_allclose(a["hf"][i], ref, rtol=1e-10, atol=1e-10)
+        zi = float(np.asarray(W.lm_head_rows([q.labels[i]]), np.float64)[0] @ ref)
+        np.testing.assert_allclose(a["z"][i], zi, rtol=1e-10, atol=1e-10)

@@ -102,3 +102,17 @@ def test_plan_batch_offsets():
     ps = op.plan_batch(qs, _pages_for(qs), group=2)
     assert [p["token_off"] for p in ps] == [0, 7, 15]
     assert [p["scratch_page0"] for p in ps] == [0, 1, 2]
+
+
+@pytest.mark.parametrize("seed", range(3))
+def test_multi_disc_rows_by_position(seed):
+    """The plan's per-item discriminant rows (R20), by a second formulation: item i's
+    discriminant is the suffix row of segment i whose POSITION is |U| + |I_i| - 1 (items
+    start at position |U| in UP; positions are pinned by tests/golden/mask_tiny.txt)."""
+    cfg = synth.model_config("tiny")
+    q = synth.make_query(seed, cfg, 2, 7 + seed, [3, 1, 4, 5][: 2 + seed], (2, 11), 2, "UP", use_cache=(seed != 1))
+    q.multi_disc = True
+    p = op.plan_query(q, _pages_for([q]), 2)
+    for i, t in enumerate(q.item_toks):
+        rows = np.nonzero((p["seg"] == i) & (p["pos"] == len(q.user_tok) + len(t) - 1))[0]
+        assert len(rows) == 1 and p["disc"][i] == rows[0]
