@@ -351,13 +351,36 @@ BAT_API bat_status bat_kv_register_remote(bat_pool p, int32_t kind, int64_t id, 
 BAT_API bat_status bat_kv_lookup_remote(bat_pool p, int32_t kind, int64_t id, int32_t* owner,
                                         int32_t* n_tokens, int32_t* pages_out, int32_t pages_cap,
                                         int32_t* n_pages);
-/* Pull the listed remote entries (deduplicated, skipping ones already local) from their
- * owners' arenas over NVLink into local pages (one copy kernel on `stream`, asynchronous:
- * work on `stream` after this call sees the pages), making them resolvable by
- * bat_bipartite_prefill.  *n_fetched = entries pulled.  The owners must not evict them while
- * the copy runs. */
+/* Pull the listed remote (cold-sharded) entries from their owners' arenas over NVLink into local
+ * pages, making them resolvable by bat_bipartite_prefill.  The copies are enqueued on
+ * `stream` — meant to be a dedicated copy stream, so the pull overlaps compute on another stream
+ * (order the compute after it with an event) — as ONE batched copy-engine memcpy
+ * (cudaMemcpyBatchAsync, overlap-with-compute hint; no SMs; runs of consecutive pages merged).
+ * Pulled copies are reference counted: an id already pulled gets one more reference, replicated /
+ * owned (local) ids are skipped; *n_fetched = entries copied by this call.  Pages a previous
+ * bat_kv_release gave back are reused behind a stream wait on their release event.  The owners
+ * must not evict the entries while the copy runs.  BAT_E_NOTFOUND for an id neither local nor
+ * registered remote; all-or-nothing. */
 BAT_API bat_status bat_kv_fetch(bat_pool p, int32_t kind, const int64_t* ids, int32_t n,
                         int32_t* n_fetched, bat_stream_t stream);
+/* Drop one reference per listed pulled entry (ids as passed to bat_kv_fetch; local ids are
+ * skipped).  An entry whose last reference goes is removed and its pages are freed IN STREAM
+ * ORDER: they become reusable once the work enqueued on `stream` so far (the batches reading them)
+ * has completed — no host synchronisation.  BAT_E_STATE for more releases than fetches or an entry
+ * a live plan pins; all-or-nothing. */
+BAT_API bat_status bat_kv_release(bat_pool p, int32_t kind, const int64_t* ids, int32_t n, bat_stream_t stream);
+
+/* Double-buffered staging for pre-built plans ("fetched ... overlapped with compute"):
+ * reserve n_slots (<= 8) slots of pages_per_slot pages each.  bat_plan_build_staged maps every
+ * cold (registered remote) prefix item of its batch to pages of one slot (deduplicated within
+ * the batch) and records the pulls; bat_plan_fetch enqueues them on a stream.  Pipelining batch
+ * k+1's pull (slot (k+1) % 2) under batch k's compute (slot k % 2) is the caller's event
+ * ordering: the pull into a slot must wait for the compute of the batch that last read it. */
+BAT_API bat_status bat_kv_staging_reserve(bat_pool p, int32_t n_slots, int64_t pages_per_slot);
+BAT_API bat_status bat_plan_build_staged(bat_pool p, bat_model m, const bat_query* queries, int32_t B,
+                                         int32_t slot, bat_stream_t stream, bat_plan* out);
+/* Enqueue a staged plan's cold-item pulls on `stream` (copy engines); *n_pages = pages pulled. */
+BAT_API bat_status bat_plan_fetch(bat_pool p, bat_plan plan, int64_t* n_pages, bat_stream_t stream);
 
 /* ------------------------------------------------------------------------------------------
  * Test-only entry points (kernel-level parity tests; not part of the serving path)

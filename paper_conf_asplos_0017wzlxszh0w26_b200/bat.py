@@ -132,6 +132,11 @@ def lib() -> ctypes.CDLL:
         "bat_score_multi": (S, [c_void_p, c_void_p, c_void_p, c_void_p, c_int32, c_int32, c_void_p, c_int32, c_void_p,
                                 c_void_p, c_void_p]),
         "bat_plan_export_device": (S, [c_void_p, c_int32, c_int32, c_void_p, c_int64, POINTER(c_int64)]),
+        "bat_kv_release": (S, [c_void_p, c_int32, POINTER(c_int64), c_int32, c_void_p]),
+        "bat_kv_staging_reserve": (S, [c_void_p, c_int32, c_int64]),
+        "bat_plan_build_staged": (S, [c_void_p, c_void_p, POINTER(bat_query), c_int32, c_int32, c_void_p,
+                                      POINTER(c_void_p)]),
+        "bat_plan_fetch": (S, [c_void_p, c_void_p, POINTER(c_int64), c_void_p]),
         "bat_sched_create": (S, [POINTER(bat_sched_cfg), POINTER(c_void_p)]),
         "bat_sched_destroy": (S, [c_void_p]),
         "bat_sched_decide": (S, [c_void_p, c_double, c_int64, c_int32, c_int32, POINTER(bat_sched_decision),
@@ -157,7 +162,8 @@ EXPORTED = ("bat_last_error", "bat_version", "bat_kernel_launch_count", "bat_mod
             "bat_plan_build", "bat_prefill_plan", "bat_profile_enable", "bat_profile_read",
             "bat_profile_reset", "bat_debug_attach_peer_pool", "bat_sched_create", "bat_sched_destroy",
             "bat_sched_decide", "bat_sched_stats", "bat_sched_is_cached", "bat_score_multi",
-            "bat_plan_export_device")
+            "bat_plan_export_device", "bat_kv_release", "bat_kv_staging_reserve", "bat_plan_build_staged",
+            "bat_plan_fetch")
 
 
 def _check(status: int) -> None:
@@ -454,6 +460,27 @@ def bat_kv_fetch(pool: int, kind: int, ids: Sequence[int], stream=None) -> int:
     a = np.ascontiguousarray(ids, dtype=np.int64)
     n = c_int32()
     _check(lib().bat_kv_fetch(pool, kind, _i64p(a), len(a), byref(n), _vp(stream)))
+    return n.value
+
+
+def bat_kv_release(pool: int, kind: int, ids: Sequence[int], stream=None) -> None:
+    a = np.ascontiguousarray(ids, dtype=np.int64)
+    _check(lib().bat_kv_release(pool, kind, _i64p(a), len(a), _vp(stream)))
+
+
+def bat_kv_staging_reserve(pool: int, n_slots: int, pages_per_slot: int) -> None:
+    _check(lib().bat_kv_staging_reserve(pool, n_slots, pages_per_slot))
+
+
+def bat_plan_build_staged(pool: int, model: int, queries: QueryArray, slot: int, stream=None) -> int:
+    out = c_void_p()
+    _check(lib().bat_plan_build_staged(pool, model, queries.arr, len(queries), slot, _vp(stream), byref(out)))
+    return out.value
+
+
+def bat_plan_fetch(pool: int, plan: int, stream=None) -> int:
+    n = c_int64()
+    _check(lib().bat_plan_fetch(pool, plan, byref(n), _vp(stream)))
     return n.value
 
 

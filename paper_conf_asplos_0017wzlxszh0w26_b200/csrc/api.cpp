@@ -30,6 +30,9 @@ struct bat_plan_s {
   bat_pool_s* pool = nullptr;              // the pool whose page ids the device image holds
   std::vector<bat::EntityKey> pinned;      // entries pinned (not evictable) while the plan lives
   std::vector<int32_t> dev_copy;           // host copy of the device image (bat_plan_export_device)
+  int32_t slot = -1;                       // staging slot of a bat_plan_build_staged plan
+  std::vector<uint64_t> pull_src;          // its cold-item pulls: peer page addresses ...
+  std::vector<int32_t> pull_dst;           // ... -> local staging pages
   ~bat_plan_s() {
     if (dev_img) cudaFree(dev_img);
   }
@@ -720,6 +723,8 @@ bat_status bat_kv_pool_destroy(bat_pool p) {
         if (p->pool.peer_arena[r] && p->pool.peer_ipc[r]) cudaIpcCloseMemHandle(p->pool.peer_arena[r]);
       if (p->pool.fetch_host) cudaFreeHost(p->pool.fetch_host);
       if (p->pool.fetch_done) cudaEventDestroy(static_cast<cudaEvent_t>(p->pool.fetch_done));
+      for (auto& f : p->pool.pending) cudaEventDestroy(f.ev);
+      for (cudaEvent_t e : p->pool.spare_events) cudaEventDestroy(e);
       cudaFree(p->pool.arena);
     }
     delete p;
@@ -731,8 +736,8 @@ int64_t bat_kv_page_bytes(bat_pool p) { return p ? p->pool.geo.page_bytes : 0; }
 bat_status bat_kv_pool_stats(bat_pool p, int64_t* free_pages, int64_t* used_pages, int64_t* n_entities) {
   return guarded([&] {
     BAT_REQUIRE(p, "null pool");
-    if (free_pages) *free_pages = int64_t(p->pool.free_pages.size());
-    if (used_pages) *used_pages = p->pool.cfg.num_pages - int64_t(p->pool.free_pages.size());
+    if (free_pages) *free_pages = p->pool.n_free();
+    if (used_pages) *used_pages = p->pool.cfg.num_pages - p->pool.n_free();
     if (n_entities) *n_entities = int64_t(p->pool.index.size());
   });
 }
@@ -1221,6 +1226,64 @@ bat_status bat_kv_lookup_remote(bat_pool p, int32_t kind, int64_t id, int32_t* o
   });
 }
 
+// Page pulls from peer-mapped arenas: one batched copy-engine memcpy (cudaMemcpyBatchAsync with
+// the overlap-with-compute hint: no SMs taken from the kernels running beside it), runs of
+// consecutive pages merged; BAT_FETCH_SM=1 selects the round-1 SM copy kernel instead.
+static void issue_page_pulls(Pool& P, const std::vector<uint64_t>& src, const std::vector<int32_t>& dst,
+                             cudaStream_t st) {
+  if (src.empty()) return;
+  static const bool use_sm = std::getenv("BAT_FETCH_SM") && std::getenv("BAT_FETCH_SM")[0] == '1';
+  const int64_t pb = P.geo.page_bytes;
+  if (use_sm) {
+    const size_t bytes = src.size() * 8 + dst.size() * 4;
+    if (!P.fetch_done) {
+      cudaEvent_t e;
+      CUDA_OK(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
+      P.fetch_done = e;
+    }
+    CUDA_OK(cudaEventSynchronize(static_cast<cudaEvent_t>(P.fetch_done)));
+    if (P.fetch_host_cap < bytes) {
+      if (P.fetch_host) cudaFreeHost(P.fetch_host);
+      P.fetch_host_cap = bytes * 2;
+      CUDA_OK(cudaMallocHost(&P.fetch_host, P.fetch_host_cap));
+    }
+    std::memcpy(P.fetch_host, src.data(), src.size() * 8);
+    std::memcpy(static_cast<char*>(P.fetch_host) + src.size() * 8, dst.data(), dst.size() * 4);
+    void* buf = nullptr;
+    CUDA_OK(cudaMallocAsync(&buf, bytes, st));
+    CUDA_OK(cudaMemcpyAsync(buf, P.fetch_host, bytes, cudaMemcpyHostToDevice, st));
+    CUDA_OK(cudaEventRecord(static_cast<cudaEvent_t>(P.fetch_done), st));
+    launch_page_copy(static_cast<const uint64_t*>(buf), reinterpret_cast<const int32_t*>(static_cast<char*>(buf) + src.size() * 8),
+                     P.arena, pb, int(src.size()), st);
+    CUDA_OK(cudaFreeAsync(buf, st));
+    return;
+  }
+  std::vector<void*> d, s;
+  std::vector<size_t> n;
+  for (size_t k = 0; k < src.size(); ++k) {
+    char* dp = P.arena + int64_t(dst[k]) * pb;
+    char* sp = reinterpret_cast<char*>(src[k]);
+    if (!d.empty() && static_cast<char*>(d.back()) + n.back() == dp && static_cast<char*>(s.back()) + n.back() == sp) {
+      n.back() += size_t(pb);
+    } else {
+      d.push_back(dp);
+      s.push_back(sp);
+      n.push_back(size_t(pb));
+    }
+  }
+  if (st == nullptr) {  // the batched API does not take the legacy default stream
+    for (size_t k = 0; k < d.size(); ++k) CUDA_OK(cudaMemcpyAsync(d[k], s[k], n[k], cudaMemcpyDefault, st));
+    return;
+  }
+  cudaMemcpyAttributes attr{};
+  attr.srcAccessOrder = cudaMemcpySrcAccessOrderStream;
+  attr.flags = cudaMemcpyFlagPreferOverlapWithCompute;
+  size_t idx0 = 0, fail_idx = 0;
+  const cudaError_t e = cudaMemcpyBatchAsync(d.data(), s.data(), n.data(), d.size(), &attr, &idx0, 1, &fail_idx, st);
+  if (e != cudaSuccess)
+    fail(BAT_E_CUDA, std::string("cudaMemcpyBatchAsync (copy ") + std::to_string(fail_idx) + "): " + cudaGetErrorString(e));
+}
+
 bat_status bat_kv_fetch(bat_pool p, int32_t kind, const int64_t* ids, int32_t n, int32_t* n_fetched,
                         bat_stream_t stream) {
   return guarded([&] {
@@ -1228,14 +1291,22 @@ bat_status bat_kv_fetch(bat_pool p, int32_t kind, const int64_t* ids, int32_t n,
     Pool& P = p->pool;
     if (P.index_only) fail(BAT_E_STATE, "index-only pool");
     DeviceGuard dg(P.device);
+    cudaStream_t st = static_cast<cudaStream_t>(stream);
     std::vector<uint64_t> src;
     std::vector<int32_t> dst;
-    std::vector<EntityKey> made;
+    std::vector<EntityKey> made, bumped;
     int32_t fetched = 0;
     try {
       for (int32_t i = 0; i < n; ++i) {
         EntityKey key{kind, ids[i]};
-        if (P.index.count(key)) continue;  // local (replicated, owned or already fetched)
+        auto loc = P.index.find(key);
+        if (loc != P.index.end()) {  // replicated / owned, or already pulled: one more holder
+          if (loc->second.fetched) {
+            ++loc->second.refs;
+            bumped.push_back(key);
+          }
+          continue;
+        }
         auto it = P.remote.find(key);
         if (it == P.remote.end()) fail(BAT_E_NOTFOUND, "entry neither local nor registered remote");
         const RemoteEntity& r = it->second;
@@ -1244,7 +1315,9 @@ bat_status bat_kv_fetch(bat_pool p, int32_t kind, const int64_t* ids, int32_t n,
         Entity en;
         en.n_tokens = r.n_tokens;
         en.fetched = true;
-        if (!P.alloc_pages(int64_t(r.pages.size()), en.pages)) {
+        en.refs = 1;
+        // pages still pending a stream-ordered release are taken behind a wait on `st`
+        if (!P.alloc_pages_on(int64_t(r.pages.size()), en.pages, st)) {
           P.release_pages(en.pages);
           fail(BAT_E_POOLFULL, "pool full while fetching");
         }
@@ -1256,34 +1329,8 @@ bat_status bat_kv_fetch(bat_pool p, int32_t kind, const int64_t* ids, int32_t n,
         made.push_back(key);
         ++fetched;
       }
-      if (!src.empty()) {
-        cudaStream_t st = static_cast<cudaStream_t>(stream);
-        const size_t bytes = src.size() * 8 + dst.size() * 4;
-        // asynchronous: descriptors go through a pool-owned pinned buffer (reused once the
-        // previous upload has read it), the device copy is freed in stream order
-        if (!P.fetch_done) {
-          cudaEvent_t e;
-          CUDA_OK(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
-          P.fetch_done = e;
-        }
-        CUDA_OK(cudaEventSynchronize(static_cast<cudaEvent_t>(P.fetch_done)));
-        if (P.fetch_host_cap < bytes) {
-          if (P.fetch_host) cudaFreeHost(P.fetch_host);
-          P.fetch_host_cap = bytes * 2;
-          CUDA_OK(cudaMallocHost(&P.fetch_host, P.fetch_host_cap));
-        }
-        std::memcpy(P.fetch_host, src.data(), src.size() * 8);
-        std::memcpy(static_cast<char*>(P.fetch_host) + src.size() * 8, dst.data(), dst.size() * 4);
-        void* buf = nullptr;
-        CUDA_OK(cudaMallocAsync(&buf, bytes, st));
-        CUDA_OK(cudaMemcpyAsync(buf, P.fetch_host, bytes, cudaMemcpyHostToDevice, st));
-        CUDA_OK(cudaEventRecord(static_cast<cudaEvent_t>(P.fetch_done), st));
-        launch_page_copy(static_cast<const uint64_t*>(buf),
-                         reinterpret_cast<const int32_t*>(static_cast<char*>(buf) + src.size() * 8), P.arena,
-                         P.geo.page_bytes, int(src.size()), st);
-        CUDA_OK(cudaFreeAsync(buf, st));
-        CUDA_OK(cudaGetLastError());
-      }
+      issue_page_pulls(P, src, dst, st);
+      CUDA_OK(cudaGetLastError());
     } catch (...) {
       for (auto& k : made) {
         auto it = P.index.find(k);
@@ -1292,12 +1339,72 @@ bat_status bat_kv_fetch(bat_pool p, int32_t kind, const int64_t* ids, int32_t n,
           P.index.erase(it);
         }
       }
+      for (auto& k : bumped) {
+        auto it = P.index.find(k);
+        if (it != P.index.end()) --it->second.refs;
+      }
       throw;
     }
     if (n_fetched) *n_fetched = fetched;
   });
 }
 
+bat_status bat_kv_release(bat_pool p, int32_t kind, const int64_t* ids, int32_t n, bat_stream_t stream) {
+  return guarded([&] {
+    BAT_REQUIRE(p && (ids || n == 0), "null argument");
+    Pool& P = p->pool;
+    if (P.index_only) fail(BAT_E_STATE, "index-only pool");
+    DeviceGuard dg(P.device);
+    // validate first (all-or-nothing)
+    std::unordered_map<EntityKey, int32_t, EntityKeyHash> drops;
+    for (int32_t i = 0; i < n; ++i) {
+      EntityKey key{kind, ids[i]};
+      auto it = P.index.find(key);
+      if (it == P.index.end()) {
+        if (P.remote.count(key)) fail(BAT_E_STATE, "remote entry released but not fetched");
+        fail(BAT_E_NOTFOUND, "entry not found");
+      }
+      if (!it->second.fetched) continue;  // replicated / owned: not a pulled copy
+      const int32_t d = ++drops[key];
+      if (d > it->second.refs) fail(BAT_E_STATE, "more releases than fetches");
+      if (d == it->second.refs && it->second.pins > 0) fail(BAT_E_STATE, "entry is referenced by a live plan");
+    }
+    std::vector<int32_t> freed;
+    for (auto& kv : drops) {
+      auto it = P.index.find(kv.first);
+      it->second.refs -= kv.second;
+      if (it->second.refs == 0) {
+        freed.insert(freed.end(), it->second.pages.begin(), it->second.pages.end());
+        P.index.erase(it);
+      }
+    }
+    if (freed.empty()) return;
+    cudaEvent_t ev;
+    if (!P.spare_events.empty()) {
+      ev = P.spare_events.back();
+      P.spare_events.pop_back();
+    } else {
+      CUDA_OK(cudaEventCreateWithFlags(&ev, cudaEventDisableTiming));
+    }
+    CUDA_OK(cudaEventRecord(ev, static_cast<cudaStream_t>(stream)));
+    P.pending.push_back(Pool::PendingFree{ev, std::move(freed)});
+  });
+}
+
+bat_status bat_kv_staging_reserve(bat_pool p, int32_t n_slots, int64_t pages_per_slot) {
+  return guarded([&] {
+    BAT_REQUIRE(p && n_slots >= 1 && n_slots <= 8 && pages_per_slot >= 1, "argument");
+    Pool& P = p->pool;
+    BAT_REQUIRE(P.staging.empty(), "staging already reserved");
+    std::vector<std::vector<int32_t>> slots(n_slots);
+    for (auto& sl : slots)
+      if (!P.alloc_pages(pages_per_slot, sl)) {
+        for (auto& x : slots) P.release_pages(x);
+        fail(BAT_E_POOLFULL, "pool too small for the staging slots");
+      }
+    P.staging = std::move(slots);
+  });
+}
 
 // ------------------------------------------------------------------------ test-only
 bat_status bat_debug_gemm(int32_t epi, int32_t M, int32_t N, int32_t K, const void* A, const void* Bw,
@@ -1389,36 +1496,65 @@ bat_status bat_debug_attention_layer(bat_pool p, bat_model mdl, const bat_query*
 
 
 // ------------------------------------------------------------------ planned execution
+static void plan_build_impl(bat_pool p, bat_model mdl, const bat_query* queries, int32_t B, int32_t slot,
+                            bat_stream_t stream, bat_plan* out) {
+  BAT_REQUIRE(p && mdl && queries && out && B >= 1, "null argument");
+  Pool& P = p->pool;
+  Model& m = mdl->m;
+  check_compat(P, m);
+  for (int b = 0; b < B; ++b) validate_tokens(queries[b], m.cfg.vocab);
+  DeviceGuard dg(P.device);
+  auto pl = std::make_unique<bat_plan_s>();
+  StagingCtx stg;
+  if (slot >= 0) {
+    BAT_REQUIRE(slot < int32_t(P.staging.size()), "staging slot (bat_kv_staging_reserve first)");
+    stg.slot_pages = &P.staging[slot];
+  }
+  build_plan(P, m.cfg.q_heads / m.cfg.kv_heads, m.cfg.kv_heads, wrap(queries, B), pl->plan, true,
+             attn_grid_slots(m.dpad, m.num_sms), slot >= 0 ? &stg : nullptr);
+  pl->pull_src = std::move(stg.src);
+  pl->pull_dst = std::move(stg.dst);
+  pl->slot = slot;
+  const size_t bytes = pl->plan.img.buf.size() * 4;
+  CUDA_OK(cudaMalloc(&pl->dev_img, size_t(pl->plan.img.total_ints) * 4));
+  CUDA_OK(cudaMemcpyAsync(pl->dev_img, pl->plan.img.buf.data(), bytes, cudaMemcpyHostToDevice,
+                          static_cast<cudaStream_t>(stream)));
+  build_masks(pl->plan, static_cast<int32_t*>(pl->dev_img), static_cast<cudaStream_t>(stream));
+  CUDA_OK(cudaStreamSynchronize(static_cast<cudaStream_t>(stream)));
+  pl->device = P.device;
+  // the device image bakes in page ids: pin every referenced entry until bat_plan_destroy
+  for (const QueryPlan& q : pl->plan.q)
+    for (const EntityKey& k : q.refs) {
+      auto it = P.index.find(k);
+      if (it != P.index.end()) {
+        ++it->second.pins;
+        pl->pinned.push_back(k);
+      }
+    }
+  pl->pool = p;
+  ++P.live_plans;
+  *out = pl.release();
+}
+
 bat_status bat_plan_build(bat_pool p, bat_model mdl, const bat_query* queries, int32_t B, bat_stream_t stream,
                           bat_plan* out) {
+  return guarded([&] { plan_build_impl(p, mdl, queries, B, -1, stream, out); });
+}
+
+bat_status bat_plan_build_staged(bat_pool p, bat_model mdl, const bat_query* queries, int32_t B, int32_t slot,
+                                 bat_stream_t stream, bat_plan* out) {
+  return guarded([&] { plan_build_impl(p, mdl, queries, B, slot, stream, out); });
+}
+
+bat_status bat_plan_fetch(bat_pool p, bat_plan plan, int64_t* n_pages, bat_stream_t stream) {
   return guarded([&] {
-    BAT_REQUIRE(p && mdl && queries && out && B >= 1, "null argument");
+    BAT_REQUIRE(p && plan, "null argument");
+    if (plan->pool != p) fail(BAT_E_STATE, "plan was built for another pool");
     Pool& P = p->pool;
-    Model& m = mdl->m;
-    check_compat(P, m);
-    for (int b = 0; b < B; ++b) validate_tokens(queries[b], m.cfg.vocab);
     DeviceGuard dg(P.device);
-    auto pl = std::make_unique<bat_plan_s>();
-    build_plan(P, m.cfg.q_heads / m.cfg.kv_heads, m.cfg.kv_heads, wrap(queries, B), pl->plan, true, attn_grid_slots(m.dpad, m.num_sms));
-    // the device image bakes in page ids: pin every referenced entry until bat_plan_destroy
-    for (const QueryPlan& q : pl->plan.q)
-      for (const EntityKey& k : q.refs) {
-        auto it = P.index.find(k);
-        if (it != P.index.end()) {
-          ++it->second.pins;
-          pl->pinned.push_back(k);
-        }
-      }
-    pl->pool = p;
-    ++P.live_plans;
-    const size_t bytes = pl->plan.img.buf.size() * 4;
-    CUDA_OK(cudaMalloc(&pl->dev_img, size_t(pl->plan.img.total_ints) * 4));
-    CUDA_OK(cudaMemcpyAsync(pl->dev_img, pl->plan.img.buf.data(), bytes, cudaMemcpyHostToDevice,
-                            static_cast<cudaStream_t>(stream)));
-    build_masks(pl->plan, static_cast<int32_t*>(pl->dev_img), static_cast<cudaStream_t>(stream));
-    CUDA_OK(cudaStreamSynchronize(static_cast<cudaStream_t>(stream)));
-    pl->device = P.device;
-    *out = pl.release();
+    issue_page_pulls(P, plan->pull_src, plan->pull_dst, static_cast<cudaStream_t>(stream));
+    CUDA_OK(cudaGetLastError());
+    if (n_pages) *n_pages = int64_t(plan->pull_dst.size());
   });
 }
 

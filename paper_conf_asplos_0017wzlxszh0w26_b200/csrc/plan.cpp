@@ -20,8 +20,34 @@ struct PrefixEnt {
   int32_t expect_n;  // tokens the request carries for it (-1: unchecked)
 };
 
-void add_prefix_pages(const Pool& pool, const PrefixEnt& e, QueryPlan& qp) {
+// A cold item of a staged plan: pages of the staging slot, the pull recorded once per plan.
+const Entity* staged_entity(const Pool& pool, const PrefixEnt& e, StagingCtx* stg) {
+  if (!stg) return nullptr;
+  const EntityKey key{e.kind, e.id};
+  auto a = stg->assigned.find(key);
+  if (a != stg->assigned.end()) return &a->second;
+  auto r = pool.remote.find(key);
+  if (r == pool.remote.end()) return nullptr;
+  const RemoteEntity& re = r->second;
+  const char* peer = pool.peer_arena[re.owner];
+  if (!peer) fail(BAT_E_STATE, "peer arena of rank " + std::to_string(re.owner) + " not attached");
+  if (stg->used + re.pages.size() > stg->slot_pages->size())
+    fail(BAT_E_POOLFULL, "staging slot too small for the batch's cold items");
+  Entity en;
+  en.n_tokens = re.n_tokens;
+  en.fetched = true;
+  for (size_t k = 0; k < re.pages.size(); ++k) {
+    const int32_t dst = (*stg->slot_pages)[stg->used++];
+    en.pages.push_back(dst);
+    stg->src.push_back(reinterpret_cast<uint64_t>(peer + int64_t(re.pages[k]) * pool.geo.page_bytes));
+    stg->dst.push_back(dst);
+  }
+  return &stg->assigned.emplace(key, std::move(en)).first->second;
+}
+
+void add_prefix_pages(const Pool& pool, const PrefixEnt& e, QueryPlan& qp, StagingCtx* stg) {
   const Entity* ent = pool.find(e.kind, e.id);
+  const bool staged = !ent && (ent = staged_entity(pool, e, stg)) != nullptr;
   if (!ent) {
     fail(BAT_E_NOTFOUND, "prefix entry (kind " + std::to_string(e.kind) + ", id " +
                              std::to_string(e.id) + ") is not in the pool");
@@ -31,7 +57,7 @@ void add_prefix_pages(const Pool& pool, const PrefixEnt& e, QueryPlan& qp) {
                           std::to_string(e.id) + ") holds " + std::to_string(ent->n_tokens) +
                           " tokens but the request has " + std::to_string(e.expect_n));
   }
-  qp.refs.push_back(EntityKey{e.kind, e.id});
+  if (!staged) qp.refs.push_back(EntityKey{e.kind, e.id});
   for (size_t pi = 0; pi < ent->pages.size(); ++pi) {
     int32_t nv = std::min<int32_t>(kPageTokens, ent->n_tokens - static_cast<int32_t>(pi) * kPageTokens);
     qp.pages.push_back(ent->pages[pi]);
@@ -45,7 +71,7 @@ void add_prefix_pages(const Pool& pool, const PrefixEnt& e, QueryPlan& qp) {
 }
 
 // Suffix tokens / positions / segments of a ranking request (readings R2, R3).
-void build_request(const Pool& pool, const bat_query& q, QueryPlan& qp) {
+void build_request(const Pool& pool, const bat_query& q, QueryPlan& qp, StagingCtx* stg) {
   BAT_REQUIRE(q.order == BAT_ORDER_UP || q.order == BAT_ORDER_IP, "order must be UP or IP");
   BAT_REQUIRE(q.n_items >= 1, "n_items >= 1");
   BAT_REQUIRE(q.n_instr >= 1, "n_instr >= 1 (the discriminant is the last token, P:173)");
@@ -76,7 +102,7 @@ void build_request(const Pool& pool, const bat_query& q, QueryPlan& qp) {
   };
   if (q.order == BAT_ORDER_UP) {
     if (q.use_cache) {
-      add_prefix_pages(pool, PrefixEnt{BAT_ENT_USER, q.user_id, SEG_USER, nu}, qp);
+      add_prefix_pages(pool, PrefixEnt{BAT_ENT_USER, q.user_id, SEG_USER, nu}, qp, stg);
     } else {
       put(q.user_tok, nu, SEG_USER, 0);
     }
@@ -84,9 +110,9 @@ void build_request(const Pool& pool, const bat_query& q, QueryPlan& qp) {
     put(q.instr_tok, nx, SEG_INSTR, nu + m);
   } else {
     if (q.use_cache) {
-      if (h > 0) add_prefix_pages(pool, PrefixEnt{BAT_ENT_HEADER, q.header_id, SEG_HEADER, h}, qp);
+      if (h > 0) add_prefix_pages(pool, PrefixEnt{BAT_ENT_HEADER, q.header_id, SEG_HEADER, h}, qp, stg);
       for (int i = 0; i < q.n_items; ++i)
-        add_prefix_pages(pool, PrefixEnt{BAT_ENT_ITEM, q.item_id[i], i, q.item_off[i + 1] - q.item_off[i]}, qp);
+        add_prefix_pages(pool, PrefixEnt{BAT_ENT_ITEM, q.item_id[i], i, q.item_off[i + 1] - q.item_off[i]}, qp, stg);
     } else {
       put(q.header_tok, h, SEG_HEADER, 0);
       put_items(h);
@@ -99,7 +125,7 @@ void build_request(const Pool& pool, const bat_query& q, QueryPlan& qp) {
 }
 
 void build_entity(const Pool& pool, const PlanRequest& r, QueryPlan& qp) {
-  if (r.ctx_kind >= 0) add_prefix_pages(pool, PrefixEnt{r.ctx_kind, r.ctx_id, SEG_HEADER, -1}, qp);
+  if (r.ctx_kind >= 0) add_prefix_pages(pool, PrefixEnt{r.ctx_kind, r.ctx_id, SEG_HEADER, -1}, qp, nullptr);
   for (int32_t j = 0; j < r.ent_n; ++j) {
     qp.tokens.push_back(r.ent_tok[j]);
     qp.seg.push_back(SEG_USER);  // one entity alone: plain causal attention
@@ -214,7 +240,8 @@ void classify_tiles(QueryPlan& qp, int32_t qt) {
 }  // namespace
 
 void build_plan(const Pool& pool, int32_t group, int32_t kv_heads,
-                const std::vector<PlanRequest>& reqs, Plan& plan, bool build_image, int32_t grid) {
+                const std::vector<PlanRequest>& reqs, Plan& plan, bool build_image, int32_t grid,
+                StagingCtx* stg) {
   BAT_REQUIRE(group >= 1 && group <= kQtileRows, "group in [1,128]");
   plan.group = group;
   plan.kv_heads = kv_heads;
@@ -234,7 +261,7 @@ void build_plan(const Pool& pool, int32_t group, int32_t kv_heads,
     QueryPlan& qp = plan.q[b];
     const PlanRequest& r = reqs[b];
     if (r.q) {
-      build_request(pool, *r.q, qp);
+      build_request(pool, *r.q, qp, stg);
     } else {
       build_entity(pool, r, qp);
       plan.entity_mode = true;

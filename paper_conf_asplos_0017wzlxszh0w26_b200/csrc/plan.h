@@ -73,7 +73,10 @@ struct Plan {
 // Build the plan of a batch.  Pool supplies the entry -> pages index.  Throws bat::Error.
 // grid > 0: order the attention work lists for a persistent grid of that many CTAs (LPT
 // balance; empty items pad the rounds).
+// stg != nullptr: prefix items that are not local but registered remote are mapped to pages of
+// the staging slot (deduplicated per plan) and their pulls recorded in *stg.
 void build_plan(const Pool& pool, int32_t group, int32_t kv_heads,
-                const std::vector<PlanRequest>& reqs, Plan& plan, bool build_image, int32_t grid = 0);
+                const std::vector<PlanRequest>& reqs, Plan& plan, bool build_image, int32_t grid = 0,
+                StagingCtx* stg = nullptr);
 
 }  // namespace bat

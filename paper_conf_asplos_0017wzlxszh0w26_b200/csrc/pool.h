@@ -2,7 +2,11 @@
 // user / item granularity, every entry a list of 16-token pages holding all layers.
 #pragma once
 
+#include <cuda_runtime.h>
+
 #include <cstdint>
+#include <deque>
+#include <string>
 #include <unordered_map>
 #include <vector>
 
@@ -82,12 +86,47 @@ struct Pool {
   void* fetch_done = nullptr;  // cudaEvent_t: last descriptor upload finished reading fetch_host
   int64_t live_plans = 0;      // bat_plan_build plans not yet destroyed
 
+  // pages released in stream order (bat_kv_release): reusable once `ev` has completed
+  struct PendingFree {
+    cudaEvent_t ev;
+    std::vector<int32_t> pages;
+  };
+  std::deque<PendingFree> pending;
+  std::vector<cudaEvent_t> spare_events;
+  // double-buffered staging of pulled cold item pages for pre-built plans (bat_kv_staging_reserve)
+  std::vector<std::vector<int32_t>> staging;
+
   const Entity* find(int32_t kind, int64_t id) const {
     auto it = index.find(EntityKey{kind, id});
     return it == index.end() ? nullptr : &it->second;
   }
-  // allocate n pages (all-or-nothing)
+  // Move pending pages back to the free list.  wait_stream != nullptr: make that stream wait for
+  // their release events (no host blocking); otherwise the host waits for the events.
+  bool reclaim(int64_t need, cudaStream_t wait_stream, bool use_stream) {
+    while (static_cast<int64_t>(free_pages.size()) < need && !pending.empty()) {
+      PendingFree& f = pending.front();
+      cudaError_t e = use_stream ? cudaStreamWaitEvent(wait_stream, f.ev, 0) : cudaEventSynchronize(f.ev);
+      if (e != cudaSuccess) return false;
+      for (auto it = f.pages.rbegin(); it != f.pages.rend(); ++it) free_pages.push_back(*it);
+      spare_events.push_back(f.ev);
+      pending.pop_front();
+    }
+    return true;
+  }
+  // allocate n pages (all-or-nothing); pages still pending a stream-ordered release are reused
+  // after a host wait on their release events (host-synchronous callers)
   bool alloc_pages(int64_t n, std::vector<int32_t>& out) {
+    if (static_cast<int64_t>(free_pages.size()) < n) reclaim(n, nullptr, false);
+    if (static_cast<int64_t>(free_pages.size()) < n) return false;
+    for (int64_t i = 0; i < n; ++i) {
+      out.push_back(free_pages.back());
+      free_pages.pop_back();
+    }
+    return true;
+  }
+  // ... for asynchronous writers on `st`: pending pages are handed out behind a stream wait
+  bool alloc_pages_on(int64_t n, std::vector<int32_t>& out, cudaStream_t st) {
+    if (static_cast<int64_t>(free_pages.size()) < n) reclaim(n, st, true);
     if (static_cast<int64_t>(free_pages.size()) < n) return false;
     for (int64_t i = 0; i < n; ++i) {
       out.push_back(free_pages.back());
@@ -98,6 +137,21 @@ struct Pool {
   void release_pages(const std::vector<int32_t>& pages) {
     for (auto it = pages.rbegin(); it != pages.rend(); ++it) free_pages.push_back(*it);
   }
+  int64_t n_free() const {
+    int64_t n = static_cast<int64_t>(free_pages.size());
+    for (const auto& f : pending) n += static_cast<int64_t>(f.pages.size());
+    return n;
+  }
+};
+
+// Cold items of a pre-built plan pulled into a staging slot (bat_plan_build_staged): the planner
+// maps every remote (cold-sharded) prefix item to pages of the slot and records the copies.
+struct StagingCtx {
+  const std::vector<int32_t>* slot_pages = nullptr;
+  size_t used = 0;
+  std::unordered_map<EntityKey, Entity, EntityKeyHash> assigned;
+  std::vector<uint64_t> src;  // peer-mapped source page addresses
+  std::vector<int32_t> dst;   // local staging page ids
 };
 
 }  // namespace bat

@@ -6,7 +6,11 @@ weight replica and serves its own requests (requests are independe
 is no per-layer collective).  Items are placed by Algorithm 1 (bat_hrcs_place): the hottest
 r·|F| items are replicated on every rank, the rest are owned round-robin by hotness rank.
 Before a batch, each rank pulls the cold items it needs but does not own from the owners'
-pools over NVLink (CUDA-IPC-mapped arenas, one page-copy kernel: bat_kv_fetch).
+pools over NVLink (CUDA-IPC-mapped arenas) with copy engines on a dedicated copy stream, one batch
+ahead of the compute: ``ColdPipeline`` (reference-counted bat_kv_fetch / stream-ordered
+bat_kv_release) for batches planned at call time, or staged pre-built plans (bat_plan_build_staged
+/ bat_plan_fetch, double-buffered slots) for the device-resident bench leg.  Requests are routed
+with user affinity for User-as-prefix requests and suffix-token balancing (``route_requests``).
 
 The collective steps here are bootstrap only: all_gather of the pools' IPC handles and of
 the owners' page tables.  Works with the "gloo" backend and index-only pools (device = -1)
@@ -80,16 +84,102 @@ def cold_items(queries: Iterable, owner: np.ndarray, rank: int) -> np.ndarray:
 
 
 def fetch_cold(pool: int, ids: np.ndarray, stream=None) -> int:
-    """Pull the cold items over NVLink into local pages (bat_kv_fetch); returns entries pulled."""
+    """Pull the cold items over NVLink into local pages (bat_kv_fetch on `stream`, copy engines;
+    reference counted); returns entries copied."""
     if len(ids) == 0:
         return 0
     return bat.bat_kv_fetch(pool, bat.BAT_ENT_ITEM, ids, stream)
 
 
+def release_cold(pool: int, ids: np.ndarray, stream=None) -> None:
+    """Drop this batch's references to its pulled items; pages freed in `stream` order."""
+    if len(ids):
+        bat.bat_kv_release(pool, bat.BAT_ENT_ITEM, ids, stream)
+
+
 def drop_fetched(pool: int, ids: np.ndarray) -> None:
-    """Release the local copies of pulled items (a per-batch staging policy)."""
+    """Evict the local copies of pulled items outright (host-ordered; no work may still read them)."""
     for i in ids:
         bat.bat_kv_evict(pool, bat.BAT_ENT_ITEM, int(i))
+
+
+class ColdPipeline:
+    """One-batch-ahead cold-item pulls on a dedicated copy stream (fetched from peer GPUs
+    "overlapped with compute").  ``prefetch(k, ids)`` enqueues batch k's pulls on the copy stream and
+    records an event; ``acquire(k)`` makes the compute stream wait for it; ``release(k)`` drops the
+    batch's references in compute-stream order after its work is enqueued.  torch streams/events are
+    plumbing only; the copies are libbat's (bat_kv_fetch / bat_kv_release)."""
+
+    def __init__(self, pool: int, compute_stream, copy_stream):
+        import torch
+        self.torch = torch
+        self.pool, self.compute, self.copy = pool, compute_stream, copy_stream
+        self.ready: Dict[int, object] = {}
+        self.ids: Dict[int, np.ndarray] = {}
+        self.pulled = 0
+
+    def prefetch(self, k: int, ids: np.ndarray) -> None:
+        ev = self.torch.cuda.Event()
+        self.pulled += fetch_cold(self.pool, ids, self.copy)
+        ev.record(self.copy)
+        self.ready[k], self.ids[k] = ev, ids
+
+    def acquire(self, k: int) -> None:
+        self.compute.wait_event(self.ready.pop(k))
+
+    def release(self, k: int) -> None:
+        release_cold(self.pool, self.ids.pop(k), self.compute)
+
+
+def measure_pull_gbs(pool: int, peer: int, peer_pages: Sequence[int], page_bytes: int, stream, reps: int = 3) -> float:
+    """Measured peer -> local pull bandwidth (GB/s) through the production pull path: the peer's
+    pages are registered as temporary remote items (ids < 0), pulled with bat_kv_fetch on
+    `stream` and timed with CUDA events, then released.  Feeds Algorithm 1's B."""
+    import torch
+    ids = np.array([-1000 - i for i in range(len(peer_pages))], dtype=np.int64)
+    for i, pg in zip(ids, peer_pages):
+        bat.bat_kv_register_remote(pool, bat.BAT_ENT_ITEM, int(i), peer, [int(pg)], 16)
+    best = 0.0
+    for _ in range(reps):
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        fetch_cold(pool, ids, stream)
+        e1.record(stream)
+        e1.synchronize()
+        release_cold(pool, ids, stream)
+        ms = e0.elapsed_time(e1)
+        best = max(best, len(ids) * page_bytes / (ms / 1e3) / 1e9)
+    torch.cuda.current_stream().synchronize()
+    stream.synchronize()
+    return best
+
+
+def route_requests(queries: Sequence, world: int, user_rank=None) -> List[List[int]]:
+    """Route a global batch over the ranks ("load-balanced manner"): a cached
+    User-as-prefix request goes to the rank holding its user's prefix (user affinity, default
+    user_id mod world); the other requests fill the least-loaded rank by suffix tokens, longest
+    first.  Returns the request indices of every rank."""
+    user_rank = user_rank or (lambda uid: int(uid) % world)
+    def suffix(q):
+        items = sum(len(t) for t in q.item_toks)
+        if not q.use_cache:
+            return len(q.user_tok) + items + len(q.instr_tok) + len(q.header_tok)
+        return (items if q.order == "UP" else len(q.user_tok)) + len(q.instr_tok)
+    out: List[List[int]] = [[] for _ in range(world)]
+    load = [0] * world
+    rest = []
+    for i, q in enumerate(queries):
+        if q.use_cache and q.order == "UP":
+            r = user_rank(q.user_id)
+            out[r].append(i)
+            load[r] += suffix(q)
+        else:
+            rest.append(i)
+    for i in sorted(rest, key=lambda i: (-suffix(queries[i]), i)):
+        r = min(range(world), key=lambda k: (load[k], k))
+        out[r].append(i)
+        load[r] += suffix(queries[i])
+    return [sorted(x) for x in out]
 
 
 def partition_requests(lengths: Sequence[int], world: int) -> List[List[int]]:

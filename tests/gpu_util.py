@@ -49,9 +49,11 @@ def prefix_entities_in_order(q):
     return out
 
 
-def oracle_attention_layer(cfg, q, entity_kv, qkv_rows, layer, rope_on=True):
+def oracle_attention_layer(cfg, q, entity_kv, qkv_rows, layer, rope_on=True, round_qk=False):
     """fp64 reference of one layer of bipartite attention for request q given the cached
-    prefix K/V (entity_kv[(kind,id)] = (K [L][n][Hkv][d], V)) and the suffix's raw qkv rows."""
+    prefix K/V (entity_kv[(kind,id)] = (K [L][n][Hkv][d], V)) and the suffix's raw qkv rows.
+    round_qk: round the RoPE'd suffix q and k to bf16 (RNE) — the tensor-core operands' own input
+    rounding — for a TIGHTER secondary check that isolates the kernel from that rounding."""
     d, Hq, Hkv = cfg["head_dim"], cfg["q_heads"], cfg["kv_heads"]
     toks, seg, pos = build_sequence(q.order, q.user_tok, q.item_toks, q.instr_tok,
                                     q.header_tok if q.order == "IP" else ())
@@ -66,6 +68,9 @@ def oracle_attention_layer(cfg, q, entity_kv, qkv_rows, layer, rope_on=True):
     if rope_on:
         qq = om.rope(qq, pos[P:], cfg["rope_theta"])
         kk = om.rope(kk, pos[P:], cfg["rope_theta"])
+    if round_qk:
+        qq = synth.bf16_round(qq.astype(np.float32)).astype(np.float64)
+        kk = synth.bf16_round(kk.astype(np.float32)).astype(np.float64)
     if ents:
         Kp = np.concatenate([entity_kv[(k, i)][0][layer] for k, i, _ in ents]).astype(np.float64)
         Vp = np.concatenate([entity_kv[(k, i)][1][layer] for k, i, _ in ents]).astype(np.float64)

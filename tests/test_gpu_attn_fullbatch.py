@@ -7,8 +7,13 @@ bat_debug_attention_layer plans the batch like bat_bipartite_prefill, RoPEs and 
 qkv rows, and runs attn_tc_kernel over the pool's pages of one layer in the production launch
 configuration (persistent grid, LPT work list, device masks).  Prefix KV is random bf16 appended
 with bat_kv_append (values do not change the indexing; the kernel reads them from the pool), q and
-k are scaled so the attention is peaked (|O| ~ 1) and the 2e-2 abs/rel tolerance is not loose
-against the outputs.  A guard asserts that a wrong mask (every key visible) would fail."""
+k are scaled by 1.5 so the attention is peaked (logit std ~2.3) and the 2e-2 abs/rel tolerance is
+not loose against the outputs.  Two checks: (1) the north_star tolerance against the exact fp64
+oracle; (2) 1e-2 abs/rel against the same oracle fed the RoPE'd suffix q/k rounded to bf16 — the
+tensor-core operands' own input rounding, which at larger logit scales (q, k x 2: logit std ~4)
+alone exceeds 2e-2 (measured: excess +0.0098 vs the exact oracle, -0.016 vs the rounded one,
+tools/diag_attn_fullbatch.py) — so (2) bounds everything the kernel adds at half the tolerance.
+A guard asserts that a wrong mask (every key visible) would fail."""
 import numpy as np
 import pytest
 
@@ -42,7 +47,7 @@ def _dummy_model(cfg):
     return DeviceModel(cfg, tensors=dict(embed=emb, lm_head=emb, final_norm=e(H), layers=layers))
 
 
-def _run(B, cfg, queries, sample, n_pages, kscale=2.0):
+def _run(B, cfg, queries, sample, n_pages, kscale=1.5):
     from paper_conf_asplos_0017wzlxszh0w26_b200.runtime import DevicePool
     L, Hkv, d, Hq = cfg["layers"], cfg["kv_heads"], cfg["head_dim"], cfg["q_heads"]
     model = _dummy_model(cfg)
@@ -71,21 +76,23 @@ def _run(B, cfg, queries, sample, n_pages, kscale=2.0):
     torch.cuda.synchronize()
     qkv_np, out_np = qkv.double().cpu().numpy(), out.double().cpu().numpy()
     offs = np.concatenate([[0], np.cumsum(S)])
-    worst, guard, rows = -1.0, -1.0, 0
+    worst, worst_r, guard, rows = -1.0, -1.0, -1.0, 0
     for b in sample:
         q = queries[b]
         x = qkv_np[offs[b]:offs[b + 1]]
         ref = oracle_attention_layer(cfg, q, ekv, x, LAYER)
         got = out_np[offs[b]:offs[b + 1]].reshape(ref.shape)
         worst = max(worst, max_excess(got, ref))
+        ref_r = oracle_attention_layer(cfg, q, ekv, x, LAYER, round_qk=True)
+        worst_r = max(worst_r, max_excess(got, ref_r, 1e-2, 1e-2))
         rows += ref.shape[0]
         if b == sample[0]:  # wrong-mask guard: every key visible
             guard = max_excess(got, _all_visible_attention(cfg, q, ekv, x))
     pool.close()
     model.close()
-    print(f"{len(sample)} requests, {rows} suffix rows x {Hq} heads: worst excess {worst:.4g}, "
-          f"wrong-mask excess {guard:.4g}")
-    return worst, guard
+    print(f"{len(sample)} requests, {rows} suffix rows x {Hq} heads: worst excess {worst:.4g} (2e-2, exact "
+          f"oracle), {worst_r:.4g} (1e-2, bf16-rounded q/k), wrong-mask excess {guard:.4g}")
+    return max(worst, worst_r), guard
 
 
 def _all_visible_attention(cfg, q, ekv, x):

@@ -41,7 +41,7 @@ def test_cold_item_pull_is_bit_exact_and_serves_identically(B):
     cold = bdist.cold_items([q], owner, 0)
     assert list(cold) == sorted(items[:20])
     assert bdist.fetch_cold(local_pool.handle, cold) == 20
-    assert bdist.fetch_cold(local_pool.handle, cold) == 0            # already local: dedup
+    assert bdist.fetch_cold(local_pool.handle, cold) == 0            # already local: one more reference
     L, Hkv, d = cfg["layers"], cfg["kv_heads"], cfg["head_dim"]
     for i in cold[:5]:
         ka = torch.empty(L, 16, Hkv, d, dtype=torch.bfloat16, device="cuda"); va = torch.empty_like(ka)
@@ -55,7 +55,152 @@ def test_cold_item_pull_is_bit_exact_and_serves_identically(B):
     B.bat_bipartite_prefill(local_pool.handle, model.handle, B.QueryArray([q]), h_local)
     torch.cuda.synchronize()
     assert torch.equal(h_owner, h_local)
-    bdist.drop_fetched(local_pool.handle, cold)
+    bdist.release_cold(local_pool.handle, cold)                      # 2 references -> 1: still there
+    B.bat_bipartite_prefill(local_pool.handle, model.handle, B.QueryArray([q]), h_local)
+    bdist.release_cold(local_pool.handle, cold)                      # last reference: freed in stream order
     with pytest.raises(B.BatError):
         B.bat_bipartite_prefill(local_pool.handle, model.handle, B.QueryArray([q]), h_local)
+    with pytest.raises(B.BatError):                                  # more releases than fetches
+        bdist.release_cold(local_pool.handle, cold)
     local_pool.close(); owner_pool.close(); model.close()
+
+
+def _two_pools(B, cfg, model, items, n_pages=2048):
+    from paper_conf_asplos_0017wzlxszh0w26_b200.runtime import DevicePool
+    owner_pool = DevicePool(cfg, n_pages, rank=1, world=2)
+    local_pool = DevicePool(cfg, n_pages, rank=0, world=2)
+    toks = [synth.item_tokens(0, i, 16, cfg["vocab"]) for i in items]
+    for s in range(0, len(items), 256):
+        B.bat_kv_prefill_entities(owner_pool.handle, model.handle, B.BAT_ENT_ITEM, items[s:s + 256], toks[s:s + 256], 0)
+    for i in items:
+        n_tok, pages = B.bat_kv_lookup(owner_pool.handle, B.BAT_ENT_ITEM, i)
+        B.bat_kv_register_remote(local_pool.handle, B.BAT_ENT_ITEM, i, 1, pages, n_tok)
+    B.bat_debug_attach_peer_pool(local_pool.handle, 1, owner_pool.handle)
+    return owner_pool, local_pool
+
+
+def _batches(cfg, items, n_batches, B_req=8, n_items=40, seed=3):
+    rng = np.random.default_rng(seed)
+    return [[synth.make_query(0, cfg, 100 * k + b, 200, rng.choice(items, n_items, replace=False), (16, 16), 4, "IP")
+             for b in range(B_req)] for k in range(n_batches)]
+
+
+def test_cold_pipeline_one_batch_ahead_overlaps_and_serves_identically(B):
+    """ColdPipeline: batch k+1's pull runs on a copy stream while batch k computes; pages of
+    released batches are reused behind stream waits.  Every batch's hidden states equal those of the
+    same batch served from the owner's pool, and the event timeline shows the pulls inside compute."""
+    from paper_conf_asplos_0017wzlxszh0w26_b200 import dist as bdist
+    from paper_conf_asplos_0017wzlxszh0w26_b200.runtime import DeviceModel
+    cfg = synth.model_config("small")
+    model = DeviceModel(cfg, synth.Weights(cfg, seed=1))
+    items = list(range(1000, 1600))
+    owner_pool, local_pool = _two_pools(B, cfg, model, items)
+    batches = _batches(cfg, items, 6)
+    owner = np.full(2000, -1, np.int32)
+    owner[items] = 1
+    compute, copy = torch.cuda.current_stream(), torch.cuda.Stream()
+    pipe = bdist.ColdPipeline(local_pool.handle, compute, copy)
+    free0 = B.bat_kv_pool_stats(local_pool.handle)[0]
+    outs, ev = [], []
+    cold = [bdist.cold_items(b, owner, 0) for b in batches]
+    t0 = torch.cuda.Event(enable_timing=True)
+    t0.record(compute)
+    pipe.prefetch(0, cold[0])
+    for k, qs in enumerate(batches):
+        if k + 1 < len(batches):
+            f0 = torch.cuda.Event(enable_timing=True); f0.record(copy)
+            pipe.prefetch(k + 1, cold[k + 1])
+            f1 = torch.cuda.Event(enable_timing=True); f1.record(copy)
+        pipe.acquire(k)
+        c0 = torch.cuda.Event(enable_timing=True); c0.record(compute)
+        h = torch.empty(len(qs), cfg["hidden"], device="cuda")
+        B.bat_bipartite_prefill(local_pool.handle, model.handle, B.QueryArray(qs), h, compute)
+        c1 = torch.cuda.Event(enable_timing=True); c1.record(compute)
+        pipe.release(k)
+        outs.append(h)
+        ev.append((c0, c1) + ((f0, f1) if k + 1 < len(batches) else ()))
+    torch.cuda.synchronize()
+    assert B.bat_kv_pool_stats(local_pool.handle)[0] == free0  # every pulled page given back
+    overlapped = 0
+    for k in range(len(batches) - 1):
+        c0, c1, f0, f1 = ev[k]
+        a, b, fa, fb = t0.elapsed_time(c0), t0.elapsed_time(c1), t0.elapsed_time(f0), t0.elapsed_time(f1)
+        overlapped += int(fa < b and fb > a)  # the pull of k+1 intersects the compute of k
+        print(f"batch {k}: compute [{a:.3f}, {b:.3f}] ms, pull of {k + 1} [{fa:.3f}, {fb:.3f}] ms")
+    assert overlapped >= len(batches) - 2
+    for qs, h in zip(batches, outs):
+        ref = torch.empty_like(h)
+        B.bat_bipartite_prefill(owner_pool.handle, model.handle, B.QueryArray(qs), ref)
+        torch.cuda.synchronize()
+        assert torch.equal(h, ref)
+    local_pool.close(); owner_pool.close(); model.close()
+
+
+def test_staged_plans_double_buffered_serve_identically(B):
+    """Pre-built plans with staged cold items (bat_plan_build_staged, 2 slots): the pull of batch
+    k+1 into slot (k+1)%2 waits for batch k-1 (same slot) and overlaps batch k; outputs equal the
+    owner-pool plans bit for bit, across two passes over the batches."""
+    from paper_conf_asplos_0017wzlxszh0w26_b200.runtime import DeviceModel
+    cfg = synth.model_config("small")
+    model = DeviceModel(cfg, synth.Weights(cfg, seed=1))
+    items = list(range(2000, 2600))
+    owner_pool, local_pool = _two_pools(B, cfg, model, items)
+    B.bat_kv_staging_reserve(local_pool.handle, 2, 8 * 40)
+    batches = _batches(cfg, items, 4, seed=5)
+    compute, copy = torch.cuda.current_stream(), torch.cuda.Stream()
+    plans = [B.bat_plan_build_staged(local_pool.handle, model.handle, B.QueryArray(qs), k % 2, compute)
+             for k, qs in enumerate(batches)]
+    ref_plans = [B.bat_plan_build(owner_pool.handle, model.handle, B.QueryArray(qs), compute) for qs in batches]
+    refs = []
+    for p, qs in zip(ref_plans, batches):
+        h = torch.empty(len(qs), cfg["hidden"], device="cuda")
+        B.bat_prefill_plan(owner_pool.handle, model.handle, p, h, compute)
+        refs.append(h)
+    n_steps = 8
+    fetched = [None] * (n_steps + 1)
+    done = [None] * n_steps
+    def pull(i):
+        if i >= 2:
+            copy.wait_event(done[i - 2])  # the slot's previous reader has finished
+        n = B.bat_plan_fetch(local_pool.handle, plans[i % 4], copy)
+        e = torch.cuda.Event(); e.record(copy)
+        fetched[i] = e
+        return n
+    assert pull(0) > 0
+    outs = []
+    for i in range(n_steps):
+        if i + 1 < n_steps:
+            pull(i + 1)
+        compute.wait_event(fetched[i])
+        h = torch.empty(len(batches[i % 4]), cfg["hidden"], device="cuda")
+        B.bat_prefill_plan(local_pool.handle, model.handle, plans[i % 4], h, compute)
+        done[i] = torch.cuda.Event(); done[i].record(compute)
+        outs.append(h)
+    torch.cuda.synchronize()
+    for i, h in enumerate(outs):
+        assert torch.equal(h, refs[i % 4]), i
+    with pytest.raises(B.BatError):  # plans built on another pool are refused
+        B.bat_prefill_plan(local_pool.handle, model.handle, ref_plans[0], outs[0], compute)
+    for p in plans + ref_plans:
+        B.bat_plan_destroy(p)
+    local_pool.close(); owner_pool.close(); model.close()
+
+
+def test_plan_pins_entries_until_destroyed(B):
+    """A pre-built plan's device image holds page ids: evicting an entry it reads is refused
+    (BAT_E_STATE) until the plan is destroyed; destroying the pool first is refused too."""
+    from paper_conf_asplos_0017wzlxszh0w26_b200.runtime import DeviceModel, DevicePool, prefill_missing_entities
+    cfg = synth.model_config("tiny")
+    model = DeviceModel(cfg, synth.Weights(cfg, seed=1))
+    pool = DevicePool(cfg, 256)
+    q = synth.make_query(0, cfg, 3, 16, [11, 22, 33, 44], (8, 8), 2, "IP")
+    prefill_missing_entities(pool, model, [q])
+    plan = B.bat_plan_build(pool.handle, model.handle, B.QueryArray([q]))
+    with pytest.raises(B.BatError) as e:
+        B.bat_kv_evict(pool.handle, B.BAT_ENT_ITEM, 22)
+    assert e.value.status == -7
+    with pytest.raises(B.BatError):
+        B.bat_kv_pool_destroy(pool.handle)
+    B.bat_plan_destroy(plan)
+    B.bat_kv_evict(pool.handle, B.BAT_ENT_ITEM, 22)
+    pool.close(); model.close()
