@@ -1,33 +1,44 @@
 #!/usr/bin/env python
 """bench.py — throughput of the BAT bipartite prefill on B200 (one JSON line on rank 0).
 
-Workload (BASELINE.json configs[1]): Qwen2-1.5B-shaped GR ranking model (28 layers, hidden
-1536, 12 Q / 2 KV heads, d 128, ffn 8960, vocab 151936; random bf16 weights), requests of
-1 user of 512 tokens + 100 candidate items of 16 tokens + 8 instruction tokens, served
-Item-as-prefix (the prefix side P:366's larger-side rule picks for |U| = 512 < 1600
-item tokens): the 100 items' KV is read from the paged pool, the 520 user + instruction
-tokens are computed through the 28 layers, then the 100 items are scored.
-A step = one batch of --batch requests (all §8(a) rows: plan, embed, 28 x [norm, QKV,
-RoPE/stage, bipartite attention, O, norm, SwiGLU MLP], last-layer trim, final norm, score).
-Items are drawn Zipf(1.093) from a corpus whose KV was precomputed with the same model
-(bat_kv_prefill_entities, the prefix-miss path) before timing.
+Workload (BASELINE.json configs[2], the largest single-GPU config): Qwen2-1.5B-shaped GR ranking
+model (28 layers, hidden 1536, 12 Q / 2 KV heads, d 128, ffn 8960, vocab 151936; random bf16
+weights); a step = one batch of --batch requests per GPU, each request 1 user of |U| ~
+lognormal(median 1500, sigma 0.8) clipped to [64, 8192] tokens (Table 1) + 200
+candidate items of 16 tokens + 8 instruction tokens; the prefix side is chosen per request by
+the cache-agnostic larger-side rule (User-as-prefix iff |U| >= 200 x 16, else
+Item-as-prefix), so a batch mixes UP requests (the user's KV cached, the 3,208 item + instruction
+tokens computed) and IP requests (the 200 items' KV cached, |U| + 8 tokens computed).  Items are
+drawn Zipf(1.093) from a corpus of --corpus items (default 262,144 = configs[3]'s
+Books-scale corpus) whose KV was precomputed by the model (bat_kv_prefill_entities) before timing;
+UP users' KV likewise.  All §8(a) rows run every step: plan, embed, 28 x [norm, QKV, RoPE/stage,
+bipartite attention, O, norm, SwiGLU MLP], last-layer trim, final norm, score + top-k.
 
-value  = requests/s with inputs resident in HBM (pre-built device plans, bat_prefill_plan).
+value  = requests/s with inputs resident in HBM (pre-built device plans: bat_plan_build_staged +
+         bat_prefill_plan + bat_score).  N > 1: the cold item pages each batch needs are pulled
+         from their owners INSIDE the timed region, one batch ahead on a copy stream (copy
+         engines, bat_plan_fetch into double-buffered staging slots), overlapped with compute.
 e2e    = requests/s through the public call with HOST inputs (bat_bipartite_prefill plans and
-         uploads every step; labels H2D from pinned memory; scores + top-k D2H every step).
-N > 1  = one process per GPU (torchrun); every rank serves its own batches (weak scaling);
-         items are placed hot-replicated / cold-sharded by Algorithm 1 and every
-         rank pulls the cold items it needs from their owners' pools over NVLink (CUDA IPC
-         mapped arenas, bat_kv_fetch) inside the timed region.
+         uploads every step; labels H2D from pinned memory; scores + top-k D2H every step; N > 1:
+         ColdPipeline's reference-counted pulls one batch ahead, stream-ordered releases).
+N > 1  = one process per GPU (torchrun), weak scaling: every step serves a global batch of
+         --batch x N requests routed over the ranks (User-as-prefix requests to the rank caching
+         their user — user affinity; the rest balanced by suffix tokens); the item corpus is
+         placed hot-replicated / cold-sharded by Algorithm 1 with the pull bandwidth B
+         and per-request prefill time t MEASURED in-run (calibration before placement).
+extras = configs[1] (|U| = 512, 100 items) at batch 64 in the IP, UP and RE (full recompute)
+         orderings and the batch-1 IP latency — the kernel-level analogs of the paper's
+         RE-vs-IP / UP-vs-IP comparisons — unless --no-extras.
 
---impl reference times the fp64 CPU oracle (oracle/, full recompute, the plain definition)
-on the host cores on a bounded sample (one layer of one request per step, x28 layers).
+--impl reference times the fp64 CPU oracle (oracle/, full recompute, the plain definition) on the
+host cores on a bounded sample (one layer of one configs[2] request per step, x28 layers).
 """
 from __future__ import annotations
 
 import argparse
 import json
 import os
+import platform
 import statistics
 import subprocess
 import sys
@@ -43,30 +54,38 @@ if ROOT not in sys.path:
 import synth  # noqa: E402
 
 METRIC = "ranking queries/sec & prefill tokens/sec per B200 at 1/2/4/8 GPUs; % tensor peak"
-WORKLOAD = ("configs[1]: Qwen2-1.5B-shaped (28 layers, hidden 1536, 12 Q / 2 KV heads, d=128), "
-            "1 user of 512 tokens + 100 items of 16 tokens, bf16, item-as-prefix")
+WORKLOAD_CFG2 = ("configs[2]: Qwen2-1.5B-shaped (28 layers, hidden 1536, 12 Q / 2 KV heads, d=128), 200 candidate "
+                 "items of 16 tokens, batch of 64 queries per GPU, |U| lognormal(1500, 0.8) in [64, 8192], mixed "
+                 "user-/item-prefix selection (P:366 larger-side rule), bf16")
+WORKLOAD_CFG3 = ("configs[3]: the configs[2] requests over an item KV pool hot-replicated/cold-sharded (Zipf item "
+                 "hotness, Algorithm 1) across {n} B200")
+WORKLOAD_CFG1 = ("configs[1]: Qwen2-1.5B-shaped, 1 user of 512 tokens + 100 items of 16 tokens, bf16, 1 GPU")
+ITEM_LEN, N_INSTR = 16, 8
+WL_ID = {"cfg2": 2, "cfg1-ip": 11, "cfg1-up": 12, "cfg1-re": 13}  # stable across processes
 
 
 def parse():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
-    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--steps", type=int, default=8)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="bat", choices=["bat", "reference"])
     ap.add_argument("--batch", type=int, default=64, help="requests per step per GPU")
-    ap.add_argument("--model", default="qwen2-1.5b", choices=["qwen2-1.5b", "qwen2-7b", "llama3-1b"],
-                    help="model shape (the driver's line is qwen2-1.5b = configs[1])")
-    ap.add_argument("--n-user", type=int, default=512)
-    ap.add_argument("--n-items", type=int, default=100)
-    ap.add_argument("--item-len", type=int, default=16)
-    ap.add_argument("--n-instr", type=int, default=8)
-    ap.add_argument("--corpus", type=int, default=8192, help="items in the corpus")
-    ap.add_argument("--plans", type=int, default=4, help="distinct pre-built batches cycled")
+    ap.add_argument("--model", default="qwen2-1.5b", choices=["qwen2-1.5b", "qwen2-7b", "llama3-1b"])
+    ap.add_argument("--workload", default="cfg2", choices=["cfg2", "cfg1-ip", "cfg1-up", "cfg1-re"],
+                    help="timed workload (the driver's line is cfg2 = configs[2])")
+    ap.add_argument("--n-items", type=int, default=None, help="candidates per request (cfg2: 200, cfg1: 100)")
+    ap.add_argument("--corpus", type=int, default=262144, help="items in the corpus")
+    ap.add_argument("--plans", type=int, default=4, help="distinct pre-built batches cycled (even)")
     ap.add_argument("--alpha", type=float, default=0.1, help="Alg. 1 communication/compute ratio")
     ap.add_argument("--seed", type=int, default=0)
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-extras", action="store_true")
     ap.add_argument("--cpu-budget", type=float, default=20.0, help="seconds of oracle time")
-    return ap.parse_args()
+    a = ap.parse_args()
+    if a.plans % 2:
+        a.plans += 1
+    return a
 
 
 def peaks():
@@ -112,7 +131,7 @@ class ClockSampler:
             self.proc.wait(timeout=5)
         except Exception:
             self.proc.kill()
-        sm, mx, reasons = [], None, set()
+        sm, mx, reasons, pw = [], None, set(), []
         names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
         for ln in self.lines:
             parts = [x.strip() for x in ln.split(",")]
@@ -121,13 +140,15 @@ class ClockSampler:
             try:
                 sm.append(float(parts[0]))
                 mx = float(parts[1])
+                pw.append(float(parts[2]))
             except ValueError:
                 continue
             for n, v in zip(names, parts[4:8]):
                 if v.lower().startswith("active"):
                     reasons.add(n)
         return dict(sm_mhz=statistics.median(sm) if sm else None, sm_max_mhz=mx,
-                    reasons=sorted(reasons), samples=len(sm))
+                    reasons=sorted(reasons), samples=len(sm),
+                    power_w_median=statistics.median(pw) if pw else None)
 
 
 # ---------------------------------------------------------------------- weights
@@ -148,13 +169,31 @@ def device_weights(cfg, seed, device):
                 layers=layers)
 
 
-def make_queries(args, cfg, rng, user0, n, zipf_p):
-    qs = []
+# ----------------------------------------------------------------------- requests
+def n_items_of(args, workload):
+    return args.n_items or (200 if workload == "cfg2" else 100)
+
+
+def global_batch(args, cfg, workload, k, n, zipf_p):
+    """The k-th global batch of n requests of `workload` (deterministic on every rank)."""
+    rng = np.random.default_rng([args.seed, 91, k, WL_ID[workload]])
+    n_items = n_items_of(args, workload)
+    if workload == "cfg2":
+        r = np.random.default_rng([args.seed, 92, k])
+        lens = np.clip(np.round(np.exp(np.log(1500.0) + 0.8 * r.standard_normal(n))), 64, 8192).astype(int)
+    else:
+        lens = np.full(n, 512)
+    out = []
     for b in range(n):
-        items = synth.distinct_label_items(args.seed, cfg, args.n_items, rng, args.corpus, zipf_p)
-        qs.append(synth.make_query(args.seed, cfg, user0 + b, args.n_user, items,
-                                   (args.item_len, args.item_len), args.n_instr, "IP"))
-    return qs
+        items = synth.distinct_label_items(args.seed, cfg, n_items, rng, args.corpus, zipf_p)
+        if workload == "cfg2":  # P:366 larger-side rule (cache-agnostic)
+            order, cache = ("UP" if lens[b] >= n_items * ITEM_LEN else "IP"), True
+        else:
+            order, cache = {"cfg1-ip": ("IP", True), "cfg1-up": ("UP", True), "cfg1-re": ("UP", False)}[workload]
+        uid = 1_000_000 * (1 + k) + 10_000 * WL_ID[workload] + b
+        out.append(synth.make_query(args.seed, cfg, uid, int(lens[b]), items, (ITEM_LEN, ITEM_LEN), N_INSTR,
+                                    order, use_cache=cache))
+    return out
 
 
 def algorithmic_flops_per_request(cfg, S, live_pairs, live_last):
@@ -169,33 +208,14 @@ def algorithmic_flops_per_request(cfg, S, live_pairs, live_last):
 
 
 # --------------------------------------------------------------------- oracle arm
-def oracle_time_per_request(args, budget_s, max_layers=None):
-    """Time the fp64 oracle (full recompute, explicit mask) on one configs[1] request,
-    layer by layer until `budget_s`; returns (seconds per request extrapolated to L layers,
-    sample description, threads)."""
-    from oracle import model as om
-    from oracle.sequence import bipartite_mask, build_sequence
-    cfg = synth.model_config(args.model)
-    W = synth.Weights(cfg, seed=args.seed)
-    q = synth.make_query(args.seed, cfg, 0, args.n_user, list(range(args.n_items)),
-                         (args.item_len, args.item_len), args.n_instr, "IP")
-    toks, seg, pos = build_sequence(q.order, q.user_tok, q.item_toks, q.instr_tok)
-    mask = bipartite_mask(seg)
-    h = np.asarray(W.embed_rows(toks), np.float64)
-    times = []
-    L = cfg["layers"]
-    for l in range(L if max_layers is None else min(L, max_layers)):
-        w = W.layer(l)  # generation outside the timed region
-        t0 = time.perf_counter()
-        h, _, _ = om.layer_forward(cfg, w, h, pos, None, None, mask)
-        times.append(time.perf_counter() - t0)
-        if sum(times) >= budget_s:
-            break
-    per_layer = statistics.mean(times)
-    threads = _blas_threads()
-    sample = (f"1 request (T={len(toks)} tokens, full recompute as the oracle defines it), "
-              f"{len(times)} of {L} layers timed, x{L} extrapolated")
-    return per_layer * L, sample, threads, times
+def cpu_model():
+    try:
+        for ln in open("/proc/cpuinfo"):
+            if ln.startswith("model name"):
+                return ln.split(":", 1)[1].strip()
+    except OSError:
+        pass
+    return platform.processor() or "unknown"
 
 
 def _blas_threads():
@@ -207,16 +227,57 @@ def _blas_threads():
         return len(os.sched_getaffinity(0))
 
 
-def run_reference(args):
-    cfg = synth.model_config(args.model)
-    S = args.n_user + args.n_instr
-    from oracle import model as om
+def _oracle_request(args, cfg):
+    """A median configs[2] request (|U| = 1500, 200 items: IP by the larger-side rule), full
+    recompute as the oracle defines it."""
     from oracle.sequence import bipartite_mask, build_sequence
-    W = synth.Weights(cfg, seed=args.seed)
-    q = synth.make_query(args.seed, cfg, 0, args.n_user, list(range(args.n_items)),
-                         (args.item_len, args.item_len), args.n_instr, "IP")
+    q = synth.make_query(args.seed, cfg, 0, 1500, list(range(n_items_of(args, "cfg2"))), (ITEM_LEN, ITEM_LEN),
+                         N_INSTR, "IP")
     toks, seg, pos = build_sequence(q.order, q.user_tok, q.item_toks, q.instr_tok)
-    mask = bipartite_mask(seg)
+    return toks, pos, bipartite_mask(seg)
+
+
+def oracle_time_per_request(args, budget_s):
+    """Time the fp64 oracle layer by layer on one configs[2] request until `budget_s`, with all
+    host cores, then one layer single-threaded; returns a cpu_baseline dict."""
+    from oracle import model as om
+    cfg = synth.model_config(args.model)
+    W = synth.Weights(cfg, seed=args.seed)
+    toks, pos, mask = _oracle_request(args, cfg)
+    h = np.asarray(W.embed_rows(toks), np.float64)
+    times = []
+    L = cfg["layers"]
+    for l in range(L):
+        w = W.layer(l)  # generation outside the timed region
+        t0 = time.perf_counter()
+        h, _, _ = om.layer_forward(cfg, w, h, pos, None, None, mask)
+        times.append(time.perf_counter() - t0)
+        if sum(times) >= budget_s:
+            break
+    per_layer = statistics.mean(times)
+    threads = _blas_threads()
+    single = None
+    try:
+        from threadpoolctl import threadpool_limits
+        with threadpool_limits(limits=1, user_api="blas"):
+            w = W.layer(0)
+            t0 = time.perf_counter()
+            om.layer_forward(cfg, w, h, pos, None, None, mask)
+            single = 1.0 / ((time.perf_counter() - t0) * L)
+    except Exception:
+        pass
+    return dict(value=1.0 / (per_layer * L), unit="requests/s", cores=threads, kind="oracle",
+                cpu_model=cpu_model(), single_thread_value=single,
+                sample=(f"1 median configs[2] request (|U| = 1500 + 200 x 16 item + 8 instruction tokens, T = {len(toks)}, "
+                        f"fp64 full recompute with explicit mask), {len(times)} of {L} layers timed with {threads} "
+                        f"threads and x{L} extrapolated; single_thread_value = 1 layer with 1 BLAS thread, x{L}"))
+
+
+def run_reference(args):
+    from oracle import model as om
+    cfg = synth.model_config(args.model)
+    W = synth.Weights(cfg, seed=args.seed)
+    toks, pos, mask = _oracle_request(args, cfg)
     h0 = np.asarray(W.embed_rows(toks), np.float64)
     w = W.layer(0)
     times = []
@@ -226,22 +287,366 @@ def run_reference(args):
         dt = time.perf_counter() - t0
         if i >= args.warmup:
             times.append(dt)
-    t_req = statistics.mean(times) * cfg["layers"]
-    value = 1.0 / t_req
+    L = cfg["layers"]
+    value = 1.0 / (statistics.mean(times) * L)
     cores = _blas_threads()
-    sample = (f"each step = 1 of 28 layers of 1 configs[1] request (T={len(toks)}, fp64 full recompute "
-              f"with explicit mask), requests/s = 1 / (28 x mean layer time)")
+    sample = (f"each step = 1 of {L} layers of 1 median configs[2] request (T = {len(toks)}, fp64 full recompute with "
+              f"explicit mask), requests/s = 1 / ({L} x mean layer time)")
     line = dict(metric=METRIC, value=value, unit="requests/s", n_gpus=args.gpus, steps=args.steps,
                 warmup=args.warmup, ms_per_step=1e3 * statistics.mean(times), higher_is_better=True,
                 scaling="weak", vs_baseline=None, dtype="f64", data="synthetic", impl="reference",
-                config=dict(workload=WORKLOAD, batch=1, prefix="IP (oracle: full recompute)"),
-                cpu_baseline=dict(value=value, unit="requests/s", cores=cores, kind="oracle", sample=sample),
+                config=dict(workload=WORKLOAD_CFG2, batch=1, prefix="oracle: full recompute"),
+                cpu_baseline=dict(value=value, unit="requests/s", cores=cores, kind="oracle", sample=sample,
+                                  cpu_model=cpu_model()),
                 e2e=dict(value=value, unit="requests/s", h2d_bytes_per_step=0, d2h_bytes_per_step=0),
-                prefill_tokens_per_s=value * (len(toks)))
+                prefill_tokens_per_s=value * len(toks))
     print(json.dumps(line))
 
 
 # ------------------------------------------------------------------------ GPU arm
+class Server:
+    """One rank's model, pool, corpus and pre-built batches (bookkeeping over the C ABI)."""
+
+    def __init__(self, args, cfg, rank, world, local, dev, red_dev):
+        import torch
+        import torch.distributed as dist
+        from paper_conf_asplos_0017wzlxszh0w26_b200 import bat
+        from paper_conf_asplos_0017wzlxszh0w26_b200 import dist as bdist
+        from paper_conf_asplos_0017wzlxszh0w26_b200.runtime import DeviceModel, DevicePool
+        self.torch, self.dist, self.bat, self.bdist = torch, dist, bat, bdist
+        self.args, self.cfg, self.rank, self.world, self.dev, self.red_dev = args, cfg, rank, world, dev, red_dev
+        self.local = local
+        self.model = DeviceModel(cfg, tensors=device_weights(cfg, 1234, dev), device=local)
+        self.page_bytes = 16 * 2 * cfg["kv_heads"] * cfg["head_dim"] * cfg["layers"] * 2
+        self.kv_tok = self.page_bytes // 16
+        self.compute = torch.cuda.current_stream(dev)
+        self.copy = torch.cuda.Stream(dev)
+        self.zipf = synth.zipf_weights(args.corpus)
+        self.hrcs = None
+        self.plan_host_bytes = {}
+
+    # -- corpus placement (Alg. 1) and prefill
+    def setup_corpus(self, batches_global):
+        args, cfg, bat, bdist = self.args, self.cfg, self.bat, self.bdist
+        world, rank = self.world, self.rank
+        # pages: local corpus share + UP users of this rank's batches + staging for cold items
+        my = [self.route(b) for b in batches_global]
+        user_pages = sum((len(q.user_tok) + 15) // 16 for qs in my for q in qs if q.use_cache and q.order == "UP")
+        owner = np.full(args.corpus, -1, np.int32)
+        calib = None
+        if world > 1:
+            calib = self.calibrate(batches_global[0])
+            r_max = bdist.rmax_for_nvlink(calib["pull_gbs"], calib["t_request_s"], args.alpha,
+                                          n_items_of(args, "cfg2"), ITEM_LEN, world, self.kv_tok)
+            r_rep, owner = bdist.place_items(self.zipf, r_max, world)
+            self.hrcs = dict(replication_ratio=r_rep, r_max=r_max, alpha=args.alpha, **calib)
+        local_items = bdist.local_items(owner, rank)
+        cold_max = 0
+        for qs in my:
+            cold_max = max(cold_max, len(bdist.cold_items(qs, owner, rank)))
+        staging = max(1, cold_max) if world > 1 else 1
+        pages = len(local_items) + user_pages + 2 * staging + 256
+        if world > 1:
+            pages += 2 * staging  # the e2e leg's reference-counted pulls (one batch ahead)
+        if world == 1 and not args.no_extras and args.workload == "cfg2":
+            pages += 2 * 64 * 32  # extras: the configs[1] UP users (|U| = 512: 32 pages each)
+        from paper_conf_asplos_0017wzlxszh0w26_b200.runtime import DevicePool
+        self.pool = DevicePool(cfg, pages, device=self.local, rank=rank, world=world)
+        bat.bat_kv_staging_reserve(self.pool.handle, 2, staging)
+        t0 = time.perf_counter()
+        for s in range(0, len(local_items), 1024):
+            ids = local_items[s:s + 1024]
+            toks = [synth.item_tokens(args.seed, i, ITEM_LEN, cfg["vocab"]) for i in ids]
+            bat.bat_kv_prefill_entities(self.pool.handle, self.model.handle, bat.BAT_ENT_ITEM, ids, toks, 0,
+                                        stream=self.compute)
+        users = {}
+        for qs in my:
+            for q in qs:
+                if q.use_cache and q.order == "UP":
+                    users[int(q.user_id)] = q.user_tok
+        uids = sorted(users)
+        for s in range(0, len(uids), 16):
+            ids = uids[s:s + 16]
+            bat.bat_kv_prefill_entities(self.pool.handle, self.model.handle, bat.BAT_ENT_USER, ids,
+                                        [users[u] for u in ids], 0, stream=self.compute)
+        self.torch.cuda.synchronize()
+        self.t_corpus = time.perf_counter() - t0
+        self.owner = owner
+        if world > 1:
+            bdist.exchange_remote(self.pool.handle, owner, rank, world)
+            self.dist.barrier()
+        self.n_local_items = len(local_items)
+        return my
+
+    def route(self, qs):
+        if self.world == 1:
+            return qs
+        parts = self.bdist.route_requests(qs, self.world)
+        return [qs[i] for i in parts[self.rank]]
+
+    def calibrate(self, batch_global):
+        """Alg. 1 inputs measured in-run: B = the pull bandwidth from a peer's arena through
+        the production copy path; t = prefill seconds per request of this rank's share of a
+        configs[2] batch, its items computed into a scratch pool first."""
+        torch, bat, bdist, cfg, args = self.torch, self.bat, self.bdist, self.cfg, self.args
+        from paper_conf_asplos_0017wzlxszh0w26_b200.runtime import DevicePool, prefill_missing_entities
+        qs = self.route(batch_global)
+        need = sum(len(q.item_ids) for q in qs) + sum((len(q.user_tok) + 15) // 16 for q in qs) + 768
+        tmp = DevicePool(cfg, need, device=self.local, rank=self.rank, world=self.world)
+        prefill_missing_entities(tmp, self.model, qs, stream=self.compute)
+        h = torch.empty(len(qs), cfg["hidden"], device=self.dev)
+        qa = bat.QueryArray(qs)
+        bat.bat_bipartite_prefill(tmp.handle, self.model.handle, qa, h, self.compute)
+        torch.cuda.synchronize()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(self.compute)
+        for _ in range(2):
+            bat.bat_bipartite_prefill(tmp.handle, self.model.handle, qa, h, self.compute)
+        e1.record(self.compute)
+        torch.cuda.synchronize()
+        t_req = e0.elapsed_time(e1) / 2 / 1e3 / max(1, len(qs))
+        # pull bandwidth: every rank pulls 512 pages from the next rank's scratch arena
+        handles = [None] * self.world
+        self.dist.all_gather_object(handles, bat.bat_pool_ipc_handle(tmp.handle))
+        peer = (self.rank + 1) % self.world
+        bat.bat_pool_attach_peer(tmp.handle, peer, handles[peer])
+        n_pg = 256
+        gbs = bdist.measure_pull_gbs(tmp.handle, peer, list(range(n_pg)), self.page_bytes, self.copy)
+        vals = torch.tensor([t_req, gbs], dtype=torch.float64, device=self.red_dev)
+        self.dist.all_reduce(vals, op=self.dist.ReduceOp.SUM)
+        t_req, gbs = float(vals[0]) / self.world, float(vals[1]) / self.world
+        self.dist.barrier()
+        tmp.close()
+        return dict(t_request_s=t_req, pull_gbs=gbs, pull_pages=n_pg)
+
+    def close(self):
+        self.pool.close()
+        self.model.close()
+
+
+def run_timed(S, batches, args, label_k=10, prof=False):
+    """Device-resident leg over the rank's pre-built batches (staged plans, pulls one ahead)."""
+    torch, bat = S.torch, S.bat
+    cfg, dev = S.cfg, S.dev
+    nb = len(batches)
+    plans, infos, labels, nits = [], [], [], []
+    n_max = max(max(q.n_items for q in qs) for qs in batches if qs) if any(batches) else 1
+    for k, qs in enumerate(batches):
+        qa = bat.QueryArray(qs)
+        plans.append(bat.bat_plan_build_staged(S.pool.handle, S.model.handle, qa, k % 2, S.compute))
+        S.plan_host_bytes[k] = bat.bat_plan_bytes(plans[-1])[0]
+        pi = bat.bat_plan_create(S.pool.handle, cfg["q_heads"] // cfg["kv_heads"], qa)
+        infos.append([bat.bat_plan_query_info(pi, b) for b in range(len(qs))])
+        bat.bat_plan_destroy(pi)
+        lab = np.zeros((len(qs), n_max), np.int32)
+        for b, q in enumerate(qs):
+            lab[b, : q.n_items] = q.labels
+        labels.append(torch.tensor(lab, device=dev))
+        nits.append(torch.tensor([q.n_items for q in qs], dtype=torch.int32, device=dev))
+    Bmax = max(len(qs) for qs in batches)
+    hidden = torch.empty(Bmax, cfg["hidden"], device=dev)
+    scores = torch.empty(Bmax, n_max, device=dev)
+    topk = torch.empty(Bmax, label_k, dtype=torch.int32, device=dev)
+    n_steps = args.warmup + args.steps
+    fetched, done = {}, {}
+    pulled_pages = [0]
+
+    def pull(i):
+        if i >= 2:
+            S.copy.wait_event(done[i - 2])  # the slot's previous reader has finished
+        n = bat.bat_plan_fetch(S.pool.handle, plans[i % nb], S.copy)
+        if i >= args.warmup:
+            pulled_pages[0] += n
+        e = torch.cuda.Event()
+        e.record(S.copy)
+        fetched[i] = e
+
+    def step(i):
+        k = i % nb
+        B = len(batches[k])
+        S.compute.wait_event(fetched.pop(i))
+        bat.bat_prefill_plan(S.pool.handle, S.model.handle, plans[k], hidden[:B], S.compute)
+        bat.bat_score(S.model.handle, hidden[:B], labels[k], nits[k], B, n_max, scores[:B], label_k, topk[:B], S.compute)
+        e = torch.cuda.Event()
+        e.record(S.compute)
+        done[i] = e
+
+    pull(0)
+    for i in range(args.warmup):
+        pull(i + 1)
+        step(i)
+    torch.cuda.synchronize()
+    if S.world > 1:
+        S.dist.barrier()
+    if prof:
+        bat.bat_profile_reset(S.model.handle)
+        bat.bat_profile_enable(S.model.handle, True)
+    clk = ClockSampler(S.local)
+    clk.start()
+    n_launch0 = bat.bat_kernel_launch_count()
+    ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    prof_range = os.environ.get("BAT_PROFILE_RANGE") == "1"  # ncu --profile-from-start off
+    torch.cuda.synchronize()
+    if prof_range:
+        torch.cuda.cudart().cudaProfilerStart()
+    ev0.record(S.compute)
+    for i in range(args.warmup, n_steps):
+        if i + 1 < n_steps:
+            pull(i + 1)
+        step(i)
+    S.compute.wait_stream(S.copy)
+    ev1.record(S.compute)
+    torch.cuda.synchronize()
+    if prof_range:
+        torch.cuda.cudart().cudaProfilerStop()
+    launches = bat.bat_kernel_launch_count() - n_launch0
+    clocks = clk.stop()
+    prof_out = None
+    if prof:
+        bat.bat_profile_enable(S.model.handle, False)
+        prof_out = bat.bat_profile_read(S.model.handle)
+    ms = ev0.elapsed_time(ev1)
+    my_req = sum(len(batches[i % nb]) for i in range(args.warmup, n_steps))
+    my_tok = sum(sum(r["S"] for r in infos[i % nb]) for i in range(args.warmup, n_steps))
+    my_flops = 0.0
+    for i in range(args.warmup, n_steps):
+        for r in infos[i % nb]:
+            my_flops += algorithmic_flops_per_request(cfg, r["S"], r["n_live_pairs"], r["n_live_pairs_last"])[0]
+    my_prefix = sum(sum(r["P"] for r in infos[i % nb]) for i in range(args.warmup, n_steps))
+    for p in plans:
+        bat.bat_plan_destroy(p)
+    tot = dict(ms=ms, req=my_req, tok=my_tok, flops=my_flops, prefix=my_prefix, pulled=pulled_pages[0])
+    if S.world > 1:
+        t = torch.tensor([ms], device=S.red_dev)
+        S.dist.all_reduce(t, op=S.dist.ReduceOp.MAX)
+        v = torch.tensor([my_req, my_tok, my_flops, my_prefix, pulled_pages[0]], dtype=torch.float64, device=S.red_dev)
+        S.dist.all_reduce(v, op=S.dist.ReduceOp.SUM)
+        tot.update(ms=float(t.item()), req=float(v[0]), tok=float(v[1]), flops=float(v[2]), prefix=float(v[3]),
+                   pulled=float(v[4]))
+    return tot, prof_out, clocks, launches
+
+
+def run_e2e(S, batches, args, label_k=10):
+    """Public-call leg: host requests through bat_bipartite_prefill every step, labels H2D from
+    pinned memory, scores + top-k D2H; N > 1: ColdPipeline pulls one batch ahead."""
+    torch, bat, bdist = S.torch, S.bat, S.bdist
+    cfg, dev = S.cfg, S.dev
+    nb = len(batches)
+    qas = [bat.QueryArray(qs) for qs in batches]
+    n_max = max(max(q.n_items for q in qs) for qs in batches)
+    labels_h, nits = [], []
+    for qs in batches:
+        lab = np.zeros((len(qs), n_max), np.int32)
+        for b, q in enumerate(qs):
+            lab[b, : q.n_items] = q.labels
+        labels_h.append(torch.tensor(lab).pin_memory())
+        nits.append(torch.tensor([q.n_items for q in qs], dtype=torch.int32, device=dev))
+    Bmax = max(len(qs) for qs in batches)
+    hidden = torch.empty(Bmax, cfg["hidden"], device=dev)
+    scores = torch.empty(Bmax, n_max, device=dev)
+    topk = torch.empty(Bmax, label_k, dtype=torch.int32, device=dev)
+    scores_h = torch.empty(Bmax, n_max).pin_memory()
+    topk_h = torch.empty(Bmax, label_k, dtype=torch.int32).pin_memory()
+    cold = [bdist.cold_items(qs, S.owner, S.rank) for qs in batches]
+    pipe = bdist.ColdPipeline(S.pool.handle, S.compute, S.copy) if S.world > 1 else None
+    n_steps = args.warmup + args.steps
+    h2d = d2h = 0
+
+    def step(i):
+        nonlocal h2d, d2h
+        k = i % nb
+        B = len(batches[k])
+        if pipe:
+            if i + 1 < n_steps:
+                pipe.prefetch(i + 1, cold[(i + 1) % nb])
+            pipe.acquire(i)
+        bat.bat_bipartite_prefill(S.pool.handle, S.model.handle, qas[k], hidden[:B], S.compute)
+        with torch.cuda.stream(S.compute):
+            lab = labels_h[k].to(dev, non_blocking=True)
+        bat.bat_score(S.model.handle, hidden[:B], lab, nits[k], B, n_max, scores[:B], label_k, topk[:B], S.compute)
+        with torch.cuda.stream(S.compute):
+            scores_h[:B].copy_(scores[:B], non_blocking=True)
+            topk_h[:B].copy_(topk[:B], non_blocking=True)
+        if pipe:
+            pipe.release(i)
+        if i == args.warmup:
+            # plan image uploaded by the call (tokens, positions, segments + page tables) + labels;
+            # scores and top-k read back
+            h2d = S.plan_host_bytes.get(k, 0) + lab.numel() * 4
+            d2h = B * n_max * 4 + B * label_k * 4
+
+    if pipe:
+        pipe.prefetch(0, cold[0])
+    for i in range(args.warmup):
+        step(i)
+    torch.cuda.synchronize()
+    if S.world > 1:
+        S.dist.barrier()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    e0.record(S.compute)
+    for i in range(args.warmup, n_steps):
+        step(i)
+    e1.record(S.compute)
+    torch.cuda.synchronize()
+    ms = e0.elapsed_time(e1)
+    req = sum(len(batches[i % nb]) for i in range(args.warmup, n_steps))
+    if S.world > 1:
+        t = torch.tensor([ms, req], dtype=torch.float64, device=S.red_dev)
+        S.dist.all_reduce(t[:1], op=S.dist.ReduceOp.MAX)
+        r = torch.tensor([req], dtype=torch.float64, device=S.red_dev)
+        S.dist.all_reduce(r, op=S.dist.ReduceOp.SUM)
+        ms, req = float(t[0]), float(r[0])
+    return req / (ms / 1e3), h2d, d2h, (pipe.pulled if pipe else 0)
+
+
+def extras(S, args, pk):
+    """configs[1] orderings at batch 64 (rank 0, N = 1 only) and the batch-1 IP latency."""
+    torch, bat = S.torch, S.bat
+    out = {}
+    import copy as _copy
+    a = _copy.copy(args)
+    a.steps, a.warmup = 4, 2
+    for wl in ("cfg1-ip", "cfg1-up", "cfg1-re"):
+        bs = [global_batch(a, S.cfg, wl, 50 + k, 64, S.zipf) for k in range(2)]
+        users = {int(q.user_id): q.user_tok for qs in bs for q in qs if q.use_cache and q.order == "UP"}
+        uids = sorted(users)
+        for s in range(0, len(uids), 16):
+            bat.bat_kv_prefill_entities(S.pool.handle, S.model.handle, bat.BAT_ENT_USER, uids[s:s + 16],
+                                        [users[u] for u in uids[s:s + 16]], 0, stream=S.compute)
+        tot, _, _, _ = run_timed(S, bs, a)
+        out[wl] = dict(requests_per_s=tot["req"] / (tot["ms"] / 1e3), ms_per_step=tot["ms"] / a.steps,
+                       prefill_tokens_per_s=tot["tok"] / (tot["ms"] / 1e3),
+                       algorithmic_tflops=tot["flops"] / (tot["ms"] / 1e3) / 1e12,
+                       suffix_tokens_per_request=tot["tok"] / tot["req"])
+        for u in uids:
+            bat.bat_kv_evict(S.pool.handle, bat.BAT_ENT_USER, u)
+    ip = out["cfg1-ip"]["requests_per_s"]
+    out["re_over_ip_time"] = ip / out["cfg1-re"]["requests_per_s"]
+    out["up_over_ip_time"] = ip / out["cfg1-up"]["requests_per_s"]
+    # batch-1 latency (configs[1] IP, one request per call, median of 40)
+    q1 = global_batch(a, S.cfg, "cfg1-ip", 60, 1, S.zipf)
+    plan = bat.bat_plan_build(S.pool.handle, S.model.handle, bat.QueryArray(q1), S.compute)
+    h = torch.empty(1, S.cfg["hidden"], device=S.dev)
+    lab = torch.tensor(np.asarray(q1[0].labels, np.int32)[None], device=S.dev)
+    nit = torch.tensor([q1[0].n_items], dtype=torch.int32, device=S.dev)
+    sc = torch.empty(1, q1[0].n_items, device=S.dev)
+    tk = torch.empty(1, 10, dtype=torch.int32, device=S.dev)
+    lat = []
+    for i in range(45):
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(S.compute)
+        bat.bat_prefill_plan(S.pool.handle, S.model.handle, plan, h, S.compute)
+        bat.bat_score(S.model.handle, h, lab, nit, 1, q1[0].n_items, sc, 10, tk, S.compute)
+        e1.record(S.compute)
+        e1.synchronize()
+        if i >= 5:
+            lat.append(e0.elapsed_time(e1))
+    bat.bat_plan_destroy(plan)
+    out["batch1_ip_latency_ms"] = dict(median=statistics.median(lat), best=min(lat))
+    out["config"] = WORKLOAD_CFG1 + "; batch 64 (extras), items Zipf from the same corpus"
+    return out
+
+
 def main():
     args = parse()
     world = int(os.environ.get("WORLD_SIZE", "1"))
@@ -256,7 +661,6 @@ def main():
     import torch
     import torch.distributed as dist
     from paper_conf_asplos_0017wzlxszh0w26_b200 import bat
-    from paper_conf_asplos_0017wzlxszh0w26_b200.runtime import DeviceModel, DevicePool
 
     # BAT_BENCH_SHARED_GPU=1 (validation only): several ranks share the visible GPUs, bootstrap
     # and the max-over-ranks reduction go over gloo — exercises the N>1 code path on one GPU
@@ -272,164 +676,14 @@ def main():
             dist.init_process_group("nccl", device_id=dev)
     cfg = synth.model_config(args.model)
     pk = peaks()
+    S = Server(args, cfg, rank, world, local, dev, red_dev)
+    batches_global = [global_batch(args, cfg, args.workload, k, args.batch * world, S.zipf) for k in range(args.plans)]
+    my = S.setup_corpus(batches_global)
 
-    # ---- model + pool
-    model = DeviceModel(cfg, tensors=device_weights(cfg, 1234, dev), device=local)
-    page_bytes = 16 * 2 * cfg["kv_heads"] * cfg["head_dim"] * cfg["layers"] * 2
-    per_item_pages = (args.item_len + 15) // 16
-    pages = args.corpus * per_item_pages * (2 if world > 1 else 1) + 1024
-    pool = DevicePool(cfg, pages, device=local, rank=rank, world=world)
-    stream = torch.cuda.current_stream(dev)
-
-    # ---- item corpus: Zipf hotness, HRCS placement (Alg. 1) for N > 1
-    from paper_conf_asplos_0017wzlxszh0w26_b200 import dist as bdist
-    zipf_p = synth.zipf_weights(args.corpus)
-    t_req_est = 0.0015  # s per request (prefill time t of Alg. 1 line 4, measured order on B200)
-    owner = np.full(args.corpus, -1, np.int32)
-    r_rep = 1.0
-    r_max = None
-    if world > 1:
-        kv_tok = 2 * cfg["kv_heads"] * cfg["head_dim"] * cfg["layers"] * 2
-        r_max = bdist.rmax_for_nvlink(770.0, t_req_est, args.alpha, args.n_items, args.item_len, world, kv_tok)
-        r_rep, owner = bdist.place_items(zipf_p, r_max, world)
-    local_items = bdist.local_items(owner, rank)
-    item_toks = {i: synth.item_tokens(args.seed, i, args.item_len, cfg["vocab"]) for i in local_items}
-    t0 = time.perf_counter()
-    for s in range(0, len(local_items), 1024):
-        ids = local_items[s:s + 1024]
-        bat.bat_kv_prefill_entities(pool.handle, model.handle, bat.BAT_ENT_ITEM, ids, [item_toks[i] for i in ids],
-                                    0, stream=stream)
-    torch.cuda.synchronize()
-    t_corpus = time.perf_counter() - t0
-    if world > 1:
-        bdist.exchange_remote(pool.handle, owner, rank, world)
-        dist.barrier()
-
-    # ---- batches
-    rng = np.random.default_rng([args.seed, rank])
-    n_batches = max(1, args.plans)
-    batches = [make_queries(args, cfg, rng, 10_000_000 * (rank + 1) + 100_000 * k, args.batch, zipf_p)
-               for k in range(n_batches)]
-    qarrays = [bat.QueryArray(b) for b in batches]
-    cold_ids = [bdist.cold_items(b, owner, rank) for b in batches]
-
-    def fetch(k):
-        return bdist.fetch_cold(pool.handle, cold_ids[k], stream) if world > 1 else 0
-
-    def drop(k):
-        if world > 1:
-            bdist.drop_fetched(pool.handle, cold_ids[k])
-
-    B = args.batch
-    n_max = args.n_items
-    hidden = torch.empty(B, cfg["hidden"], device=dev)
-    labels_h = [torch.tensor(np.stack([q.labels for q in b]), dtype=torch.int32).pin_memory() for b in batches]
-    labels_d = [l.to(dev) for l in labels_h]
-    n_items_d = torch.full((B,), args.n_items, dtype=torch.int32, device=dev)
-    scores = torch.empty(B, n_max, device=dev)
-    topk = torch.empty(B, 10, dtype=torch.int32, device=dev)
-    scores_h = torch.empty(B, n_max).pin_memory()
-    topk_h = torch.empty(B, 10, dtype=torch.int32).pin_memory()
-
-    # plan info (suffix tokens, visible pairs) for the FLOP count
-    plans = []
-    info = []
-    for k in range(n_batches):
-        fetch(k)
-        plans.append(bat.bat_plan_build(pool.handle, model.handle, qarrays[k], stream))
-        pi = bat.bat_plan_create(pool.handle, cfg["q_heads"] // cfg["kv_heads"], qarrays[k])
-        info.append([bat.bat_plan_query_info(pi, b) for b in range(B)])
-        bat.bat_plan_destroy(pi)
-    # NOTE: for N > 1 the device plans reference fetched pages; they stay resident (no drop)
-    flops_step = []
-    toks_step = []
-    for inf in info:
-        f = 0.0
-        for r in inf:
-            # the last layer's attention covers only the last q-tile's rows (a8)
-            f += algorithmic_flops_per_request(cfg, r["S"], r["n_live_pairs"], r["n_live_pairs_last"])[0]
-        flops_step.append(f)
-        toks_step.append(sum(r["S"] for r in inf))
-
-    def step_device(k):
-        bat.bat_prefill_plan(pool.handle, model.handle, plans[k % n_batches], hidden, stream)
-        bat.bat_score(model.handle, hidden, labels_d[k % n_batches], n_items_d, B, n_max, scores, 10, topk, stream)
-
-    # ---- device-resident timing
-    for i in range(args.warmup):
-        step_device(i)
-    torch.cuda.synchronize()
-    if world > 1:
-        dist.barrier()
-    bat.bat_profile_reset(model.handle)
-    bat.bat_profile_enable(model.handle, True)
-    clk = ClockSampler(local)
-    clk.start()
-    n_launch0 = bat.bat_kernel_launch_count()
-    ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-    prof_range = os.environ.get("BAT_PROFILE_RANGE") == "1"  # ncu --profile-from-start off
-    torch.cuda.synchronize()
-    if prof_range:
-        torch.cuda.cudart().cudaProfilerStart()
-    ev0.record(stream)
-    for i in range(args.steps):
-        step_device(i)
-    ev1.record(stream)
-    torch.cuda.synchronize()
-    if prof_range:
-        torch.cuda.cudart().cudaProfilerStop()
-    launches = bat.bat_kernel_launch_count() - n_launch0
-    clocks = clk.stop()
-    bat.bat_profile_enable(model.handle, False)
-    prof = bat.bat_profile_read(model.handle)
-    ms = ev0.elapsed_time(ev1)
-    if world > 1:
-        t = torch.tensor([ms], device=red_dev)
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-        ms = float(t.item())
-    ms_step = ms / args.steps
-    total_req = args.steps * B * world
-    value = total_req / (ms / 1e3)
-    alg_flops = sum(flops_step[i % n_batches] for i in range(args.steps))
-    sfx_tokens = sum(toks_step[i % n_batches] for i in range(args.steps))
-
-    # ---- end-to-end through the public call with host inputs
-    for k in range(n_batches):
-        bat.bat_plan_destroy(plans[k])
-    h2d = d2h = 0
-    for i in range(args.warmup):
-        k = i % n_batches
-        bat.bat_bipartite_prefill(pool.handle, model.handle, qarrays[k], hidden, stream)
-    torch.cuda.synchronize()
-    if world > 1:  # release every pulled copy once (batches share cold items)
-        all_cold = np.unique(np.concatenate([c for c in cold_ids] + [np.zeros(0, np.int64)]))
-        bdist.drop_fetched(pool.handle, all_cold)
-        dist.barrier()
-    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-    e0.record(stream)
-    for i in range(args.steps):
-        k = i % n_batches
-        nf = fetch(k)
-        bat.bat_bipartite_prefill(pool.handle, model.handle, qarrays[k], hidden, stream)
-        lab = labels_h[k].to(dev, non_blocking=True)
-        bat.bat_score(model.handle, hidden, lab, n_items_d, B, n_max, scores, 10, topk, stream)
-        scores_h.copy_(scores, non_blocking=True)
-        topk_h.copy_(topk, non_blocking=True)
-        if i == 0:
-            # plan image uploaded by the call + labels; results read back
-            h2d = sum(4 * (2 * r["S"] + 8) for r in info[k]) + lab.numel() * 4
-            d2h = scores_h.numel() * 4 + topk_h.numel() * 4
-        if world > 1:
-            torch.cuda.current_stream(dev).synchronize()
-            drop(k)
-    e1.record(stream)
-    torch.cuda.synchronize()
-    ems = e0.elapsed_time(e1)
-    if world > 1:
-        t = torch.tensor([ems], device=red_dev)
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-        ems = float(t.item())
-    e2e = total_req / (ems / 1e3)
+    tot, prof, clocks, launches = run_timed(S, my, args, prof=True)
+    ms = tot["ms"]
+    value = tot["req"] / (ms / 1e3)
+    e2e, h2d, d2h, e2e_pulled = run_e2e(S, my, args)
 
     # ---- roofline of the dominant kernel (largest share of the step)
     dom = max(prof, key=lambda k: prof[k]["ms"])
@@ -437,8 +691,10 @@ def main():
     achieved = dp["flops"] / (dp["ms"] / 1e3) / 1e12 if dp["ms"] > 0 else 0.0
     traffic = None
     tp = os.path.join(ROOT, "profiles", "ncu_traffic.json")
-    if os.path.exists(tp) and B == 64:  # captured at this batch (layer-0 launch, one ncu --set full)
-        traffic = json.load(open(tp))["dram_bytes_per_launch"].get(dom)
+    if os.path.exists(tp):
+        t = json.load(open(tp))
+        if t.get("workload") == args.workload and t.get("batch") == args.batch:
+            traffic = t["dram_bytes_per_launch"].get(dom)
     roof = dict(kernel=dom, bound="tensor", achieved=achieved, peak=pk["bf16_sus"], unit="TFLOP/s",
                 frac=achieved / pk["bf16_sus"], traffic=traffic,
                 traffic_unit="DRAM bytes per launch (ncu dram__bytes_read.sum + dram__bytes_write.sum)",
@@ -452,31 +708,39 @@ def main():
                        gbs=(v["bytes"] / (v["ms"] / 1e3) / 1e9) if v["ms"] > 0 else None)
                for k, v in prof.items() if v["launches"]}
 
+    ext = None
+    if world == 1 and not args.no_extras and args.workload == "cfg2":
+        ext = extras(S, args, pk)
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
-        t_req, sample, threads, _ = oracle_time_per_request(args, args.cpu_budget)
-        cpu = dict(value=1.0 / t_req, unit="requests/s", cores=threads, kind="oracle", sample=sample)
+        cpu = oracle_time_per_request(args, args.cpu_budget)
 
     if rank == 0:
+        n_up = sum(q.order == "UP" and q.use_cache for qs in batches_global for q in qs)
+        n_all = sum(len(qs) for qs in batches_global)
+        wl = {"cfg2": WORKLOAD_CFG2 if world == 1 else WORKLOAD_CFG2 + "; " + WORKLOAD_CFG3.format(n=world)}.get(
+            args.workload, WORKLOAD_CFG1 + f" ({args.workload})")
+        alg = tot["flops"] / (ms / 1e3) / 1e12
         line = dict(
             metric=METRIC, value=value, unit="requests/s", n_gpus=world, steps=args.steps, warmup=args.warmup,
-            ms_per_step=ms_step, higher_is_better=True, scaling="weak", vs_baseline=None, dtype="bf16",
-            data="synthetic (random-init weights, seeded synthetic requests; item KV computed by the model)",
-            config=dict(workload=WORKLOAD if args.model == "qwen2-1.5b" else
-                        f"{args.model}-shaped, 1 user of {args.n_user} tokens + {args.n_items} items of "
-                        f"{args.item_len} tokens, bf16, item-as-prefix", batch_per_gpu=B, global_batch=B * world, seq_len=args.n_user + args.n_items * args.item_len + args.n_instr,
-                        suffix_tokens_per_request=args.n_user + args.n_instr, prefix_tokens_per_request=args.n_items * args.item_len,
-                        corpus_items=args.corpus, item_hotness="Zipf s=1.093", parallelism=f"dp{world}",
-                        hrcs=dict(replication_ratio=r_rep, r_max=r_max, alpha=args.alpha, t_request_s=0.0015,
-                                  link_gbs=770.0, cold_items_per_step=float(np.mean([len(c) for c in cold_ids])))
-                        if world > 1 else None,
+            ms_per_step=ms / args.steps, higher_is_better=True, scaling="weak", vs_baseline=None, dtype="bf16",
+            data=("synthetic (random-init weights, seeded synthetic requests; item and user KV computed by the "
+                  "model before timing)"),
+            config=dict(workload=wl, model=args.model, batch_per_gpu=args.batch, global_batch=args.batch * world,
+                        n_items=n_items_of(args, args.workload), item_tokens=ITEM_LEN, instr_tokens=N_INSTR,
+                        up_fraction=n_up / max(1, n_all), suffix_tokens_per_request=tot["tok"] / tot["req"],
+                        prefix_tokens_per_request=tot["prefix"] / tot["req"], corpus_items=args.corpus,
+                        item_hotness="Zipf s=1.093", parallelism=f"dp{world}",
+                        routing="UP user affinity + suffix-token balancing" if world > 1 else None,
+                        hrcs=(dict(S.hrcs, cold_pages_pulled_per_step=tot["pulled"] / args.steps / world,
+                                   pull_bytes_per_step=tot["pulled"] * S.page_bytes / args.steps,
+                                   local_items_rank0=S.n_local_items) if world > 1 else None),
                         l2="inputs larger than L2 (2.6 GB of weights streamed every step)"),
-            prefill_tokens_per_s=sfx_tokens * world / (ms / 1e3),
-            served_tokens_per_s=total_req * (args.n_user + args.n_instr + args.n_items * args.item_len) / (ms / 1e3),
-            algorithmic_tflops=alg_flops * world / (ms / 1e3) / 1e12,
-            mfu=dict(of_measured_burst=alg_flops / (ms / 1e3) / 1e12 / pk["bf16"],
-                     of_measured_sustained=alg_flops / (ms / 1e3) / 1e12 / pk["bf16_sus"],
-                     of_spec_2250=alg_flops / (ms / 1e3) / 1e12 / 2250.0),
+            prefill_tokens_per_s=tot["tok"] / (ms / 1e3),
+            served_tokens_per_s=(tot["tok"] + tot["prefix"]) / (ms / 1e3),
+            algorithmic_tflops=alg,
+            mfu=dict(of_measured_burst=alg / world / pk["bf16"], of_measured_sustained=alg / world / pk["bf16_sus"],
+                     of_spec_2250=alg / world / 2250.0),
             roofline=roof,
             attention=dict(tflops=attn_ach, frac_of_sustained=attn_ach / pk["bf16_sus"],
                            frac_of_burst=attn_ach / pk["bf16"], ms_per_step=at["ms"] / args.steps),
@@ -485,9 +749,11 @@ def main():
             gpu_launches=launches,
             clocks=clocks,
             cpu_baseline=cpu,
-            corpus_prefill_s=t_corpus,
+            extras=ext,
+            corpus_prefill_s=S.t_corpus,
         )
         print(json.dumps(line))
+    S.close()
     if world > 1:
         dist.barrier()
         dist.destroy_process_group()

@@ -354,8 +354,8 @@ BAT_API bat_status bat_kv_lookup_remote(bat_pool p, int32_t kind, int64_t id, in
 /* Pull the listed remote (cold-sharded) entries from their owners' arenas over NVLink into local
  * pages, making them resolvable by bat_bipartite_prefill.  The copies are enqueued on
  * `stream` — meant to be a dedicated copy stream, so the pull overlaps compute on another stream
- * (order the compute after it with an event) — as ONE batched copy-engine memcpy
- * (cudaMemcpyBatchAsync, overlap-with-compute hint; no SMs; runs of consecutive pages merged).
+ * (order the compute after it with an event) — as copy-engine memcpys, one per run of
+ * consecutive pages (no SMs taken from the kernels).
  * Pulled copies are reference counted: an id already pulled gets one more reference, replicated /
  * owned (local) ids are skipped; *n_fetched = entries copied by this call.  Pages a previous
  * bat_kv_release gave back are reused behind a stream wait on their release event.  The owners
@@ -379,6 +379,9 @@ BAT_API bat_status bat_kv_release(bat_pool p, int32_t kind, const int64_t* ids, 
 BAT_API bat_status bat_kv_staging_reserve(bat_pool p, int32_t n_slots, int64_t pages_per_slot);
 BAT_API bat_status bat_plan_build_staged(bat_pool p, bat_model m, const bat_query* queries, int32_t B,
                                          int32_t slot, bat_stream_t stream, bat_plan* out);
+/* Bytes of a plan's image: *host_bytes uploaded from the host per call (bat_bipartite_prefill
+ * uploads this much for the same batch), *device_bytes its device footprint incl. the masks. */
+BAT_API bat_status bat_plan_bytes(bat_plan plan, int64_t* host_bytes, int64_t* device_bytes);
 /* Enqueue a staged plan's cold-item pulls on `stream` (copy engines); *n_pages = pages pulled. */
 BAT_API bat_status bat_plan_fetch(bat_pool p, bat_plan plan, int64_t* n_pages, bat_stream_t stream);
 

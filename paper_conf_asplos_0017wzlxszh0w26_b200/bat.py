@@ -137,6 +137,7 @@ def lib() -> ctypes.CDLL:
         "bat_plan_build_staged": (S, [c_void_p, c_void_p, POINTER(bat_query), c_int32, c_int32, c_void_p,
                                       POINTER(c_void_p)]),
         "bat_plan_fetch": (S, [c_void_p, c_void_p, POINTER(c_int64), c_void_p]),
+        "bat_plan_bytes": (S, [c_void_p, POINTER(c_int64), POINTER(c_int64)]),
         "bat_sched_create": (S, [POINTER(bat_sched_cfg), POINTER(c_void_p)]),
         "bat_sched_destroy": (S, [c_void_p]),
         "bat_sched_decide": (S, [c_void_p, c_double, c_int64, c_int32, c_int32, POINTER(bat_sched_decision),
@@ -163,7 +164,7 @@ EXPORTED = ("bat_last_error", "bat_version", "bat_kernel_launch_count", "bat_mod
             "bat_profile_reset", "bat_debug_attach_peer_pool", "bat_sched_create", "bat_sched_destroy",
             "bat_sched_decide", "bat_sched_stats", "bat_sched_is_cached", "bat_score_multi",
             "bat_plan_export_device", "bat_kv_release", "bat_kv_staging_reserve", "bat_plan_build_staged",
-            "bat_plan_fetch")
+            "bat_plan_fetch", "bat_plan_bytes")
 
 
 def _check(status: int) -> None:
@@ -476,6 +477,13 @@ def bat_plan_build_staged(pool: int, model: int, queries: QueryArray, slot: int,
     out = c_void_p()
     _check(lib().bat_plan_build_staged(pool, model, queries.arr, len(queries), slot, _vp(stream), byref(out)))
     return out.value
+
+
+def bat_plan_bytes(plan: int):
+    """(host image bytes uploaded per call, device image bytes)"""
+    h, d = c_int64(), c_int64()
+    _check(lib().bat_plan_bytes(plan, byref(h), byref(d)))
+    return h.value, d.value
 
 
 def bat_plan_fetch(pool: int, plan: int, stream=None) -> int:

@@ -1226,9 +1226,9 @@ bat_status bat_kv_lookup_remote(bat_pool p, int32_t kind, int64_t id, int32_t* o
   });
 }
 
-// Page pulls from peer-mapped arenas: one batched copy-engine memcpy (cudaMemcpyBatchAsync with
-// the overlap-with-compute hint: no SMs taken from the kernels running beside it), runs of
-// consecutive pages merged; BAT_FETCH_SM=1 selects the round-1 SM copy kernel instead.
+// Page pulls from peer-mapped arenas on the copy engines: one cudaMemcpyAsync per run of
+// consecutive pages (no SMs taken from the kernels running beside it; the host-side enqueue is
+// asynchronous); BAT_FETCH_SM=1 selects the round-1 SM copy kernel instead.
 static void issue_page_pulls(Pool& P, const std::vector<uint64_t>& src, const std::vector<int32_t>& dst,
                              cudaStream_t st) {
   if (src.empty()) return;
@@ -1271,17 +1271,7 @@ static void issue_page_pulls(Pool& P, const std::vector<uint64_t>& src, const st
       n.push_back(size_t(pb));
     }
   }
-  if (st == nullptr) {  // the batched API does not take the legacy default stream
-    for (size_t k = 0; k < d.size(); ++k) CUDA_OK(cudaMemcpyAsync(d[k], s[k], n[k], cudaMemcpyDefault, st));
-    return;
-  }
-  cudaMemcpyAttributes attr{};
-  attr.srcAccessOrder = cudaMemcpySrcAccessOrderStream;
-  attr.flags = cudaMemcpyFlagPreferOverlapWithCompute;
-  size_t idx0 = 0, fail_idx = 0;
-  const cudaError_t e = cudaMemcpyBatchAsync(d.data(), s.data(), n.data(), d.size(), &attr, &idx0, 1, &fail_idx, st);
-  if (e != cudaSuccess)
-    fail(BAT_E_CUDA, std::string("cudaMemcpyBatchAsync (copy ") + std::to_string(fail_idx) + "): " + cudaGetErrorString(e));
+  for (size_t k = 0; k < d.size(); ++k) CUDA_OK(cudaMemcpyAsync(d[k], s[k], n[k], cudaMemcpyDefault, st));
 }
 
 bat_status bat_kv_fetch(bat_pool p, int32_t kind, const int64_t* ids, int32_t n, int32_t* n_fetched,
@@ -1544,6 +1534,14 @@ bat_status bat_plan_build(bat_pool p, bat_model mdl, const bat_query* queries, i
 bat_status bat_plan_build_staged(bat_pool p, bat_model mdl, const bat_query* queries, int32_t B, int32_t slot,
                                  bat_stream_t stream, bat_plan* out) {
   return guarded([&] { plan_build_impl(p, mdl, queries, B, slot, stream, out); });
+}
+
+bat_status bat_plan_bytes(bat_plan plan, int64_t* host_bytes, int64_t* device_bytes) {
+  return guarded([&] {
+    BAT_REQUIRE(plan, "null plan");
+    if (host_bytes) *host_bytes = int64_t(plan->plan.img.buf.size()) * 4;
+    if (device_bytes) *device_bytes = plan->plan.img.total_ints * 4;
+  });
 }
 
 bat_status bat_plan_fetch(bat_pool p, bat_plan plan, int64_t* n_pages, bat_stream_t stream) {
