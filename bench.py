@@ -435,9 +435,7 @@ def run_timed(S, batches, args, label_k=10, prof=False):
         qa = bat.QueryArray(qs)
         plans.append(bat.bat_plan_build_staged(S.pool.handle, S.model.handle, qa, k % 2, S.compute))
         S.plan_host_bytes[k] = bat.bat_plan_bytes(plans[-1])[0]
-        pi = bat.bat_plan_create(S.pool.handle, cfg["q_heads"] // cfg["kv_heads"], qa)
-        infos.append([bat.bat_plan_query_info(pi, b) for b in range(len(qs))])
-        bat.bat_plan_destroy(pi)
+        infos.append([bat.bat_plan_query_info(plans[-1], b) for b in range(len(qs))])
         lab = np.zeros((len(qs), n_max), np.int32)
         for b, q in enumerate(qs):
             lab[b, : q.n_items] = q.labels
@@ -473,8 +471,8 @@ def run_timed(S, batches, args, label_k=10, prof=False):
 
     pull(0)
     for i in range(args.warmup):
-        pull(i + 1)
         step(i)
+        pull(i + 1)
     torch.cuda.synchronize()
     if S.world > 1:
         S.dist.barrier()
@@ -491,9 +489,9 @@ def run_timed(S, batches, args, label_k=10, prof=False):
         torch.cuda.cudart().cudaProfilerStart()
     ev0.record(S.compute)
     for i in range(args.warmup, n_steps):
+        step(i)  # compute first: the GPU starts while the host enqueues the next batch's pulls
         if i + 1 < n_steps:
             pull(i + 1)
-        step(i)
     S.compute.wait_stream(S.copy)
     ev1.record(S.compute)
     torch.cuda.synchronize()
@@ -557,8 +555,6 @@ def run_e2e(S, batches, args, label_k=10):
         k = i % nb
         B = len(batches[k])
         if pipe:
-            if i + 1 < n_steps:
-                pipe.prefetch(i + 1, cold[(i + 1) % nb])
             pipe.acquire(i)
         bat.bat_bipartite_prefill(S.pool.handle, S.model.handle, qas[k], hidden[:B], S.compute)
         with torch.cuda.stream(S.compute):
@@ -567,7 +563,9 @@ def run_e2e(S, batches, args, label_k=10):
         with torch.cuda.stream(S.compute):
             scores_h[:B].copy_(scores[:B], non_blocking=True)
             topk_h[:B].copy_(topk[:B], non_blocking=True)
-        if pipe:
+        if pipe:  # next batch's pulls ride under this batch's compute; then drop this batch's refs
+            if i + 1 < n_steps:
+                pipe.prefetch(i + 1, cold[(i + 1) % nb])
             pipe.release(i)
         if i == args.warmup:
             # plan image uploaded by the call (tokens, positions, segments + page tables) + labels;

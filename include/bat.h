@@ -340,6 +340,20 @@ BAT_API bat_status bat_sched_stats(bat_sched s, int64_t out[7]);
 /* Whether user_id's prefix is cached. */
 BAT_API int32_t bat_sched_is_cached(bat_sched s, int64_t user_id);
 
+/* Background placement update (P:312 Step 3: "replace the KV cache item according to ad hoc
+ * hotness in a background process ... update these items in the replicate area"; footnote P:322:
+ * new items "by a similar background compute and update strategy"; reading DESIGN.md R21).
+ * owner_old[0..n_old): the current placement (-1 replicated, else the owning rank); freq_new
+ * [0..n_new): new access frequencies, ids >= n_old are new items.  owner_new[0..n_new): the
+ * replicated area keeps floor(r * n_new + 1/2) items — the top ones by freq_new (descending, lower id
+ * first, Algorithm 1 line 8) — cold items keep their owner, and items leaving the replicated
+ * area or new cold items go to the rank owning the fewest cold items (ties: lowest rank),
+ * hottest first.  Moves follow from the diff: promoted items are pulled by every other rank
+ * (bat_kv_replicate), demoted ones dropped (bat_kv_evict) by every rank but the new owner, new
+ * items computed (bat_kv_prefill_entities) by their owner, or by every rank if replicated. */
+BAT_API bat_status bat_hrcs_refresh(const int32_t* owner_old, int64_t n_old, const double* freq_new, int64_t n_new,
+                                    double r, int32_t world, int32_t* owner_new);
+
 /* CUDA-IPC export of the pool arena (64-byte handle) and import of a peer's arena. */
 BAT_API bat_status bat_pool_ipc_handle(bat_pool p, void* handle_out64);
 BAT_API bat_status bat_pool_attach_peer(bat_pool p, int32_t peer_rank, const void* handle64);
@@ -363,6 +377,10 @@ BAT_API bat_status bat_kv_lookup_remote(bat_pool p, int32_t kind, int64_t id, in
  * registered remote; all-or-nothing. */
 BAT_API bat_status bat_kv_fetch(bat_pool p, int32_t kind, const int64_t* ids, int32_t n,
                         int32_t* n_fetched, bat_stream_t stream);
+/* Pull the listed remote entries as REGULAR local entries (a replicated-area refresh): as
+ * bat_kv_fetch on `stream`, but the copies are not reference counted (bat_kv_evict drops them);
+ * local ids are skipped; BAT_E_STATE for an id currently held as a pulled (counted) copy. */
+BAT_API bat_status bat_kv_replicate(bat_pool p, int32_t kind, const int64_t* ids, int32_t n, bat_stream_t stream);
 /* Drop one reference per listed pulled entry (ids as passed to bat_kv_fetch; local ids are
  * skipped).  An entry whose last reference goes is removed and its pages are freed IN STREAM
  * ORDER: they become reusable once the work enqueued on `stream` so far (the batches reading them)

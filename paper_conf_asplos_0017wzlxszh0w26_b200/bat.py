@@ -138,6 +138,9 @@ def lib() -> ctypes.CDLL:
                                       POINTER(c_void_p)]),
         "bat_plan_fetch": (S, [c_void_p, c_void_p, POINTER(c_int64), c_void_p]),
         "bat_plan_bytes": (S, [c_void_p, POINTER(c_int64), POINTER(c_int64)]),
+        "bat_hrcs_refresh": (S, [POINTER(c_int32), c_int64, POINTER(c_double), c_int64, c_double, c_int32,
+                                 POINTER(c_int32)]),
+        "bat_kv_replicate": (S, [c_void_p, c_int32, POINTER(c_int64), c_int32, c_void_p]),
         "bat_sched_create": (S, [POINTER(bat_sched_cfg), POINTER(c_void_p)]),
         "bat_sched_destroy": (S, [c_void_p]),
         "bat_sched_decide": (S, [c_void_p, c_double, c_int64, c_int32, c_int32, POINTER(bat_sched_decision),
@@ -164,7 +167,7 @@ EXPORTED = ("bat_last_error", "bat_version", "bat_kernel_launch_count", "bat_mod
             "bat_profile_reset", "bat_debug_attach_peer_pool", "bat_sched_create", "bat_sched_destroy",
             "bat_sched_decide", "bat_sched_stats", "bat_sched_is_cached", "bat_score_multi",
             "bat_plan_export_device", "bat_kv_release", "bat_kv_staging_reserve", "bat_plan_build_staged",
-            "bat_plan_fetch", "bat_plan_bytes")
+            "bat_plan_fetch", "bat_plan_bytes", "bat_hrcs_refresh", "bat_kv_replicate")
 
 
 def _check(status: int) -> None:
@@ -429,6 +432,20 @@ def bat_hrcs_place(freq: Sequence[float], r_max: float, world: int):
     _check(lib().bat_hrcs_place(f.ctypes.data_as(POINTER(c_double)), len(f), r_max, world,
                                 _i32p(owner), byref(r)))
     return r.value, owner
+
+
+def bat_hrcs_refresh(owner_old: Sequence[int], freq_new: Sequence[float], r: float, world: int) -> np.ndarray:
+    o = np.ascontiguousarray(owner_old, dtype=np.int32)
+    f = np.ascontiguousarray(freq_new, dtype=np.float64)
+    out = np.zeros(len(f), dtype=np.int32)
+    _check(lib().bat_hrcs_refresh(_i32p(o) if len(o) else None, len(o), f.ctypes.data_as(POINTER(c_double)), len(f),
+                                  r, world, _i32p(out)))
+    return out
+
+
+def bat_kv_replicate(pool: int, kind: int, ids: Sequence[int], stream=None) -> None:
+    a = np.ascontiguousarray(ids, dtype=np.int64)
+    _check(lib().bat_kv_replicate(pool, kind, _i64p(a), len(a), _vp(stream)))
 
 
 def bat_pool_ipc_handle(pool: int) -> bytes:

@@ -1163,6 +1163,41 @@ bat_status bat_hrcs_place(const double* freq, int64_t n, double r_max, int32_t w
   });
 }
 
+// Background placement update (P:312 Step 3, footnote P:322; R21): replicated area =
+// top round(r n_new) by the new frequencies; cold items keep their owner; demoted and new cold
+// items go to the rank owning the fewest cold items (ties: lowest rank), hottest first.
+bat_status bat_hrcs_refresh(const int32_t* owner_old, int64_t n_old, const double* freq_new, int64_t n_new,
+                            double r, int32_t world, int32_t* owner_new) {
+  return guarded([&] {
+    BAT_REQUIRE(freq_new && owner_new && (owner_old || n_old == 0) && n_new >= n_old && n_new >= 1 && world >= 1,
+                "argument");
+    BAT_REQUIRE(r >= 0.0 && r <= 1.0, "r in [0, 1]");
+    std::vector<int64_t> order(n_new);
+    std::iota(order.begin(), order.end(), 0);
+    std::stable_sort(order.begin(), order.end(), [&](int64_t a, int64_t b) { return freq_new[a] > freq_new[b]; });
+    const int64_t n_rep = static_cast<int64_t>(std::floor(r * double(n_new) + 0.5));  // round half up
+    std::vector<uint8_t> rep(n_new, 0);
+    for (int64_t k = 0; k < n_rep; ++k) rep[order[k]] = 1;
+    std::vector<int64_t> load(world, 0);
+    for (int64_t i = 0; i < n_old; ++i) {
+      BAT_REQUIRE(owner_old[i] >= -1 && owner_old[i] < world, "owner_old out of range");
+      if (!rep[i] && owner_old[i] >= 0) {
+        owner_new[i] = owner_old[i];
+        ++load[owner_old[i]];
+      }
+    }
+    for (int64_t i : order) {
+      if (rep[i]) {
+        owner_new[i] = -1;
+      } else if (i >= n_old || owner_old[i] < 0) {
+        const int32_t k = static_cast<int32_t>(std::min_element(load.begin(), load.end()) - load.begin());
+        owner_new[i] = k;
+        ++load[k];
+      }
+    }
+  });
+}
+
 // ------------------------------------------------------------- NVLink page pull (a10)
 bat_status bat_pool_ipc_handle(bat_pool p, void* out64) {
   return guarded([&] {
@@ -1336,6 +1371,28 @@ bat_status bat_kv_fetch(bat_pool p, int32_t kind, const int64_t* ids, int32_t n,
       throw;
     }
     if (n_fetched) *n_fetched = fetched;
+  });
+}
+
+bat_status bat_kv_replicate(bat_pool p, int32_t kind, const int64_t* ids, int32_t n, bat_stream_t stream) {
+  return guarded([&] {
+    BAT_REQUIRE(p && (ids || n == 0), "null argument");
+    Pool& P = p->pool;
+    for (int32_t i = 0; i < n; ++i) {
+      auto it = P.index.find(EntityKey{kind, ids[i]});
+      if (it != P.index.end() && it->second.fetched)
+        fail(BAT_E_STATE, "entry is a pulled (reference-counted) copy; release it first");
+    }
+    int32_t nf = 0;
+    const bat_status st = bat_kv_fetch(p, kind, ids, n, &nf, stream);
+    if (st != BAT_OK) fail(st, last_error());
+    for (int32_t i = 0; i < n; ++i) {  // the new copies become regular local (replicated) entries
+      auto it = P.index.find(EntityKey{kind, ids[i]});
+      if (it != P.index.end() && it->second.fetched) {
+        it->second.fetched = false;
+        it->second.refs = 0;
+      }
+    }
   });
 }
 

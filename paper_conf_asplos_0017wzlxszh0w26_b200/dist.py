@@ -107,7 +107,9 @@ class ColdPipeline:
     """One-batch-ahead cold-item pulls on a dedicated copy stream (fetched from peer GPUs
     "overlapped with compute").  ``prefetch(k, ids)`` enqueues batch k's pulls on the copy stream and
     records an event; ``acquire(k)`` makes the compute stream wait for it; ``release(k)`` drops the
-    batch's references in compute-stream order after its work is enqueued.  torch streams/events are
+    batch's references in compute-stream order after its work is enqueued.  Per step:
+    acquire(k), enqueue batch k's compute, prefetch(k + 1) (its copies run under batch k's
+    compute; items batch k also holds only gain a reference), release(k).  torch streams/events are
     plumbing only; the copies are libbat's (bat_kv_fetch / bat_kv_release)."""
 
     def __init__(self, pool: int, compute_stream, copy_stream):

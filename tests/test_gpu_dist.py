@@ -95,7 +95,7 @@ def test_cold_pipeline_one_batch_ahead_overlaps_and_serves_identically(B):
     model = DeviceModel(cfg, synth.Weights(cfg, seed=1))
     items = list(range(1000, 1600))
     owner_pool, local_pool = _two_pools(B, cfg, model, items)
-    batches = _batches(cfg, items, 6)
+    batches = _batches(cfg, items, 6, B_req=24, n_items=24)  # compute long enough to hide a pull
     owner = np.full(2000, -1, np.int32)
     owner[items] = 1
     compute, copy = torch.cuda.current_stream(), torch.cuda.Stream()
@@ -106,16 +106,17 @@ def test_cold_pipeline_one_batch_ahead_overlaps_and_serves_identically(B):
     t0 = torch.cuda.Event(enable_timing=True)
     t0.record(compute)
     pipe.prefetch(0, cold[0])
+    qas = [B.QueryArray(qs) for qs in batches]
     for k, qs in enumerate(batches):
+        pipe.acquire(k)
+        c0 = torch.cuda.Event(enable_timing=True); c0.record(compute)
+        h = torch.empty(len(qs), cfg["hidden"], device="cuda")
+        B.bat_bipartite_prefill(local_pool.handle, model.handle, qas[k], h, compute)
+        c1 = torch.cuda.Event(enable_timing=True); c1.record(compute)
         if k + 1 < len(batches):
             f0 = torch.cuda.Event(enable_timing=True); f0.record(copy)
             pipe.prefetch(k + 1, cold[k + 1])
             f1 = torch.cuda.Event(enable_timing=True); f1.record(copy)
-        pipe.acquire(k)
-        c0 = torch.cuda.Event(enable_timing=True); c0.record(compute)
-        h = torch.empty(len(qs), cfg["hidden"], device="cuda")
-        B.bat_bipartite_prefill(local_pool.handle, model.handle, B.QueryArray(qs), h, compute)
-        c1 = torch.cuda.Event(enable_timing=True); c1.record(compute)
         pipe.release(k)
         outs.append(h)
         ev.append((c0, c1) + ((f0, f1) if k + 1 < len(batches) else ()))

@@ -43,9 +43,10 @@ def test_two_process_cold_item_pull_and_serving(tmp_path):
 
 
 def test_bench_two_ranks_on_one_gpu_prints_a_valid_line():
-    """bench.py's N > 1 path (torchrun, HRCS placement, IPC exchange, per-step cold pulls,
-    max-over-ranks timing) end to end with two ranks sharing the GPU (BAT_BENCH_SHARED_GPU=1:
-    gloo bootstrap).  Only the contract is checked — two ranks on one GPU time nothing real."""
+    """bench.py's N > 1 path (torchrun, in-run calibration of Alg. 1's B and t, HRCS placement, IPC
+    exchange, request routing, staged cold pulls one batch ahead inside the timed region,
+    max-over-ranks timing) end to end with two ranks sharing the GPU (BAT_BENCH_SHARED_GPU=1: gloo
+    bootstrap).  Only the contract is checked — two ranks on one GPU time nothing real."""
     if not torch.cuda.is_available():
         pytest.skip("no CUDA device")
     import json
@@ -59,4 +60,6 @@ def test_bench_two_ranks_on_one_gpu_prints_a_valid_line():
     assert len(lines) == 1  # rank 0 only
     d = json.loads(lines[0])
     assert d["n_gpus"] == 2 and d["config"]["global_batch"] == 8 and d["value"] > 0
-    assert d["config"]["hrcs"]["cold_items_per_step"] > 0 and d["e2e"]["value"] > 0
+    h = d["config"]["hrcs"]
+    assert h["cold_pages_pulled_per_step"] > 0 and d["e2e"]["value"] > 0
+    assert h["pull_gbs"] > 0 and h["t_request_s"] > 0  # Alg. 1 inputs measured in-run

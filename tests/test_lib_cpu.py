@@ -211,3 +211,20 @@ def test_hrcs_matches_oracle(B, seed):
             exp = np.array([-1 if i in set(rep) else own[i] for i in range(n)], dtype=np.int32)
             np.testing.assert_array_equal(owner, exp)
     assert B.bat_hrcs_rmax(100, 2, 0.1, 10, 5, 4) == pytest.approx(ohrcs.rmax_paper(100, 2, 0.1, 10, 5, 4), rel=1e-15)
+
+
+@pytest.mark.parametrize("seed", range(5))
+def test_hrcs_refresh_matches_oracle(B, seed):
+    rng = np.random.default_rng(50 + seed)
+    n_old = int(rng.integers(1, 300))
+    n_new = n_old + int(rng.integers(0, 40))
+    for world in (1, 2, 8):
+        for r in (0.0, 0.1, 0.5, 1.0):
+            F_old = rng.pareto(1.1, size=n_old) + 1e-3
+            F_old[rng.integers(0, n_old, size=n_old // 4)] = F_old[0]  # ties
+            rep, own = ohrcs.place(F_old, r, world)
+            owner_old = [-1 if i in set(rep) else own[i] for i in range(n_old)]
+            F_new = rng.pareto(1.1, size=n_new) + 1e-3
+            F_new[rng.integers(0, n_new, size=n_new // 4)] = F_new[-1]
+            got = B.bat_hrcs_refresh(owner_old, F_new, r, world)
+            np.testing.assert_array_equal(got, np.array(ohrcs.refresh(owner_old, F_new, r, world), np.int32))

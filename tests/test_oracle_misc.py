@@ -125,3 +125,43 @@ def test_simulation_degenerate_policies_are_closed_forms():
     # zero capacity: hotness never admits, so it is IP for every request
     _, t_h = scheduler.simulate(tr, "hotness", 0, 5.0)
     assert t_h["ip"] == len(tr) and t_h["hits"] == 0
+
+
+# ------------------------------------------------ placement refresh (footnote P:322; R21)
+def test_refresh_hand_case():
+    """5 placed items, 1 new; r = 1/3 of 6 -> 2 replicated.  New order: 1 (.5), 2 (.2), 0 (.1),
+    5 (.1, new), 3, 4 (.05).  Replicated {1, 2}; 3 and 4 keep owners 0 / 1 (loads 1, 1); demoted
+    item 0 -> rank 0 (tie -> lower rank), new item 5 -> rank 1."""
+    assert hrcs.refresh([-1, 0, 1, 0, 1], [0.1, 0.5, 0.2, 0.05, 0.05, 0.1], 1 / 3, 2) == [0, -1, -1, 0, 1, 1]
+
+
+@pytest.mark.parametrize("seed", range(6))
+def test_refresh_invariants(seed):
+    """The replicated area is exactly Algorithm 1's top-r set under the new frequencies (the
+    same set place() picks); items cold before and after never move; every rank's cold load
+    differs by at most the imbalance it already had (new assignments go to the least loaded)."""
+    rng = np.random.default_rng(seed)
+    n_old, n_new, N = int(rng.integers(10, 200)), 0, int(rng.integers(1, 6))
+    n_new = n_old + int(rng.integers(0, 30))
+    F_old = rng.pareto(1.1, size=n_old) + 1e-3
+    r = float(rng.uniform(0, 0.5))
+    rep, own = hrcs.place(F_old, r, N)
+    owner_old = [-1 if i in set(rep) else own[i] for i in range(n_old)]
+    F_new = rng.pareto(1.1, size=n_new) + 1e-3
+    owner_new = hrcs.refresh(owner_old, F_new, r, N)
+    rep_new, _ = hrcs.place(F_new, r, N)
+    assert {i for i in range(n_new) if owner_new[i] < 0} == set(rep_new)
+    for i in range(n_old):
+        if owner_old[i] >= 0 and owner_new[i] >= 0:
+            assert owner_new[i] == owner_old[i]
+    loads = [sum(1 for o in owner_new if o == k) for k in range(N)]
+    kept = [sum(1 for i in range(n_old) if owner_old[i] == k and owner_new[i] == k) for k in range(N)]
+    assert max(loads) - min(loads) <= max(1, max(kept) - min(kept))
+
+
+def test_refresh_without_change_is_identity():
+    """Same frequencies, same r, no new items: the placement of Algorithm 1 is a fixed point."""
+    F = np.arange(50, 0, -1, dtype=float)
+    rep, own = hrcs.place(F, 0.2, 3)
+    owner = [-1 if i in set(rep) else own[i] for i in range(50)]
+    assert hrcs.refresh(owner, F, 0.2, 3) == owner
