@@ -900,7 +900,8 @@ bat_status bat_kv_prefill_entities(bat_pool p, bat_model mdl, int32_t kind, int3
         reqs[e].ent_pages = &pages[e];
       }
       Plan plan;
-      build_plan(P, m.cfg.q_heads / m.cfg.kv_heads, m.cfg.kv_heads, reqs, plan, true, attn_grid_slots(m.dpad, m.num_sms));
+      build_plan(P, m.cfg.q_heads / m.cfg.kv_heads, m.cfg.kv_heads, reqs, plan, true, attn_grid_slots(m.dpad, m.num_sms),
+                 nullptr, attn_qtiles_per_item());
       run_plan(P, m, plan, nullptr, static_cast<cudaStream_t>(stream));
       CUDA_OK(cudaStreamSynchronize(static_cast<cudaStream_t>(stream)));
     } catch (...) {
@@ -944,7 +945,8 @@ bat_status bat_bipartite_prefill(bat_pool p, bat_model mdl, const bat_query* que
     for (int b = 0; b < B; ++b) validate_tokens(queries[b], m.cfg.vocab);
     DeviceGuard dg(P.device);
     Plan plan;
-    build_plan(P, m.cfg.q_heads / m.cfg.kv_heads, m.cfg.kv_heads, wrap(queries, B), plan, true, attn_grid_slots(m.dpad, m.num_sms));
+    build_plan(P, m.cfg.q_heads / m.cfg.kv_heads, m.cfg.kv_heads, wrap(queries, B), plan, true, attn_grid_slots(m.dpad, m.num_sms),
+               nullptr, attn_qtiles_per_item());
     run_plan(P, m, plan, out_hidden, static_cast<cudaStream_t>(stream));
   });
 }
@@ -1485,7 +1487,8 @@ bat_status bat_debug_attention_layer(bat_pool p, bat_model mdl, const bat_query*
     DeviceGuard dg(P.device);
     cudaStream_t st = static_cast<cudaStream_t>(stream);
     Plan plan;
-    build_plan(P, m.cfg.q_heads / m.cfg.kv_heads, m.cfg.kv_heads, wrap(queries, B), plan, true, attn_grid_slots(m.dpad, m.num_sms));
+    build_plan(P, m.cfg.q_heads / m.cfg.kv_heads, m.cfg.kv_heads, wrap(queries, B), plan, true, attn_grid_slots(m.dpad, m.num_sms),
+               nullptr, attn_qtiles_per_item());
     const int32_t* I = prepare(P, m, plan, st);
     StageParams sp = stage_params(P, m, plan, I);
     sp.qkv = static_cast<const __nv_bfloat16*>(qkv);
@@ -1558,7 +1561,7 @@ static void plan_build_impl(bat_pool p, bat_model mdl, const bat_query* queries,
     stg.slot_pages = &P.staging[slot];
   }
   build_plan(P, m.cfg.q_heads / m.cfg.kv_heads, m.cfg.kv_heads, wrap(queries, B), pl->plan, true,
-             attn_grid_slots(m.dpad, m.num_sms), slot >= 0 ? &stg : nullptr);
+             attn_grid_slots(m.dpad, m.num_sms), slot >= 0 ? &stg : nullptr, attn_qtiles_per_item());
   pl->pull_src = std::move(stg.src);
   pl->pull_dst = std::move(stg.dst);
   pl->slot = slot;

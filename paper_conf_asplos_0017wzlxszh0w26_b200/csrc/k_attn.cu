@@ -30,6 +30,7 @@
 //               moves when a row's exponent would exceed 2^8 (lazy rescaling).
 // TMEM (512 columns): S0 [0,128) S1 [128,256) O0 [256,384) O1 [384,512).
 #include <cstdlib>
+#include <string>
 #include <cuda_bf16.h>
 #include <cuda_runtime.h>
 
@@ -384,7 +385,7 @@ __device__ __forceinline__ void attn_loaders(const AttnParams& p, uint8_t* smem,
 }
 
 // MMA issuer (warp 1).  P_HALF_COLS: TMEM column offset of the P of key half 1 within an S
-// buffer (v1: P of half h at [64h, 64h+32); v2: all 128 keys' P in [0, 64), half 1 at 32).
+// buffer (P of half h at [64h, 64h+32)).
 template <int DP, int P_HALF_COLS>
 __device__ __forceinline__ void attn_mma(const AttnParams& p, uint8_t* smem, AttnBars* bars, uint32_t tmem,
                                          uint32_t lane) {
@@ -770,209 +771,11 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) attn_tc_kernel(const __grid_co
 // ready; V2_POLY of the 64 pairs of a full tile take exp2 on the FMA pipe.  The two teams
 // alternate naturally: team 0's softmax runs while the tensor pipe does q-tile 1's P.V and next
 // S, and vice versa (tools/fa4_chain.cu measures the bare chain).
-constexpr int V2_THREADS = 384;
-#ifndef BAT_V2_POLY
-#define BAT_V2_POLY 16
-#endif
-
-template <int DP>
-__global__ void __launch_bounds__(V2_THREADS, 1) attn_v2_kernel(const __grid_constant__ AttnParams p) {
-  using L = AttnSmem<DP>;
-  extern __shared__ uint8_t smem_raw[];
-  uint8_t* smem = smem_raw + ((1024u - (ptx::smem_u32(smem_raw) & 1023u)) & 1023u);
-  AttnBars* bars = reinterpret_cast<AttnBars*>(smem + L::BAR_OFF);
-  const uint32_t warp = ptx::warp_id(), lane = ptx::lane_id();
-  if (warp == 0 && lane == 0) {
-    ptx::mbar_init(&bars->q_full, 1);
-    ptx::mbar_init(&bars->q_empty, 1);
-    for (int i = 0; i < 3; ++i) {
-      ptx::mbar_init(&bars->k_full[i], 1);
-      ptx::mbar_init(&bars->k_empty[i], 1);
-      ptx::mbar_init(&bars->v_full[i], 1);
-      ptx::mbar_init(&bars->v_empty[i], 1);
-    }
-    for (int i = 0; i < 2; ++i) {
-      ptx::mbar_init(&bars->s_full[i], 1);
-      ptx::mbar_init(&bars->p_full[i], 4);
-      ptx::mbar_init(&bars->o_full[i], 1);
-      ptx::mbar_init(&bars->o_empty[i], 4);
-    }
-    ptx::fence_mbar_init();
-  }
-  if (warp == 1) ptx::tmem_alloc(&bars->tmem_base, 512);
-  ptx::tc_fence_before();
-  __syncthreads();
-  ptx::tc_fence_after();
-  const uint32_t tmem = bars->tmem_base;
-  const int32_t* img = p.img;
-  const int32_t* work = img + p.off_work;
-
-  if (warp == 0 || warp == 2 || warp == 3) {
-    attn_loaders<DP>(p, smem, bars, warp, lane);
-  } else if (warp == 1) {
-    attn_mma<DP, 32>(p, smem, bars, tmem, lane);
-  } else if (warp >= 4) {  // ------------------------------------------------ softmax teams
-    const int wg = (warp - 4) >> 2;  // q-tile of the pair
-    const uint32_t sub = warp & 3;
-    const int row = sub * 32 + lane;
-    const uint32_t lane_base = (sub * 32) << 16;
-    const uint32_t tS = tmem + wg * 128 + lane_base;
-    const uint32_t tO = tmem + 256 + wg * 128 + lane_base;
-    constexpr int OCH = DP / 32;  // 32-column O chunks
-    uint32_t sc = 0, oc = 0;
-    const float scale = p.scale_log2;
-    for (int w = blockIdx.x; w < p.n_work; w += gridDim.x) {
-      const WorkItem wi = load_work(work, w);
-      const int qi = wg == 0 ? wi.q0 : wi.q1;
-      if (qi < 0 || wi.kt_n == 0) continue;
-      const int32_t* q_info = img + p.off_qinfo + int64_t(wi.b) * 8;
-      const int tok_off = q_info[0], S = q_info[1];
-      const int tok_local = qi * p.qt + row / p.group;
-      const bool valid_row = row < p.qt * p.group && tok_local < S;
-      const int mrow = valid_row ? row / p.group : p.qt;  // this row's line in the masks
-      const int32_t* ktl = img + wi.kt_off;
-      auto mask_of = [&](int mid) {
-        return __ldg(reinterpret_cast<const uint4*>(img + p.off_masks + (int64_t(mid) * (p.qt + 1) + mrow) * 4));
-      };
-      float m_ref = -INFINITY, l_sum = 0.0f;
-      int n_state = (ktl[0] >> (24 + 2 * wg)) & 3;
-      int n_mid = img[wi.km_off + wg];
-      uint4 n_mv = make_uint4(~0u, ~0u, ~0u, ~0u);
-      if (n_state == 2) n_mv = mask_of(n_mid);
-      for (int x = 0; x < wi.kt_n; ++x) {
-        const int state = n_state;
-        const uint4 mv = n_mv;
-        if (x + 1 < wi.kt_n) {  // next tile's state and mask id, in flight during this tile
-          n_state = (ktl[x + 1] >> (24 + 2 * wg)) & 3;
-          n_mid = img[wi.km_off + 2 * (x + 1) + wg];
-        } else {
-          n_state = 0;
-        }
-        ptx::mbar_wait(&bars->s_full[wg], sc & 1);
-        ++sc;
-        ptx::tc_fence_after();
-        if (state == 0) {  // no visible pair in this (q-tile, k-tile): P = 0
-#pragma unroll
-          for (int c = 0; c < 4; ++c)
-            asm volatile(
-                "tcgen05.st.sync.aligned.32x32b.x16.b32 [%0], "
-                "{%1,%1,%1,%1,%1,%1,%1,%1,%1,%1,%1,%1,%1,%1,%1,%1};" ::"r"(tS + c * 16), "r"(0u));
-        } else {
-          uint32_t s[128];
-          ptx::tmem_ld32(tS, *reinterpret_cast<uint32_t(*)[32]>(s));
-          ptx::tmem_ld32(tS + 32, *reinterpret_cast<uint32_t(*)[32]>(s + 32));
-          ptx::tmem_ld32(tS + 64, *reinterpret_cast<uint32_t(*)[32]>(s + 64));
-          ptx::tmem_ld32(tS + 96, *reinterpret_cast<uint32_t(*)[32]>(s + 96));
-          ptx::tmem_ld_wait();
-          const bool masked = state == 2;
-          if (masked) {
-            const uint32_t vw[4] = {mv.x, mv.y, mv.z, mv.w};
-#pragma unroll
-            for (int i = 0; i < 128; ++i) s[i] = ((vw[i >> 5] >> (i & 31)) & 1u) ? s[i] : 0xff800000u;
-          }
-          float m0 = -INFINITY, m1 = -INFINITY, m2 = -INFINITY, m3 = -INFINITY;
-#pragma unroll
-          for (int i = 0; i < 128; i += 8) {
-            m0 = fmax3(m0, __uint_as_float(s[i]), __uint_as_float(s[i + 1]));
-            m1 = fmax3(m1, __uint_as_float(s[i + 2]), __uint_as_float(s[i + 3]));
-            m2 = fmax3(m2, __uint_as_float(s[i + 4]), __uint_as_float(s[i + 5]));
-            m3 = fmax3(m3, __uint_as_float(s[i + 6]), __uint_as_float(s[i + 7]));
-          }
-          const float mt = fmaxf(fmaxf(m0, m1), fmaxf(m2, m3)) * scale;  // -inf: nothing visible
-          const bool grow = mt > m_ref + kRescaleThreshold;
-          const bool need_o = grow && m_ref != -INFINITY && x > 0;
-          if (grow) {
-            const float alpha = ex2(m_ref - mt);  // 0 when m_ref = -inf
-            l_sum *= alpha;
-            if (__any_sync(0xffffffffu, need_o)) {
-              // O (complete: P.V of the previous tile was issued before this S) *= alpha
-              const float a = need_o ? alpha : 1.0f;
-#pragma unroll 1
-              for (int c = 0; c < OCH; ++c) {
-                uint32_t r[32];
-                ptx::tmem_ld32(tO + c * 32, r);
-                ptx::tmem_ld_wait();
-#pragma unroll
-                for (int i = 0; i < 32; ++i) r[i] = __float_as_uint(__uint_as_float(r[i]) * a);
-                ptx::tmem_st32(tO + c * 32, r);
-              }
-            }
-            m_ref = mt;
-          }
-          const float mr = m_ref == -INFINITY ? 0.0f : m_ref;
-          const uint64_t sc2 = pk2(scale, scale), nm2 = pk2(-mr, -mr);
-          uint64_t acc0 = pk2(0.f, 0.f), acc1 = acc0;
-#pragma unroll
-          for (int c = 0; c < 4; ++c) {
-            uint32_t pk[16];
-#pragma unroll
-            for (int j = 0; j < 16; ++j) {
-              const int i = c * 16 + j;  // key pair (2i, 2i + 1)
-              const uint64_t xv = ffma2(pk2(__uint_as_float(s[2 * i]), __uint_as_float(s[2 * i + 1])), sc2, nm2);
-              uint64_t e;
-              if (i < BAT_V2_POLY && !masked) {  // the polynomial would turn -inf into 2^-127
-                e = exp2_poly2(xv);
-              } else {
-                float x0, x1;
-                up2(xv, x0, x1);
-                e = pk2(ex2(x0), ex2(x1));  // ex2(-inf) = 0
-              }
-              if (j & 1) acc1 = fadd2(acc1, e);
-              else acc0 = fadd2(acc0, e);
-              float p0, p1;
-              up2(e, p0, p1);
-              pk[j] = ptx::pack_bf16x2(p0, p1);
-            }
-            ptx::tmem_st16(tS + c * 16, pk);
-          }
-          float a0, a1, b0, b1;
-          up2(acc0, a0, a1);
-          up2(acc1, b0, b1);
-          l_sum += (a0 + a1) + (b0 + b1);
-        }
-        ptx::tmem_st_wait();
-        ptx::tc_fence_before();
-        __syncwarp();
-        if (lane == 0) ptx::mbar_arrive(&bars->p_full[wg]);
-        n_mv = make_uint4(~0u, ~0u, ~0u, ~0u);
-        if (n_state == 2) n_mv = mask_of(n_mid);
-      }
-      // ---- epilogue: O / l -> bf16 (this row's head vector)
-      ptx::mbar_wait(&bars->o_full[wg], oc & 1);
-      ++oc;
-      ptx::tc_fence_after();
-      const float inv = (l_sum > 0.0f) ? 1.0f / l_sum : 0.0f;
-      const int head = wi.kvh * p.group + row % p.group;
-      __nv_bfloat16* dst = p.out + int64_t(tok_off + tok_local) * p.ldo + int64_t(head) * p.head_dim;
-#pragma unroll 1
-      for (int c = 0; c < OCH; ++c) {
-        const int col0 = c * 32;
-        uint32_t r[32];
-        ptx::tmem_ld32(tO + c * 32, r);
-        ptx::tmem_ld_wait();
-        if (valid_row && col0 < p.head_dim) {
-          uint32_t pk[16];
-#pragma unroll
-          for (int i = 0; i < 16; ++i)
-            pk[i] = ptx::pack_bf16x2(__uint_as_float(r[2 * i]) * inv, __uint_as_float(r[2 * i + 1]) * inv);
-          const int n16 = min(4, (p.head_dim - col0) / 8);
-          uint4* d4 = reinterpret_cast<uint4*>(dst + col0);
-          for (int i = 0; i < n16; ++i) d4[i] = make_uint4(pk[4 * i], pk[4 * i + 1], pk[4 * i + 2], pk[4 * i + 3]);
-        }
-      }
-      ptx::tc_fence_before();
-      __syncwarp();
-      if (lane == 0) ptx::mbar_arrive(&bars->o_empty[wg]);
-    }
-  }
-  ptx::tc_fence_before();
-  __syncthreads();
-  if (warp == 1) ptx::tmem_dealloc(tmem, 512);
-}
-
 }  // namespace
 
 int attn_grid_slots(int, int num_sms) { return num_sms; }
+
+int attn_qtiles_per_item() { return 2; }
 
 size_t attn_smem_bytes(int dpad) {
   return 1024 + (dpad == 128 ? AttnSmem<128>::TOTAL : AttnSmem<64>::TOTAL);
@@ -982,19 +785,12 @@ void launch_attention(int dpad, const AttnParams& p, int num_sms, cudaStream_t s
   const int grid = p.n_work < num_sms ? p.n_work : num_sms;
   if (grid <= 0) return;
   const size_t smem = attn_smem_bytes(dpad);
-  // BAT_ATTN=v1: the round-1 kernel (two softmax threads per row), kept for A/B measurement
-  static const bool v1 = std::getenv("BAT_ATTN") && std::getenv("BAT_ATTN")[0] == 'v' &&
-                         std::getenv("BAT_ATTN")[1] == '1';
-  auto run = [&](auto kern, int threads) {
-    set_smem_attr(kern, smem);
-    kern<<<grid, threads, smem, stream>>>(p);
-  };
   if (dpad == 128) {
-    if (v1) run(attn_tc_kernel<128>, NUM_THREADS);
-    else run(attn_v2_kernel<128>, V2_THREADS);
+    set_smem_attr(attn_tc_kernel<128>, smem);
+    attn_tc_kernel<128><<<grid, NUM_THREADS, smem, stream>>>(p);
   } else {
-    if (v1) run(attn_tc_kernel<64>, NUM_THREADS);
-    else run(attn_v2_kernel<64>, V2_THREADS);
+    set_smem_attr(attn_tc_kernel<64>, smem);
+    attn_tc_kernel<64><<<grid, NUM_THREADS, smem, stream>>>(p);
   }
   count_launch();
 }

@@ -60,6 +60,8 @@ size_t attn_smem_bytes(int dpad);
 
 // number of persistent work slots the planner balances the attention work list over
 int attn_grid_slots(int dpad, int num_sms);
+// q-tiles per attention work item of the kernel launch_attention runs (2: pairs, 1: singles)
+int attn_qtiles_per_item();
 
 // Visibility masks of the plan's partial (q-tile, k-tile) pairs (PlanImage::off_mdesc): one block
 // per mask, bit (32 c + i) of row r's word c = key slot 32 c + i of the k-tile visible to token

@@ -241,7 +241,7 @@ void classify_tiles(QueryPlan& qp, int32_t qt) {
 
 void build_plan(const Pool& pool, int32_t group, int32_t kv_heads,
                 const std::vector<PlanRequest>& reqs, Plan& plan, bool build_image, int32_t grid,
-                StagingCtx* stg) {
+                StagingCtx* stg, int32_t qtiles_per_item) {
   BAT_REQUIRE(group >= 1 && group <= kQtileRows, "group in [1,128]");
   plan.group = group;
   plan.kv_heads = kv_heads;
@@ -379,7 +379,8 @@ void build_plan(const Pool& pool, int32_t group, int32_t kv_heads,
       std::vector<std::pair<int32_t, int32_t>> pairs;
       if (last_only) pairs.push_back({qp.n_qtiles - 1, -1});
       else
-        for (int32_t i = 0; i < qp.n_qtiles; i += 2) pairs.push_back({i, i + 1 < qp.n_qtiles ? i + 1 : -1});
+        for (int32_t i = 0; i < qp.n_qtiles; i += qtiles_per_item)
+          pairs.push_back({i, (qtiles_per_item == 2 && i + 1 < qp.n_qtiles) ? i + 1 : -1});
       for (auto& pr : pairs) {
         std::vector<int32_t> kt;
         for (int32_t j = 0; j < qp.n_ktiles; ++j) {

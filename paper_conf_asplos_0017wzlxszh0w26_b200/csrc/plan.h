@@ -75,8 +75,10 @@ struct Plan {
 // balance; empty items pad the rounds).
 // stg != nullptr: prefix items that are not local but registered remote are mapped to pages of
 // the staging slot (deduplicated per plan) and their pulls recorded in *stg.
+// qtiles_per_item: 2 = attention work items are q-tile PAIRS sharing every K/V tile (the v1/v2
+// kernels), 1 = single q-tiles with their own exact k-tile lists (the v3 kernel).
 void build_plan(const Pool& pool, int32_t group, int32_t kv_heads,
                 const std::vector<PlanRequest>& reqs, Plan& plan, bool build_image, int32_t grid = 0,
-                StagingCtx* stg = nullptr);
+                StagingCtx* stg = nullptr, int32_t qtiles_per_item = 2);
 
 }  // namespace bat

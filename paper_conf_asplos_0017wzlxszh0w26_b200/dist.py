@@ -184,6 +184,35 @@ def route_requests(queries: Sequence, world: int, user_rank=None) -> List[List[i
     return [sorted(x) for x in out]
 
 
+def refresh_placement(owner_old: Sequence[int], freq_new: Sequence[float], r: float, world: int) -> np.ndarray:
+    """Background placement update (P:312 Step 3, footnote P:322): bat_hrcs_refresh."""
+    return bat.bat_hrcs_refresh(owner_old, freq_new, r, world)
+
+
+def apply_refresh(pool: int, model: int, owner_old: Sequence[int], owner_new: Sequence[int], rank: int,
+                  token_fn, pos0: int = 0, stream=None) -> Dict[str, int]:
+    """Apply a placement refresh on this rank's pool: items promoted into the replicated area are
+    pulled from their owner as regular local entries (bat_kv_replicate), items demoted from it
+    are dropped unless this rank is their new owner (bat_kv_evict), and new items this rank
+    stores (owned or replicated) are computed by the prefix-miss path (bat_kv_prefill_entities;
+    token_fn(id) gives an item's tokens).  Afterwards every rank calls exchange_remote with
+    owner_new so the remote tables name the new owners.  Returns the move counts."""
+    import torch
+    n_old = len(owner_old)
+    promote = [i for i in range(n_old) if owner_old[i] >= 0 and owner_new[i] < 0 and owner_old[i] != rank]
+    drop = [i for i in range(n_old) if owner_old[i] < 0 and owner_new[i] >= 0 and owner_new[i] != rank]
+    new = [i for i in range(n_old, len(owner_new)) if owner_new[i] < 0 or owner_new[i] == rank]
+    if promote:
+        bat.bat_kv_replicate(pool, bat.BAT_ENT_ITEM, promote, stream)
+    torch.cuda.synchronize()  # background refresh: nothing may still read the dropped pages
+    for i in drop:
+        bat.bat_kv_evict(pool, bat.BAT_ENT_ITEM, int(i))
+    for s in range(0, len(new), 256):
+        ids = new[s:s + 256]
+        bat.bat_kv_prefill_entities(pool, model, bat.BAT_ENT_ITEM, ids, [token_fn(i) for i in ids], pos0, stream=stream)
+    return dict(promoted=len(promote), dropped=len(drop), computed=len(new))
+
+
 def partition_requests(lengths: Sequence[int], world: int) -> List[List[int]]:
     """Greedy load balance of requests over ranks by suffix tokens, longest first (the paper's
     "load-balanced manner").  Returns the request indices of every rank."""

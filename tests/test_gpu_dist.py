@@ -6,6 +6,7 @@ import numpy as np
 import pytest
 
 import synth
+from oracle import hrcs as ohrcs
 
 pytestmark = pytest.mark.gpu
 torch = pytest.importorskip("torch")
@@ -205,3 +206,74 @@ def test_plan_pins_entries_until_destroyed(B):
     B.bat_plan_destroy(plan)
     B.bat_kv_evict(pool.handle, B.BAT_ENT_ITEM, 22)
     pool.close(); model.close()
+
+
+def test_placement_refresh_and_new_items_serve_identically(B):
+    """NEXT-1 (P:312 Step 3, footnote P:322): after a burst changes item hotness and new items
+    join the corpus, bat_hrcs_refresh's placement is applied on both 'ranks' (two pools on one
+    GPU): promoted items pulled into the replicated area, demoted ones dropped by non-owners, new
+    items computed by their owner.  Requests over old and new items then serve bit-identically
+    to a pool that computed every item itself, before and after the refresh."""
+    from paper_conf_asplos_0017wzlxszh0w26_b200 import dist as bdist
+    from paper_conf_asplos_0017wzlxszh0w26_b200.runtime import DeviceModel, DevicePool
+    cfg = synth.model_config("small")
+    model = DeviceModel(cfg, synth.Weights(cfg, seed=1))
+    tok = lambda i: synth.item_tokens(0, int(i), 16, cfg["vocab"])
+    n_old, n_new, r = 60, 70, 0.2
+    F = synth.zipf_weights(n_old)
+    rep, own = ohrcs.place(F, r, 2)
+    owner = np.array([-1 if i in set(rep) else own[i] for i in range(n_old)], np.int32)
+    pools = [DevicePool(cfg, 1024, rank=k, world=2) for k in range(2)]
+    for k in range(2):
+        B.bat_debug_attach_peer_pool(pools[k].handle, 1 - k, pools[1 - k].handle)
+        mine = bdist.local_items(owner, k)
+        B.bat_kv_prefill_entities(pools[k].handle, model.handle, B.BAT_ENT_ITEM, mine, [tok(i) for i in mine], 0)
+
+    def register(owner_vec):
+        for k in range(2):
+            for i in np.nonzero(owner_vec == 1 - k)[0]:
+                n_tok, pages = B.bat_kv_lookup(pools[1 - k].handle, B.BAT_ENT_ITEM, int(i))
+                B.bat_kv_register_remote(pools[k].handle, B.BAT_ENT_ITEM, int(i), 1 - k, pages, n_tok)
+
+    register(owner)
+    ref_pool = DevicePool(cfg, 1024)
+    B.bat_kv_prefill_entities(ref_pool.handle, model.handle, B.BAT_ENT_ITEM, list(range(n_new)),
+                              [tok(i) for i in range(n_new)], 0)
+
+    def serve_and_compare(owner_vec, items_range):
+        rng = np.random.default_rng(9)
+        for k in range(2):
+            qs = [synth.make_query(0, cfg, 40 + b, 30, rng.choice(items_range, 12, replace=False), (16, 16), 2, "IP")
+                  for b in range(3)]
+            cold = bdist.cold_items(qs, owner_vec, k)
+            bdist.fetch_cold(pools[k].handle, cold)
+            h = torch.empty(3, cfg["hidden"], device="cuda")
+            ref = torch.empty_like(h)
+            B.bat_bipartite_prefill(pools[k].handle, model.handle, B.QueryArray(qs), h)
+            B.bat_bipartite_prefill(ref_pool.handle, model.handle, B.QueryArray(qs), ref)
+            bdist.release_cold(pools[k].handle, cold, torch.cuda.current_stream())
+            torch.cuda.synchronize()
+            assert torch.equal(h, ref)
+
+    serve_and_compare(owner, np.arange(n_old))
+    F_new = np.concatenate([F, np.full(n_new - n_old, F[3])])
+    F_new[[40, 50, 55]] = F.max() * 2  # burst hotspots (P:312)
+    owner_new = bdist.refresh_placement(owner, F_new, r, 2)
+    np.testing.assert_array_equal(owner_new, np.array(ohrcs.refresh(list(owner), F_new, r, 2), np.int32))
+    assert owner[40] >= 0 and owner_new[40] == -1  # a cold item promoted by the burst
+    moves = [bdist.apply_refresh(pools[k].handle, model.handle, owner, owner_new, k, tok) for k in range(2)]
+    assert sum(m["promoted"] for m in moves) > 0 and sum(m["computed"] for m in moves) >= n_new - n_old
+    register(owner_new)
+    for k in range(2):  # every item is stored where the new placement says
+        for i in range(n_new):
+            local = owner_new[i] < 0 or owner_new[i] == k
+            try:
+                B.bat_kv_lookup(pools[k].handle, B.BAT_ENT_ITEM, i)
+                assert local, (k, i)
+            except B.BatError:
+                assert not local, (k, i)
+    serve_and_compare(owner_new, np.arange(n_new))
+    for p_ in pools + [ref_pool]:
+        p_.close()
+    model.close()
+

@@ -12,7 +12,8 @@ dev = torch.device("cuda", 0)
 model = DeviceModel(cfg, tensors=device_weights(cfg, 1, dev))
 pool = DevicePool(cfg, 20000)
 rng = np.random.default_rng(0)
-qs = [synth.make_query(0, cfg, 1000 + b, 512, rng.choice(4000, 100, replace=False), (16, 16), 8, order) for b in range(B)]
+NU = int(os.environ.get("NU", "512")); NI = int(os.environ.get("NI", "100"))
+qs = [synth.make_query(0, cfg, 1000 + b, NU, rng.choice(4000, NI, replace=False), (16, 16), 8, order) for b in range(B)]
 L, Hkv, d = cfg["layers"], cfg["kv_heads"], cfg["head_dim"]
 seen = set()
 for q in qs:
@@ -43,13 +44,13 @@ e1.record(); torch.cuda.synchronize()
 ms = e0.elapsed_time(e1) / 10
 print(f"{order} B={B}: stage+attention {ms:.3f} ms/layer (host sync included); flops {4*128*12*live/1e9:.1f} GF -> {4*128*12*live/ms/1e9:.0f} TFLOP/s lower bound")
 t = np.loadtxt("gpurun_out/attn_timeline.txt").astype(np.int64)
-names = ["ld_top", "ld_kfree", "ld_kiss", "ld_vfree", "ld_viss", "mma_top", "mma_p0", "mma_vful",
-         "mma_kful", "mma_p1", "mma_end", "sm0_s", "sm0_fast", "sm0_p", "sm1_s", "sm1_p",
-         "sm0_meta", "sm0_vis", "sm0_cmp", "sm0_agr"]
+names = ["ld_kwait", "ld_kgot", "ld_kiss", "ld_vbwait", "ld_vbgot", "mma_top", "mma_p0", "mma_vful",
+         "mma_pvdone", "mma_Skful", "mma_end", "sm0_s", "sm0_fast", "sm0_p", "sm1_s", "sm1_p",
+         "sm0_16", "sm0_17", "sm0_max", "sm0_pst"]
 t0 = t[t > 0].min()
-n = int((t[3] > 0).sum())
+n = int(max((t[e] > 0).sum() for e in range(t.shape[0])))
 print("tile " + " ".join(f"{nm:>10}" for nm in names))
-for x in range(min(n, 24)):
+for x in range(min(n, 64)):
     print(f"{x:4d} " + " ".join(f"{(t[e, x] - t0) if t[e, x] else -1:10d}" for e in range(20)))
 
 # ---- per-work-item records (BAT_ATTN_ITEMS): where the time per item goes, per CTA

@@ -1,11 +1,7 @@
 #!/bin/bash
-# exp2 MUFU/FMA split sweep for both attention kernels (bench attention TFLOP/s)
 cd $GRAFT_REPO_ROOT
-mkdir -p gpurun_out
-for v in 0 2 8; do
-  for k in pair tc; do
-    if [ $k = tc ]; then E="BAT_ATTN=tc"; else E=""; fi
-    env $E BAT_LIB=$PWD/paper_conf_asplos_0017wzlxszh0w26_b200/libbat_pp$v.so timeout 300 python bench.py --steps 4 --warmup 3 --no-cpu-baseline > gpurun_out/poly_${k}_$v.json 2>/dev/null
-    python -c "import json;d=json.loads(open('gpurun_out/poly_${k}_$v.json').read().strip().splitlines()[-1]);print('$k poly $v', round(d['attention']['tflops'],1), round(d['value'],1))"
-  done
+export PYTHONUNBUFFERED=1
+for v in p0 p8 p32; do
+  echo "== $v"; BAT_LIB=$PWD/paper_conf_asplos_0017wzlxszh0w26_b200/libbat_$v.so B=8 NU=8192 NI=20 ORDER=UP timeout 300 python tools/attn_timeline.py 2>&1 | sed -n 18,23p | cut -c1-240
 done
+echo "== p16"; B=8 NU=8192 NI=20 ORDER=UP timeout 300 python tools/attn_timeline.py 2>&1 | sed -n 18,23p | cut -c1-240

@@ -1,0 +1,6 @@
+#!/bin/bash
+cd $GRAFT_REPO_ROOT
+export PYTHONUNBUFFERED=1
+B=8 NU=8192 NI=20 ORDER=UP timeout 300 python tools/attn_timeline.py > gpurun_out/tl4_up.txt 2>&1
+ORDER=IP timeout 300 python tools/attn_timeline.py > gpurun_out/tl4_ip.txt 2>&1
+for f in gpurun_out/tl4_up.txt gpurun_out/tl4_ip.txt; do echo $f; head -1 $f; sed -n 20,24p $f | cut -c1-200; tail -1 $f; done
