@@ -400,6 +400,12 @@ BAT_API bat_status bat_plan_build_staged(bat_pool p, bat_model m, const bat_quer
 /* Bytes of a plan's image: *host_bytes uploaded from the host per call (bat_bipartite_prefill
  * uploads this much for the same batch), *device_bytes its device footprint incl. the masks. */
 BAT_API bat_status bat_plan_bytes(bat_plan plan, int64_t* host_bytes, int64_t* device_bytes);
+/* Attention work-list shape of a plan (host): out[0] work items of layers 1..L-1 (CTA-sized units
+ * the persistent kernel balances over the SMs), out[1] of the last layer, out[2] / out[3] split-KV
+ * groups / partial slots of the main list, out[4] / out[5] of the last-layer list.  A list with
+ * fewer items than SMs has its long items split into k-tile chunks on separate CTAs (log-sum-exp
+ * combine); BAT_SPLITKV=0 disables it. */
+BAT_API bat_status bat_plan_work_info(bat_plan plan, int64_t out[6]);
 /* Enqueue a staged plan's cold-item pulls on `stream` (copy engines); *n_pages = pages pulled. */
 BAT_API bat_status bat_plan_fetch(bat_pool p, bat_plan plan, int64_t* n_pages, bat_stream_t stream);
 

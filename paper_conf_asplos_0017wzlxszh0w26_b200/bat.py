@@ -138,6 +138,7 @@ def lib() -> ctypes.CDLL:
                                       POINTER(c_void_p)]),
         "bat_plan_fetch": (S, [c_void_p, c_void_p, POINTER(c_int64), c_void_p]),
         "bat_plan_bytes": (S, [c_void_p, POINTER(c_int64), POINTER(c_int64)]),
+        "bat_plan_work_info": (S, [c_void_p, POINTER(c_int64)]),
         "bat_hrcs_refresh": (S, [POINTER(c_int32), c_int64, POINTER(c_double), c_int64, c_double, c_int32,
                                  POINTER(c_int32)]),
         "bat_kv_replicate": (S, [c_void_p, c_int32, POINTER(c_int64), c_int32, c_void_p]),
@@ -167,7 +168,8 @@ EXPORTED = ("bat_last_error", "bat_version", "bat_kernel_launch_count", "bat_mod
             "bat_profile_reset", "bat_debug_attach_peer_pool", "bat_sched_create", "bat_sched_destroy",
             "bat_sched_decide", "bat_sched_stats", "bat_sched_is_cached", "bat_score_multi",
             "bat_plan_export_device", "bat_kv_release", "bat_kv_staging_reserve", "bat_plan_build_staged",
-            "bat_plan_fetch", "bat_plan_bytes", "bat_hrcs_refresh", "bat_kv_replicate")
+            "bat_plan_fetch", "bat_plan_bytes", "bat_hrcs_refresh", "bat_kv_replicate",
+            "bat_plan_work_info")
 
 
 def _check(status: int) -> None:
@@ -501,6 +503,13 @@ def bat_plan_bytes(plan: int):
     h, d = c_int64(), c_int64()
     _check(lib().bat_plan_bytes(plan, byref(h), byref(d)))
     return h.value, d.value
+
+
+def bat_plan_work_info(plan: int) -> dict:
+    out = (c_int64 * 6)()
+    _check(lib().bat_plan_work_info(plan, out))
+    return dict(zip(("n_work", "n_work_last", "split_groups", "split_slots", "split_groups_last",
+                     "split_slots_last"), [int(x) for x in out]))
 
 
 def bat_plan_fetch(pool: int, plan: int, stream=None) -> int:

@@ -120,7 +120,7 @@ struct DevBuf {
 };
 
 struct Workspace {
-  DevBuf h, xn, qkv, qp, scratch, o, act, hc, xc, oc, actc, img, small;
+  DevBuf h, xn, qkv, qp, scratch, o, act, hc, xc, oc, actc, img, small, part_o, part_ml;
   void* img_host = nullptr;
   size_t img_host_cap = 0;
   cudaEvent_t img_done = nullptr;
@@ -292,6 +292,11 @@ static const int32_t* prepare(Pool& pool, Model& m, Plan& plan, cudaStream_t st,
   ws.xc.ensure(D * H * es, st);
   ws.oc.ensure(D * nq * es, st);
   ws.actc.ensure(D * F * es, st);
+  const int64_t slots = std::max(plan.img.n_slots, plan.img.n_slots_last);
+  if (slots > 0 && !m.f32) {  // split-KV partials (small batches)
+    ws.part_o.ensure(size_t(slots) * 2 * 128 * m.dpad * 4, st);
+    ws.part_ml.ensure(size_t(slots) * 2 * 128 * 8, st);
+  }
   if (dev_img) return dev_img;
   const size_t img_bytes = plan.img.buf.size() * 4;
   ws.img.ensure(size_t(plan.img.total_ints) * 4, st);
@@ -336,12 +341,23 @@ static AttnParams attn_params(const Pool& pool, const Model& m, const Plan& plan
   ap.out = m.ws.o.as<__nv_bfloat16>();
   ap.scale_log2 = float(1.4426950408889634 / std::sqrt(double(c.head_dim)));
   ap.off_masks = im.off_masks;
+  ap.off_wslot = im.off_wslot;
+  const bool split = std::max(im.n_slots, im.n_slots_last) > 0;
+  ap.part_o = split ? m.ws.part_o.as<float>() : nullptr;
+  ap.part_ml = split ? m.ws.part_ml.as<float>() : nullptr;
   return ap;
 }
 
-// a5 launch (persistent tcgen05 kernel, one CTA per SM)
-static void run_attention(const Pool&, const Model& m, const Plan&, const AttnParams& ap, cudaStream_t st) {
+// a5 launch (persistent tcgen05 kernel, one CTA per SM) over the main (last = false) or the
+// last-layer work list, then the split-KV combine of that list's split items (if any)
+static void run_attention(const Pool&, const Model& m, const Plan& plan, AttnParams ap, bool last, cudaStream_t st) {
+  const PlanImage& im = plan.img;
+  ap.off_work = last ? im.off_work_last : im.off_work;
+  ap.n_work = last ? plan.n_work_last : plan.n_work;
+  ap.off_wslot = last ? im.off_wslot_last : im.off_wslot;
   launch_attention(m.dpad, ap, m.num_sms, st);
+  if (ap.part_o) launch_attention_combine(m.dpad, ap, last ? im.off_sgrp_last : im.off_sgrp,
+                                          last ? im.n_sgrp_last : im.n_sgrp, st);
 }
 
 static StageParams stage_params(const Pool& pool, const Model& m, const Plan& plan, const int32_t* I) {
@@ -509,8 +525,6 @@ static void run_plan(Pool& pool, Model& m, Plan& plan, float* out_hidden, cudaSt
     if (last && plan.entity_mode) break;  // entity prefill: only this layer's K/V are needed
     ap.pool_layer_off = int64_t(l) * pool.geo.layer_bytes;
     if (!last) {
-      ap.off_work = im.off_work;
-      ap.n_work = plan.n_work;
       // debug (BAT_ATTN_ITEMS=file, BAT_ATTN_LAYER=l): per-work-item clock64 records of one layer
       static const char* items_file = std::getenv("BAT_ATTN_ITEMS");
       static const int items_layer = std::getenv("BAT_ATTN_LAYER") ? std::atoi(std::getenv("BAT_ATTN_LAYER")) : 1;
@@ -521,7 +535,7 @@ static void run_plan(Pool& pool, Model& m, Plan& plan, float* out_hidden, cudaSt
       }
       ap.dbg_items = dbi;
       pf.begin(st);
-      run_attention(pool, m, plan, ap, st);
+      run_attention(pool, m, plan, ap, false, st);
       pf.end(st, BAT_K_ATTN, attn_fl, attn_by);
       ap.dbg_items = nullptr;
       if (dbi) {
@@ -558,10 +572,8 @@ static void run_plan(Pool& pool, Model& m, Plan& plan, float* out_hidden, cudaSt
     } else {
       // a8: after the last layer's K/V only the discriminant rows matter; with one
       // discriminant per item they are spread over the suffix: attend for every row
-      ap.off_work = plan.multi_disc ? im.off_work : im.off_work_last;
-      ap.n_work = plan.multi_disc ? plan.n_work : plan.n_work_last;
       pf.begin(st);
-      run_attention(pool, m, plan, ap, st);
+      run_attention(pool, m, plan, ap, !plan.multi_disc, st);
       pf.end(st, BAT_K_ATTN, plan.multi_disc ? attn_fl : attn_fl_last, attn_by);
       const int32_t* disc = I + im.off_disc;
       pf.begin(st);
@@ -1512,7 +1524,7 @@ bat_status bat_debug_attention_layer(bat_pool p, bat_model mdl, const bat_query*
       CUDA_OK(cudaMemsetAsync(dbi, 0, size_t(ap.n_work) * 6 * sizeof(long long), st));
       ap.dbg_items = dbi;
     }
-    run_attention(P, m, plan, ap, st);
+    run_attention(P, m, plan, ap, false, st);
     CUDA_OK(cudaGetLastError());
     CUDA_OK(cudaStreamSynchronize(st));
     if (dbg) {
@@ -1594,6 +1606,16 @@ bat_status bat_plan_build(bat_pool p, bat_model mdl, const bat_query* queries, i
 bat_status bat_plan_build_staged(bat_pool p, bat_model mdl, const bat_query* queries, int32_t B, int32_t slot,
                                  bat_stream_t stream, bat_plan* out) {
   return guarded([&] { plan_build_impl(p, mdl, queries, B, slot, stream, out); });
+}
+
+bat_status bat_plan_work_info(bat_plan plan, int64_t out[6]) {
+  return guarded([&] {
+    BAT_REQUIRE(plan && out, "null argument");
+    const Plan& pl = plan->plan;
+    const int64_t v[6] = {pl.n_work, pl.n_work_last, pl.img.n_sgrp, pl.img.n_slots, pl.img.n_sgrp_last,
+                          pl.img.n_slots_last};
+    std::copy(v, v + 6, out);
+  });
 }
 
 bat_status bat_plan_bytes(bat_plan plan, int64_t* host_bytes, int64_t* device_bytes) {

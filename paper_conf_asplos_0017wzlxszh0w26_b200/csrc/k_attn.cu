@@ -731,8 +731,28 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) attn_tc_kernel(const __grid_co
       const float inv = (l_tot > 0.0f) ? 1.0f / l_tot : 0.0f;
       const int head = wi.kvh * p.group + row % p.group;
       __nv_bfloat16* dst = p.out + int64_t(tok_off + tok_local) * p.ldo + int64_t(head) * p.head_dim;
+      // split-KV chunk: O / l in fp32 and the row's (m, l) go to the item's partial slot instead
+      const int slot = p.part_o ? img[p.off_wslot + w] : -1;
+      if (slot >= 0) {
+        const int64_t pr = (int64_t(slot) * 2 + wg) * 128 + row;
+        if (h == 0) reinterpret_cast<float2*>(p.part_ml)[pr] = make_float2(m_ref, l_tot);
+        float* po = p.part_o + pr * DP + h * (DP / 2);
 #pragma unroll 1
-      for (int c = 0; c < OCH; ++c) {
+        for (int c = 0; c < OCH; ++c) {
+          uint32_t r[32];
+          ptx::tmem_ld32(tO + c * 32, r);
+          ptx::tmem_ld_wait();
+          if (valid_row) {
+            float4* d4 = reinterpret_cast<float4*>(po + c * 32);
+#pragma unroll
+            for (int i = 0; i < 8; ++i)
+              d4[i] = make_float4(__uint_as_float(r[4 * i]) * inv, __uint_as_float(r[4 * i + 1]) * inv,
+                                  __uint_as_float(r[4 * i + 2]) * inv, __uint_as_float(r[4 * i + 3]) * inv);
+          }
+        }
+      }
+#pragma unroll 1
+      for (int c = 0; c < (slot >= 0 ? 0 : OCH); ++c) {
         const int col0 = h * (DP / 2) + c * 32;
         uint32_t r[32];
         ptx::tmem_ld32(tO + c * 32, r);
@@ -771,6 +791,49 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) attn_tc_kernel(const __grid_co
 // ready; V2_POLY of the 64 pairs of a full tile take exp2 on the FMA pipe.  The two teams
 // alternate naturally: team 0's softmax runs while the tensor pipe does q-tile 1's P.V and next
 // S, and vice versa (tools/fa4_chain.cu measures the bare chain).
+// Split-KV combine: one warp per (split group, q-tile of the pair, row); O = sum_p w_p O_p /
+// sum_p w_p with w_p = l_p 2^(m_p - max m) over the group's parts (O_p already divided by l_p).
+template <int DP>
+__global__ void attn_combine_kernel(const AttnParams p, int64_t off_sgrp) {
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int rid = blockIdx.x * (blockDim.x >> 5) + warp;  // (group, q-tile, row)
+  const int g = rid / 256, qsel = (rid >> 7) & 1, row = rid & 127;
+  const int32_t* gr = p.img + off_sgrp + int64_t(g) * 6;
+  const int b = gr[0], kvh = gr[1], qi = qsel ? gr[3] : gr[2], slot0 = gr[4], parts = gr[5];
+  if (qi < 0) return;
+  const int32_t* q_info = p.img + p.off_qinfo + int64_t(b) * 8;
+  const int tok_off = q_info[0], S = q_info[1];
+  const int tok_local = qi * p.qt + row / p.group;
+  if (row >= p.qt * p.group || tok_local >= S) return;
+  const float2* ml = reinterpret_cast<const float2*>(p.part_ml);
+  float m = -INFINITY;
+  for (int k = 0; k < parts; ++k) {
+    const float2 v = ml[(int64_t(slot0 + k) * 2 + qsel) * 128 + row];
+    if (v.y > 0.0f) m = fmaxf(m, v.x);
+  }
+  constexpr int PER = DP / 32;
+  float acc[PER];
+#pragma unroll
+  for (int i = 0; i < PER; ++i) acc[i] = 0.0f;
+  float wsum = 0.0f;
+  for (int k = 0; k < parts; ++k) {
+    const int64_t pr = (int64_t(slot0 + k) * 2 + qsel) * 128 + row;
+    const float2 v = ml[pr];
+    if (!(v.y > 0.0f)) continue;
+    const float wgt = v.y * ex2(v.x - m);
+    wsum += wgt;
+    const float* po = p.part_o + pr * DP;
+#pragma unroll
+    for (int i = 0; i < PER; ++i) acc[i] = fmaf(wgt, po[lane + 32 * i], acc[i]);
+  }
+  const float inv = wsum > 0.0f ? 1.0f / wsum : 0.0f;
+  const int head = kvh * p.group + row % p.group;
+  __nv_bfloat16* dst = p.out + int64_t(tok_off + tok_local) * p.ldo + int64_t(head) * p.head_dim;
+#pragma unroll
+  for (int i = 0; i < PER; ++i)
+    if (lane + 32 * i < p.head_dim) dst[lane + 32 * i] = __float2bfloat16_rn(acc[i] * inv);
+}
+
 }  // namespace
 
 int attn_grid_slots(int, int num_sms) { return num_sms; }
@@ -779,6 +842,14 @@ int attn_qtiles_per_item() { return 2; }
 
 size_t attn_smem_bytes(int dpad) {
   return 1024 + (dpad == 128 ? AttnSmem<128>::TOTAL : AttnSmem<64>::TOTAL);
+}
+
+void launch_attention_combine(int dpad, const AttnParams& p, int64_t off_sgrp, int n_sgrp, cudaStream_t stream) {
+  if (n_sgrp <= 0) return;
+  const int blocks = n_sgrp * 256 / 8;  // 8 warps (rows) per block
+  if (dpad == 128) attn_combine_kernel<128><<<blocks, 256, 0, stream>>>(p, off_sgrp);
+  else attn_combine_kernel<64><<<blocks, 256, 0, stream>>>(p, off_sgrp);
+  count_launch();
 }
 
 void launch_attention(int dpad, const AttnParams& p, int num_sms, cudaStream_t stream) {

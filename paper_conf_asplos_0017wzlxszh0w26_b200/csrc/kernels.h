@@ -55,6 +55,9 @@ struct AttnParams {
   long long* dbg;           // optional timeline (clock64) of CTA 0's first work item
   long long* dbg_items;     // optional per-work-item record [n_work][6] (see k_attn.cu)
   int64_t off_masks;        // visibility masks of the partial tiles (launch_masks)
+  int64_t off_wslot;        // split-KV: per work item its partial slot (-1: direct output)
+  float* part_o;            // split-KV partials [slot][2][128][Dp] (O / l, fp32); nullptr: no split
+  float* part_ml;           // [slot][2][128] (m, l)
 };
 size_t attn_smem_bytes(int dpad);
 
@@ -70,6 +73,8 @@ int attn_qtiles_per_item();
 void launch_masks(int32_t* img, int64_t off_mdesc, int64_t off_qinfo, int64_t off_kmeta, int64_t off_rseg,
                   int64_t off_masks, int32_t n_masks, int32_t qt, cudaStream_t s);
 void launch_attention(int dpad, const AttnParams& p, int num_sms, cudaStream_t stream);
+// merge the split-KV partials of n_sgrp groups (PlanImage::off_sgrp) into p.out
+void launch_attention_combine(int dpad, const AttnParams& p, int64_t off_sgrp, int n_sgrp, cudaStream_t stream);
 
 // --------------------------------------------------------------------- small kernels
 void launch_embed(const __nv_bfloat16* E, const int32_t* tok, float* h, int M, int H,

@@ -360,7 +360,7 @@ void build_plan(const Pool& pool, int32_t group, int32_t kv_heads,
   }
   // work items: (b, kvh, q-tile pair) sharing every K/V tile, with the union of the two
   // q-tiles' live k-tiles and a state per q-tile; longest first (LPT over the SMs)
-  struct W { int32_t b, kvh, q0, q1, n; std::vector<int32_t> kt; };
+  struct W { int32_t b, kvh, q0, q1, n; std::vector<int32_t> kt; int32_t slot = -1; };
   std::unordered_map<int64_t, int32_t> mask_id;  // (b, q-tile, k-tile) -> mask
   std::vector<int32_t> mdesc;
   auto mask_of = [&](int32_t b, int32_t qi, int32_t j) {
@@ -372,7 +372,13 @@ void build_plan(const Pool& pool, int32_t group, int32_t kv_heads,
     mdesc.insert(mdesc.end(), {b, qi, j, 0});
     return id;
   };
-  auto make_work = [&](bool last_only, int64_t& off_work, int32_t& n_work) {
+  // split-KV: when a list has fewer items than the persistent grid, a long item's k-tile list is
+  // cut into contiguous chunks (>= kSplitMin tiles) run by different CTAs; each chunk writes its
+  // O / l and (m, l) to a partial slot and a combine kernel merges them (log-sum-exp weights)
+  static const bool split_on = !(std::getenv("BAT_SPLITKV") && std::getenv("BAT_SPLITKV")[0] == '0');
+  constexpr int32_t kSplitMin = 2;
+  auto make_work = [&](bool last_only, int64_t& off_work, int32_t& n_work, int64_t& off_wslot, int64_t& off_sgrp,
+                       int32_t& n_sgrp, int32_t& n_slots) {
     std::vector<W> ws;
     for (int32_t b = 0; b < B; ++b) {
       const QueryPlan& qp = plan.q[b];
@@ -391,6 +397,26 @@ void build_plan(const Pool& pool, int32_t group, int32_t kv_heads,
         if (kt.empty()) continue;  // cannot happen for real rows (each row sees itself)
         for (int32_t h = 0; h < kv_heads; ++h) ws.push_back(W{b, h, pr.first, pr.second, int32_t(kt.size()), kt});
       }
+    }
+    std::vector<int32_t> groups;  // [g][6]
+    n_slots = 0;
+    if (split_on && grid > 0 && !ws.empty() && static_cast<int32_t>(ws.size()) < grid) {
+      const int32_t want = static_cast<int32_t>(ceil_div(grid, static_cast<int64_t>(ws.size())));
+      std::vector<W> out;
+      for (W& w : ws) {
+        const int32_t c = std::min(want, w.n / kSplitMin);
+        if (c <= 1) {
+          out.push_back(std::move(w));
+          continue;
+        }
+        groups.insert(groups.end(), {w.b, w.kvh, w.q0, w.q1, n_slots, c});
+        for (int32_t k = 0; k < c; ++k) {
+          const int32_t t0 = k * w.n / c, t1 = (k + 1) * w.n / c;
+          W part{w.b, w.kvh, w.q0, w.q1, t1 - t0, std::vector<int32_t>(w.kt.begin() + t0, w.kt.begin() + t1), n_slots++};
+          out.push_back(std::move(part));
+        }
+      }
+      ws.swap(out);
     }
     // cost of an item in k-tile-pair units: its tiles, with a fixed prologue / epilogue share
     // (BAT_LPT_SINGLE, BAT_LPT_ITEM: experiment knobs for the per-tile weight of single-q-tile
@@ -422,11 +448,16 @@ void build_plan(const Pool& pool, int32_t group, int32_t kv_heads,
       out.reserve(rounds * grid);
       for (size_t r = 0; r < rounds; ++r)
         for (int32_t c = 0; c < grid; ++c)
-          out.push_back(r < per[c].size() ? ws[per[c][r]] : W{0, 0, -1, -1, 0, {}});
+          out.push_back(r < per[c].size() ? ws[per[c][r]] : W{0, 0, -1, -1, 0, {}, -1});
       ws.swap(out);
     }
     n_work = static_cast<int32_t>(ws.size());
     off_work = reserve_at(int64_t(n_work) * 8);
+    off_wslot = reserve_at(std::max<int64_t>(1, n_work));
+    for (int32_t w = 0; w < n_work; ++w) v[off_wslot + w] = ws[w].slot;
+    n_sgrp = static_cast<int32_t>(groups.size() / 6);
+    off_sgrp = reserve_at(std::max<int64_t>(1, int64_t(groups.size())));
+    std::copy(groups.begin(), groups.end(), v.begin() + off_sgrp);
     int64_t total_kt = 0;
     for (auto& w : ws) total_kt += w.n;
     int64_t off_kt = reserve_at(total_kt);
@@ -451,8 +482,9 @@ void build_plan(const Pool& pool, int32_t group, int32_t kv_heads,
       }
     }
   };
-  make_work(false, im.off_work, plan.n_work);
-  make_work(true, im.off_work_last, plan.n_work_last);
+  make_work(false, im.off_work, plan.n_work, im.off_wslot, im.off_sgrp, im.n_sgrp, im.n_slots);
+  make_work(true, im.off_work_last, plan.n_work_last, im.off_wslot_last, im.off_sgrp_last, im.n_sgrp_last,
+            im.n_slots_last);
   im.n_masks = static_cast<int32_t>(mdesc.size() / 4);
   im.off_mdesc = reserve_at(std::max<int64_t>(1, int64_t(mdesc.size())));
   std::copy(mdesc.begin(), mdesc.end(), v.begin() + im.off_mdesc);

@@ -48,6 +48,11 @@ struct PlanImage {
   int64_t off_qtiles = 0;                           // [n_qtiles_total][4] {b, t0, ntok, 0}
   int64_t off_spages = 0;                           // [n_spages][4] {b, t0, ntok, target}
   int64_t off_work = 0, off_work_last = 0;          // [W][8] {b, kvh, q0, q1|-1, kt_off, kt_n, tp_off, km_off}
+  // split-KV (small batches): per work item its partial-result slot (-1: writes O directly);
+  // per split group {b, kvh, q0, q1, first slot, parts} for the combine kernel
+  int64_t off_wslot = 0, off_wslot_last = 0;        // [W]
+  int64_t off_sgrp = 0, off_sgrp_last = 0;          // [groups][6]
+  int32_t n_sgrp = 0, n_sgrp_last = 0, n_slots = 0, n_slots_last = 0;
   int64_t off_ktl = 0;                              // kt list: ktile | state0 << 24 | state1 << 26
   int64_t off_disc = 0;                             // [B][n_disc] global discriminant rows
   // Visibility masks of the partial (state 2) (q-tile, k-tile) pairs, shared by all KV heads and

@@ -137,3 +137,26 @@ def test_attention_layer_config2_mixed_batch_sampled(B):
     worst, guard = _run(B, cfg, qs, sample, pages)
     assert worst <= 0
     assert guard > 0
+
+
+def test_attention_layer_config1_batch1_split_kv(B):
+    """A single configs[1] request: 26 q-tile-pair work items for 148 SMs, so every long item is
+    split into k-tile chunks on separate CTAs and merged by the log-sum-exp combine (split-KV,
+    SURVEY §5).  Every row against the oracle; the plan must fill >= 120 SMs."""
+    cfg = synth.model_config("qwen2-1.5b")
+    rng = np.random.default_rng(21)
+    zp = synth.zipf_weights(8192)
+    qs = [synth.make_query(0, cfg, 4242, 512, synth.distinct_label_items(0, cfg, 100, rng, 8192, zp),
+                           (16, 16), 8, "IP")]
+    worst, guard = _run(B, cfg, qs, [0], 1024)
+    assert worst <= 0 and guard > 0
+    from paper_conf_asplos_0017wzlxszh0w26_b200.runtime import DevicePool
+    model, pool = _dummy_model(cfg), DevicePool(cfg, 256)
+    for i, t in zip(qs[0].item_ids, qs[0].item_toks):
+        B.bat_kv_reserve(pool.handle, B.BAT_ENT_ITEM, int(i), len(t))
+    plan = B.bat_plan_build(pool.handle, model.handle, B.QueryArray(qs), torch.cuda.current_stream())
+    info = B.bat_plan_work_info(plan)
+    B.bat_plan_destroy(plan)
+    pool.close(); model.close()
+    print("batch-1 work list:", info)
+    assert info["split_groups"] > 0 and info["n_work"] >= 120
