@@ -47,10 +47,10 @@ def launches(tag):
         n, t = tot.get(k, (0, 0.0))
         tot[k] = (n + 1, t + v * scale)
     total = sum(t for _, t in tot.values())
-    out = [f"# ncu launch list ({tag}): bench.py --steps 2 --warmup 1 --plans 1 --corpus 2048, timed region only",
+    out = [f"# ncu launch list ({tag}): {os.environ.get('NCU_CMD', 'bench.py --steps 2 --warmup 1')}, timed region only",
            "# (--profile-from-start off; --metrics gpu__time_duration.sum --clock-control none).  Per-launch times",
            "# are cold-cache and serialised: compare SHARES with bench.py's live CUDA-event kernel table.",
-           f"# raw unit {sorted(unit)}; 2 steps of a 64-request configs[1] IP batch",
+           f"# raw unit {sorted(unit)}; workload: {os.environ.get('NCU_WORKLOAD', 'configs[1] IP batch 64')}",
            f"{'kernel':40s} {'launches':>9s} {'total_ms':>10s} {'share':>7s}"]
     for k, (n, t) in sorted(tot.items(), key=lambda kv: -kv[1][1]):
         out.append(f"{k:40s} {n:9d} {t:10.3f} {100 * t / total:6.1f}%")
@@ -65,7 +65,7 @@ def full(tag):
     hdr, units, data = rows[0], rows[1], rows[2:]
     col = {h: i for i, h in enumerate(hdr)}
     out = [f"# ncu --set full --clock-control none ({tag}): first launches of bench.py's timed region",
-           "# (configs[1] IP, batch 64); attention + GEMM kernels (-k regex:attn|gemm)."]
+           f"# ({os.environ.get('NCU_WORKLOAD', 'configs[1] IP, batch 64')}); kernels {os.environ.get('NCU_KERNELS', 'attn|gemm')}."]
     traffic = collections.OrderedDict()
     for r in data:
         name = r[col["Kernel Name"]]
