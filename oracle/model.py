@@ -147,7 +147,7 @@ def run_query(cfg: dict, W, q, mode: str = "full", rope_on: bool = True, k: int 
     Returns dict(hf, z, s, topk, h_last).  ``mask_fn`` overrides the bipartite mask (only
     for the mask-sensitivity guard test)."""
     tokens, seg, pos = build_sequence(q.order, q.user_tok, q.item_toks, q.instr_tok,
-                                      q.header_tok if q.order == "IP" else ())
+                                      q.header_tok if q.order == "IP" else (), _pic(q))
     mask = (mask_fn or bipartite_mask)(seg)
     if mode == "full" or not q.use_cache:
         h, _ = forward_full(cfg, W, tokens, pos, mask, rope_on)
@@ -189,10 +189,16 @@ def run_query_multi(cfg: dict, W, q, mode: str = "full", rope_on: bool = True, k
     return dict(hf=hf, z=z, s=s, topk=np.asarray(order, np.int64))
 
 
+def _pic(q) -> int:
+    """Selective-recompute tail length of an IP request (reading R25; 0 = plain IP)."""
+    return int(getattr(q, "pic_tail", 0) or 0) if q.order == "IP" else 0
+
+
 def _prefix_len(q) -> int:
     if q.order == "UP":
         return len(q.user_tok)
-    return len(q.header_tok) + sum(len(t) for t in q.item_toks)
+    k = _pic(q)
+    return len(q.header_tok) + sum(len(t) - min(k, len(t)) for t in q.item_toks)
 
 
 def _prefix_kv(cfg: dict, W, q, rope_on: bool = True):
@@ -203,8 +209,12 @@ def _prefix_kv(cfg: dict, W, q, rope_on: bool = True):
     parts = []
     if len(hdr):
         parts.append(entity_kv(cfg, W, hdr, 0, (), rope_on))
+    k = _pic(q)
     for t in q.item_toks:
-        parts.append(entity_kv(cfg, W, t, len(hdr), hdr, rope_on))
+        # the cached head of an item = the first |I| - k rows of its standalone KV (causal)
+        kv = entity_kv(cfg, W, t, len(hdr), hdr, rope_on)
+        n = len(t) - min(k, len(t))
+        parts.append([(kk[:n], vv[:n]) for kk, vv in kv])
     L = cfg["layers"]
     return [(np.concatenate([p[l][0] for p in parts]), np.concatenate([p[l][1] for p in parts]))
             for l in range(L)]

@@ -53,18 +53,26 @@ def prefix_entities(q) -> List[Tuple[int, int, int]]:
 
 def plan_query(q, entity_pages: Dict[Tuple[int, int], Tuple[Sequence[int], int]],
                group: int, scratch_page0: int = 0) -> dict:
+    pic = int(getattr(q, "pic_tail", 0) or 0) if q.order == "IP" else 0
     tokens, seg, pos = build_sequence(q.order, q.user_tok, q.item_toks, q.instr_tok,
-                                      q.header_tok if q.order == "IP" else ())
+                                      q.header_tok if q.order == "IP" else (), pic)
+
+    def used(kind, eid):  # prefix tokens served from an entry: an item's head under PIC (R25)
+        n = entity_pages[(kind, eid)][1]
+        return n - min(pic, n) if kind == ENT_ITEM else n
+
     ents = prefix_entities(q)
-    P = sum(entity_pages[(k, i)][1] for (k, i, _) in ents)
+    P = sum(used(k, i) for (k, i, _) in ents)
     S = len(tokens) - P
     pages: List[int] = []
     valid: List[int] = []
     kseg: List[int] = []
     kord: List[int] = []
     for (kind, eid, sg) in ents:
-        plist, n = entity_pages[(kind, eid)]
-        assert len(plist) == (n + PAGE - 1) // PAGE
+        plist, n_all = entity_pages[(kind, eid)]
+        assert len(plist) == (n_all + PAGE - 1) // PAGE
+        n = used(kind, eid)
+        plist = plist[: (n + PAGE - 1) // PAGE]
         for pi, p in enumerate(plist):
             nv = min(PAGE, n - pi * PAGE)
             pages.append(int(p))

@@ -17,7 +17,7 @@ INSTR = -2
 HEADER = -3
 
 
-def build_sequence(order: str, user_tok, item_toks, instr_tok, header_tok=()):
+def build_sequence(order: str, user_tok, item_toks, instr_tok, header_tok=(), pic_tail: int = 0):
     """Return (tokens, seg, pos) of the full prompt as int64 arrays.
 
     seg: USER / INSTR / HEADER, or the candidate index i >= 0 for item tokens.
@@ -25,6 +25,11 @@ def build_sequence(order: str, user_tok, item_toks, instr_tok, header_tok=()):
          IP  — header: 0..h-1; item i token j: h + j; U token p: h + m + p;
                Instr k: h + m + |U| + k
     where m = max_i |I_i| (reading R2) and h = len(header_tok) (reading R3, IP only).
+
+    pic_tail = k > 0 (IP only; selective recompute, P:265 / P:476, reading R25): the last
+    k_i = min(k, |I_i|) tokens of every item move after U — order [header, item heads, U,
+    item tails (candidate order), Instr] — at positions h + m + |U| + j for item token j, and
+    Instr continues at h + m + |U| + m + k'; item heads keep h + j.  k = 0 is plain IP.
     """
     user_tok = np.asarray(user_tok, dtype=np.int64)
     instr_tok = np.asarray(instr_tok, dtype=np.int64)
@@ -49,10 +54,14 @@ def build_sequence(order: str, user_tok, item_toks, instr_tok, header_tok=()):
     elif order == "IP":
         h = len(header_tok)
         put(header_tok, HEADER, np.arange(h))
-        for i, t in enumerate(items):
-            put(t, i, h + np.arange(len(t)))
+        tails = [min(int(pic_tail), len(t)) for t in items]
+        for i, t in enumerate(items):                 # cached heads (all of every item when k = 0)
+            put(t[: len(t) - tails[i]], i, h + np.arange(len(t) - tails[i]))
         put(user_tok, USER, h + m + np.arange(nu))
-        put(instr_tok, INSTR, h + m + nu + np.arange(nx))
+        for i, t in enumerate(items):                 # recomputed tails, after U
+            put(t[len(t) - tails[i]:], i, h + m + nu + np.arange(len(t) - tails[i], len(t)))
+        x0 = h + m + nu + (m if sum(tails) > 0 else 0)
+        put(instr_tok, INSTR, x0 + np.arange(nx))
     else:
         raise ValueError(order)
     return np.concatenate(toks), np.concatenate(segs), np.concatenate(poss)
@@ -82,8 +91,8 @@ def causal_mask(T: int) -> np.ndarray:
     return np.tril(np.ones((T, T), dtype=bool))
 
 
-def prefix_length(order: str, user_tok, item_toks, header_tok=()) -> int:
+def prefix_length(order: str, user_tok, item_toks, header_tok=(), pic_tail: int = 0) -> int:
     """P: number of prompt tokens that are served from the prefix cache."""
     if order == "UP":
         return len(user_tok)
-    return len(header_tok) + sum(len(t) for t in item_toks)
+    return len(header_tok) + sum(len(t) - min(int(pic_tail), len(t)) for t in item_toks)

@@ -235,6 +235,7 @@ class Query:
     header_id: int = -1
     header_tok: np.ndarray = field(default_factory=lambda: np.zeros(0, np.int32))
     multi_disc: bool = False  # one discriminant token per item (UP only)
+    pic_tail: int = 0         # IP selective recompute: last k tokens of every item (reading R25)
 
     @property
     def n_items(self) -> int:

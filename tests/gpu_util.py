@@ -55,10 +55,13 @@ def oracle_attention_layer(cfg, q, entity_kv, qkv_rows, layer, rope_on=True, rou
     round_qk: round the RoPE'd suffix q and k to bf16 (RNE) — the tensor-core operands' own input
     rounding — for a TIGHTER secondary check that isolates the kernel from that rounding."""
     d, Hq, Hkv = cfg["head_dim"], cfg["q_heads"], cfg["kv_heads"]
+    pic = int(getattr(q, "pic_tail", 0) or 0) if q.order == "IP" else 0
     toks, seg, pos = build_sequence(q.order, q.user_tok, q.item_toks, q.instr_tok,
-                                    q.header_tok if q.order == "IP" else ())
+                                    q.header_tok if q.order == "IP" else (), pic)
     ents = prefix_entities_in_order(q)
-    P = sum(len(t) for _, _, t in ents)
+    # under PIC (reading R25) an item serves only its head from the cache
+    used = {(k, i): (len(t) - min(pic, len(t)) if k == 1 else len(t)) for k, i, t in ents}
+    P = sum(used.values())
     S = len(toks) - P
     x = np.asarray(qkv_rows, np.float64)
     assert x.shape[0] == S
@@ -72,8 +75,8 @@ def oracle_attention_layer(cfg, q, entity_kv, qkv_rows, layer, rope_on=True, rou
         qq = synth.bf16_round(qq.astype(np.float32)).astype(np.float64)
         kk = synth.bf16_round(kk.astype(np.float32)).astype(np.float64)
     if ents:
-        Kp = np.concatenate([entity_kv[(k, i)][0][layer] for k, i, _ in ents]).astype(np.float64)
-        Vp = np.concatenate([entity_kv[(k, i)][1][layer] for k, i, _ in ents]).astype(np.float64)
+        Kp = np.concatenate([entity_kv[(k, i)][0][layer][: used[(k, i)]] for k, i, _ in ents]).astype(np.float64)
+        Vp = np.concatenate([entity_kv[(k, i)][1][layer][: used[(k, i)]] for k, i, _ in ents]).astype(np.float64)
         K = np.concatenate([Kp, kk])
         V = np.concatenate([Vp, vv])
     else:
