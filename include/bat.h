@@ -181,6 +181,12 @@ typedef struct {
                          item, whose hidden state has attended to U and its own item; requires
                          order UP (the items must be computed) and the same value for the whole
                          batch.  0: the last sequence token is the discriminant. */
+  int32_t pic_tail;   /* IP only: selective recompute (PIC, P:265 / P:476; R25).  k > 0:
+                         the last min(k, |I_i|) tokens of every item are recomputed after U (they
+                         attend to the header, their item's cached head, U and their earlier tail
+                         tokens), at positions h + m + |U| + j; the instruction tokens then start
+                         at h + m + |U| + m.  Each item serves only its head from the cache (the
+                         first |I_i| - k rows of the same entry).  0 = plain IP. */
 } bat_query;
 
 /* Run the L layers for B requests (data-parallel batch): every request's suffix

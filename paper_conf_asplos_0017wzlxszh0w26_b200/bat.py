@@ -57,7 +57,7 @@ class bat_query(Structure):
                 ("item_id", POINTER(c_int64)), ("item_off", POINTER(c_int32)),
                 ("item_tok", POINTER(c_int32)), ("instr_tok", POINTER(c_int32)),
                 ("n_instr", c_int32), ("header_id", c_int64), ("header_tok", POINTER(c_int32)),
-                ("n_header", c_int32), ("multi_disc", c_int32)]
+                ("n_header", c_int32), ("multi_disc", c_int32), ("pic_tail", c_int32)]
 
 
 _lib = None
@@ -323,6 +323,7 @@ class QueryArray:
             s.header_tok = _i32p(ht)
             s.n_header = len(q.header_tok)
             s.multi_disc = 1 if getattr(q, "multi_disc", False) else 0
+            s.pic_tail = int(getattr(q, "pic_tail", 0) or 0)
 
     def __len__(self):
         return len(self.arr)

@@ -18,6 +18,7 @@ struct PrefixEnt {
   int64_t id;
   int32_t seg;
   int32_t expect_n;  // tokens the request carries for it (-1: unchecked)
+  int32_t use_n = -1;  // tokens served from the entry (PIC: an item's head); -1: all
 };
 
 // A cold item of a staged plan: pages of the staging slot, the pull recorded once per plan.
@@ -57,9 +58,12 @@ void add_prefix_pages(const Pool& pool, const PrefixEnt& e, QueryPlan& qp, Stagi
                           std::to_string(e.id) + ") holds " + std::to_string(ent->n_tokens) +
                           " tokens but the request has " + std::to_string(e.expect_n));
   }
+  const int32_t use = e.use_n >= 0 ? std::min(e.use_n, ent->n_tokens) : ent->n_tokens;
+  if (use == 0) return;  // PIC: the whole item is recomputed
   if (!staged) qp.refs.push_back(EntityKey{e.kind, e.id});
-  for (size_t pi = 0; pi < ent->pages.size(); ++pi) {
-    int32_t nv = std::min<int32_t>(kPageTokens, ent->n_tokens - static_cast<int32_t>(pi) * kPageTokens);
+  const size_t n_pages = static_cast<size_t>(ceil_div(use, kPageTokens));
+  for (size_t pi = 0; pi < n_pages; ++pi) {
+    int32_t nv = std::min<int32_t>(kPageTokens, use - static_cast<int32_t>(pi) * kPageTokens);
     qp.pages.push_back(ent->pages[pi]);
     qp.valid.push_back(nv);
     for (int j = 0; j < kPageTokens; ++j) {
@@ -67,7 +71,7 @@ void add_prefix_pages(const Pool& pool, const PrefixEnt& e, QueryPlan& qp, Stagi
       qp.kord.push_back(j < nv ? 0 : kInvalidOrd);
     }
   }
-  qp.P += ent->n_tokens;
+  qp.P += use;
 }
 
 // Suffix tokens / positions / segments of a ranking request (readings R2, R3).
@@ -77,6 +81,9 @@ void build_request(const Pool& pool, const bat_query& q, QueryPlan& qp, StagingC
   BAT_REQUIRE(q.n_instr >= 1, "n_instr >= 1 (the discriminant is the last token, P:173)");
   BAT_REQUIRE(q.n_user >= 0 && q.n_header >= 0, "negative length");
   BAT_REQUIRE(q.n_header == 0 || q.order == BAT_ORDER_IP, "header tokens are IP-only (P:257)");
+  BAT_REQUIRE(q.pic_tail >= 0, "pic_tail >= 0");
+  BAT_REQUIRE(q.pic_tail == 0 || q.order == BAT_ORDER_IP, "pic_tail (selective recompute) is IP-only");
+  BAT_REQUIRE(q.pic_tail == 0 || !q.multi_disc, "pic_tail and multi_disc do not combine");
   BAT_REQUIRE(q.item_off && q.item_id, "item arrays");
   BAT_REQUIRE(q.n_user == 0 || q.user_tok, "user_tok");
   BAT_REQUIRE(q.instr_tok, "instr_tok");
@@ -109,16 +116,30 @@ void build_request(const Pool& pool, const bat_query& q, QueryPlan& qp, StagingC
     put_items(nu);
     put(q.instr_tok, nx, SEG_INSTR, nu + m);
   } else {
+    // PIC (reading R25): item i keeps its first n_i - k_i tokens in the prefix, its last k_i
+    // tokens are recomputed after U at positions h + m + |U| + j
+    auto tail = [&](int i) { return std::min(q.pic_tail, q.item_off[i + 1] - q.item_off[i]); };
+    int32_t any_tail = 0;
+    for (int i = 0; i < q.n_items; ++i) any_tail += tail(i);
     if (q.use_cache) {
       if (h > 0) add_prefix_pages(pool, PrefixEnt{BAT_ENT_HEADER, q.header_id, SEG_HEADER, h}, qp, stg);
-      for (int i = 0; i < q.n_items; ++i)
-        add_prefix_pages(pool, PrefixEnt{BAT_ENT_ITEM, q.item_id[i], i, q.item_off[i + 1] - q.item_off[i]}, qp, stg);
+      for (int i = 0; i < q.n_items; ++i) {
+        const int32_t n = q.item_off[i + 1] - q.item_off[i];
+        PrefixEnt pe{BAT_ENT_ITEM, q.item_id[i], i, n};
+        pe.use_n = n - tail(i);
+        add_prefix_pages(pool, pe, qp, stg);
+      }
     } else {
       put(q.header_tok, h, SEG_HEADER, 0);
-      put_items(h);
+      for (int i = 0; i < q.n_items; ++i)
+        put(q.item_tok + q.item_off[i], q.item_off[i + 1] - q.item_off[i] - tail(i), i, h);
     }
     put(q.user_tok, nu, SEG_USER, h + m);
-    put(q.instr_tok, nx, SEG_INSTR, h + m + nu);
+    for (int i = 0; i < q.n_items; ++i) {
+      const int32_t n = q.item_off[i + 1] - q.item_off[i], k = tail(i);
+      put(q.item_tok + q.item_off[i] + (n - k), k, i, h + m + nu + (n - k));
+    }
+    put(q.instr_tok, nx, SEG_INSTR, h + m + nu + (any_tail > 0 ? m : 0));
   }
   qp.n_prefix_pages = static_cast<int32_t>(qp.pages.size());
   qp.S = static_cast<int32_t>(qp.tokens.size());

@@ -121,7 +121,20 @@ def prefill_missing_entities(pool: DevicePool, model: DeviceModel, queries, stre
             pass
         bat.bat_kv_prefill_entities(pool.handle, model.handle, kind, [eid], [toks], 0, stream=stream)
         n += 1
-    hdr_len = {int(q.header_id): len(q.header_tok) for q in queries if q.order == "IP" and len(q.header_tok)}
+    # an item's KV is computed in the context its requests give it: after their header (reading
+    # R3) or alone; the context of every item is the header id of the IP requests using it
+    item_ctx: Dict[int, int] = {}
+    hdr_len: Dict[int, int] = {}
+    for q in queries:
+        if not (q.use_cache and q.order == "IP"):
+            continue
+        h = int(q.header_id) if len(q.header_tok) else -1
+        if h >= 0:
+            hdr_len[h] = len(q.header_tok)
+        for iid in q.item_ids:
+            prev = item_ctx.setdefault(int(iid), h)
+            if prev != h:
+                raise ValueError(f"item {int(iid)} is used after different headers in one batch")
     for kind in (bat.BAT_ENT_USER, bat.BAT_ENT_ITEM):
         todo = []
         for (k, eid), toks in ents.items():
@@ -131,17 +144,15 @@ def prefill_missing_entities(pool: DevicePool, model: DeviceModel, queries, stre
                 bat.bat_kv_lookup(pool.handle, kind, eid)
             except bat.BatError:
                 todo.append((eid, toks))
-        # items with a header context are grouped by header
         groups: Dict[int, List] = {}
         for eid, toks in todo:
-            groups.setdefault(-1, []).append((eid, toks))
-        for _, lst in groups.items():
+            groups.setdefault(item_ctx.get(int(eid), -1) if kind == bat.BAT_ENT_ITEM else -1, []).append((eid, toks))
+        for hid, lst in groups.items():
             for s in range(0, len(lst), batch):
                 chunk = lst[s:s + batch]
-                if kind == bat.BAT_ENT_ITEM and hdr_len:
-                    hid, hl = next(iter(hdr_len.items()))
+                if hid >= 0:
                     bat.bat_kv_prefill_entities(pool.handle, model.handle, kind, [e for e, _ in chunk],
-                                                [t for _, t in chunk], hl, bat.BAT_ENT_HEADER, hid, stream)
+                                                [t for _, t in chunk], hdr_len[hid], bat.BAT_ENT_HEADER, hid, stream)
                 else:
                     bat.bat_kv_prefill_entities(pool.handle, model.handle, kind, [e for e, _ in chunk],
                                                 [t for _, t in chunk], 0, stream=stream)

@@ -52,17 +52,19 @@ def _run_check(B, cfg_name, queries, k=3):
     for b, q in enumerate(queries):
         labels[b, : q.n_items] = q.labels
     scores = torch.empty(Bn, n_max, device="cuda")
+    logits = torch.empty(Bn, n_max, device="cuda")
     topk = torch.empty(Bn, k, dtype=torch.int32, device="cuda")
     B.bat_score(model.handle, hidden, torch.tensor(labels, device="cuda"),
                 torch.tensor([q.n_items for q in queries], dtype=torch.int32, device="cuda"), Bn, n_max, scores,
-                k, topk)
+                k, topk, logits=logits)
     torch.cuda.synchronize()
     hf_all, s_all, tk = hidden.double().cpu().numpy(), scores.double().cpu().numpy(), topk.cpu().numpy()
+    z_all = logits.double().cpu().numpy()
     pool.close()
     worst = {}
     for b, q in enumerate(queries):
         ref = om.run_query(cfg, W, q, "full", k=k)
-        z = np.asarray(W.lm_head_rows(q.labels), np.float64) @ hf_all[b]
+        z = z_all[b, : q.n_items]  # the score kernel's own logits
         for name, got, want in (("hf", hf_all[b], ref["hf"]), ("z", z, ref["z"]),
                                 ("s", s_all[b, : q.n_items], ref["s"])):
             worst[name] = max(worst.get(name, -1.0), max_excess(got, want, TOL, TOL))

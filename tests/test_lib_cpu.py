@@ -228,3 +228,42 @@ def test_hrcs_refresh_matches_oracle(B, seed):
             F_new[rng.integers(0, n_new, size=n_new // 4)] = F_new[-1]
             got = B.bat_hrcs_refresh(owner_old, F_new, r, world)
             np.testing.assert_array_equal(got, np.array(ohrcs.refresh(owner_old, F_new, r, world), np.int32))
+
+
+@pytest.mark.parametrize("seed", range(4))
+def test_plan_pic_bit_exact_vs_oracle(B, seed):
+    """Selective recompute (PIC, reading R25): item heads served from the cached entries (pages
+    trimmed to |I| - k tokens), the tails recomputed after U — the C++ plan bit-exact against the
+    oracle's plan over random ragged items, headers, RE and plain IP neighbours."""
+    cfg = synth.model_config("tiny")
+    rng = np.random.default_rng(300 + seed)
+    item_len = (1, 37)
+    queries = []
+    for k in range(5):
+        q = synth.make_query(seed, cfg, user_id=10 + k, n_user=int(rng.integers(0, 60)),
+                             item_ids=rng.choice(40, size=int(rng.integers(1, 9)), replace=False),
+                             item_len=item_len, n_instr=int(rng.integers(1, 5)), order="IP",
+                             use_cache=(k != 4), n_header=3 if k == 2 else 0)
+        q.pic_tail = [0, 1, 5, 17, 40][k]
+        queries.append(q)
+    pool = _index_pool(B, cfg)
+    try:
+        ep = _reserve_for(B, pool, queries)
+        refs = oplan.plan_batch(queries, ep, 2)
+        plan = B.bat_plan_create(pool, 2, B.QueryArray(queries))
+        try:
+            for b, ref in enumerate(refs):
+                _compare_plan(B, plan, b, ref)
+        finally:
+            B.bat_plan_destroy(plan)
+    finally:
+        B.bat_kv_pool_destroy(pool)
+    with pytest.raises(B.BatError):  # PIC is an Item-as-prefix notion
+        q = synth.make_query(0, cfg, 1, 5, [1, 2], (4, 4), 1, "UP")
+        q.pic_tail = 2
+        pool = _index_pool(B, cfg)
+        try:
+            _reserve_for(B, pool, [q])
+            B.bat_plan_create(pool, 2, B.QueryArray([q]))
+        finally:
+            B.bat_kv_pool_destroy(pool)
