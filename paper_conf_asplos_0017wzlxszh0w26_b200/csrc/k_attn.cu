@@ -57,6 +57,14 @@ constexpr float kRescaleThreshold = 8.0f;  // log2 units: P <= 2^8 between resca
 #ifndef BAT_SUMCHECK
 #define BAT_SUMCHECK 0  // 1: fast-path bound from the row-half sum instead of a per-element max (measured equal: 598.7 vs 601.0 TFLOP/s)
 #endif
+#ifndef BAT_LOADER_SLEEP
+#define BAT_LOADER_SLEEP 0  // 1: loader warps wait on their ring barriers with a suspend hint
+#endif
+#if BAT_LOADER_SLEEP
+#define BAT_LWAIT(b, ph) ptx::mbar_wait_sleep(b, ph)
+#else
+#define BAT_LWAIT(b, ph) ptx::mbar_wait(b, ph)
+#endif
 #ifndef BAT_POLY_PAIRS
 #define BAT_POLY_PAIRS 2  // of every 16 column pairs, exp2 on the FMA pipe (rest: MUFU); swept 0/2/4/8: 600/613/604/542 TFLOP/s
 #endif
@@ -313,7 +321,7 @@ __device__ __forceinline__ void attn_loaders(const AttnParams& p, uint8_t* smem,
       const int qtile0 = q_info[2];
       int32_t pa = ids(wi, nx, 0), pb = ids(wi, nx, 1), pc = ids(wi, nx, 2);
       if (role == 0 && lane == 0) {
-        ptx::mbar_wait(&bars->q_empty, (qc & 1) ^ 1);
+        BAT_LWAIT(&bars->q_empty, (qc & 1) ^ 1);
         const int nq = wi.q1 >= 0 ? 2 : 1;
         ptx::mbar_expect_tx(&bars->q_full, nq * L::TILE_BYTES);
         const char* qbase = reinterpret_cast<const char*>(p.qp);
@@ -339,7 +347,7 @@ __device__ __forceinline__ void attn_loaders(const AttnParams& p, uint8_t* smem,
             const uint32_t ks = ring_slot(kc);
             uint8_t* sk = smem + L::K_OFF + ks * L::TILE_BYTES;
             DBG(0, x);
-            ptx::mbar_wait(&bars->k_empty[ks], ring_phase(kc) ^ 1);
+            BAT_LWAIT(&bars->k_empty[ks], ring_phase(kc) ^ 1);
             DBG(1, x);
             if (BAT_ATTN_NOLOAD) {  // timing experiment only: K never loaded (results are garbage)
               ptx::mbar_arrive(&bars->k_full[ks]);
@@ -361,7 +369,7 @@ __device__ __forceinline__ void attn_loaders(const AttnParams& p, uint8_t* smem,
             const uint32_t vi = 2 * kc + hf, vs = ring_slot(vi);
             uint8_t* sv = smem + L::V_OFF + vs * L::HALF_BYTES;
             if (hf == 0) DBG(3, x);
-            ptx::mbar_wait(&bars->v_empty[vs], ring_phase(vi) ^ 1);
+            BAT_LWAIT(&bars->v_empty[vs], ring_phase(vi) ^ 1);
             if (hf == 0) DBG(4, x);
             if (BAT_ATTN_NOLOAD) {
               ptx::mbar_arrive(&bars->v_full[vs]);

@@ -76,6 +76,17 @@ __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
       : "memory");
 }
 #endif
+// The same wait with a suspend-time hint (ns): the thread sleeps in the barrier instead of
+// re-polling, leaving its SMSP's issue slots to the warps doing arithmetic.
+__device__ __forceinline__ void mbar_wait_sleep(uint64_t* bar, uint32_t parity) {
+  asm volatile(
+      "{\n\t.reg .pred p;\n\t"
+      "LAB_WAITS_%=:\n\t"
+      "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1, %2;\n\t"
+      "@!p bra LAB_WAITS_%=;\n\t}\n" ::"r"(smem_u32(bar)),
+      "r"(parity), "r"(0x10000u)
+      : "memory");
+}
 // non-blocking: true iff the phase of the given parity has completed
 __device__ __forceinline__ bool mbar_test(uint64_t* bar, uint32_t parity) {
   uint32_t ok;

@@ -6,12 +6,15 @@
 //   mode 0: one q-tile chain (8 softmax warps)
 //   mode 1: one chain, softmax replaced by an immediate hand-off (MMA + barrier round trips only)
 //   mode 2: two independent q-tile chains (16 softmax warps), the default kernel's structure
+//   mode 3: mode 0 + warp 2 keeping the tensor pipe busy with unrelated MMAs into other TMEM
+//           columns (is a lone softmax slowed by concurrent tensor work / TMEM traffic?)
 // build: nvcc -gencode arch=compute_100a,code=sm_100a -O3 -std=c++17 --expt-relaxed-constexpr
 //        -I paper_conf_asplos_0017wzlxszh0w26_b200/csrc -I include tools/chain_rate.cu -o tools/chain_rate -lcuda
 #include "../paper_conf_asplos_0017wzlxszh0w26_b200/csrc/k_attn.cu"
 
 namespace bat {
 void count_launch(int) {}
+void set_smem_attr_raw(const void*, int) {}
 namespace {
 
 template <int MODE>
@@ -22,14 +25,16 @@ __global__ void __launch_bounds__(640, 1) chain(long long* out, int iters) {
   __shared__ int okx[2][2][4];
   const uint32_t warp = ptx::warp_id(), lane = ptx::lane_id();
   constexpr int NQ = MODE == 2 ? 2 : 1;
+  __shared__ int bg_stop;
   if (threadIdx.x == 0) {
     for (int q = 0; q < 2; ++q) {
       ptx::mbar_init(&s_full[q], 1);
-      ptx::mbar_init(&p_full[q], 8);
+      ptx::mbar_init(&p_full[q], (MODE == 3 && q == 1) ? 1 : 8);
     }
     ptx::fence_mbar_init();
   }
   for (int i = threadIdx.x; i < 131072 / 16; i += blockDim.x) reinterpret_cast<uint4*>(smem)[i] = make_uint4(0, 0, 0, 0);
+  if (threadIdx.x == 0) bg_stop = 0;
   ptx::fence_proxy_async_smem();
   if (warp == 1) ptx::tmem_alloc(&tbase, 512);
   ptx::tc_fence_before();
@@ -67,6 +72,23 @@ __global__ void __launch_bounds__(640, 1) chain(long long* out, int iters) {
     ptx::mbar_wait(&s_full[0], (iters + (NQ == 1 ? 0 : 0)) & 1);
     const long long t1 = clock64();
     if (lane == 0 && blockIdx.x == 0) out[0] = t1 - t0;
+    if (MODE == 3 && lane == 0) atomicExch(&bg_stop, 1);
+  } else if (MODE == 3 && warp == 2) {  // background tensor work: S-shaped SS MMAs into cols 384+
+    const uint32_t sq = ptx::smem_u32(smem), sk = sq + 65536;
+    constexpr uint32_t IS = ptx::idesc_bf16(128, 128, 0, 0);
+    long long n = 0;
+    while (!*(volatile int*)&bg_stop) {
+#pragma unroll
+      for (int kk = 0; kk < 8; ++kk)
+        ptx::mma_ss_elect(tmem + 384, ptx::desc_sw128(sq + (kk >> 2) * 16384 + (kk & 3) * 32, 16, 1024),
+                          ptx::desc_sw128(sk + (kk >> 2) * 1024 + (kk & 3) * 32, 16, 2048), IS, kk ? 1u : 0u);
+      ++n;
+      if ((n & 7) == 0) {  // bound the queue: wait for this batch of MMAs
+        ptx::mma_commit_elect(&p_full[1]);
+        ptx::mbar_wait(&p_full[1], ((n >> 3) - 1) & 1);
+      }
+    }
+    if (lane == 0 && blockIdx.x == 0) out[2] = n;
   } else if (warp >= 4 && warp < 4 + 8 * NQ) {
     const int wgi = (warp - 4) >> 2;
     const int q = NQ == 2 ? (wgi & 1) : 0, h = NQ == 2 ? (wgi >> 1) : wgi;
@@ -74,8 +96,10 @@ __global__ void __launch_bounds__(640, 1) chain(long long* out, int iters) {
     const uint32_t tS = tmem + q * 128 + h * 64 + ((sub * 32) << 16);
     const uint64_t sc2 = pk2(0.01f, 0.01f), nm2 = pk2(-1.0f, -1.0f);
     float acc = 0.0f;
+    long long soft = 0;
     for (int i = 0; i < iters; ++i) {
       ptx::mbar_wait(&s_full[q], i & 1);
+      const long long ts = clock64();
       ptx::tc_fence_after();
       if (MODE != 1) {
         uint32_t vis[2] = {~0u, ~0u};
@@ -92,8 +116,10 @@ __global__ void __launch_bounds__(640, 1) chain(long long* out, int iters) {
       ptx::tc_fence_before();
       __syncwarp();
       if (lane == 0) ptx::mbar_arrive(&p_full[q]);
+      soft += clock64() - ts;
     }
     if (acc == 12345.0f) out[1] = 1;
+    if (warp == 4 && lane == 0 && blockIdx.x == 0) out[3] = soft;
   }
   ptx::tc_fence_before();
   __syncthreads();
@@ -116,11 +142,12 @@ int main() {
     cudaError_t e = cudaDeviceSynchronize();
     long long h[8];
     cudaMemcpy(h, d, sizeof(h), cudaMemcpyDeviceToHost);
-    printf("%-46s %s  clk per chain step %.0f  (tensor work per step %d clk)\n", name, cudaGetErrorString(e),
-           double(h[0]) / iters, 1024 * nq);
+    printf("%-46s %s  clk per chain step %.0f  (tensor work per step %d clk); softmax S->P %.0f clk\n", name,
+           cudaGetErrorString(e), double(h[0]) / iters, 1024 * nq, double(h[3]) / iters);
   };
   run(chain<0>, "1 q-tile: S -> softmax -> P.V -> S", 1);
   run(chain<1>, "1 q-tile, softmax skipped (MMA + hand-offs)", 1);
   run(chain<2>, "2 q-tiles (default kernel structure)", 2);
+  run(chain<3>, "1 q-tile + background MMAs on other TMEM cols", 1);
   return 0;
 }
