@@ -120,7 +120,7 @@ struct DevBuf {
 };
 
 struct Workspace {
-  DevBuf h, xn, qkv, qp, scratch, o, act, hc, xc, oc, actc, img, small, part_o, part_ml;
+  DevBuf h, xn, qkv, qp, scratch, o, act, hc, xc, oc, actc, img, small, part_o, part_ml, gpart;
   void* img_host = nullptr;
   size_t img_host_cap = 0;
   cudaEvent_t img_done = nullptr;
@@ -503,6 +503,24 @@ static void run_plan(Pool& pool, Model& m, Plan& plan, float* out_hidden, cudaSt
   const CUtensorMap tC_actc = make_tmap(ws.actc.p, Dr, F, F, 32);
   AttnParams ap = attn_params(pool, m, plan, I);
   StageParams sp = stage_params(pool, m, plan, I);
+  // a dense projection; split-K (deterministic fp32 partials + an ordered reduce) when its tile
+  // grid would leave SMs idle — batch-1 requests, the last layer's discriminant rows
+  auto gemm = [&](int epi, const CUtensorMap& tA, const CUtensorMap& tB, const CUtensorMap& tC, const GemmParams& gp) {
+    int mpad = 0;
+    const int ks = (epi == EPI_RESID_F32 || epi == EPI_BF16_BIAS) ? gemm_ksplit(epi, gp.M, gp.N, gp.K, m.num_sms, &mpad) : 1;
+    if (ks <= 1) {
+      launch_gemm(epi, tA, tB, tC, gp, m.num_sms, st);
+      return;
+    }
+    ws.gpart.ensure(size_t(ks) * mpad * gp.N * 4, st);
+    const CUtensorMap tP = make_tmap(ws.gpart.p, int64_t(ks) * mpad, gp.N, gp.N, 32, true);
+    GemmParams pp = gp;
+    pp.ksplit = ks;
+    pp.mpad = mpad;
+    launch_gemm(EPI_PART_F32, tA, tB, tP, pp, m.num_sms, st);
+    launch_gemm_reduce(ws.gpart.as<float>(), ks, mpad, gp.M, gp.N, gp.out, gp.ldo,
+                       epi == EPI_BF16_BIAS ? gp.bias : nullptr, epi == EPI_RESID_F32 ? 0 : 1, st);
+  };
 
   pf.begin(st);
   launch_embed(m.embed, I + im.off_tok, ws.h.as<float>(), M, H, st);
@@ -516,7 +534,7 @@ static void run_plan(Pool& pool, Model& m, Plan& plan, float* out_hidden, cudaSt
     GemmParams gp{M, m.nqkv(), H, ws.qkv.p, m.nqkv(), Lw.bqkv, 0};
     auto fq = gemm_fb(M, m.nqkv(), H, 2);
     pf.begin(st);
-    launch_gemm(EPI_BF16_BIAS, tA_xn, Lw.t_qkv, tC_qkv, gp, m.num_sms, st);
+    gemm(EPI_BF16_BIAS, tA_xn, Lw.t_qkv, tC_qkv, gp);
     pf.end(st, BAT_K_GEMM_QKV, fq.first, fq.second);
     sp.pool_layer_off = int64_t(l) * pool.geo.layer_bytes;
     pf.begin(st);
@@ -554,7 +572,7 @@ static void run_plan(Pool& pool, Model& m, Plan& plan, float* out_hidden, cudaSt
       GemmParams go{M, H, nq, ws.h.p, H, nullptr, 0};
       auto fo = gemm_fb(M, H, nq, 8);
       pf.begin(st);
-      launch_gemm(EPI_RESID_F32, tA_o, Lw.t_o, tC_h, go, m.num_sms, st);
+      gemm(EPI_RESID_F32, tA_o, Lw.t_o, tC_h, go);
       pf.end(st, BAT_K_GEMM_O, fo.first, fo.second);
       pf.begin(st);
       launch_rmsnorm_bf16(ws.h.as<float>(), Lw.ln2, ws.xn.as<__nv_bfloat16>(), M, H, c.rms_eps, st);
@@ -567,7 +585,7 @@ static void run_plan(Pool& pool, Model& m, Plan& plan, float* out_hidden, cudaSt
       GemmParams gd{M, H, F, ws.h.p, H, nullptr, 0};
       auto fd = gemm_fb(M, H, F, 8);
       pf.begin(st);
-      launch_gemm(EPI_RESID_F32, tA_act, Lw.t_d, tC_h, gd, m.num_sms, st);
+      gemm(EPI_RESID_F32, tA_act, Lw.t_d, tC_h, gd);
       pf.end(st, BAT_K_GEMM_DOWN, fd.first, fd.second);
     } else {
       // a8: after the last layer's K/V only the discriminant rows matter; with one
@@ -583,7 +601,7 @@ static void run_plan(Pool& pool, Model& m, Plan& plan, float* out_hidden, cudaSt
       GemmParams go{Dr, H, nq, ws.hc.p, H, nullptr, 0};
       auto fo = gemm_fb(Dr, H, nq, 8);
       pf.begin(st);
-      launch_gemm(EPI_RESID_F32, tA_oc, Lw.t_o, tC_hc, go, m.num_sms, st);
+      gemm(EPI_RESID_F32, tA_oc, Lw.t_o, tC_hc, go);
       pf.end(st, BAT_K_GEMM_O, fo.first, fo.second);
       pf.begin(st);
       launch_rmsnorm_bf16(ws.hc.as<float>(), Lw.ln2, ws.xc.as<__nv_bfloat16>(), Dr, H, c.rms_eps, st);
@@ -596,7 +614,7 @@ static void run_plan(Pool& pool, Model& m, Plan& plan, float* out_hidden, cudaSt
       GemmParams gd{Dr, H, F, ws.hc.p, H, nullptr, 0};
       auto fd = gemm_fb(Dr, H, F, 8);
       pf.begin(st);
-      launch_gemm(EPI_RESID_F32, tA_actc, Lw.t_d, tC_hc, gd, m.num_sms, st);
+      gemm(EPI_RESID_F32, tA_actc, Lw.t_d, tC_hc, gd);
       pf.end(st, BAT_K_GEMM_DOWN, fd.first, fd.second);
       pf.begin(st);
       launch_rmsnorm_f32out(ws.hc.as<float>(), m.final_norm, out_hidden, Dr, H, c.rms_eps, st);

@@ -94,6 +94,7 @@ struct Epilogue {
     __syncwarp();
     if (lane == 0) {
       if (EPI == EPI_RESID_F32) ptx::tma_reduce_add_2d(tmC, buf, col, row);
+      else if (EPI == EPI_PART_F32) ptx::tma_store_2d(tmC, buf, col, row);
       else if (p->hints & 2) ptx::tma_store_2d_hint(tmC, buf, col, row, ptx::policy_evict_first());
       else ptx::tma_store_2d(tmC, buf, col, row);
       ptx::bulk_commit();
@@ -124,7 +125,7 @@ struct Epilogue {
         }
         flush(buf, n * (BN / 2) + c, row0);
       }
-    } else if constexpr (EPI == EPI_RESID_F32) {
+    } else if constexpr (EPI == EPI_RESID_F32 || EPI == EPI_PART_F32) {
 #pragma unroll 1
       for (int c = 0; c < BN; c += 32) {  // 32 fp32 columns per staging buffer
         uint8_t* buf = next_buf();
@@ -188,6 +189,8 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
   const int num_n = (p.N + out_bn - 1) / out_bn;
   const int num_tiles = num_m * num_n;
   const int num_kb = (p.K + BK - 1) / BK;
+  const int ksplit = EPI == EPI_PART_F32 ? p.ksplit : 1;
+  const int num_work = num_tiles * ksplit;  // (K slice, tile) work units, slice-major
 
   if (warp == 0 && lane == 0) {
     for (int s = 0; s < STAGES1; ++s) {
@@ -214,10 +217,11 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
       const uint64_t pol_b = ptx::policy_evict_last();
       int stage = 0;
       uint32_t phase = 0;
-      for (int t = blockIdx.x; t < num_tiles; t += gridDim.x) {
+      for (int t = blockIdx.x; t < num_work; t += gridDim.x) {
         int m, n;
-        tile_coords(t, num_m, num_n, p.group_m, m, n);
-        for (int kb = 0; kb < num_kb; ++kb) {
+        tile_coords(t % num_tiles, num_m, num_n, p.group_m, m, n);
+        const int ks = t / num_tiles;
+        for (int kb = ks * num_kb / ksplit; kb < (ks + 1) * num_kb / ksplit; ++kb) {
           ptx::mbar_wait(&bars->empty[stage], phase ^ 1);
           uint8_t* sa = smem + stage * STAGE1_BYTES;
           uint8_t* sb = sa + A_BYTES;
@@ -240,11 +244,12 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
       uint32_t phase = 0;
       int acc = 0;
       uint32_t acc_phase = 0;
-      for (int t = blockIdx.x; t < num_tiles; t += gridDim.x) {
+      for (int t = blockIdx.x; t < num_work; t += gridDim.x) {
         ptx::mbar_wait(&bars->tempty[acc], acc_phase ^ 1);
         ptx::tc_fence_after();
         const uint32_t d_tmem = tmem + acc * BN;
-        for (int kb = 0; kb < num_kb; ++kb) {
+        const int ks = t / num_tiles, kb0 = ks * num_kb / ksplit;
+        for (int kb = kb0; kb < (ks + 1) * num_kb / ksplit; ++kb) {
           ptx::mbar_wait(&bars->full[stage], phase);
           ptx::tc_fence_after();
           const uint32_t sa = ptx::smem_u32(smem + stage * STAGE1_BYTES);
@@ -253,7 +258,7 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
           for (int kk = 0; kk < BK / 16; ++kk) {
             uint64_t da = ptx::desc_sw128(sa + kk * 32, 16, 1024);
             uint64_t db = ptx::desc_sw128(sb + kk * 32, 16, 1024);
-            ptx::mma_ss(d_tmem, da, db, IDESC, (kb | kk) ? 1u : 0u);
+            ptx::mma_ss(d_tmem, da, db, IDESC, (kb != kb0 || kk) ? 1u : 0u);
           }
           ptx::mma_commit(&bars->empty[stage]);
           if (++stage == STAGES1) { stage = 0; phase ^= 1; }
@@ -267,12 +272,13 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
     Epilogue<EPI> epi{&tmC, &p, smem + STG1_OFF + (warp - 2) * 2 * STG_BYTES, lane};
     int acc = 0;
     uint32_t acc_phase = 0;
-    for (int t = blockIdx.x; t < num_tiles; t += gridDim.x) {
+    for (int t = blockIdx.x; t < num_work; t += gridDim.x) {
       int m, n;
-      tile_coords(t, num_m, num_n, p.group_m, m, n);
+      tile_coords(t % num_tiles, num_m, num_n, p.group_m, m, n);
+      const int slab = EPI == EPI_PART_F32 ? (t / num_tiles) * p.mpad : 0;
       ptx::mbar_wait(&bars->tfull[acc], acc_phase);
       ptx::tc_fence_after();
-      epi.run(tmem + ((sub * 32) << 16) + acc * BN, n, m * 128 + sub * 32);
+      epi.run(tmem + ((sub * 32) << 16) + acc * BN, n, slab + m * 128 + sub * 32);
       ptx::tc_fence_before();
       __syncwarp();
       if (lane == 0) ptx::mbar_arrive(&bars->tempty[acc]);
@@ -303,6 +309,8 @@ gemm2_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__
   const int num_n = (p.N + out_bn - 1) / out_bn;
   const int num_tiles = num_m * num_n;
   const int num_kb = (p.K + BK - 1) / BK;
+  const int ksplit = EPI == EPI_PART_F32 ? p.ksplit : 1;
+  const int num_work = num_tiles * ksplit;
   const int pair = blockIdx.x >> 1, n_pairs = gridDim.x >> 1;
 
   if (warp == 0 && lane == 0) {
@@ -330,10 +338,11 @@ gemm2_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__
     if (lane == 0) {  // ---------------- TMA producer (both CTAs): my 128 rows of A and of B
       int stage = 0;
       uint32_t phase = 0;
-      for (int t = pair; t < num_tiles; t += n_pairs) {
+      for (int t = pair; t < num_work; t += n_pairs) {
         int m, n;
-        tile_coords(t, num_m, num_n, p.group_m, m, n);
-        for (int kb = 0; kb < num_kb; ++kb) {
+        tile_coords(t % num_tiles, num_m, num_n, p.group_m, m, n);
+        const int ks = t / num_tiles;
+        for (int kb = ks * num_kb / ksplit; kb < (ks + 1) * num_kb / ksplit; ++kb) {
           ptx::mbar_wait(&bars->empty[stage], phase ^ 1);
           uint8_t* sa = smem + stage * STAGE2_BYTES;
           uint8_t* sb = sa + A_BYTES;
@@ -351,11 +360,12 @@ gemm2_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__
       uint32_t phase = 0;
       int acc = 0;
       uint32_t acc_phase = 0;
-      for (int t = pair; t < num_tiles; t += n_pairs) {
+      for (int t = pair; t < num_work; t += n_pairs) {
         ptx::mbar_wait(&bars->tempty[acc], acc_phase ^ 1);
         ptx::tc_fence_after();
         const uint32_t d_tmem = tmem + acc * BN;
-        for (int kb = 0; kb < num_kb; ++kb) {
+        const int ks = t / num_tiles, kb0 = ks * num_kb / ksplit;
+        for (int kb = kb0; kb < (ks + 1) * num_kb / ksplit; ++kb) {
           ptx::mbar_wait(&bars->full[stage], phase);
           ptx::tc_fence_after();
           const uint32_t sa = ptx::smem_u32(smem + stage * STAGE2_BYTES);
@@ -364,7 +374,7 @@ gemm2_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__
           for (int kk = 0; kk < BK / 16; ++kk) {
             uint64_t da = ptx::desc_sw128(sa + kk * 32, 16, 1024);
             uint64_t db = ptx::desc_sw128(sb + kk * 32, 16, 1024);
-            ptx::mma2_ss(d_tmem, da, db, IDESC, (kb | kk) ? 1u : 0u);
+            ptx::mma2_ss(d_tmem, da, db, IDESC, (kb != kb0 || kk) ? 1u : 0u);
           }
           ptx::mma2_commit(&bars->empty[stage], 3);
           if (++stage == STAGES2) { stage = 0; phase ^= 1; }
@@ -378,12 +388,13 @@ gemm2_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__
     Epilogue<EPI> epi{&tmC, &p, smem + STG2_OFF + (warp - 2) * 2 * STG_BYTES, lane};
     int acc = 0;
     uint32_t acc_phase = 0;
-    for (int t = pair; t < num_tiles; t += n_pairs) {
+    for (int t = pair; t < num_work; t += n_pairs) {
       int m, n;
-      tile_coords(t, num_m, num_n, p.group_m, m, n);
+      tile_coords(t % num_tiles, num_m, num_n, p.group_m, m, n);
+      const int slab = EPI == EPI_PART_F32 ? (t / num_tiles) * p.mpad : 0;
       ptx::mbar_wait(&bars->tfull[acc], acc_phase);
       ptx::tc_fence_after();
-      epi.run(tmem + ((sub * 32) << 16) + acc * BN, n, m * 256 + int(rank) * 128 + sub * 32);
+      epi.run(tmem + ((sub * 32) << 16) + acc * BN, n, slab + m * 256 + int(rank) * 128 + sub * 32);
       ptx::tc_fence_before();
       __syncwarp();
       if (lane == 0) ptx::mbar_arrive_cluster(ptx::mapa(ptx::smem_u32(&bars->tempty[acc]), 0));
@@ -423,8 +434,9 @@ void launch_gemm(int epi, const CUtensorMap& tmA, const CUtensorMap& tmB, const 
   const int n_tiles = (p.N + out_bn - 1) / out_bn;
   // the SwiGLU GEMM stays on 1-CTA tiles: measured in the bench step, its pair version ran
   // slower (1.18 vs 1.24 PFLOP/s) although both tie when timed alone
+  const int ks = epi == EPI_PART_F32 ? p.ksplit : 1;
   if (p.M >= 256 && num_sms >= 2 && epi != EPI_SWIGLU) {
-    const int tiles = ((p.M + 255) / 256) * n_tiles;
+    const int tiles = ((p.M + 255) / 256) * n_tiles * ks;
     const int pairs = tiles < num_sms / 2 ? tiles : num_sms / 2;
     auto launch = [&](auto kern) {
       set_smem_attr(kern, kGemmSmem2);
@@ -435,9 +447,10 @@ void launch_gemm(int epi, const CUtensorMap& tmA, const CUtensorMap& tmB, const 
       case EPI_BF16_BIAS: launch(gemm2_tc_kernel<EPI_BF16_BIAS>); break;
       case EPI_RESID_F32: launch(gemm2_tc_kernel<EPI_RESID_F32>); break;
       case EPI_SWIGLU: launch(gemm2_tc_kernel<EPI_SWIGLU>); break;
+      case EPI_PART_F32: launch(gemm2_tc_kernel<EPI_PART_F32>); break;
     }
   } else {
-    const int tiles = ((p.M + 127) / 128) * n_tiles;
+    const int tiles = ((p.M + 127) / 128) * n_tiles * ks;
     const int grid = tiles < num_sms ? tiles : num_sms;
     if (grid <= 0) return;
     auto launch = [&](auto kern) {
@@ -449,8 +462,61 @@ void launch_gemm(int epi, const CUtensorMap& tmA, const CUtensorMap& tmB, const 
       case EPI_BF16_BIAS: launch(gemm_tc_kernel<EPI_BF16_BIAS>); break;
       case EPI_RESID_F32: launch(gemm_tc_kernel<EPI_RESID_F32>); break;
       case EPI_SWIGLU: launch(gemm_tc_kernel<EPI_SWIGLU>); break;
+      case EPI_PART_F32: launch(gemm_tc_kernel<EPI_PART_F32>); break;
     }
   }
+  count_launch();
+}
+
+int gemm_ksplit(int epi, int M, int N, int K, int num_sms, int* mpad) {
+  static const bool off = std::getenv("BAT_GEMM_SPLITK") && std::getenv("BAT_GEMM_SPLITK")[0] == '0';
+  if (mpad) *mpad = 0;
+  if (off || epi == EPI_SWIGLU || M <= 0) return 1;
+  const bool pair = M >= 256 && num_sms >= 2;
+  const int rows = pair ? 256 : 128;
+  const int units = ((M + rows - 1) / rows) * ((N + BN - 1) / BN);  // CTA pairs or CTAs
+  const int slots = pair ? num_sms / 2 : num_sms;
+  const int num_kb = (K + BK - 1) / BK;
+  int ks = slots / units;            // fill the idle SMs...
+  ks = ks < num_kb / 4 ? ks : num_kb / 4;  // ...keeping >= 4 k-blocks (256 of K) per slice
+  ks = ks < 8 ? ks : 8;
+  if (ks < 2) return 1;
+  if (mpad) *mpad = ((M + rows - 1) / rows) * rows;
+  return ks;
+}
+
+__global__ void gemm_reduce_kernel(const float* __restrict__ part, int ksplit, int64_t slab, int M, int N,
+                                   void* __restrict__ out, int ldo, const __nv_bfloat16* __restrict__ bias,
+                                   int mode) {
+  const int64_t n4 = int64_t(M) * (N / 4);
+  for (int64_t e = blockIdx.x * int64_t(blockDim.x) + threadIdx.x; e < n4; e += int64_t(gridDim.x) * blockDim.x) {
+    const int m = int(e / (N / 4)), c = int(e % (N / 4)) * 4;
+    const float4* src = reinterpret_cast<const float4*>(part + int64_t(m) * N + c);
+    float4 a = src[0];
+    for (int s = 1; s < ksplit; ++s) {  // slice order: deterministic
+      const float4 b = src[s * slab / 4];
+      a.x += b.x; a.y += b.y; a.z += b.z; a.w += b.w;
+    }
+    if (mode == 0) {
+      float4* h = reinterpret_cast<float4*>(static_cast<float*>(out) + int64_t(m) * ldo + c);
+      float4 v = *h;
+      v.x += a.x; v.y += a.y; v.z += a.z; v.w += a.w;
+      *h = v;
+    } else {
+      __nv_bfloat16* o = static_cast<__nv_bfloat16*>(out) + int64_t(m) * ldo + c;
+      o[0] = __float2bfloat16_rn(a.x + (bias ? __bfloat162float(bias[c]) : 0.0f));
+      o[1] = __float2bfloat16_rn(a.y + (bias ? __bfloat162float(bias[c + 1]) : 0.0f));
+      o[2] = __float2bfloat16_rn(a.z + (bias ? __bfloat162float(bias[c + 2]) : 0.0f));
+      o[3] = __float2bfloat16_rn(a.w + (bias ? __bfloat162float(bias[c + 3]) : 0.0f));
+    }
+  }
+}
+
+void launch_gemm_reduce(const float* part, int ksplit, int mpad, int M, int N, void* out, int ldo,
+                        const __nv_bfloat16* bias, int mode, cudaStream_t stream) {
+  const int64_t n4 = int64_t(M) * (N / 4);
+  const int blocks = int((n4 + 255) / 256 < 1184 ? (n4 + 255) / 256 : 1184);
+  gemm_reduce_kernel<<<blocks, 256, 0, stream>>>(part, ksplit, int64_t(mpad) * N, M, N, out, ldo, bias, mode);
   count_launch();
 }
 

@@ -21,7 +21,7 @@ inline void set_smem_attr(K* kern, size_t bytes) {
 }
 
 // ------------------------------------------------------------------------ tcgen05 GEMM
-enum GemmEpi { EPI_BF16 = 0, EPI_BF16_BIAS = 1, EPI_RESID_F32 = 2, EPI_SWIGLU = 3 };
+enum GemmEpi { EPI_BF16 = 0, EPI_BF16_BIAS = 1, EPI_RESID_F32 = 2, EPI_SWIGLU = 3, EPI_PART_F32 = 4 };
 struct GemmParams {
   int M, N, K;        // N = output columns (SWIGLU: the ffn width F)
   void* out;          // bf16 [M][ldo] or fp32 residual [M][ldo]
@@ -30,7 +30,16 @@ struct GemmParams {
   int up_row0;        // EPI_SWIGLU: first "up" row of B (= F)
   int group_m = 0;    // M-tiles per rasterisation group (0: launch_gemm's default)
   int hints = 0;      // 1-CTA kernel L2 hints: bit 0 B loads evict_last, bit 1 bf16 C stores evict_first
+  int ksplit = 1;     // EPI_PART_F32: K split in ksplit slices; slice s stores its fp32 partial at
+  int mpad = 0;       // rows [s * mpad, s * mpad + M) of the partial buffer (tmC)
 };
+// Split-K for grids that would leave SMs idle (small M: batch-1 requests, the last layer's
+// discriminant rows): slices per tile (1 = no split) for a GEMM of this shape and the row pitch of
+// its partial slabs.  Deterministic: the partials are summed in slice order by launch_gemm_reduce.
+int gemm_ksplit(int epi, int M, int N, int K, int num_sms, int* mpad);
+// out = sum_s part[s] (+ bias), mode 0: fp32 residual h += ..., mode 1: bf16 out = .. + bias
+void launch_gemm_reduce(const float* part, int ksplit, int mpad, int M, int N, void* out, int ldo,
+                        const __nv_bfloat16* bias, int mode, cudaStream_t stream);
 size_t gemm_smem_bytes();
 // tmC: output tensor map — bf16 [M][ldo] with box {64, 32} (EPI_BF16*, EPI_SWIGLU) or fp32
 // [M][ldo] with box {32, 32} (EPI_RESID_F32, TMA reduce-add), 128-byte swizzle

@@ -149,3 +149,15 @@ def test_small64_llama_head_shape(B, order):
                            "UP" if order == "UP" else "IP", use_cache=(order != "RE"))]
     cfg, W, out = _run(B, "small64", qs)
     _check(cfg, W, qs, out)
+
+
+def test_small_batch_paths_are_deterministic(B):
+    """A batch-1 request runs the small-batch paths (split-KV attention chunks + log-sum-exp
+    combine, split-K projections with fp32 partials summed in slice order): two runs must agree
+    bit for bit, and match the oracle."""
+    cfg = synth.model_config("small")
+    qs = [synth.make_query(9, cfg, 77, 300, list(range(500, 540)), (16, 16), 8, "IP")]
+    cfg, W, out1 = _run(B, "small", qs)
+    _, _, out2 = _run(B, "small", qs)
+    assert np.array_equal(out1["hf"], out2["hf"]) and np.array_equal(out1["z"], out2["z"])
+    _check(cfg, W, qs, out1)

@@ -17,7 +17,7 @@ void count_launch(int) {}
 void set_smem_attr_raw(const void*, int) {}
 namespace {
 
-template <int MODE>
+template <int MODE, bool RANDOM_DATA = false>
 __global__ void __launch_bounds__(640, 1) chain(long long* out, int iters) {
   extern __shared__ __align__(1024) uint8_t smem[];
   __shared__ uint64_t s_full[2], p_full[2];
@@ -33,7 +33,20 @@ __global__ void __launch_bounds__(640, 1) chain(long long* out, int iters) {
     }
     ptx::fence_mbar_init();
   }
-  for (int i = threadIdx.x; i < 131072 / 16; i += blockDim.x) reinterpret_cast<uint4*>(smem)[i] = make_uint4(0, 0, 0, 0);
+  for (int i = threadIdx.x; i < 131072 / 16; i += blockDim.x) {
+    if (RANDOM_DATA) {  // pseudo-random bf16 operands in ~[-1, 1): realistic S values
+      uint32_t w[4];
+      for (int j = 0; j < 4; ++j) {
+        uint32_t x = (i * 4 + j) * 2654435761u;
+        x ^= x >> 13; x *= 0x5bd1e995u; x ^= x >> 15;
+        const float a = (float(x & 0xffff) / 32768.0f) - 1.0f, b = (float(x >> 16) / 32768.0f) - 1.0f;
+        w[j] = ptx::pack_bf16x2(a, b);
+      }
+      reinterpret_cast<uint4*>(smem)[i] = make_uint4(w[0], w[1], w[2], w[3]);
+    } else {
+      reinterpret_cast<uint4*>(smem)[i] = make_uint4(0, 0, 0, 0);
+    }
+  }
   if (threadIdx.x == 0) bg_stop = 0;
   ptx::fence_proxy_async_smem();
   if (warp == 1) ptx::tmem_alloc(&tbase, 512);
@@ -149,5 +162,7 @@ int main() {
   run(chain<1>, "1 q-tile, softmax skipped (MMA + hand-offs)", 1);
   run(chain<2>, "2 q-tiles (default kernel structure)", 2);
   run(chain<3>, "1 q-tile + background MMAs on other TMEM cols", 1);
+  run(chain<0, true>, "1 q-tile, random Q/K/V (realistic S)", 1);
+  run(chain<2, true>, "2 q-tiles, random Q/K/V (realistic S)", 2);
   return 0;
 }
