@@ -65,6 +65,14 @@ constexpr float kRescaleThreshold = 8.0f;  // log2 units: P <= 2^8 between resca
 #else
 #define BAT_LWAIT(b, ph) ptx::mbar_wait(b, ph)
 #endif
+#ifndef BAT_SOFT_SLEEP
+#define BAT_SOFT_SLEEP 0  // 1: softmax warps wait for S / O with a suspend hint instead of re-polling
+#endif
+#if BAT_SOFT_SLEEP
+#define BAT_SWAIT(b, ph) ptx::mbar_wait_sleep(b, ph)
+#else
+#define BAT_SWAIT(b, ph) ptx::mbar_wait(b, ph)
+#endif
 #ifndef BAT_POLY_PAIRS
 #define BAT_POLY_PAIRS 2  // of every 16 column pairs, exp2 on the FMA pipe (rest: MUFU); swept 0/2/4/8: 600/613/604/542 TFLOP/s
 #endif
@@ -656,7 +664,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) attn_tc_kernel(const __grid_co
           n_state = 0;
         }
         const bool dbg_first = (kc == 0) && row == 0 && h == 0;
-        ptx::mbar_wait(&bars->s_full[wg], sc & 1);
+        BAT_SWAIT(&bars->s_full[wg], sc & 1);
         DBG(11 + 3 * wg, x);
         ++sc;
         seq_wait();
@@ -731,7 +739,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) attn_tc_kernel(const __grid_co
       kc += wi.kt_n;
       // ---- epilogue: O / l -> bf16, my half of the head's columns
       xch->lsum[wg][h][row] = l_sum;
-      ptx::mbar_wait(&bars->o_full[wg], oc & 1);
+      BAT_SWAIT(&bars->o_full[wg], oc & 1);
       ++oc;
       ptx::tc_fence_after();
       ptx::bar_sync(pair_bar, 64);
