@@ -225,6 +225,13 @@ BAT_API bat_status bat_score_multi(bat_model m, const float* hidden, const int32
  * bat_kv_evict / bat_kv_release of a pinned entry fail with BAT_E_STATE until bat_plan_destroy,
  * and bat_kv_pool_destroy fails while the pool has live plans.  bat_prefill_plan returns
  * BAT_E_STATE for a plan built on another pool.
+ * CUDA graphs (opt-in: BAT_GRAPH=1 in the environment; measured neutral on a B200, where the
+ * batch-1 prefill is GPU-bound): on a non-default stream (and with kernel profiling off) bat_prefill_plan runs a
+ * plan's first call eagerly (sizing the model's workspace), captures its second call into a CUDA
+ * graph and replays that graph on later calls with the same out_hidden, as long as no workspace
+ * buffer was reallocated since (a larger plan run in between forces one eager call and a new
+ * capture).  Results are bit-identical to eager runs.  The legacy default stream (stream = NULL)
+ * always runs eagerly.
  * ---------------------------------------------------------------------------------------- */
 typedef struct bat_plan_s* bat_plan;
 BAT_API bat_status bat_plan_build(bat_pool p, bat_model m, const bat_query* queries, int32_t B,

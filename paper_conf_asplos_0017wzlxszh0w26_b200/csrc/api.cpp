@@ -6,6 +6,7 @@
 #include <algorithm>
 #include <cmath>
 #include <cstdio>
+#include <atomic>
 #include <cstdlib>
 #include <cstring>
 #include <memory>
@@ -33,7 +34,17 @@ struct bat_plan_s {
   int32_t slot = -1;                       // staging slot of a bat_plan_build_staged plan
   std::vector<uint64_t> pull_src;          // its cold-item pulls: peer page addresses ...
   std::vector<int32_t> pull_dst;           // ... -> local staging pages
+  // CUDA graph of this plan's prefill (bat_prefill_plan, BAT_GRAPH != 0): captured on the second
+  // call (the first sizes the workspace), replayed while the workspace buffers, the output
+  // pointer and the model are those it was captured with
+  cudaGraphExec_t gexec = nullptr;
+  uint64_t warm_gen = 0, graph_gen = 0;
+  bool warm = false;
+  const void* graph_model = nullptr;
+  float* graph_out = nullptr;
+  int64_t graph_launches = 0;
   ~bat_plan_s() {
+    if (gexec) cudaGraphExecDestroy(gexec);
     if (dev_img) cudaFree(dev_img);
   }
 };
@@ -91,6 +102,10 @@ static CUtensorMap make_tmap(const void* ptr, int64_t rows, int64_t cols, int64_
 
 
 // ------------------------------------------------------------------------ device buffer
+// bumped whenever a workspace buffer or the RoPE table is (re)allocated: a captured prefill
+// graph holds their addresses (bat_prefill_plan)
+static std::atomic<uint64_t> g_buf_gen{1};
+
 struct DevBuf {
   void* p = nullptr;
   size_t cap = 0;
@@ -100,6 +115,7 @@ struct DevBuf {
   // stream kind — a legacy-default-stream memset would not be with a non-blocking stream)
   void ensure(size_t bytes, cudaStream_t st, bool zero = false) {
     if (bytes <= cap) return;
+    ++g_buf_gen;
     if (p) {
       CUDA_OK(cudaStreamSynchronize(st));  // the old buffer may still be read by queued work
       cudaFree(p);
@@ -230,6 +246,7 @@ static void ensure_rope(Model& m, int need_pos, cudaStream_t st) {
   if (need_pos <= m.max_pos) return;
   int np = std::max(32768, m.max_pos);
   while (np < need_pos) np *= 2;
+  ++g_buf_gen;
   if (m.rope) {
     CUDA_OK(cudaStreamSynchronize(st));
     cudaFree(m.rope);
@@ -1666,8 +1683,52 @@ bat_status bat_prefill_plan(bat_pool p, bat_model mdl, bat_plan plan, float* out
     BAT_REQUIRE(!plan->plan.entity_mode && plan->plan.kv_heads == m.cfg.kv_heads, "plan / model mismatch");
     if (plan->pool != p) fail(BAT_E_STATE, "plan was built for another pool");
     DeviceGuard dg(P.device);
-    run_plan(P, m, plan->plan, out_hidden, static_cast<cudaStream_t>(stream),
-             static_cast<const int32_t*>(plan->dev_img));
+    cudaStream_t st = static_cast<cudaStream_t>(stream);
+    const int32_t* img = static_cast<const int32_t*>(plan->dev_img);
+    // CUDA graph replay of the ~12 launches per layer (launch-bound at small batches); not on the
+    // legacy default stream (not capturable) nor while kernel profiling records events
+    const char* gv = std::getenv("BAT_GRAPH");  // opt-in: measured neutral (batch-1 5.038 vs 5.038 ms)
+    const bool use_graph = gv && std::atoi(gv) != 0;
+    if (!use_graph || st == nullptr || m.prof.on) {
+      run_plan(P, m, plan->plan, out_hidden, st, img);
+      return;
+    }
+    const uint64_t gen = g_buf_gen.load();
+    if (plan->gexec && plan->graph_gen == gen && plan->graph_out == out_hidden && plan->graph_model == &m) {
+      CUDA_OK(cudaGraphLaunch(plan->gexec, st));
+      count_launch(int(plan->graph_launches));
+      return;
+    }
+    if (plan->gexec) {
+      CUDA_OK(cudaGraphExecDestroy(plan->gexec));
+      plan->gexec = nullptr;
+    }
+    if (!plan->warm || plan->warm_gen != gen) {  // size the workspace first: nothing may allocate during capture
+      run_plan(P, m, plan->plan, out_hidden, st, img);
+      plan->warm = true;
+      plan->warm_gen = g_buf_gen.load();
+      return;
+    }
+    const int64_t n0 = launch_count();
+    CUDA_OK(cudaStreamBeginCapture(st, cudaStreamCaptureModeThreadLocal));
+    cudaGraph_t g = nullptr;
+    try {
+      run_plan(P, m, plan->plan, out_hidden, st, img);
+    } catch (...) {
+      cudaStreamEndCapture(st, &g);
+      if (g) cudaGraphDestroy(g);
+      throw;
+    }
+    CUDA_OK(cudaStreamEndCapture(st, &g));
+    const cudaError_t ie = cudaGraphInstantiate(&plan->gexec, g, 0);
+    cudaGraphDestroy(g);
+    CUDA_OK(ie);
+    plan->graph_gen = g_buf_gen.load();
+    if (plan->graph_gen != gen) fail(BAT_E_CUDA, "workspace reallocated during graph capture");
+    plan->graph_out = out_hidden;
+    plan->graph_model = &m;
+    plan->graph_launches = launch_count() - n0;
+    CUDA_OK(cudaGraphLaunch(plan->gexec, st));
   });
 }
 

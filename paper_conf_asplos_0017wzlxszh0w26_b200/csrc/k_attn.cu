@@ -73,6 +73,9 @@ constexpr float kRescaleThreshold = 8.0f;  // log2 units: P <= 2^8 between resca
 #else
 #define BAT_SWAIT(b, ph) ptx::mbar_wait(b, ph)
 #endif
+#ifndef BAT_ATTN_DBE
+#define BAT_ATTN_DBE 1  // 1: decide-before-exp softmax (row max -> halves exchange -> P per chunk); 0: single pass + vote
+#endif
 #ifndef BAT_POLY_PAIRS
 #define BAT_POLY_PAIRS 2  // of every 16 column pairs, exp2 on the FMA pipe (rest: MUFU); swept 0/2/4/8: 600/613/604/542 TFLOP/s
 #endif
@@ -281,6 +284,74 @@ __device__ __forceinline__ bool row_exp_opt(uint32_t tS, const uint32_t (&vis)[N
         "r"(pk[c * 16 + 14]), "r"(pk[c * 16 + 15]));
   lsum = (a0 + a1) + (b0 + b1);
   return true;
+}
+
+// Decide-before-exp (BAT_ATTN_DBE): the row half's 64 S values are loaded once (two tcgen05.ld,
+// one wait) and kept in registers; their raw max goes to `decide`, which exchanges it with the
+// other half, moves the reference when the row max grew by > 2^8 (rescaling O) and returns the
+// reference every P of this tile is taken against (0 while the row has seen no visible key);
+// P = exp2(s * scale - ref) is then written per 32-column chunk as soon as it is packed, so the
+// first chunk's tcgen05.st overlaps the second chunk's math.  Returns the row-half sum.
+template <bool MASKED, class Decide>
+__device__ __forceinline__ float row_softmax_dbe(uint32_t tS, const uint32_t (&vis)[2], float scale,
+                                                 Decide&& decide) {
+  uint32_t r[2][32];
+  ptx::tmem_ld32(tS, r[0]);
+  ptx::tmem_ld32(tS + 32, r[1]);
+  ptx::tmem_ld_wait();
+  if (MASKED) {
+#pragma unroll
+    for (int c = 0; c < 2; ++c)
+#pragma unroll
+      for (int i = 0; i < 32; ++i) r[c][i] = ((vis[c] >> i) & 1u) ? r[c][i] : 0xff800000u;  // -inf
+  }
+  float m0 = -INFINITY, m1 = -INFINITY;
+#pragma unroll
+  for (int c = 0; c < 2; ++c)
+#pragma unroll
+    for (int i = 0; i < 32; i += 4) {
+      m0 = fmax3(m0, __uint_as_float(r[c][i]), __uint_as_float(r[c][i + 1]));
+      m1 = fmax3(m1, __uint_as_float(r[c][i + 2]), __uint_as_float(r[c][i + 3]));
+    }
+  const float ref = decide(fmaxf(m0, m1));
+  const uint64_t sc2 = pk2(scale, scale), nm2 = pk2(-ref, -ref);
+  uint64_t acc0 = pk2(0.0f, 0.0f), acc1 = acc0;
+#pragma unroll
+  for (int c = 0; c < 2; ++c) {
+    uint32_t pk[16];
+#pragma unroll
+    for (int i = 0; i < 16; ++i) {
+      const uint64_t xv = ffma2(pk2(__uint_as_float(r[c][2 * i]), __uint_as_float(r[c][2 * i + 1])), sc2, nm2);
+      float x0, x1;
+      up2(xv, x0, x1);
+      uint64_t e;
+      if (i < BAT_POLY_PAIRS) {
+        e = exp2_poly2(xv);
+        if (MASKED) {  // the polynomial clamps at -127: re-zero masked lanes
+          float p0, p1;
+          up2(e, p0, p1);
+          e = pk2(x0 == -INFINITY ? 0.0f : p0, x1 == -INFINITY ? 0.0f : p1);
+        }
+      } else {
+        e = pk2(ex2(x0), ex2(x1));  // ex2(-inf) = 0
+      }
+      float p0, p1;
+      up2(e, p0, p1);
+      if (i & 1) acc1 = fadd2(acc1, e);
+      else acc0 = fadd2(acc0, e);
+      pk[i] = ptx::pack_bf16x2(p0, p1);
+    }
+    asm volatile(
+        "tcgen05.st.sync.aligned.32x32b.x16.b32 [%0], "
+        "{%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,%16};" ::"r"(tS + c * 16),
+        "r"(pk[0]), "r"(pk[1]), "r"(pk[2]), "r"(pk[3]), "r"(pk[4]), "r"(pk[5]), "r"(pk[6]), "r"(pk[7]),
+        "r"(pk[8]), "r"(pk[9]), "r"(pk[10]), "r"(pk[11]), "r"(pk[12]), "r"(pk[13]), "r"(pk[14]),
+        "r"(pk[15]));
+  }
+  float a0, a1, b0, b1;
+  up2(acc0, a0, a1);
+  up2(acc1, b0, b1);
+  return (a0 + a1) + (b0 + b1);
 }
 
 template <int NC>
@@ -670,9 +741,52 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) attn_tc_kernel(const __grid_co
         seq_wait();
         ptx::tc_fence_after();
         const uint32_t vis[NCH] = {mv.x, mv.y};
+        float lsum = 0.0f;
+#if BAT_ATTN_DBE
+        if (state == 0) {
+          row_zero_p<NCH>(tS);
+        } else {
+          // the row's reference for this tile: both halves' raw maxima through smem, then the
+          // same lazy-rescale decision in both (so they agree without a vote)
+          bool need_o = false;
+          float alpha = 1.0f;
+          auto decide = [&](float mt) {
+            if (wg == 0) DBG(18, x);
+            xch->rmax[s][wg][h][row] = mt;
+            ptx::bar_sync(pair_bar, 64);
+            if (wg == 0) DBG(19, x);
+            mt = fmaxf(mt, xch->rmax[s][wg][h ^ 1][row]);
+            const float m_new = fmaxf(m_ref, mt * p.scale_log2);
+            if (m_new > m_ref + kRescaleThreshold) {
+              alpha = ex2(m_ref - m_new);  // 0 when m_ref = -inf
+              l_sum *= alpha;
+              need_o = (m_ref != -INFINITY) && (x > 0);
+              m_ref = m_new;
+            }
+            return (m_ref == -INFINITY) ? 0.0f : m_ref;
+          };
+          lsum = (state == 1) ? row_softmax_dbe<false>(tS, vis, p.scale_log2, decide)
+                              : row_softmax_dbe<true>(tS, vis, p.scale_log2, decide);
+          // O rows of this warp rescaled (my half of the columns) before P is handed over: the
+          // previous P.V of this q-tile is complete (issued before this S, in-order tensor pipe)
+          // and this tile's P.V waits for the hand-off
+          if (__any_sync(0xffffffffu, need_o)) {
+            const float a = need_o ? alpha : 1.0f;
+#pragma unroll 1
+            for (int c = 0; c < OCH; ++c) {
+              uint32_t r[32];
+              ptx::tmem_ld32(tO + c * 32, r);
+              ptx::tmem_ld_wait();
+#pragma unroll
+              for (int i = 0; i < 32; ++i) r[i] = __float_as_uint(__uint_as_float(r[i]) * a);
+              ptx::tmem_st32(tO + c * 32, r);
+            }
+          }
+        }
+        if (wg == 0) DBG(12, x);
+#else
         // fast path: one pass against the settled reference max; both halves must agree
         bool done = false;
-        float lsum = 0.0f;
         if (state == 0) {
           row_zero_p<NCH>(tS);
           done = true;
@@ -726,6 +840,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) attn_tc_kernel(const __grid_co
           const uint64_t sc2 = pk2(p.scale_log2, p.scale_log2), nm2 = pk2(-mref, -mref);
           lsum = (state == 1) ? row_exp<false>(tS, vis, sc2, nm2) : row_exp<true>(tS, vis, sc2, nm2);
         }
+#endif
         l_sum += lsum;
         ptx::tmem_st_wait();
         ptx::tc_fence_before();
