@@ -118,6 +118,7 @@ struct __align__(8) AttnBars {
 static_assert(sizeof(AttnBars) <= 256, "barrier area");
 #ifndef BAT_ATTN_SEQ
 #define BAT_ATTN_SEQ 0  // 1: the two q-tile softmax teams take turns (FA4-style); measured 543 vs 600 TFLOP/s
+                        // 2: only their exp phases (DBE: after the reference decision, until P is stored) take turns
 #endif
 
 // ring positions: K tile g -> slot g % 3; V half h (= 2 g + {0,1}) -> slot h % 3
@@ -738,13 +739,17 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) attn_tc_kernel(const __grid_co
         BAT_SWAIT(&bars->s_full[wg], sc & 1);
         DBG(11 + 3 * wg, x);
         ++sc;
-        seq_wait();
+        if (BAT_ATTN_SEQ == 1) seq_wait();
         ptx::tc_fence_after();
         const uint32_t vis[NCH] = {mv.x, mv.y};
         float lsum = 0.0f;
 #if BAT_ATTN_DBE
         if (state == 0) {
           row_zero_p<NCH>(tS);
+          if (BAT_ATTN_SEQ == 2) {
+            seq_wait();
+            seq_pass();
+          }
         } else {
           // the row's reference for this tile: both halves' raw maxima through smem, then the
           // same lazy-rescale decision in both (so they agree without a vote)
@@ -763,10 +768,12 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) attn_tc_kernel(const __grid_co
               need_o = (m_ref != -INFINITY) && (x > 0);
               m_ref = m_new;
             }
+            if (BAT_ATTN_SEQ == 2) seq_wait();  // the exp phases of the two teams take turns
             return (m_ref == -INFINITY) ? 0.0f : m_ref;
           };
           lsum = (state == 1) ? row_softmax_dbe<false>(tS, vis, p.scale_log2, decide)
                               : row_softmax_dbe<true>(tS, vis, p.scale_log2, decide);
+          if (BAT_ATTN_SEQ == 2) seq_pass();
           // O rows of this warp rescaled (my half of the columns) before P is handed over: the
           // previous P.V of this q-tile is complete (issued before this S, in-order tensor pipe)
           // and this tile's P.V waits for the hand-off
@@ -846,7 +853,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) attn_tc_kernel(const __grid_co
         ptx::tc_fence_before();
         __syncwarp();
         if (lane == 0) ptx::mbar_arrive(&bars->p_full[wg]);
-        seq_pass();
+        if (BAT_ATTN_SEQ == 1) seq_pass();
         DBG(13 + 2 * wg, x);
         n_mv = make_uint2(0xffffffffu, 0xffffffffu);
         if (n_state == 2) n_mv = mask_of(n_mid);
