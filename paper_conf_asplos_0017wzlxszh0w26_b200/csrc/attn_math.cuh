@@ -39,11 +39,14 @@ __device__ __forceinline__ float fmax3(float a, float b, float c) {
 }
 // 2^x for a pair on the FMA pipe (offloads the MUFU): x = j + f, j = rint(x) by the
 // 1.5*2^23 trick, 2^f on [-0.5, 0.5] by a degree-3 minimax polynomial (rel. err 1.1e-4, far
-// below the bf16 rounding of P), exponent inserted with an integer multiply-add.
+// below the bf16 rounding of P), exponent inserted with an integer multiply-add.  x is clamped
+// at -126 so the inserted exponent never underflows the field: p(0) = 0.99992 < 1 has biased
+// exponent 126, so j = -127 would wrap into the sign bit (a NaN, seen with rows whose scores
+// span > 126 log2 units — tests/test_gpu_attn_rescale.py); 2^-126 is far below P's bf16 ulp.
 __device__ __forceinline__ uint64_t exp2_poly2(uint64_t x) {
   float x0, x1;
   up2(x, x0, x1);
-  x = pk2(fmaxf(x0, -127.0f), fmaxf(x1, -127.0f));
+  x = pk2(fmaxf(x0, -126.0f), fmaxf(x1, -126.0f));
   const uint64_t magic = pk2(12582912.0f, 12582912.0f);
   const uint64_t t = fadd2(x, magic);
   const uint64_t jf = fadd2(t, pk2(-12582912.0f, -12582912.0f));

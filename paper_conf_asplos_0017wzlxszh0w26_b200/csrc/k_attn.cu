@@ -250,7 +250,7 @@ __device__ __forceinline__ bool row_exp_opt(uint32_t tS, const uint32_t (&vis)[N
       uint64_t e;
       if (i < BAT_POLY_PAIRS) {
         e = exp2_poly2(xv);
-        if (MASKED) {  // the polynomial clamps at -127: re-zero masked lanes
+        if (MASKED) {  // the polynomial clamps at -126: re-zero masked lanes
           float p0, p1;
           up2(e, p0, p1);
           e = pk2(x0 == -INFINITY ? 0.0f : p0, x1 == -INFINITY ? 0.0f : p1);
@@ -328,7 +328,7 @@ __device__ __forceinline__ float row_softmax_dbe(uint32_t tS, const uint32_t (&v
       uint64_t e;
       if (i < BAT_POLY_PAIRS) {
         e = exp2_poly2(xv);
-        if (MASKED) {  // the polynomial clamps at -127: re-zero masked lanes
+        if (MASKED) {  // the polynomial clamps at -126: re-zero masked lanes
           float p0, p1;
           up2(e, p0, p1);
           e = pk2(x0 == -INFINITY ? 0.0f : p0, x1 == -INFINITY ? 0.0f : p1);

@@ -17,7 +17,7 @@ void count_launch(int) {}
 void set_smem_attr_raw(const void*, int) {}
 namespace {
 
-template <int MODE, bool RANDOM_DATA = false>
+template <int MODE, bool RANDOM_DATA = false, bool DBE = false>
 __global__ void __launch_bounds__(640, 1) chain(long long* out, int iters) {
   extern __shared__ __align__(1024) uint8_t smem[];
   __shared__ uint64_t s_full[2], p_full[2];
@@ -122,7 +122,17 @@ __global__ void __launch_bounds__(640, 1) chain(long long* out, int iters) {
           ptx::bar_sync(1 + q * 4 + sub, 64);
           return ok && okx[q][h ^ 1][sub] != 0;
         };
-        row_exp_opt<false>(tS, vis, sc2, nm2, INFINITY, lsum, agree);
+        if (DBE) {
+          __shared__ float rmx[2][2][128];
+          auto decide = [&](float mt) {
+            rmx[q][h][sub * 32 + lane] = mt;
+            ptx::bar_sync(1 + q * 4 + sub, 64);
+            return fmaxf(mt, rmx[q][h ^ 1][sub * 32 + lane]) * 0.0f + 1.0f;
+          };
+          lsum = row_softmax_dbe<false>(tS, vis, 0.01f, decide);
+        } else {
+          row_exp_opt<false>(tS, vis, sc2, nm2, INFINITY, lsum, agree);
+        }
         acc += lsum;
         ptx::tmem_st_wait();
       }
@@ -164,5 +174,7 @@ int main() {
   run(chain<3>, "1 q-tile + background MMAs on other TMEM cols", 1);
   run(chain<0, true>, "1 q-tile, random Q/K/V (realistic S)", 1);
   run(chain<2, true>, "2 q-tiles, random Q/K/V (realistic S)", 2);
+  run(chain<0, true, true>, "1 q-tile, DBE softmax (k_attn default)", 1);
+  run(chain<2, true, true>, "2 q-tiles, DBE softmax (k_attn default)", 2);
   return 0;
 }
