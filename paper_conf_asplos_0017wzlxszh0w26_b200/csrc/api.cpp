@@ -136,7 +136,7 @@ struct DevBuf {
 };
 
 struct Workspace {
-  DevBuf h, xn, qkv, qp, scratch, o, act, hc, xc, oc, actc, img, small, part_o, part_ml, gpart;
+  DevBuf h, xn, qkv, qp, scratch, o, act, hc, xc, oc, actc, img, small, part_o, part_ml, gpart, ss;
   void* img_host = nullptr;
   size_t img_host_cap = 0;
   cudaEvent_t img_done = nullptr;
@@ -539,16 +539,49 @@ static void run_plan(Pool& pool, Model& m, Plan& plan, float* out_hidden, cudaSt
                        epi == EPI_BF16_BIAS ? gp.bias : nullptr, epi == EPI_RESID_F32 ? 0 : 1, st);
   };
 
+  // RMSNorm fused across the residual updates (GemmParams::norm_g / ss_in; opt-in BAT_FUSED_NORM=1,
+  // large batches only: no projection of a full-row layer on the split-K path).  Measured in the
+  // configs[2] step it is a net loss (the O GEMM's epilogue, short K, slows by more than the 8 ms
+  // of norm passes it removes: profiles/r2_gemm_epilogue.txt), so the standalone norm is the default
+  const char* fuse_e = std::getenv("BAT_FUSED_NORM");  // read per call: tests A/B both paths
+  const bool fuse_env = fuse_e && fuse_e[0] == '1';
+  const bool fuse_ok = fuse_env && (H % 32) == 0 &&
+                         gemm_ksplit(EPI_BF16_BIAS, M, m.nqkv(), H, m.num_sms, nullptr) <= 1 &&
+                         gemm_ksplit(EPI_RESID_F32, M, H, nq, m.num_sms, nullptr) <= 1 &&
+                         gemm_ksplit(EPI_RESID_F32, M, H, F, m.num_sms, nullptr) <= 1;
+  const int ss_parts_resid = (H + 255) / 256 * gemm_epi_col_splits();  // (N-tile, slice) partial sums
+  const bool fuse_norm = fuse_ok && ss_parts_resid <= 32;                  // row_rstd loads <= 32 parts
+  if (fuse_norm) ws.ss.ensure(size_t(ss_parts_resid) * M * 4, st);
+  auto set_norm_out = [&](GemmParams& g, const __nv_bfloat16* gnext) {  // producer: h += .., xn, ss
+    g.norm_g = gnext;
+    g.xg_out = ws.xn.as<__nv_bfloat16>();
+    g.ss_out = ws.ss.as<float>();
+    g.norm_h = H;
+  };
+  auto set_norm_in = [&](GemmParams& g, int parts) {  // consumer: rows scaled by rsqrt(mean h^2 + eps)
+    g.ss_in = ws.ss.as<float>();
+    g.ss_parts = parts;
+    g.norm_h = H;
+    g.eps = c.rms_eps;
+  };
   pf.begin(st);
-  launch_embed(m.embed, I + im.off_tok, ws.h.as<float>(), M, H, st);
-  pf.end(st, BAT_K_EMBED, 0, 6.0 * M * H);
+  if (fuse_norm)
+    launch_embed_norm(m.embed, I + im.off_tok, ws.h.as<float>(), m.layers[0].ln1, ws.xn.as<__nv_bfloat16>(),
+                      ws.ss.as<float>(), M, H, st);
+  else
+    launch_embed(m.embed, I + im.off_tok, ws.h.as<float>(), M, H, st);
+  pf.end(st, BAT_K_EMBED, 0, (fuse_norm ? 8.0 : 6.0) * M * H);
   for (int l = 0; l < c.layers; ++l) {
     const Model::Layer& Lw = m.layers[l];
     const bool last = (l == c.layers - 1);
-    pf.begin(st);
-    launch_rmsnorm_bf16(ws.h.as<float>(), Lw.ln1, ws.xn.as<__nv_bfloat16>(), M, H, c.rms_eps, st);
-    pf.end(st, BAT_K_RMSNORM, 0, 6.0 * M * H);
     GemmParams gp{M, m.nqkv(), H, ws.qkv.p, m.nqkv(), Lw.bqkv, 0};
+    if (fuse_norm) {
+      set_norm_in(gp, l == 0 ? 1 : ss_parts_resid);
+    } else {
+      pf.begin(st);
+      launch_rmsnorm_bf16(ws.h.as<float>(), Lw.ln1, ws.xn.as<__nv_bfloat16>(), M, H, c.rms_eps, st);
+      pf.end(st, BAT_K_RMSNORM, 0, 6.0 * M * H);
+    }
     auto fq = gemm_fb(M, m.nqkv(), H, 2);
     pf.begin(st);
     gemm(EPI_BF16_BIAS, tA_xn, Lw.t_qkv, tC_qkv, gp);
@@ -587,20 +620,27 @@ static void run_plan(Pool& pool, Model& m, Plan& plan, float* out_hidden, cudaSt
         cudaFree(dbi);
       }
       GemmParams go{M, H, nq, ws.h.p, H, nullptr, 0};
-      auto fo = gemm_fb(M, H, nq, 8);
+      if (fuse_norm) set_norm_out(go, Lw.ln2);
+      auto fo = gemm_fb(M, H, nq, fuse_norm ? 10 : 8);
       pf.begin(st);
       gemm(EPI_RESID_F32, tA_o, Lw.t_o, tC_h, go);
       pf.end(st, BAT_K_GEMM_O, fo.first, fo.second);
-      pf.begin(st);
-      launch_rmsnorm_bf16(ws.h.as<float>(), Lw.ln2, ws.xn.as<__nv_bfloat16>(), M, H, c.rms_eps, st);
-      pf.end(st, BAT_K_RMSNORM, 0, 6.0 * M * H);
       GemmParams gg{M, F, H, ws.act.p, F, nullptr, F};
+      if (fuse_norm) {
+        set_norm_in(gg, ss_parts_resid);
+      } else {
+        pf.begin(st);
+        launch_rmsnorm_bf16(ws.h.as<float>(), Lw.ln2, ws.xn.as<__nv_bfloat16>(), M, H, c.rms_eps, st);
+        pf.end(st, BAT_K_RMSNORM, 0, 6.0 * M * H);
+      }
       auto fg = gemm_fb(M, 2 * F, H, 1);
       pf.begin(st);
       launch_gemm(EPI_SWIGLU, tA_xn, Lw.t_gu, tC_act, gg, m.num_sms, st);
       pf.end(st, BAT_K_GEMM_GU, fg.first, fg.second);
       GemmParams gd{M, H, F, ws.h.p, H, nullptr, 0};
-      auto fd = gemm_fb(M, H, F, 8);
+      // the next layer's RMSNorm rides on this residual update (its K/V are needed: not the last)
+      if (fuse_norm) set_norm_out(gd, m.layers[l + 1].ln1);
+      auto fd = gemm_fb(M, H, F, fuse_norm ? 10 : 8);
       pf.begin(st);
       gemm(EPI_RESID_F32, tA_act, Lw.t_d, tC_h, gd);
       pf.end(st, BAT_K_GEMM_DOWN, fd.first, fd.second);

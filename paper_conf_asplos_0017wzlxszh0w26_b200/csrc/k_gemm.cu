@@ -21,6 +21,7 @@
 // Tiles are rasterised in groups of M-tiles (GROUP_M; 32 for SwiGLU) so concurrently running CTAs
 // share operand tiles in L2.
 #include <cuda.h>
+#include <algorithm>
 #include <cstdlib>
 #include <cuda_bf16.h>
 #include <cuda_runtime.h>
@@ -37,26 +38,36 @@ constexpr int A_BYTES = 128 * BK * 2;           // 16 KB: 128 rows of A per CTA
 // run back to back (down GEMM DRAM reads 1.43 GB at 8, 1.27 at 4, 1.12 at 1, 2.26 at 32 per launch,
 // profiles/r1_gemm_raster.txt); BAT_GEMM_GROUP_M / _SWIGLU override
 constexpr int GROUP_M = 1;
-constexpr int GROUP_M_SWIGLU = 32;
-constexpr int NUM_THREADS = 192;
+constexpr int GROUP_M_SWIGLU = 32;       // 1-CTA SwiGLU kernel (128-row M-tiles)
+constexpr int GROUP_M_SWIGLU_PAIR = 4;   // CTA-pair SwiGLU kernel (256-row M-tiles)
+// Epilogue warps per CTA: 4 (one per TMEM lane quarter) or 8 (two per quarter, splitting the
+// accumulator's columns).  The SwiGLU GEMM (short K = hidden, MUFU-heavy epilogue) runs 8 and
+// gains 5% over 4; the others keep 4 warps and one more ring stage (their K loops are long or
+// their epilogues light: 8 warps measured 1-4% slower there, profiles/r2_gemm_epilogue.txt)
+constexpr int epi_warps(int epi) { return epi == EPI_SWIGLU ? 8 : 4; }
 constexpr int STG_BYTES = 4096;  // per-warp epilogue staging buffer: [32 rows][128 B], 128B-swizzled
 
-// 1-CTA kernel: 128 x 256 tiles
-constexpr int STAGES1 = 4;
-constexpr int STAGE1_BYTES = A_BYTES + BN * BK * 2;  // 48 KB
-constexpr int STG1_OFF = STAGES1 * STAGE1_BYTES;
-// CTA-pair kernel: 256 x 256 tiles, each CTA 128 rows of A + 128 rows of B per stage
-constexpr int STAGES2 = 6;
-constexpr int STAGE2_BYTES = A_BYTES + BROWS * BK * 2;  // 32 KB
-constexpr int STG2_OFF = STAGES2 * STAGE2_BYTES;
+constexpr int STAGE1_BYTES = A_BYTES + BN * BK * 2;  // 1-CTA kernel (128 x 256 tiles): 48 KB per stage
+constexpr int STAGE2_BYTES = A_BYTES + BROWS * BK * 2;  // CTA pair (256 x 256 tiles, 128 rows of A + B per CTA): 32 KB
 
 struct __align__(8) GemmSmemBars {
   uint64_t full[8], empty[8], tfull[2], tempty[2];
   uint32_t tmem_base;
 };
-constexpr size_t kGemmSmem1 = 1024 /*align slack*/ + STG1_OFF + 4 * 2 * STG_BYTES + sizeof(GemmSmemBars);
-constexpr size_t kGemmSmem2 = 1024 /*align slack*/ + STG2_OFF + 4 * 2 * STG_BYTES + sizeof(GemmSmemBars);
-static_assert(kGemmSmem1 <= 232448 && kGemmSmem2 <= 232448, "GEMM shared memory");
+template <int EW>
+struct GemmCfg {
+  static constexpr int THREADS = 64 + 32 * EW;
+  static constexpr int SPLIT = EW / 4;  // column slices of an accumulator
+  static constexpr int STAGES1 = EW == 8 ? 3 : 4;
+  static constexpr int STG1_OFF = STAGES1 * STAGE1_BYTES;
+  static constexpr int STAGES2 = EW == 8 ? 5 : 6;
+  static constexpr int STG2_OFF = STAGES2 * STAGE2_BYTES;
+  static constexpr size_t SMEM1 = 1024 /*align slack*/ + STG1_OFF + EW * 2 * STG_BYTES + sizeof(GemmSmemBars);
+  static constexpr size_t SMEM2 = 1024 /*align slack*/ + STG2_OFF + EW * 2 * STG_BYTES + sizeof(GemmSmemBars);
+  static_assert(EW == 4 || EW == 8, "epilogue warps");
+  static_assert(SMEM1 <= 232448 && SMEM2 <= 232448, "GEMM shared memory");
+  static_assert(STAGES2 <= 8, "barrier array");
+};
 
 __device__ __forceinline__ void tile_coords(int t, int num_m, int num_n, int group_m, int& m, int& n) {
   const int per_group = group_m * num_n;
@@ -67,7 +78,19 @@ __device__ __forceinline__ void tile_coords(int t, int num_m, int num_n, int gro
   n = r / rows;
 }
 
-__device__ __forceinline__ float silu(float x) { return x / (1.0f + __expf(-x)); }
+__device__ __forceinline__ float rcp_approx(float x) {
+  float y;
+  asm("rcp.approx.ftz.f32 %0, %1;" : "=f"(y) : "f"(x));
+  return y;
+}
+__device__ __forceinline__ float ex2_approx(float x) {
+  float y;
+  asm("ex2.approx.ftz.f32 %0, %1;" : "=f"(y) : "f"(x));
+  return y;
+}
+// silu(x) = x / (1 + e^-x) with MUFU ex2 and rcp (both ~1 ulp; an IEEE division cost ~10 more
+// instructions per output in the epilogue, which paces the short-K SwiGLU GEMM)
+__device__ __forceinline__ float silu(float x) { return x * rcp_approx(1.0f + ex2_approx(x * -1.44269504f)); }
 
 // Epilogue of one accumulator (this warp's 32 TMEM lanes = output rows row0 .. row0 + 31):
 // TMEM -> registers -> (bias / SwiGLU) -> 128B-swizzled smem staging -> TMA store (bf16) or
@@ -93,7 +116,8 @@ struct Epilogue {
     ptx::fence_proxy_async_smem();
     __syncwarp();
     if (lane == 0) {
-      if (EPI == EPI_RESID_F32) ptx::tma_reduce_add_2d(tmC, buf, col, row);
+      if (EPI == EPI_RESID_F32 && p->norm_g) ptx::tma_store_2d(tmC, buf, col, row);  // h_new computed here
+      else if (EPI == EPI_RESID_F32) ptx::tma_reduce_add_2d(tmC, buf, col, row);
       else if (EPI == EPI_PART_F32) ptx::tma_store_2d(tmC, buf, col, row);
       else if (p->hints & 2) ptx::tma_store_2d_hint(tmC, buf, col, row, ptx::policy_evict_first());
       else ptx::tma_store_2d(tmC, buf, col, row);
@@ -101,11 +125,85 @@ struct Epilogue {
     }
     sbuf ^= 1;
   }
-  // tbase: TMEM address of this warp's lanes, column 0 of the accumulator; n: output N-tile
-  __device__ __forceinline__ void run(uint32_t tbase, int n, int row0) {
+  // fused RMSNorm, consumer side: this lane's row scale rsqrt(mean(h^2) + eps) (1 without ss_in);
+  // the partial sums are loaded together (independent loads), summed in a fixed order
+  __device__ __forceinline__ float row_rstd(int row) const {
+    if (!p->ss_in || row >= p->M) return 1.0f;
+    float v[32];
+#pragma unroll
+    for (int j = 0; j < 32; ++j) v[j] = j < p->ss_parts ? p->ss_in[int64_t(j) * p->M + row] : 0.0f;
+    float ss = 0.0f;
+#pragma unroll
+    for (int j = 0; j < 32; ++j) ss += v[j];
+    return rsqrtf(ss / float(p->norm_h) + p->eps);
+  }
+  // fused RMSNorm, producer side (EPI_RESID_F32 with norm_g): h_new = h + acc for this lane's row,
+  // 32 columns per chunk; h_old is read directly (128 B per lane, one chunk ahead), h_new leaves
+  // through the swizzled staging buffer and a TMA store, xg = bf16(h_new * g) with 16-byte stores
+  __device__ __forceinline__ void run_resid_norm(uint32_t tbase, int n, int row0, int c_lo, int c_hi, int part) {
+    const int row = row0 + int(lane);
+    const bool ok = row < p->M;
+    const int col_base = n * BN;
+    const float* hrow = static_cast<const float*>(p->out) + int64_t(ok ? row : 0) * p->ldo;
+    float4 hv[8], hn[8];
+    auto load_h = [&](int c, float4 (&dst)[8]) {
+#pragma unroll
+      for (int i = 0; i < 8; ++i)
+        dst[i] = ok && col_base + c < p->N ? __ldcs(reinterpret_cast<const float4*>(hrow + col_base + c) + i)
+                                           : make_float4(0.f, 0.f, 0.f, 0.f);
+    };
+    load_h(c_lo, hv);
+    float ss = 0.0f;
+#pragma unroll 1
+    for (int c = c_lo; c < c_hi; c += 32) {
+      if (c + 32 < c_hi) load_h(c + 32, hn);
+      uint8_t* buf = next_buf();
+      uint32_t r[32];
+      ptx::tmem_ld32(tbase + c, r);
+      ptx::tmem_ld_wait();
+      const int col = col_base + c;
+      const uint4* g4 = reinterpret_cast<const uint4*>(p->norm_g + (col < p->N ? col : 0));
+      uint32_t pk[16];
+#pragma unroll
+      for (int j = 0; j < 8; ++j) {
+        const float4 o = hv[j];
+        const float v0 = o.x + __uint_as_float(r[4 * j]), v1 = o.y + __uint_as_float(r[4 * j + 1]);
+        const float v2 = o.z + __uint_as_float(r[4 * j + 2]), v3 = o.w + __uint_as_float(r[4 * j + 3]);
+        ss += v0 * v0 + v1 * v1 + v2 * v2 + v3 * v3;
+        stage_row(buf, j, __float_as_uint(v0), __float_as_uint(v1), __float_as_uint(v2), __float_as_uint(v3));
+        const uint4 gq = __ldg(g4 + (j >> 1));
+        const uint32_t ga = (j & 1) ? gq.z : gq.x, gb = (j & 1) ? gq.w : gq.y;
+        const float2 g01 = __bfloat1622float2(*reinterpret_cast<const __nv_bfloat162*>(&ga));
+        const float2 g23 = __bfloat1622float2(*reinterpret_cast<const __nv_bfloat162*>(&gb));
+        pk[2 * j] = ptx::pack_bf16x2(v0 * g01.x, v1 * g01.y);
+        pk[2 * j + 1] = ptx::pack_bf16x2(v2 * g23.x, v3 * g23.y);
+      }
+      if (ok && col < p->N) {
+        uint4* xd = reinterpret_cast<uint4*>(p->xg_out + int64_t(row) * p->norm_h + col);
+#pragma unroll
+        for (int i = 0; i < 4; ++i) xd[i] = make_uint4(pk[4 * i], pk[4 * i + 1], pk[4 * i + 2], pk[4 * i + 3]);
+      }
+      flush(buf, col, row0);
+#pragma unroll
+      for (int i = 0; i < 8; ++i) hv[i] = hn[i];
+    }
+    if (ok) p->ss_out[int64_t(n * GemmCfg<epi_warps(EPI)>::SPLIT + part) * p->M + row] = ss;
+  }
+  // tbase: TMEM address of this warp's lanes, column 0 of the accumulator; n: output N-tile;
+  // part: this warp's column slice of the accumulator (EPI_SPLIT slices); rs: the row's fused-norm
+  // scale (row_rstd, loaded before the accumulator wait)
+  __device__ __forceinline__ void run(uint32_t tbase, int n, int row0, int part, float rs) {
+    constexpr int W = BN / GemmCfg<epi_warps(EPI)>::SPLIT;  // accumulator columns per slice
+    const int c_lo = part * W, c_hi = c_lo + W;
+    if constexpr (EPI == EPI_RESID_F32) {
+      if (p->norm_g) {
+        run_resid_norm(tbase, n, row0, c_lo, c_hi, part);
+        return;
+      }
+    }
     if constexpr (EPI == EPI_SWIGLU) {
 #pragma unroll 1
-      for (int c = 0; c < BN / 2; c += 64) {  // 64 output columns per staging buffer
+      for (int c = c_lo / 2; c < c_hi / 2; c += 64) {  // 64 output columns per staging buffer
         uint8_t* buf = next_buf();
 #pragma unroll
         for (int h = 0; h < 2; ++h) {
@@ -116,8 +214,8 @@ struct Epilogue {
           uint32_t pk[16];
 #pragma unroll
           for (int i = 0; i < 16; ++i) {
-            float g0 = __uint_as_float(g[2 * i]), g1 = __uint_as_float(g[2 * i + 1]);
-            float u0 = __uint_as_float(u[2 * i]), u1 = __uint_as_float(u[2 * i + 1]);
+            float g0 = __uint_as_float(g[2 * i]) * rs, g1 = __uint_as_float(g[2 * i + 1]) * rs;
+            float u0 = __uint_as_float(u[2 * i]) * rs, u1 = __uint_as_float(u[2 * i + 1]) * rs;
             pk[i] = ptx::pack_bf16x2(silu(g0) * u0, silu(g1) * u1);
           }
 #pragma unroll
@@ -127,7 +225,7 @@ struct Epilogue {
       }
     } else if constexpr (EPI == EPI_RESID_F32 || EPI == EPI_PART_F32) {
 #pragma unroll 1
-      for (int c = 0; c < BN; c += 32) {  // 32 fp32 columns per staging buffer
+      for (int c = c_lo; c < c_hi; c += 32) {  // 32 fp32 columns per staging buffer
         uint8_t* buf = next_buf();
         uint32_t r[32];
         ptx::tmem_ld32(tbase + c, r);
@@ -138,7 +236,7 @@ struct Epilogue {
       }
     } else {
 #pragma unroll 1
-      for (int c = 0; c < BN; c += 64) {  // 64 bf16 columns per staging buffer
+      for (int c = c_lo; c < c_hi; c += 64) {  // 64 bf16 columns per staging buffer
         uint8_t* buf = next_buf();
 #pragma unroll
         for (int h = 0; h < 2; ++h) {
@@ -149,7 +247,7 @@ struct Epilogue {
           uint32_t pk[16];
 #pragma unroll
           for (int i = 0; i < 16; ++i) {
-            float v0 = __uint_as_float(r[2 * i]), v1 = __uint_as_float(r[2 * i + 1]);
+            float v0 = __uint_as_float(r[2 * i]) * rs, v1 = __uint_as_float(r[2 * i + 1]) * rs;
             if (EPI == EPI_BF16_BIAS && col + 2 * i + 1 < p->N) {
               v0 += __bfloat162float(p->bias[col + 2 * i]);
               v1 += __bfloat162float(p->bias[col + 2 * i + 1]);
@@ -173,14 +271,16 @@ __device__ __forceinline__ int b_row(const GemmParams& p, int n, int h) {
 
 // ------------------------------------------------------------------- 1-CTA, 128 x 256 tiles
 template <int EPI>
-__global__ void __launch_bounds__(NUM_THREADS, 1)
+__global__ void __launch_bounds__(GemmCfg<epi_warps(EPI)>::THREADS, 1)
 gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
                const __grid_constant__ CUtensorMap tmC, GemmParams p) {
   extern __shared__ uint8_t smem_raw[];
   // 1 KB-align by offsetting the __shared__ array itself (keeps the shared address space, so
   // the compiler emits LDS/STS rather than generic loads and stores)
   uint8_t* smem = smem_raw + ((1024u - (ptx::smem_u32(smem_raw) & 1023u)) & 1023u);
-  GemmSmemBars* bars = reinterpret_cast<GemmSmemBars*>(smem + STG1_OFF + 4 * 2 * STG_BYTES);
+  using C = GemmCfg<epi_warps(EPI)>;
+  constexpr int STAGES1 = C::STAGES1, STG1_OFF = C::STG1_OFF, EPI_WARPS = epi_warps(EPI);
+  GemmSmemBars* bars = reinterpret_cast<GemmSmemBars*>(smem + STG1_OFF + EPI_WARPS * 2 * STG_BYTES);
   const uint32_t warp = ptx::warp_id(), lane = ptx::lane_id();
   constexpr uint32_t IDESC = ptx::idesc_bf16(128, BN, 0, 0);
 
@@ -199,7 +299,7 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
     }
     for (int a = 0; a < 2; ++a) {
       ptx::mbar_init(&bars->tfull[a], 1);
-      ptx::mbar_init(&bars->tempty[a], 4);
+      ptx::mbar_init(&bars->tempty[a], EPI_WARPS);
     }
     ptx::fence_mbar_init();
     ptx::prefetch_tmap(&tmA);
@@ -267,8 +367,9 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
         if (++acc == 2) { acc = 0; acc_phase ^= 1; }
       }
     }
-  } else {  // ------------------------------ epilogue warps 2..5
+  } else {  // ------------------------------ epilogue warps 2 .. 1 + EPI_WARPS
     const uint32_t sub = warp & 3;  // TMEM sub-partition this warp may access
+    const int part = int(warp - 2) / 4;  // column slice
     Epilogue<EPI> epi{&tmC, &p, smem + STG1_OFF + (warp - 2) * 2 * STG_BYTES, lane};
     int acc = 0;
     uint32_t acc_phase = 0;
@@ -276,9 +377,11 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
       int m, n;
       tile_coords(t % num_tiles, num_m, num_n, p.group_m, m, n);
       const int slab = EPI == EPI_PART_F32 ? (t / num_tiles) * p.mpad : 0;
+      const int row0 = slab + m * 128 + int(sub) * 32;
+      const float rs = (EPI == EPI_SWIGLU || EPI == EPI_BF16_BIAS) ? epi.row_rstd(row0 + int(lane)) : 1.0f;
       ptx::mbar_wait(&bars->tfull[acc], acc_phase);
       ptx::tc_fence_after();
-      epi.run(tmem + ((sub * 32) << 16) + acc * BN, n, slab + m * 128 + sub * 32);
+      epi.run(tmem + ((sub * 32) << 16) + acc * BN, n, row0, part, rs);
       ptx::tc_fence_before();
       __syncwarp();
       if (lane == 0) ptx::mbar_arrive(&bars->tempty[acc]);
@@ -294,12 +397,14 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
 
 // ------------------------------------------------------------ CTA pair, 256 x 256 tiles
 template <int EPI>
-__global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(NUM_THREADS, 1)
+__global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(GemmCfg<epi_warps(EPI)>::THREADS, 1)
 gemm2_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
                 const __grid_constant__ CUtensorMap tmC, GemmParams p) {
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = smem_raw + ((1024u - (ptx::smem_u32(smem_raw) & 1023u)) & 1023u);
-  GemmSmemBars* bars = reinterpret_cast<GemmSmemBars*>(smem + STG2_OFF + 4 * 2 * STG_BYTES);
+  using C = GemmCfg<epi_warps(EPI)>;
+  constexpr int STAGES2 = C::STAGES2, STG2_OFF = C::STG2_OFF, EPI_WARPS = epi_warps(EPI);
+  GemmSmemBars* bars = reinterpret_cast<GemmSmemBars*>(smem + STG2_OFF + EPI_WARPS * 2 * STG_BYTES);
   const uint32_t warp = ptx::warp_id(), lane = ptx::lane_id();
   const uint32_t rank = ptx::cluster_ctarank();  // 0 = leader (issues the pair MMAs)
   constexpr uint32_t IDESC = ptx::idesc_bf16(256, BN, 0, 0);
@@ -320,7 +425,7 @@ gemm2_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__
     }
     for (int a = 0; a < 2; ++a) {
       ptx::mbar_init(&bars->tfull[a], 1);   // pair commit
-      ptx::mbar_init(&bars->tempty[a], 8);  // leader: the 4 epilogue warps of both CTAs
+      ptx::mbar_init(&bars->tempty[a], 2 * EPI_WARPS);  // leader: the epilogue warps of both CTAs
     }
     ptx::fence_mbar_init();
     ptx::prefetch_tmap(&tmA);
@@ -336,6 +441,7 @@ gemm2_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__
 
   if (warp == 0) {
     if (lane == 0) {  // ---------------- TMA producer (both CTAs): my 128 rows of A and of B
+      const uint64_t pol_b = ptx::policy_evict_last();
       int stage = 0;
       uint32_t phase = 0;
       for (int t = pair; t < num_work; t += n_pairs) {
@@ -349,7 +455,10 @@ gemm2_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__
           const uint32_t full_leader = ptx::mapa(ptx::smem_u32(&bars->full[stage]), 0);
           if (rank == 0) ptx::mbar_expect_tx(&bars->full[stage], 2 * STAGE2_BYTES);
           ptx::tma_load_2d_pair(sa, &tmA, kb * BK, m * 256 + int(rank) * 128, full_leader);
-          ptx::tma_load_2d_pair(sb, &tmB, kb * BK, b_row<EPI>(p, n, int(rank)), full_leader);
+          if (p.hints & 1)
+            ptx::tma_load_2d_pair_hint(sb, &tmB, kb * BK, b_row<EPI>(p, n, int(rank)), full_leader, pol_b);
+          else
+            ptx::tma_load_2d_pair(sb, &tmB, kb * BK, b_row<EPI>(p, n, int(rank)), full_leader);
           if (++stage == STAGES2) { stage = 0; phase ^= 1; }
         }
       }
@@ -383,8 +492,9 @@ gemm2_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__
         if (++acc == 2) { acc = 0; acc_phase ^= 1; }
       }
     }
-  } else {  // ------------------------------ epilogue warps 2..5 (both CTAs): my 128 rows
+  } else {  // ------------------------------ epilogue warps (both CTAs): my 128 rows
     const uint32_t sub = warp & 3;
+    const int part = int(warp - 2) / 4;  // column slice
     Epilogue<EPI> epi{&tmC, &p, smem + STG2_OFF + (warp - 2) * 2 * STG_BYTES, lane};
     int acc = 0;
     uint32_t acc_phase = 0;
@@ -392,9 +502,11 @@ gemm2_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__
       int m, n;
       tile_coords(t % num_tiles, num_m, num_n, p.group_m, m, n);
       const int slab = EPI == EPI_PART_F32 ? (t / num_tiles) * p.mpad : 0;
+      const int row0 = slab + m * 256 + int(rank) * 128 + int(sub) * 32;
+      const float rs = (EPI == EPI_SWIGLU || EPI == EPI_BF16_BIAS) ? epi.row_rstd(row0 + int(lane)) : 1.0f;
       ptx::mbar_wait(&bars->tfull[acc], acc_phase);
       ptx::tc_fence_after();
-      epi.run(tmem + ((sub * 32) << 16) + acc * BN, n, slab + m * 256 + int(rank) * 128 + sub * 32);
+      epi.run(tmem + ((sub * 32) << 16) + acc * BN, n, row0, part, rs);
       ptx::tc_fence_before();
       __syncwarp();
       if (lane == 0) ptx::mbar_arrive_cluster(ptx::mapa(ptx::smem_u32(&bars->tempty[acc]), 0));
@@ -411,7 +523,12 @@ gemm2_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__
 
 }  // namespace
 
-size_t gemm_smem_bytes() { return kGemmSmem2 > kGemmSmem1 ? kGemmSmem2 : kGemmSmem1; }
+int gemm_epi_col_splits() { return GemmCfg<epi_warps(EPI_RESID_F32)>::SPLIT; }
+
+size_t gemm_smem_bytes() {
+  const size_t a = std::max(GemmCfg<4>::SMEM1, GemmCfg<4>::SMEM2), b = std::max(GemmCfg<8>::SMEM1, GemmCfg<8>::SMEM2);
+  return std::max(a, b);
+}
 
 static int env_group(const char* name) {
   const char* v = std::getenv(name);
@@ -424,45 +541,51 @@ void launch_gemm(int epi, const CUtensorMap& tmA, const CUtensorMap& tmB, const 
   static const int hints = env_group("BAT_GEMM_HINTS");
   GemmParams p = p_in;
   if (!p.hints) p.hints = hints;
-  // SwiGLU (1-CTA, 128-row tiles, 55 MB of gate/up weights re-streamed once per group): groups of
-  // 32 M-tiles with evict_last weight loads read 574 MB of DRAM per launch instead of 705 MB at
-  // equal speed (profiles/r1_gemm_raster.txt)
+  // SwiGLU on CTA pairs by default (BAT_GEMM_SWIGLU_PAIR=0: 1-CTA 128-row tiles): 8 epilogue warps
+  // and MUFU ex2 / rcp silu, 1,202 -> 1,375-1,389 TFLOP/s in the configs[2] step against the 1-CTA
+  // kernel with the same epilogue (profiles/r2_gemm_epilogue.txt); rasterisation groups of 4 pair
+  // M-tiles (1,024 rows) or 32 1-CTA M-tiles, evict_last weight loads (the 55 MB of gate/up
+  // weights are re-streamed once per group; profiles/r1_gemm_raster.txt)
+  static const char* sp_env = std::getenv("BAT_GEMM_SWIGLU_PAIR");
+  static const bool swiglu_pair = !(sp_env && sp_env[0] == '0');
+  const bool pair = p.M >= 256 && num_sms >= 2 && (epi != EPI_SWIGLU || swiglu_pair);
   if (p.group_m <= 0)
-    p.group_m = epi == EPI_SWIGLU ? (g_swiglu ? g_swiglu : GROUP_M_SWIGLU) : (g_all ? g_all : GROUP_M);
+    p.group_m = epi == EPI_SWIGLU ? (g_swiglu ? g_swiglu : (pair ? GROUP_M_SWIGLU_PAIR : GROUP_M_SWIGLU))
+                                  : (g_all ? g_all : GROUP_M);
   if (epi == EPI_SWIGLU && !std::getenv("BAT_GEMM_HINTS")) p.hints |= 1;
   const int out_bn = (epi == EPI_SWIGLU) ? BN / 2 : BN;
   const int n_tiles = (p.N + out_bn - 1) / out_bn;
-  // the SwiGLU GEMM stays on 1-CTA tiles: measured in the bench step, its pair version ran
-  // slower (1.18 vs 1.24 PFLOP/s) although both tie when timed alone
   const int ks = epi == EPI_PART_F32 ? p.ksplit : 1;
-  if (p.M >= 256 && num_sms >= 2 && epi != EPI_SWIGLU) {
+  if (pair) {
     const int tiles = ((p.M + 255) / 256) * n_tiles * ks;
     const int pairs = tiles < num_sms / 2 ? tiles : num_sms / 2;
-    auto launch = [&](auto kern) {
-      set_smem_attr(kern, kGemmSmem2);
-      kern<<<2 * pairs, NUM_THREADS, kGemmSmem2, stream>>>(tmA, tmB, tmC, p);
+    auto launch = [&](auto kern, auto cfg) {
+      using C = decltype(cfg);
+      set_smem_attr(kern, C::SMEM2);
+      kern<<<2 * pairs, C::THREADS, C::SMEM2, stream>>>(tmA, tmB, tmC, p);
     };
     switch (epi) {
-      case EPI_BF16: launch(gemm2_tc_kernel<EPI_BF16>); break;
-      case EPI_BF16_BIAS: launch(gemm2_tc_kernel<EPI_BF16_BIAS>); break;
-      case EPI_RESID_F32: launch(gemm2_tc_kernel<EPI_RESID_F32>); break;
-      case EPI_SWIGLU: launch(gemm2_tc_kernel<EPI_SWIGLU>); break;
-      case EPI_PART_F32: launch(gemm2_tc_kernel<EPI_PART_F32>); break;
+      case EPI_BF16: launch(gemm2_tc_kernel<EPI_BF16>, GemmCfg<epi_warps(EPI_BF16)>{}); break;
+      case EPI_BF16_BIAS: launch(gemm2_tc_kernel<EPI_BF16_BIAS>, GemmCfg<epi_warps(EPI_BF16_BIAS)>{}); break;
+      case EPI_RESID_F32: launch(gemm2_tc_kernel<EPI_RESID_F32>, GemmCfg<epi_warps(EPI_RESID_F32)>{}); break;
+      case EPI_SWIGLU: launch(gemm2_tc_kernel<EPI_SWIGLU>, GemmCfg<epi_warps(EPI_SWIGLU)>{}); break;
+      case EPI_PART_F32: launch(gemm2_tc_kernel<EPI_PART_F32>, GemmCfg<epi_warps(EPI_PART_F32)>{}); break;
     }
   } else {
     const int tiles = ((p.M + 127) / 128) * n_tiles * ks;
     const int grid = tiles < num_sms ? tiles : num_sms;
     if (grid <= 0) return;
-    auto launch = [&](auto kern) {
-      set_smem_attr(kern, kGemmSmem1);
-      kern<<<grid, NUM_THREADS, kGemmSmem1, stream>>>(tmA, tmB, tmC, p);
+    auto launch = [&](auto kern, auto cfg) {
+      using C = decltype(cfg);
+      set_smem_attr(kern, C::SMEM1);
+      kern<<<grid, C::THREADS, C::SMEM1, stream>>>(tmA, tmB, tmC, p);
     };
     switch (epi) {
-      case EPI_BF16: launch(gemm_tc_kernel<EPI_BF16>); break;
-      case EPI_BF16_BIAS: launch(gemm_tc_kernel<EPI_BF16_BIAS>); break;
-      case EPI_RESID_F32: launch(gemm_tc_kernel<EPI_RESID_F32>); break;
-      case EPI_SWIGLU: launch(gemm_tc_kernel<EPI_SWIGLU>); break;
-      case EPI_PART_F32: launch(gemm_tc_kernel<EPI_PART_F32>); break;
+      case EPI_BF16: launch(gemm_tc_kernel<EPI_BF16>, GemmCfg<epi_warps(EPI_BF16)>{}); break;
+      case EPI_BF16_BIAS: launch(gemm_tc_kernel<EPI_BF16_BIAS>, GemmCfg<epi_warps(EPI_BF16_BIAS)>{}); break;
+      case EPI_RESID_F32: launch(gemm_tc_kernel<EPI_RESID_F32>, GemmCfg<epi_warps(EPI_RESID_F32)>{}); break;
+      case EPI_SWIGLU: launch(gemm_tc_kernel<EPI_SWIGLU>, GemmCfg<epi_warps(EPI_SWIGLU)>{}); break;
+      case EPI_PART_F32: launch(gemm_tc_kernel<EPI_PART_F32>, GemmCfg<epi_warps(EPI_PART_F32)>{}); break;
     }
   }
   count_launch();

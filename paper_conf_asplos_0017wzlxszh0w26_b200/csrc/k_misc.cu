@@ -68,6 +68,40 @@ __global__ void embed_kernel(const __nv_bfloat16* __restrict__ E, const int32_t*
   }
 }
 
+// fused-norm embedding: one warp per row; h0 = E[x_m] (fp32), xg = bf16(h0 * g), ss[m] = sum h0^2
+// (the first layer's RMSNorm is finished in the QKV GEMM epilogue, GemmParams::ss_in)
+__global__ void embed_norm_kernel(const __nv_bfloat16* __restrict__ E, const int32_t* __restrict__ tok,
+                                  float* __restrict__ h, const __nv_bfloat16* __restrict__ g,
+                                  __nv_bfloat16* __restrict__ xg, float* __restrict__ ss_out, int M, int H) {
+  const int m = blockIdx.x * 8 + (threadIdx.x >> 5);
+  const int lane = threadIdx.x & 31;
+  if (m >= M) return;
+  const int64_t src = int64_t(tok[m]) * H;
+  float ss = 0.0f;
+  for (int c = lane * 8; c < H; c += 256) {
+    const uint4 raw = *reinterpret_cast<const uint4*>(E + src + c);
+    const uint4 graw = *reinterpret_cast<const uint4*>(g + c);
+    const __nv_bfloat162* b2 = reinterpret_cast<const __nv_bfloat162*>(&raw);
+    const __nv_bfloat162* g2 = reinterpret_cast<const __nv_bfloat162*>(&graw);
+    float v[8];
+    uint32_t pk[4];
+#pragma unroll
+    for (int i = 0; i < 4; ++i) {
+      const float2 f = __bfloat1622float2(b2[i]), gg = __bfloat1622float2(g2[i]);
+      v[2 * i] = f.x;
+      v[2 * i + 1] = f.y;
+      ss += f.x * f.x + f.y * f.y;
+      pk[i] = ptx::pack_bf16x2(f.x * gg.x, f.y * gg.y);
+    }
+    float4* d = reinterpret_cast<float4*>(h + int64_t(m) * H + c);
+    d[0] = make_float4(v[0], v[1], v[2], v[3]);
+    d[1] = make_float4(v[4], v[5], v[6], v[7]);
+    *reinterpret_cast<uint4*>(xg + int64_t(m) * H + c) = make_uint4(pk[0], pk[1], pk[2], pk[3]);
+  }
+  ss = warp_sum(ss);
+  if (lane == 0) ss_out[m] = ss;
+}
+
 // one warp per row: y = x / sqrt(mean(x^2) + eps) * g
 template <bool F32OUT>
 __global__ void rmsnorm_kernel(const float* __restrict__ x, const __nv_bfloat16* __restrict__ g,
@@ -410,6 +444,12 @@ void launch_masks(int32_t* img, int64_t off_mdesc, int64_t off_qinfo, int64_t of
 void launch_embed(const __nv_bfloat16* E, const int32_t* tok, float* h, int M, int H, cudaStream_t s) {
   if (M <= 0) return;
   embed_kernel<<<M, 128, 0, s>>>(E, tok, h, M, H);
+  count_launch();
+}
+void launch_embed_norm(const __nv_bfloat16* E, const int32_t* tok, float* h, const __nv_bfloat16* g,
+                       __nv_bfloat16* xg, float* ss, int M, int H, cudaStream_t s) {
+  if (M <= 0) return;
+  embed_norm_kernel<<<(M + 7) / 8, 256, 0, s>>>(E, tok, h, g, xg, ss, M, H);
   count_launch();
 }
 void launch_rmsnorm_bf16(const float* x, const __nv_bfloat16* g, __nv_bfloat16* y, int M, int H,

@@ -32,6 +32,19 @@ struct GemmParams {
   int hints = 0;      // 1-CTA kernel L2 hints: bit 0 B loads evict_last, bit 1 bf16 C stores evict_first
   int ksplit = 1;     // EPI_PART_F32: K split in ksplit slices; slice s stores its fp32 partial at
   int mpad = 0;       // rows [s * mpad, s * mpad + M) of the partial buffer (tmC)
+  // RMSNorm fused across the residual update (a3 / a7, P:169 layer structure): the producer
+  // (EPI_RESID_F32 with norm_g set) writes h_new = h + acc by TMA store instead of reduce-add,
+  // xg = bf16(h_new * g) for the next projection's A operand and, per N-tile j, the partial sum of
+  // squares ss_out[j * M + row] of its columns; the consumer (EPI_BF16_BIAS / EPI_SWIGLU with ss_in
+  // set) scales each accumulator row by rsqrt(sum_j ss_in[j * M + row] / norm_h + eps) before its
+  // bias / SwiGLU — RMSNorm(h) W^T = rstd * ((h * g) W^T) with no separate norm pass.
+  const __nv_bfloat16* norm_g = nullptr;
+  __nv_bfloat16* xg_out = nullptr;
+  float* ss_out = nullptr;
+  const float* ss_in = nullptr;
+  int ss_parts = 0;
+  int norm_h = 0;
+  float eps = 0.0f;
 };
 // Split-K for grids that would leave SMs idle (small M: batch-1 requests, the last layer's
 // discriminant rows): slices per tile (1 = no split) for a GEMM of this shape and the row pitch of
@@ -41,6 +54,8 @@ int gemm_ksplit(int epi, int M, int N, int K, int num_sms, int* mpad);
 void launch_gemm_reduce(const float* part, int ksplit, int mpad, int M, int N, void* out, int ldo,
                         const __nv_bfloat16* bias, int mode, cudaStream_t stream);
 size_t gemm_smem_bytes();
+// column slices per accumulator in the epilogue (fused-norm partial sums per N-tile)
+int gemm_epi_col_splits();
 // tmC: output tensor map — bf16 [M][ldo] with box {64, 32} (EPI_BF16*, EPI_SWIGLU) or fp32
 // [M][ldo] with box {32, 32} (EPI_RESID_F32, TMA reduce-add), 128-byte swizzle
 void launch_gemm(int epi, const CUtensorMap& tmA, const CUtensorMap& tmB, const CUtensorMap& tmC,
@@ -86,6 +101,9 @@ void launch_attention(int dpad, const AttnParams& p, int num_sms, cudaStream_t s
 void launch_attention_combine(int dpad, const AttnParams& p, int64_t off_sgrp, int n_sgrp, cudaStream_t stream);
 
 // --------------------------------------------------------------------- small kernels
+// fused-norm form: also xg = bf16(h0 * g) and ss[m] = sum h0^2 (the first layer's RMSNorm inputs)
+void launch_embed_norm(const __nv_bfloat16* E, const int32_t* tok, float* h, const __nv_bfloat16* g,
+                       __nv_bfloat16* xg, float* ss, int M, int H, cudaStream_t s);
 void launch_embed(const __nv_bfloat16* E, const int32_t* tok, float* h, int M, int H,
                   cudaStream_t s);
 // y = x * rsqrt(mean(x^2) + eps) * g  (rows given by idx when idx != nullptr)
