@@ -33,7 +33,7 @@ def _queries(cfg, n, n_user, seed=7):
         items = rng.choice(5000, size=20, replace=False) + 1 + 100000 * b  # header or not: own items
         order = "UP" if b % 4 == 3 else "IP"
         qs.append(synth.make_query(seed, cfg, 100 + b, n_user + 37 * b, items, (9, 16), 8, order,
-                                   n_header=(4 if b % 2 else 0)))
+                                   n_header=(4 if b % 2 and order == "IP" else 0)))
     return qs
 
 

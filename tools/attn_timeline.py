@@ -47,6 +47,9 @@ t = np.loadtxt("gpurun_out/attn_timeline.txt").astype(np.int64)
 names = ["ld_kwait", "ld_kgot", "ld_kiss", "ld_vbwait", "ld_vbgot", "mma_top", "mma_p0", "mma_vful",
          "mma_pvdone", "mma_Skful", "mma_end", "sm0_s", "sm0_fast", "sm0_p", "sm1_s", "sm1_p",
          "sm0_16", "sm0_17", "sm0_max", "sm0_pst"]
+if os.environ.get("H64"):  # the h64 kernel's events (per 64-key half tile)
+    names = ["vfull0", "pv0iss", "s0_kwait", "s0_kgot", "-", "mma_top", "mma_p0", "mma_p1", "mma_s0", "-", "mma_end", "t0_s", "-",
+             "t0_p", "t1_s", "t1_p", "-", "-", "t0_dec", "t0_refok"]
 t0 = t[t > 0].min()
 n = int(max((t[e] > 0).sum() for e in range(t.shape[0])))
 print("tile " + " ".join(f"{nm:>10}" for nm in names))
