@@ -405,6 +405,7 @@ static StageParams stage_params(const Pool& pool, const Model& m, const Plan& pl
   sp.scratch_page_bytes = pool.geo.layer_bytes;
   sp.scratch_layer_off = 0;
   sp.head_bytes = pool.geo.head_bytes;
+  sp.n_req = static_cast<int32_t>(plan.q.size());
   return sp;
 }
 
@@ -549,6 +550,11 @@ static void run_plan(Pool& pool, Model& m, Plan& plan, float* out_hidden, cudaSt
                          gemm_ksplit(EPI_BF16_BIAS, M, m.nqkv(), H, m.num_sms, nullptr) <= 1 &&
                          gemm_ksplit(EPI_RESID_F32, M, H, nq, m.num_sms, nullptr) <= 1 &&
                          gemm_ksplit(EPI_RESID_F32, M, H, F, m.num_sms, nullptr) <= 1;
+  // a4 (RoPE + q-tile / page staging) fused into the QKV epilogue unless BAT_FUSED_STAGE=0 or the
+  // QKV projection takes the split-K path (small batches: partial sums, then stage_kernel)
+  const char* fst_e = std::getenv("BAT_FUSED_STAGE");
+  const bool fuse_stage = !(fst_e && fst_e[0] == '0') && gemm_qkv_stage_fusable(c.head_dim) &&
+                          gemm_ksplit(EPI_BF16_BIAS, M, m.nqkv(), H, m.num_sms, nullptr) <= 1;
   const int ss_parts_resid = (H + 255) / 256 * gemm_epi_col_splits();  // (N-tile, slice) partial sums
   const bool fuse_norm = fuse_ok && ss_parts_resid <= 32;                  // row_rstd loads <= 32 parts
   if (fuse_norm) ws.ss.ensure(size_t(ss_parts_resid) * M * 4, st);
@@ -583,13 +589,19 @@ static void run_plan(Pool& pool, Model& m, Plan& plan, float* out_hidden, cudaSt
       pf.end(st, BAT_K_RMSNORM, 0, 6.0 * M * H);
     }
     auto fq = gemm_fb(M, m.nqkv(), H, 2);
+    sp.pool_layer_off = int64_t(l) * pool.geo.layer_bytes;
+    if (fuse_stage) {  // a4 in the QKV epilogue: q-tiles and suffix pages written directly
+      gp.stage_on = 1;
+      gp.stage = sp;
+    }
     pf.begin(st);
     gemm(EPI_BF16_BIAS, tA_xn, Lw.t_qkv, tC_qkv, gp);
     pf.end(st, BAT_K_GEMM_QKV, fq.first, fq.second);
-    sp.pool_layer_off = int64_t(l) * pool.geo.layer_bytes;
-    pf.begin(st);
-    launch_stage(sp, st);
-    pf.end(st, BAT_K_STAGE, 0, 4.0 * M * m.nqkv());
+    if (!fuse_stage) {
+      pf.begin(st);
+      launch_stage(sp, st);
+      pf.end(st, BAT_K_STAGE, 0, 4.0 * M * m.nqkv());
+    }
     if (last && plan.entity_mode) break;  // entity prefill: only this layer's K/V are needed
     ap.pool_layer_off = int64_t(l) * pool.geo.layer_bytes;
     if (!last) {

@@ -44,7 +44,18 @@ constexpr int GROUP_M_SWIGLU_PAIR = 4;   // CTA-pair SwiGLU kernel (256-row M-ti
 // accumulator's columns).  The SwiGLU GEMM (short K = hidden, MUFU-heavy epilogue) runs 8 and
 // gains 5% over 4; the others keep 4 warps and one more ring stage (their K loops are long or
 // their epilogues light: 8 warps measured 1-4% slower there, profiles/r2_gemm_epilogue.txt)
-constexpr int epi_warps(int epi) { return epi == EPI_SWIGLU ? 8 : 4; }
+#ifndef BAT_GEMM_RESID_EW
+#define BAT_GEMM_RESID_EW 4  // epilogue warps of the fp32 residual GEMMs (O, down)
+#endif
+#ifndef BAT_GEMM_QKV_EW
+#define BAT_GEMM_QKV_EW 4  // epilogue warps of the bf16 (+bias) GEMMs (QKV)
+#endif
+constexpr int epi_warps(int epi) {
+  return epi == EPI_SWIGLU ? 8 : (epi == EPI_RESID_F32 || epi == EPI_PART_F32) ? BAT_GEMM_RESID_EW : BAT_GEMM_QKV_EW;
+}
+// staging buffers per epilogue warp: two (double-buffered TMA stores) unless 8 warps would cost a
+// ring stage; SwiGLU keeps two (its 8 warps run with one stage fewer)
+constexpr int epi_nbuf(int epi) { return (epi_warps(epi) == 8 && epi != EPI_SWIGLU) ? 1 : 2; }
 constexpr int STG_BYTES = 4096;  // per-warp epilogue staging buffer: [32 rows][128 B], 128B-swizzled
 
 constexpr int STAGE1_BYTES = A_BYTES + BN * BK * 2;  // 1-CTA kernel (128 x 256 tiles): 48 KB per stage
@@ -54,16 +65,19 @@ struct __align__(8) GemmSmemBars {
   uint64_t full[8], empty[8], tfull[2], tempty[2];
   uint32_t tmem_base;
 };
-template <int EW>
+template <int EPI>
 struct GemmCfg {
+  static constexpr int EW = epi_warps(EPI), NB = epi_nbuf(EPI);
   static constexpr int THREADS = 64 + 32 * EW;
   static constexpr int SPLIT = EW / 4;  // column slices of an accumulator
-  static constexpr int STAGES1 = EW == 8 ? 3 : 4;
+  static constexpr int STG = EW * NB * STG_BYTES;  // epilogue staging
+  static constexpr int BUDGET = 232448 - 1024 /*align slack*/ - 256 /*barriers*/ - STG;
+  static constexpr int STAGES1 = BUDGET / STAGE1_BYTES < 4 ? BUDGET / STAGE1_BYTES : 4;
   static constexpr int STG1_OFF = STAGES1 * STAGE1_BYTES;
-  static constexpr int STAGES2 = EW == 8 ? 5 : 6;
+  static constexpr int STAGES2 = BUDGET / STAGE2_BYTES < 6 ? BUDGET / STAGE2_BYTES : 6;
   static constexpr int STG2_OFF = STAGES2 * STAGE2_BYTES;
-  static constexpr size_t SMEM1 = 1024 /*align slack*/ + STG1_OFF + EW * 2 * STG_BYTES + sizeof(GemmSmemBars);
-  static constexpr size_t SMEM2 = 1024 /*align slack*/ + STG2_OFF + EW * 2 * STG_BYTES + sizeof(GemmSmemBars);
+  static constexpr size_t SMEM1 = 1024 /*align slack*/ + STG1_OFF + STG + sizeof(GemmSmemBars);
+  static constexpr size_t SMEM2 = 1024 /*align slack*/ + STG2_OFF + STG + sizeof(GemmSmemBars);
   static_assert(EW == 4 || EW == 8, "epilogue warps");
   static_assert(SMEM1 <= 232448 && SMEM2 <= 232448, "GEMM shared memory");
   static_assert(STAGES2 <= 8, "barrier array");
@@ -108,7 +122,10 @@ struct Epilogue {
   }
   __device__ __forceinline__ uint8_t* next_buf() {
     uint8_t* buf = stg + sbuf * STG_BYTES;
-    if (lane == 0) ptx::bulk_wait_read<1>();  // the group that last used this buffer is done
+    if (lane == 0) {  // the group that last used this buffer is done reading it
+      if (GemmCfg<EPI>::NB == 2) ptx::bulk_wait_read<1>();
+      else ptx::bulk_wait_read<0>();
+    }
     __syncwarp();
     return buf;
   }
@@ -123,7 +140,7 @@ struct Epilogue {
       else ptx::tma_store_2d(tmC, buf, col, row);
       ptx::bulk_commit();
     }
-    sbuf ^= 1;
+    sbuf ^= GemmCfg<EPI>::NB - 1;
   }
   // fused RMSNorm, consumer side: this lane's row scale rsqrt(mean(h^2) + eps) (1 without ss_in);
   // the partial sums are loaded together (independent loads), summed in a fixed order
@@ -187,13 +204,116 @@ struct Epilogue {
 #pragma unroll
       for (int i = 0; i < 8; ++i) hv[i] = hn[i];
     }
-    if (ok) p->ss_out[int64_t(n * GemmCfg<epi_warps(EPI)>::SPLIT + part) * p->M + row] = ss;
+    if (ok) p->ss_out[int64_t(n * GemmCfg<EPI>::SPLIT + part) * p->M + row] = ss;
+  }
+  // a4 fused (GemmParams::stage): this lane's row = one suffix token; the N-tile holds 256 / d whole
+  // heads (q, then k, then v).  Per head: (x rs) + bias, RoPE of the column pairs (c, c + d/2) at the
+  // token's plan position in fp32 (q and k), one bf16 rounding, 16-byte stores into the GQA-packed,
+  // 128B-swizzled q-tile row (token x head-in-group) or the suffix page block (K / V) — the layouts
+  // stage_kernel writes (k_misc.cu).  The row's plan lookups (request, q-tile, page) are issued
+  // before the accumulator wait (StageRow), the (cos, sin) of a column block once for all heads.
+  struct StageRow {
+    bool ok;
+    int t, pos, gq;     // token index in the request's suffix, plan position, global q-tile
+    const char* page;   // the suffix page holding the token's K / V
+  };
+  __device__ __forceinline__ StageRow stage_row(int row_in) const {
+    const StageParams& sp = p->stage;
+    StageRow r;
+    r.ok = row_in < p->M;
+    const int row = r.ok ? row_in : p->M - 1;  // lanes past the batch: same loads, no stores
+    const int32_t* img = sp.img;
+    int lo = 0, hi = sp.n_req - 1;  // the last request with token_off <= row
+    while (lo < hi) {
+      const int mid = (lo + hi + 1) >> 1;
+      if (__ldg(img + sp.off_qinfo + int64_t(mid) * 8) <= row) lo = mid;
+      else hi = mid - 1;
+    }
+    const int32_t* qi = img + sp.off_qinfo + int64_t(lo) * 8;
+    r.t = row - __ldg(qi);
+    r.pos = min(__ldg(img + sp.off_pos + row), sp.max_pos - 1);
+    r.gq = __ldg(qi + 2) + r.t / sp.qt;
+    const int target = __ldg(img + sp.off_spages + int64_t(__ldg(qi + 6) + r.t / 16) * 4 + 3);
+    r.page = target >= 0 ? sp.pool + int64_t(target) * sp.pool_page_bytes + sp.pool_layer_off
+                         : sp.scratch + int64_t(-target - 1) * sp.scratch_page_bytes + sp.scratch_layer_off;
+    return r;
+  }
+  __device__ __forceinline__ void run_stage(uint32_t tbase, int n, const StageRow& sr, float rs, int part) {
+    const StageParams& sp = p->stage;
+    const int d = sp.head_dim, half = d / 2;
+    const int nh = BN / d;  // heads of this N-tile; this warp's: [part, part + 1) * nh / SPLIT
+    constexpr int SPLIT = GemmCfg<EPI>::SPLIT;
+    const uint32_t chunks = uint32_t(sp.dpad / 64);
+    const float4* cs4 = reinterpret_cast<const float4*>(sp.rope + int64_t(sr.pos) * half);
+#pragma unroll 1
+    for (int c = 0; c < half; c += 32) {  // column pairs (c + i, c + half + i), i < 32, of every head
+      float4 rot[16];  // (cos, sin) of pairs c + 2k, c + 2k + 1
+#pragma unroll
+      for (int k = 0; k < 16; ++k) rot[k] = __ldg(cs4 + (c >> 1) + k);
+#pragma unroll 1
+      for (int hh = part * nh / SPLIT; hh < (part + 1) * nh / SPLIT; ++hh) {
+        const int head = n * nh + hh;  // 0 .. Hq-1: q, then Hkv k heads, then Hkv v heads
+        if (head >= sp.q_heads + 2 * sp.kv_heads) break;
+        const bool is_q = head < sp.q_heads;
+        const int kvi = is_q ? 0 : head - sp.q_heads;  // k: [0, Hkv), v: [Hkv, 2 Hkv)
+        const bool rope = sp.rope_enabled && kvi < sp.kv_heads;
+        const int rq = (sr.t % sp.qt) * sp.group + head % sp.group;  // q-tile row
+        char* dst = is_q ? reinterpret_cast<char*>(sp.qp) +
+                               (int64_t(sr.gq) * sp.kv_heads + head / sp.group) * (sp.dpad / 64) * 16384 + int64_t(rq) * 128
+                         : const_cast<char*>(sr.page) + (int64_t(kvi / sp.kv_heads) * sp.kv_heads + kvi % sp.kv_heads) * sp.head_bytes;
+        uint32_t a[32], b[32];
+        ptx::tmem_ld32(tbase + hh * d + c, a);
+        ptx::tmem_ld32(tbase + hh * d + half + c, b);
+        const int col = n * BN + hh * d + c;
+        const uint4* b1 = reinterpret_cast<const uint4*>(p->bias + col);
+        const uint4* b2 = reinterpret_cast<const uint4*>(p->bias + col + half);
+        ptx::tmem_ld_wait();
+        uint32_t pa[16], pb[16];
+#pragma unroll
+        for (int j = 0; j < 4; ++j) {  // 8 columns per bias vector
+          const uint4 v1 = __ldg(b1 + j), v2 = __ldg(b2 + j);
+          const uint32_t w1[4] = {v1.x, v1.y, v1.z, v1.w}, w2[4] = {v2.x, v2.y, v2.z, v2.w};
+#pragma unroll
+          for (int k = 0; k < 4; ++k) {
+            const int i = 8 * j + 2 * k;
+            const float2 g1 = __bfloat1622float2(*reinterpret_cast<const __nv_bfloat162*>(&w1[k]));
+            const float2 g2 = __bfloat1622float2(*reinterpret_cast<const __nv_bfloat162*>(&w2[k]));
+            float x10 = fmaf(__uint_as_float(a[i]), rs, g1.x), x11 = fmaf(__uint_as_float(a[i + 1]), rs, g1.y);
+            float x20 = fmaf(__uint_as_float(b[i]), rs, g2.x), x21 = fmaf(__uint_as_float(b[i + 1]), rs, g2.y);
+            if (rope) {
+              const float4 t4 = rot[i >> 1];
+              const float o10 = x10 * t4.x - x20 * t4.y, o20 = x20 * t4.x + x10 * t4.y;
+              const float o11 = x11 * t4.z - x21 * t4.w, o21 = x21 * t4.z + x11 * t4.w;
+              x10 = o10; x20 = o20; x11 = o11; x21 = o21;
+            }
+            pa[i / 2] = ptx::pack_bf16x2(x10, x11);
+            pb[i / 2] = ptx::pack_bf16x2(x20, x21);
+          }
+        }
+        if (sr.ok) {
+#pragma unroll
+          for (int j = 0; j < 4; ++j) {  // 8-column chunks of the two column ranges
+            const int c1 = c + 8 * j, c2 = c + half + 8 * j;
+            uint32_t o1, o2;
+            if (is_q) {
+              o1 = (c1 >> 6) * 16384 + ((((c1 & 63) >> 3) ^ (uint32_t(rq) & 7u)) << 4);
+              o2 = (c2 >> 6) * 16384 + ((((c2 & 63) >> 3) ^ (uint32_t(rq) & 7u)) << 4);
+            } else {
+              o1 = ptx::page_blk_off(uint32_t(sr.t % 16), uint32_t(c1), chunks);
+              o2 = ptx::page_blk_off(uint32_t(sr.t % 16), uint32_t(c2), chunks);
+            }
+            *reinterpret_cast<uint4*>(dst + o1) = make_uint4(pa[4 * j], pa[4 * j + 1], pa[4 * j + 2], pa[4 * j + 3]);
+            *reinterpret_cast<uint4*>(dst + o2) = make_uint4(pb[4 * j], pb[4 * j + 1], pb[4 * j + 2], pb[4 * j + 3]);
+          }
+        }
+      }
+    }
   }
   // tbase: TMEM address of this warp's lanes, column 0 of the accumulator; n: output N-tile;
   // part: this warp's column slice of the accumulator (EPI_SPLIT slices); rs: the row's fused-norm
   // scale (row_rstd, loaded before the accumulator wait)
   __device__ __forceinline__ void run(uint32_t tbase, int n, int row0, int part, float rs) {
-    constexpr int W = BN / GemmCfg<epi_warps(EPI)>::SPLIT;  // accumulator columns per slice
+    constexpr int W = BN / GemmCfg<EPI>::SPLIT;  // accumulator columns per slice
     const int c_lo = part * W, c_hi = c_lo + W;
     if constexpr (EPI == EPI_RESID_F32) {
       if (p->norm_g) {
@@ -201,6 +321,7 @@ struct Epilogue {
         return;
       }
     }
+
     if constexpr (EPI == EPI_SWIGLU) {
 #pragma unroll 1
       for (int c = c_lo / 2; c < c_hi / 2; c += 64) {  // 64 output columns per staging buffer
@@ -271,16 +392,16 @@ __device__ __forceinline__ int b_row(const GemmParams& p, int n, int h) {
 
 // ------------------------------------------------------------------- 1-CTA, 128 x 256 tiles
 template <int EPI>
-__global__ void __launch_bounds__(GemmCfg<epi_warps(EPI)>::THREADS, 1)
+__global__ void __launch_bounds__(GemmCfg<EPI>::THREADS, 1)
 gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
                const __grid_constant__ CUtensorMap tmC, GemmParams p) {
   extern __shared__ uint8_t smem_raw[];
   // 1 KB-align by offsetting the __shared__ array itself (keeps the shared address space, so
   // the compiler emits LDS/STS rather than generic loads and stores)
   uint8_t* smem = smem_raw + ((1024u - (ptx::smem_u32(smem_raw) & 1023u)) & 1023u);
-  using C = GemmCfg<epi_warps(EPI)>;
-  constexpr int STAGES1 = C::STAGES1, STG1_OFF = C::STG1_OFF, EPI_WARPS = epi_warps(EPI);
-  GemmSmemBars* bars = reinterpret_cast<GemmSmemBars*>(smem + STG1_OFF + EPI_WARPS * 2 * STG_BYTES);
+  using C = GemmCfg<EPI>;
+  constexpr int STAGES1 = C::STAGES1, STG1_OFF = C::STG1_OFF, EPI_WARPS = C::EW;
+  GemmSmemBars* bars = reinterpret_cast<GemmSmemBars*>(smem + STG1_OFF + C::STG);
   const uint32_t warp = ptx::warp_id(), lane = ptx::lane_id();
   constexpr uint32_t IDESC = ptx::idesc_bf16(128, BN, 0, 0);
 
@@ -370,7 +491,7 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
   } else {  // ------------------------------ epilogue warps 2 .. 1 + EPI_WARPS
     const uint32_t sub = warp & 3;  // TMEM sub-partition this warp may access
     const int part = int(warp - 2) / 4;  // column slice
-    Epilogue<EPI> epi{&tmC, &p, smem + STG1_OFF + (warp - 2) * 2 * STG_BYTES, lane};
+    Epilogue<EPI> epi{&tmC, &p, smem + STG1_OFF + (warp - 2) * C::NB * STG_BYTES, lane};
     int acc = 0;
     uint32_t acc_phase = 0;
     for (int t = blockIdx.x; t < num_work; t += gridDim.x) {
@@ -379,9 +500,21 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
       const int slab = EPI == EPI_PART_F32 ? (t / num_tiles) * p.mpad : 0;
       const int row0 = slab + m * 128 + int(sub) * 32;
       const float rs = (EPI == EPI_SWIGLU || EPI == EPI_BF16_BIAS) ? epi.row_rstd(row0 + int(lane)) : 1.0f;
-      ptx::mbar_wait(&bars->tfull[acc], acc_phase);
-      ptx::tc_fence_after();
-      epi.run(tmem + ((sub * 32) << 16) + acc * BN, n, row0, part, rs);
+      bool staged = false;
+      if constexpr (EPI == EPI_BF16_BIAS) {
+        if (p.stage_on) {  // a4 fused: the row's plan lookups overlap the accumulator wait
+          const auto sr = epi.stage_row(row0 + int(lane));
+          ptx::mbar_wait(&bars->tfull[acc], acc_phase);
+          ptx::tc_fence_after();
+          epi.run_stage(tmem + ((sub * 32) << 16) + acc * BN, n, sr, rs, part);
+          staged = true;
+        }
+      }
+      if (!staged) {
+        ptx::mbar_wait(&bars->tfull[acc], acc_phase);
+        ptx::tc_fence_after();
+        epi.run(tmem + ((sub * 32) << 16) + acc * BN, n, row0, part, rs);
+      }
       ptx::tc_fence_before();
       __syncwarp();
       if (lane == 0) ptx::mbar_arrive(&bars->tempty[acc]);
@@ -397,14 +530,14 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
 
 // ------------------------------------------------------------ CTA pair, 256 x 256 tiles
 template <int EPI>
-__global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(GemmCfg<epi_warps(EPI)>::THREADS, 1)
+__global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(GemmCfg<EPI>::THREADS, 1)
 gemm2_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
                 const __grid_constant__ CUtensorMap tmC, GemmParams p) {
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = smem_raw + ((1024u - (ptx::smem_u32(smem_raw) & 1023u)) & 1023u);
-  using C = GemmCfg<epi_warps(EPI)>;
-  constexpr int STAGES2 = C::STAGES2, STG2_OFF = C::STG2_OFF, EPI_WARPS = epi_warps(EPI);
-  GemmSmemBars* bars = reinterpret_cast<GemmSmemBars*>(smem + STG2_OFF + EPI_WARPS * 2 * STG_BYTES);
+  using C = GemmCfg<EPI>;
+  constexpr int STAGES2 = C::STAGES2, STG2_OFF = C::STG2_OFF, EPI_WARPS = C::EW;
+  GemmSmemBars* bars = reinterpret_cast<GemmSmemBars*>(smem + STG2_OFF + C::STG);
   const uint32_t warp = ptx::warp_id(), lane = ptx::lane_id();
   const uint32_t rank = ptx::cluster_ctarank();  // 0 = leader (issues the pair MMAs)
   constexpr uint32_t IDESC = ptx::idesc_bf16(256, BN, 0, 0);
@@ -495,7 +628,7 @@ gemm2_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__
   } else {  // ------------------------------ epilogue warps (both CTAs): my 128 rows
     const uint32_t sub = warp & 3;
     const int part = int(warp - 2) / 4;  // column slice
-    Epilogue<EPI> epi{&tmC, &p, smem + STG2_OFF + (warp - 2) * 2 * STG_BYTES, lane};
+    Epilogue<EPI> epi{&tmC, &p, smem + STG2_OFF + (warp - 2) * C::NB * STG_BYTES, lane};
     int acc = 0;
     uint32_t acc_phase = 0;
     for (int t = pair; t < num_work; t += n_pairs) {
@@ -504,9 +637,21 @@ gemm2_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__
       const int slab = EPI == EPI_PART_F32 ? (t / num_tiles) * p.mpad : 0;
       const int row0 = slab + m * 256 + int(rank) * 128 + int(sub) * 32;
       const float rs = (EPI == EPI_SWIGLU || EPI == EPI_BF16_BIAS) ? epi.row_rstd(row0 + int(lane)) : 1.0f;
-      ptx::mbar_wait(&bars->tfull[acc], acc_phase);
-      ptx::tc_fence_after();
-      epi.run(tmem + ((sub * 32) << 16) + acc * BN, n, row0, part, rs);
+      bool staged = false;
+      if constexpr (EPI == EPI_BF16_BIAS) {
+        if (p.stage_on) {  // a4 fused: the row's plan lookups overlap the accumulator wait
+          const auto sr = epi.stage_row(row0 + int(lane));
+          ptx::mbar_wait(&bars->tfull[acc], acc_phase);
+          ptx::tc_fence_after();
+          epi.run_stage(tmem + ((sub * 32) << 16) + acc * BN, n, sr, rs, part);
+          staged = true;
+        }
+      }
+      if (!staged) {
+        ptx::mbar_wait(&bars->tfull[acc], acc_phase);
+        ptx::tc_fence_after();
+        epi.run(tmem + ((sub * 32) << 16) + acc * BN, n, row0, part, rs);
+      }
       ptx::tc_fence_before();
       __syncwarp();
       if (lane == 0) ptx::mbar_arrive_cluster(ptx::mapa(ptx::smem_u32(&bars->tempty[acc]), 0));
@@ -523,11 +668,21 @@ gemm2_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__
 
 }  // namespace
 
-int gemm_epi_col_splits() { return GemmCfg<epi_warps(EPI_RESID_F32)>::SPLIT; }
+bool gemm_qkv_stage_fusable(int head_dim) {
+  // whole heads per epilogue warp, 32-column blocks of each half head
+  return head_dim % 64 == 0 && (BN / head_dim) % GemmCfg<EPI_BF16_BIAS>::SPLIT == 0;
+}
+
+int gemm_epi_col_splits() { return GemmCfg<EPI_RESID_F32>::SPLIT; }
 
 size_t gemm_smem_bytes() {
-  const size_t a = std::max(GemmCfg<4>::SMEM1, GemmCfg<4>::SMEM2), b = std::max(GemmCfg<8>::SMEM1, GemmCfg<8>::SMEM2);
-  return std::max(a, b);
+  size_t m = 0;
+  for (size_t v : {GemmCfg<EPI_BF16>::SMEM1, GemmCfg<EPI_BF16>::SMEM2, GemmCfg<EPI_BF16_BIAS>::SMEM1,
+                   GemmCfg<EPI_BF16_BIAS>::SMEM2, GemmCfg<EPI_RESID_F32>::SMEM1, GemmCfg<EPI_RESID_F32>::SMEM2,
+                   GemmCfg<EPI_SWIGLU>::SMEM1, GemmCfg<EPI_SWIGLU>::SMEM2, GemmCfg<EPI_PART_F32>::SMEM1,
+                   GemmCfg<EPI_PART_F32>::SMEM2})
+    m = std::max(m, v);
+  return m;
 }
 
 static int env_group(const char* name) {
@@ -565,11 +720,11 @@ void launch_gemm(int epi, const CUtensorMap& tmA, const CUtensorMap& tmB, const 
       kern<<<2 * pairs, C::THREADS, C::SMEM2, stream>>>(tmA, tmB, tmC, p);
     };
     switch (epi) {
-      case EPI_BF16: launch(gemm2_tc_kernel<EPI_BF16>, GemmCfg<epi_warps(EPI_BF16)>{}); break;
-      case EPI_BF16_BIAS: launch(gemm2_tc_kernel<EPI_BF16_BIAS>, GemmCfg<epi_warps(EPI_BF16_BIAS)>{}); break;
-      case EPI_RESID_F32: launch(gemm2_tc_kernel<EPI_RESID_F32>, GemmCfg<epi_warps(EPI_RESID_F32)>{}); break;
-      case EPI_SWIGLU: launch(gemm2_tc_kernel<EPI_SWIGLU>, GemmCfg<epi_warps(EPI_SWIGLU)>{}); break;
-      case EPI_PART_F32: launch(gemm2_tc_kernel<EPI_PART_F32>, GemmCfg<epi_warps(EPI_PART_F32)>{}); break;
+      case EPI_BF16: launch(gemm2_tc_kernel<EPI_BF16>, GemmCfg<EPI_BF16>{}); break;
+      case EPI_BF16_BIAS: launch(gemm2_tc_kernel<EPI_BF16_BIAS>, GemmCfg<EPI_BF16_BIAS>{}); break;
+      case EPI_RESID_F32: launch(gemm2_tc_kernel<EPI_RESID_F32>, GemmCfg<EPI_RESID_F32>{}); break;
+      case EPI_SWIGLU: launch(gemm2_tc_kernel<EPI_SWIGLU>, GemmCfg<EPI_SWIGLU>{}); break;
+      case EPI_PART_F32: launch(gemm2_tc_kernel<EPI_PART_F32>, GemmCfg<EPI_PART_F32>{}); break;
     }
   } else {
     const int tiles = ((p.M + 127) / 128) * n_tiles * ks;
@@ -581,11 +736,11 @@ void launch_gemm(int epi, const CUtensorMap& tmA, const CUtensorMap& tmB, const 
       kern<<<grid, C::THREADS, C::SMEM1, stream>>>(tmA, tmB, tmC, p);
     };
     switch (epi) {
-      case EPI_BF16: launch(gemm_tc_kernel<EPI_BF16>, GemmCfg<epi_warps(EPI_BF16)>{}); break;
-      case EPI_BF16_BIAS: launch(gemm_tc_kernel<EPI_BF16_BIAS>, GemmCfg<epi_warps(EPI_BF16_BIAS)>{}); break;
-      case EPI_RESID_F32: launch(gemm_tc_kernel<EPI_RESID_F32>, GemmCfg<epi_warps(EPI_RESID_F32)>{}); break;
-      case EPI_SWIGLU: launch(gemm_tc_kernel<EPI_SWIGLU>, GemmCfg<epi_warps(EPI_SWIGLU)>{}); break;
-      case EPI_PART_F32: launch(gemm_tc_kernel<EPI_PART_F32>, GemmCfg<epi_warps(EPI_PART_F32)>{}); break;
+      case EPI_BF16: launch(gemm_tc_kernel<EPI_BF16>, GemmCfg<EPI_BF16>{}); break;
+      case EPI_BF16_BIAS: launch(gemm_tc_kernel<EPI_BF16_BIAS>, GemmCfg<EPI_BF16_BIAS>{}); break;
+      case EPI_RESID_F32: launch(gemm_tc_kernel<EPI_RESID_F32>, GemmCfg<EPI_RESID_F32>{}); break;
+      case EPI_SWIGLU: launch(gemm_tc_kernel<EPI_SWIGLU>, GemmCfg<EPI_SWIGLU>{}); break;
+      case EPI_PART_F32: launch(gemm_tc_kernel<EPI_PART_F32>, GemmCfg<EPI_PART_F32>{}); break;
     }
   }
   count_launch();

@@ -20,6 +20,25 @@ inline void set_smem_attr(K* kern, size_t bytes) {
   set_smem_attr_raw(reinterpret_cast<const void*>(kern), static_cast<int>(bytes));
 }
 
+// a4 staging parameters (RoPE + q-tile / suffix-page layout), shared by stage_kernel and the
+// QKV GEMM epilogue that fuses it (GemmParams::stage)
+struct StageParams {
+  const __nv_bfloat16* qkv;  // [M][(Hq+2Hkv)*d]
+  const int32_t* img;
+  int64_t off_pos, off_qinfo, off_qtiles, off_spages;
+  int32_t n_qtiles, n_spages;
+  const float2* rope;        // [max_pos][d/2] (cos, sin)
+  int32_t rope_enabled, max_pos;
+  int32_t q_heads, kv_heads, head_dim, dpad, group, qt;
+  __nv_bfloat16* qp;         // q-tiles out
+  char* pool;                // target pages: pool page p (>= 0) or scratch page s (-(s+1))
+  int64_t pool_page_bytes, pool_layer_off;
+  char* scratch;
+  int64_t scratch_page_bytes, scratch_layer_off;
+  int64_t head_bytes;
+  int32_t n_req;             // requests of the plan (q_info rows)
+};
+
 // ------------------------------------------------------------------------ tcgen05 GEMM
 enum GemmEpi { EPI_BF16 = 0, EPI_BF16_BIAS = 1, EPI_RESID_F32 = 2, EPI_SWIGLU = 3, EPI_PART_F32 = 4 };
 struct GemmParams {
@@ -45,6 +64,11 @@ struct GemmParams {
   int ss_parts = 0;
   int norm_h = 0;
   float eps = 0.0f;
+  // a4 fused into the QKV epilogue (EPI_BF16_BIAS, stage_on): each row's q / k / v heads are
+  // rotated (RoPE at the plan position) in fp32 and written straight into the q-tiles and suffix
+  // pages; the qkv activation is never stored
+  int stage_on = 0;
+  StageParams stage{};
 };
 // Split-K for grids that would leave SMs idle (small M: batch-1 requests, the last layer's
 // discriminant rows): slices per tile (1 = no split) for a GEMM of this shape and the row pitch of
@@ -56,6 +80,8 @@ void launch_gemm_reduce(const float* part, int ksplit, int mpad, int M, int N, v
 size_t gemm_smem_bytes();
 // column slices per accumulator in the epilogue (fused-norm partial sums per N-tile)
 int gemm_epi_col_splits();
+// the QKV epilogue can run a4 (one warp per TMEM lane quarter holds whole rows of a head)
+bool gemm_qkv_stage_fusable(int head_dim);
 // tmC: output tensor map — bf16 [M][ldo] with box {64, 32} (EPI_BF16*, EPI_SWIGLU) or fp32
 // [M][ldo] with box {32, 32} (EPI_RESID_F32, TMA reduce-add), 128-byte swizzle
 void launch_gemm(int epi, const CUtensorMap& tmA, const CUtensorMap& tmB, const CUtensorMap& tmC,
@@ -113,21 +139,6 @@ void launch_rmsnorm_f32out(const float* x, const __nv_bfloat16* g, float* y, int
                            float eps, cudaStream_t s);
 void launch_rope_table(float2* tab, int max_pos, int d, double theta, cudaStream_t s);
 
-struct StageParams {
-  const __nv_bfloat16* qkv;  // [M][(Hq+2Hkv)*d]
-  const int32_t* img;
-  int64_t off_pos, off_qinfo, off_qtiles, off_spages;
-  int32_t n_qtiles, n_spages;
-  const float2* rope;        // [max_pos][d/2] (cos, sin)
-  int32_t rope_enabled, max_pos;
-  int32_t q_heads, kv_heads, head_dim, dpad, group, qt;
-  __nv_bfloat16* qp;         // q-tiles out
-  char* pool;                // target pages: pool page p (>= 0) or scratch page s (-(s+1))
-  int64_t pool_page_bytes, pool_layer_off;
-  char* scratch;
-  int64_t scratch_page_bytes, scratch_layer_off;
-  int64_t head_bytes;
-};
 void launch_stage(const StageParams& p, cudaStream_t s);
 
 void launch_gather_rows_bf16(const __nv_bfloat16* src, const int32_t* idx, __nv_bfloat16* dst,

@@ -1,9 +1,11 @@
-"""RMSNorm fused across the residual updates (a3 / a7): at batch sizes where no
+"""Fused epilogues.  (1) RMSNorm fused across the residual updates (a3 / a7): at batch sizes where no
 projection takes the split-K path, the O and down GEMMs write h_new = h + acc, xg = bf16(h_new * g)
 and per-N-tile sums of squares, and the QKV / gate-up GEMMs scale their rows by
 rsqrt(mean(h^2) + eps) — the standalone norm kernel is not launched.  Both paths are checked
 against the fp64 oracle's full recompute (2e-2 abs/rel on hf, z, s; R11) and against
-each other; the launch count proves which path ran (2L - 1 norm launches fewer when fused)."""
+each other; the launch count proves which path ran (2L - 1 norm launches fewer when fused).
+(2) a4 (RoPE + q-tile / suffix-page staging) fused into the QKV GEMM epilogue (default for batches
+whose QKV projection is not split-K): the same checks, L stage launches fewer."""
 import os
 
 import numpy as np
@@ -37,13 +39,13 @@ def _queries(cfg, n, n_user, seed=7):
     return qs
 
 
-def _prefill(B, cfg, W, model, queries, fused):
+def _prefill(B, cfg, W, model, queries, fused, var="BAT_FUSED_NORM"):
     from paper_conf_asplos_0017wzlxszh0w26_b200.runtime import DevicePool, prefill_missing_entities
     pool = DevicePool(cfg, 8192)
     prefill_missing_entities(pool, model, queries)
     hidden = torch.empty(len(queries), cfg["hidden"], device="cuda")
-    old = os.environ.get("BAT_FUSED_NORM")
-    os.environ["BAT_FUSED_NORM"] = "1" if fused else "0"
+    old = os.environ.get(var)
+    os.environ[var] = "1" if fused else "0"
     try:
         torch.cuda.synchronize()
         n0 = B.bat_kernel_launch_count()
@@ -52,9 +54,9 @@ def _prefill(B, cfg, W, model, queries, fused):
         n = B.bat_kernel_launch_count() - n0
     finally:
         if old is None:
-            del os.environ["BAT_FUSED_NORM"]
+            del os.environ[var]
         else:
-            os.environ["BAT_FUSED_NORM"] = old
+            os.environ[var] = old
     pool.close()
     return hidden.double().cpu().numpy(), n
 
@@ -95,4 +97,27 @@ def test_small_batch_keeps_standalone_norm(B):
     assert np.array_equal(hf_f, hf_u)
     ref = om.run_query(cfg, W, qs[0], "full", k=1)
     assert max_excess(hf_f[0], ref["hf"]) <= 0.0
+    model.close()
+
+
+@pytest.mark.parametrize("cfg_name", ["small", "small7", "small64"])
+def test_fused_stage_matches_oracle_and_unfused(B, cfg_name):
+    """QKV epilogue staging (bias + RoPE in fp32, one bf16 rounding, q-tile / page stores) vs
+    the separate stage kernel (bf16 qkv, then RoPE): both within the oracle tolerance, each other
+    at 1e-2, and exactly L stage launches apart.  small7: 11 heads of 128 (a half-empty last
+    N-tile); small64: d = 64 (four heads per N-tile)."""
+    from paper_conf_asplos_0017wzlxszh0w26_b200.runtime import DeviceModel
+    cfg = synth.model_config(cfg_name)
+    W = synth.Weights(cfg, seed=5)
+    model = DeviceModel(cfg, W)
+    qs = _queries(cfg, 10, 420, seed=11)
+    hf_f, n_f = _prefill(B, cfg, W, model, qs, True, "BAT_FUSED_STAGE")
+    hf_u, n_u = _prefill(B, cfg, W, model, qs, False, "BAT_FUSED_STAGE")
+    assert n_u - n_f == cfg["layers"], (n_u, n_f)
+    assert max_excess(hf_f, hf_u, atol=1e-2, rtol=1e-2) <= 0.0
+    worst = -1.0
+    for b, q in enumerate(qs):
+        ref = om.run_query(cfg, W, q, "full", k=1)
+        worst = max(worst, max_excess(hf_f[b], ref["hf"]), max_excess(hf_u[b], ref["hf"]))
+    assert worst <= 0.0, worst
     model.close()
