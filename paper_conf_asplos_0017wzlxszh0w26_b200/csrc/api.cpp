@@ -540,12 +540,14 @@ static void run_plan(Pool& pool, Model& m, Plan& plan, float* out_hidden, cudaSt
                        epi == EPI_BF16_BIAS ? gp.bias : nullptr, epi == EPI_RESID_F32 ? 0 : 1, st);
   };
 
-  // RMSNorm fused across the residual updates (GemmParams::norm_g / ss_in; opt-in BAT_FUSED_NORM=1,
-  // large batches only: no projection of a full-row layer on the split-K path).  Measured in the
-  // configs[2] step it is a net loss (the O GEMM's epilogue, short K, slows by more than the 8 ms
-  // of norm passes it removes: profiles/r2_gemm_epilogue.txt), so the standalone norm is the default
-  const char* fuse_e = std::getenv("BAT_FUSED_NORM");  // read per call: tests A/B both paths
-  const bool fuse_env = fuse_e && fuse_e[0] == '1';
+  // RMSNorm fused across the residual updates (GemmParams::norm_g / ss_in; large batches only: no
+  // projection of a full-row layer on the split-K path).  BAT_FUSED_NORM=d: the attention-block
+  // norm (ln1) rides on the down GEMM's epilogue (long K: slack to absorb it) and the embedding;
+  // =1: also ln2 on the O GEMM (short K: its epilogue becomes the bottleneck, a net loss,
+  // profiles/r2_gemm_epilogue.txt); =0: standalone norm kernels
+  const char* fuse_e = std::getenv("BAT_FUSED_NORM");  // read per call: tests A/B the paths
+  const char fuse_mode = fuse_e ? fuse_e[0] : '0';
+  const bool fuse_env = fuse_mode == '1' || fuse_mode == 'd';
   const bool fuse_ok = fuse_env && (H % 32) == 0 &&
                          gemm_ksplit(EPI_BF16_BIAS, M, m.nqkv(), H, m.num_sms, nullptr) <= 1 &&
                          gemm_ksplit(EPI_RESID_F32, M, H, nq, m.num_sms, nullptr) <= 1 &&
@@ -557,6 +559,7 @@ static void run_plan(Pool& pool, Model& m, Plan& plan, float* out_hidden, cudaSt
                           gemm_ksplit(EPI_BF16_BIAS, M, m.nqkv(), H, m.num_sms, nullptr) <= 1;
   const int ss_parts_resid = (H + 255) / 256 * gemm_epi_col_splits();  // (N-tile, slice) partial sums
   const bool fuse_norm = fuse_ok && ss_parts_resid <= 32;                  // row_rstd loads <= 32 parts
+  const bool fuse_norm2 = fuse_norm && fuse_mode == '1';                   // ln2 through the O GEMM too
   if (fuse_norm) ws.ss.ensure(size_t(ss_parts_resid) * M * 4, st);
   auto set_norm_out = [&](GemmParams& g, const __nv_bfloat16* gnext) {  // producer: h += .., xn, ss
     g.norm_g = gnext;
@@ -632,13 +635,13 @@ static void run_plan(Pool& pool, Model& m, Plan& plan, float* out_hidden, cudaSt
         cudaFree(dbi);
       }
       GemmParams go{M, H, nq, ws.h.p, H, nullptr, 0};
-      if (fuse_norm) set_norm_out(go, Lw.ln2);
-      auto fo = gemm_fb(M, H, nq, fuse_norm ? 10 : 8);
+      if (fuse_norm2) set_norm_out(go, Lw.ln2);
+      auto fo = gemm_fb(M, H, nq, fuse_norm2 ? 10 : 8);
       pf.begin(st);
       gemm(EPI_RESID_F32, tA_o, Lw.t_o, tC_h, go);
       pf.end(st, BAT_K_GEMM_O, fo.first, fo.second);
       GemmParams gg{M, F, H, ws.act.p, F, nullptr, F};
-      if (fuse_norm) {
+      if (fuse_norm2) {
         set_norm_in(gg, ss_parts_resid);
       } else {
         pf.begin(st);

@@ -50,7 +50,7 @@ def launches(tag):
     out = [f"# ncu launch list ({tag}): {os.environ.get('NCU_CMD', 'bench.py --steps 2 --warmup 1')}, timed region only",
            "# (--profile-from-start off; --metrics gpu__time_duration.sum --clock-control none).  Per-launch times",
            "# are cold-cache and serialised: compare SHARES with bench.py's live CUDA-event kernel table.",
-           f"# raw unit {sorted(unit)}; workload: {os.environ.get('NCU_WORKLOAD', 'configs[1] IP batch 64')}",
+           f"# raw unit {sorted(unit)}; workload: {os.environ.get('NCU_WORKLOAD', 'configs[2] batch 64 (bench.py default)')}",
            f"{'kernel':40s} {'launches':>9s} {'total_ms':>10s} {'share':>7s}"]
     for k, (n, t) in sorted(tot.items(), key=lambda kv: -kv[1][1]):
         out.append(f"{k:40s} {n:9d} {t:10.3f} {100 * t / total:6.1f}%")
