@@ -541,12 +541,13 @@ static void run_plan(Pool& pool, Model& m, Plan& plan, float* out_hidden, cudaSt
   };
 
   // RMSNorm fused across the residual updates (GemmParams::norm_g / ss_in; large batches only: no
-  // projection of a full-row layer on the split-K path).  BAT_FUSED_NORM=d: the attention-block
-  // norm (ln1) rides on the down GEMM's epilogue (long K: slack to absorb it) and the embedding;
-  // =1: also ln2 on the O GEMM (short K: its epilogue becomes the bottleneck, a net loss,
-  // profiles/r2_gemm_epilogue.txt); =0: standalone norm kernels
+  // projection of a full-row layer on the split-K path).  Default (BAT_FUSED_NORM=d): the
+  // attention-block norm (ln1) rides on the down GEMM's epilogue (long K: slack to absorb it) and
+  // the embedding, the MLP norm (ln2) stays a kernel; =1: ln2 on the O GEMM too (short K: its
+  // epilogue becomes the bottleneck, a net loss); =0: standalone norm kernels
+  // (profiles/r2_gemm_epilogue.txt)
   const char* fuse_e = std::getenv("BAT_FUSED_NORM");  // read per call: tests A/B the paths
-  const char fuse_mode = fuse_e ? fuse_e[0] : '0';
+  const char fuse_mode = fuse_e ? fuse_e[0] : 'd';
   const bool fuse_env = fuse_mode == '1' || fuse_mode == 'd';
   const bool fuse_ok = fuse_env && (H % 32) == 0 &&
                          gemm_ksplit(EPI_BF16_BIAS, M, m.nqkv(), H, m.num_sms, nullptr) <= 1 &&

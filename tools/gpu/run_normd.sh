@@ -12,3 +12,7 @@ for rep in 1 2 3; do
   run none_$rep BAT_FUSED_NORM=0
   run d_$rep BAT_FUSED_NORM=d
 done
+for rep in 1 2; do
+  run g16_$rep BAT_GEMM_GROUP_SWIGLU=16
+  run g1_$rep BAT_GEMM_GROUP_SWIGLU=1
+done
