@@ -157,23 +157,32 @@ struct Epilogue {
   // fused RMSNorm, producer side (EPI_RESID_F32 with norm_g): h_new = h + acc for this lane's row,
   // 32 columns per chunk; h_old is read directly (128 B per lane, one chunk ahead), h_new leaves
   // through the swizzled staging buffer and a TMA store, xg = bf16(h_new * g) with 16-byte stores
+  // h_old of this lane's row, PD 32-column chunks ahead (the first PD issued before the
+  // accumulator wait: resid_prefetch), so ~PD x 4 KB per warp are in flight against DRAM latency
+  static constexpr int PD = 4;
+  static constexpr int NCHK = BN / GemmCfg<EPI>::SPLIT / 32;  // chunks of this warp's column slice
+  float4 hpre[PD][8];
+  __device__ __forceinline__ void load_h_chunk(int row, int col, float4 (&dst)[8]) {
+    const bool ok = row < p->M && col < p->N;
+    const float4* src = reinterpret_cast<const float4*>(static_cast<const float*>(p->out) +
+                                                        int64_t(ok ? row : 0) * p->ldo + (ok ? col : 0));
+#pragma unroll
+    for (int i = 0; i < 8; ++i) dst[i] = ok ? __ldcs(src + i) : make_float4(0.f, 0.f, 0.f, 0.f);
+  }
+  __device__ __forceinline__ void resid_prefetch(int row0, int n, int part) {
+    const int c_lo = part * (BN / GemmCfg<EPI>::SPLIT);
+#pragma unroll
+    for (int k = 0; k < PD && k < NCHK; ++k) load_h_chunk(row0 + int(lane), n * BN + c_lo + 32 * k, hpre[k]);
+  }
   __device__ __forceinline__ void run_resid_norm(uint32_t tbase, int n, int row0, int c_lo, int c_hi, int part) {
     const int row = row0 + int(lane);
     const bool ok = row < p->M;
     const int col_base = n * BN;
-    const float* hrow = static_cast<const float*>(p->out) + int64_t(ok ? row : 0) * p->ldo;
-    float4 hv[8], hn[8];
-    auto load_h = [&](int c, float4 (&dst)[8]) {
-#pragma unroll
-      for (int i = 0; i < 8; ++i)
-        dst[i] = ok && col_base + c < p->N ? __ldcs(reinterpret_cast<const float4*>(hrow + col_base + c) + i)
-                                           : make_float4(0.f, 0.f, 0.f, 0.f);
-    };
-    load_h(c_lo, hv);
     float ss = 0.0f;
-#pragma unroll 1
-    for (int c = c_lo; c < c_hi; c += 32) {
-      if (c + 32 < c_hi) load_h(c + 32, hn);
+#pragma unroll
+    for (int k = 0; k < NCHK; ++k) {
+      const int c = c_lo + 32 * k;
+      float4 (&hv)[8] = hpre[k % PD];
       uint8_t* buf = next_buf();
       uint32_t r[32];
       ptx::tmem_ld32(tbase + c, r);
@@ -195,15 +204,15 @@ struct Epilogue {
         pk[2 * j] = ptx::pack_bf16x2(v0 * g01.x, v1 * g01.y);
         pk[2 * j + 1] = ptx::pack_bf16x2(v2 * g23.x, v3 * g23.y);
       }
+      if (k + PD < NCHK) load_h_chunk(row, col + 32 * PD, hv);  // refill the slot PD chunks ahead
       if (ok && col < p->N) {
         uint4* xd = reinterpret_cast<uint4*>(p->xg_out + int64_t(row) * p->norm_h + col);
 #pragma unroll
         for (int i = 0; i < 4; ++i) xd[i] = make_uint4(pk[4 * i], pk[4 * i + 1], pk[4 * i + 2], pk[4 * i + 3]);
       }
       flush(buf, col, row0);
-#pragma unroll
-      for (int i = 0; i < 8; ++i) hv[i] = hn[i];
     }
+    (void)c_hi;
     if (ok) p->ss_out[int64_t(n * GemmCfg<EPI>::SPLIT + part) * p->M + row] = ss;
   }
   // a4 fused (GemmParams::stage): this lane's row = one suffix token; the N-tile holds 256 / d whole
@@ -500,6 +509,9 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
       const int slab = EPI == EPI_PART_F32 ? (t / num_tiles) * p.mpad : 0;
       const int row0 = slab + m * 128 + int(sub) * 32;
       const float rs = (EPI == EPI_SWIGLU || EPI == EPI_BF16_BIAS) ? epi.row_rstd(row0 + int(lane)) : 1.0f;
+      if constexpr (EPI == EPI_RESID_F32) {
+        if (p.norm_g) epi.resid_prefetch(row0, n, part);  // h_old in flight during the accumulator wait
+      }
       bool staged = false;
       if constexpr (EPI == EPI_BF16_BIAS) {
         if (p.stage_on) {  // a4 fused: the row's plan lookups overlap the accumulator wait
@@ -637,6 +649,9 @@ gemm2_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__
       const int slab = EPI == EPI_PART_F32 ? (t / num_tiles) * p.mpad : 0;
       const int row0 = slab + m * 256 + int(rank) * 128 + int(sub) * 32;
       const float rs = (EPI == EPI_SWIGLU || EPI == EPI_BF16_BIAS) ? epi.row_rstd(row0 + int(lane)) : 1.0f;
+      if constexpr (EPI == EPI_RESID_F32) {
+        if (p.norm_g) epi.resid_prefetch(row0, n, part);  // h_old in flight during the accumulator wait
+      }
       bool staged = false;
       if constexpr (EPI == EPI_BF16_BIAS) {
         if (p.stage_on) {  // a4 fused: the row's plan lookups overlap the accumulator wait
