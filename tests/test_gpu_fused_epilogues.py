@@ -122,3 +122,50 @@ def test_fused_stage_matches_oracle_and_unfused(B, cfg_name):
         worst = max(worst, max_excess(hf_f[b], ref["hf"]), max_excess(hf_u[b], ref["hf"]))
     assert worst <= 0.0, worst
     model.close()
+
+
+def test_fused_stage_entity_pages_and_no_stray_writes(B):
+    """Entity precompute (the prefix-miss path writes the new entries' K/V straight into pool pages)
+    on a batch large enough for the fused QKV-epilogue staging: the pages match the stage-kernel
+    path within two bf16 roundings (1e-2), and an unrelated entry appended beforehand stays
+    byte-identical in both pools (no stray 16-byte stores from the epilogue's scattered writes)."""
+    from paper_conf_asplos_0017wzlxszh0w26_b200.runtime import DeviceModel, DevicePool, prefill_missing_entities
+    cfg = synth.model_config("small")
+    W = synth.Weights(cfg, seed=9)
+    model = DeviceModel(cfg, W)
+    L, Hkv, d = cfg["layers"], cfg["kv_heads"], cfg["head_dim"]
+    g = torch.Generator(device="cpu").manual_seed(4)
+    ck = torch.randn(L, 37, Hkv, d, generator=g).to(torch.bfloat16).cuda()
+    cv = torch.randn(L, 37, Hkv, d, generator=g).to(torch.bfloat16).cuda()
+    qs = [synth.make_query(13, cfg, 500 + b, 64, np.arange(20) + 1 + 20 * b, (16, 16), 8, "IP") for b in range(12)]
+    kv = {}
+    for fused in (True, False):
+        pool = DevicePool(cfg, 8192)
+        B.bat_kv_append(pool.handle, B.BAT_ENT_USER, 999999, ck, cv, 37)
+        old = os.environ.get("BAT_FUSED_STAGE")
+        os.environ["BAT_FUSED_STAGE"] = "1" if fused else "0"
+        try:
+            prefill_missing_entities(pool, model, qs)  # 240 items x 16 tokens per entity call
+            torch.cuda.synchronize()
+        finally:
+            if old is None:
+                del os.environ["BAT_FUSED_STAGE"]
+            else:
+                os.environ["BAT_FUSED_STAGE"] = old
+        ko = torch.empty(L, 37, Hkv, d, dtype=torch.bfloat16, device="cuda")
+        vo = torch.empty_like(ko)
+        B.bat_kv_read(pool.handle, B.BAT_ENT_USER, 999999, ko, vo)
+        torch.cuda.synchronize()
+        assert torch.equal(ko, ck) and torch.equal(vo, cv), f"canary entry changed (fused={fused})"
+        items = {}
+        for iid in range(1, 241):
+            k = torch.empty(L, 16, Hkv, d, dtype=torch.bfloat16, device="cuda")
+            v = torch.empty_like(k)
+            B.bat_kv_read(pool.handle, B.BAT_ENT_ITEM, iid, k, v)
+            items[iid] = (k.float().cpu().numpy(), v.float().cpu().numpy())
+        kv[fused] = items
+        pool.close()
+    worst = max(max(max_excess(kv[True][i][j], kv[False][i][j], atol=1e-2, rtol=1e-2) for j in (0, 1))
+                for i in kv[True])
+    assert worst <= 0.0, worst
+    model.close()
