@@ -907,7 +907,8 @@ __global__ void __launch_bounds__(NUM_THREADS, 1) attn_tc_kernel(const __grid_co
       }
       ptx::tc_fence_before();
       __syncwarp();
-      if (lane == 0) ptx::mbar_arrive(&bars->o_empty[wg]);
+      // relaxed: orders this warp's TMEM reads of O (waited above), not its global O stores
+      if (lane == 0) ptx::mbar_arrive_relaxed(&bars->o_empty[wg]);
       if (p.dbg_items && wg == 0 && h == 0 && sub == 0 && lane == 0) p.dbg_items[int64_t(w) * 6 + 3] = clock64();
     }
   }

@@ -276,11 +276,17 @@ struct Epilogue {
         const int col = n * BN + hh * d + c;
         const uint4* b1 = reinterpret_cast<const uint4*>(p->bias + col);
         const uint4* b2 = reinterpret_cast<const uint4*>(p->bias + col + half);
+        uint4 bv1[4], bv2[4];  // the block's bias, in flight with the TMEM loads
+#pragma unroll
+        for (int j = 0; j < 4; ++j) {
+          bv1[j] = __ldg(b1 + j);
+          bv2[j] = __ldg(b2 + j);
+        }
         ptx::tmem_ld_wait();
         uint32_t pa[16], pb[16];
 #pragma unroll
         for (int j = 0; j < 4; ++j) {  // 8 columns per bias vector
-          const uint4 v1 = __ldg(b1 + j), v2 = __ldg(b2 + j);
+          const uint4 v1 = bv1[j], v2 = bv2[j];
           const uint32_t w1[4] = {v1.x, v1.y, v1.z, v1.w}, w2[4] = {v2.x, v2.y, v2.z, v2.w};
 #pragma unroll
           for (int k = 0; k < 4; ++k) {
@@ -529,7 +535,7 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
       }
       ptx::tc_fence_before();
       __syncwarp();
-      if (lane == 0) ptx::mbar_arrive(&bars->tempty[acc]);
+      if (lane == 0) ptx::mbar_arrive_relaxed(&bars->tempty[acc]);  // orders the TMEM reads only
       if (++acc == 2) { acc = 0; acc_phase ^= 1; }
     }
     if (lane == 0) ptx::bulk_wait<0>();
@@ -669,7 +675,7 @@ gemm2_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__
       }
       ptx::tc_fence_before();
       __syncwarp();
-      if (lane == 0) ptx::mbar_arrive_cluster(ptx::mapa(ptx::smem_u32(&bars->tempty[acc]), 0));
+      if (lane == 0) ptx::mbar_arrive_cluster_relaxed(ptx::mapa(ptx::smem_u32(&bars->tempty[acc]), 0));
       if (++acc == 2) { acc = 0; acc_phase ^= 1; }
     }
     if (lane == 0) ptx::bulk_wait<0>();
