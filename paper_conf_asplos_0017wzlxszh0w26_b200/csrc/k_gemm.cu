@@ -160,7 +160,6 @@ struct Epilogue {
   // h_old of this lane's row, PD 32-column chunks ahead (the first PD issued before the
   // accumulator wait: resid_prefetch), so ~PD x 4 KB per warp are in flight against DRAM latency
   static constexpr int PD = 4;
-  static constexpr int NCHK = BN / GemmCfg<EPI>::SPLIT / 32;  // chunks of this warp's column slice
   float4 hpre[PD][8];
   __device__ __forceinline__ void load_h_chunk(int row, int col, float4 (&dst)[8]) {
     const bool ok = row < p->M && col < p->N;
@@ -170,6 +169,7 @@ struct Epilogue {
     for (int i = 0; i < 8; ++i) dst[i] = ok ? __ldcs(src + i) : make_float4(0.f, 0.f, 0.f, 0.f);
   }
   __device__ __forceinline__ void resid_prefetch(int row0, int n, int part) {
+    constexpr int NCHK = BN / GemmCfg<EPI>::SPLIT / 32;  // chunks of this warp's column slice
     const int c_lo = part * (BN / GemmCfg<EPI>::SPLIT);
 #pragma unroll
     for (int k = 0; k < PD && k < NCHK; ++k) load_h_chunk(row0 + int(lane), n * BN + c_lo + 32 * k, hpre[k]);
@@ -178,6 +178,7 @@ struct Epilogue {
     const int row = row0 + int(lane);
     const bool ok = row < p->M;
     const int col_base = n * BN;
+    constexpr int NCHK = BN / GemmCfg<EPI>::SPLIT / 32;
     float ss = 0.0f;
 #pragma unroll
     for (int k = 0; k < NCHK; ++k) {
