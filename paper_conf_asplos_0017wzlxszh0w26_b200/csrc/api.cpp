@@ -406,6 +406,7 @@ static StageParams stage_params(const Pool& pool, const Model& m, const Plan& pl
   sp.scratch_layer_off = 0;
   sp.head_bytes = pool.geo.head_bytes;
   sp.n_req = static_cast<int32_t>(plan.q.size());
+  sp.off_rowreq = im.off_rowreq;
   return sp;
 }
 

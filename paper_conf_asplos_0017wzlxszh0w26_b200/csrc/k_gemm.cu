@@ -116,6 +116,7 @@ struct Epilogue {
   uint8_t* stg;  // this warp's 2 staging buffers
   uint32_t lane;
   int sbuf = 0;
+  uint32_t sbias = 0;  // fused a4: shared-memory copy of the QKV bias (0: read it from global)
 
   __device__ __forceinline__ void stage_row(uint8_t* buf, int chunk16, uint32_t a, uint32_t b, uint32_t c, uint32_t d) {
     ptx::st_shared_v4(buf + lane * 128 + ((chunk16 ^ (lane & 7)) << 4), a, b, c, d);
@@ -233,13 +234,7 @@ struct Epilogue {
     r.ok = row_in < p->M;
     const int row = r.ok ? row_in : p->M - 1;  // lanes past the batch: same loads, no stores
     const int32_t* img = sp.img;
-    int lo = 0, hi = sp.n_req - 1;  // the last request with token_off <= row
-    while (lo < hi) {
-      const int mid = (lo + hi + 1) >> 1;
-      if (__ldg(img + sp.off_qinfo + int64_t(mid) * 8) <= row) lo = mid;
-      else hi = mid - 1;
-    }
-    const int32_t* qi = img + sp.off_qinfo + int64_t(lo) * 8;
+    const int32_t* qi = img + sp.off_qinfo + int64_t(__ldg(img + sp.off_rowreq + row)) * 8;  // the row's request
     r.t = row - __ldg(qi);
     r.pos = min(__ldg(img + sp.off_pos + row), sp.max_pos - 1);
     r.gq = __ldg(qi + 2) + r.t / sp.qt;
@@ -280,8 +275,8 @@ struct Epilogue {
         uint4 bv1[4], bv2[4];  // the block's bias, in flight with the TMEM loads
 #pragma unroll
         for (int j = 0; j < 4; ++j) {
-          bv1[j] = __ldg(b1 + j);
-          bv2[j] = __ldg(b2 + j);
+          bv1[j] = sbias ? ptx::ld_shared_v4(sbias + uint32_t(col) * 2 + 16 * j) : __ldg(b1 + j);
+          bv2[j] = sbias ? ptx::ld_shared_v4(sbias + uint32_t(col + half) * 2 + 16 * j) : __ldg(b2 + j);
         }
         ptx::tmem_ld_wait();
         uint32_t pa[16], pb[16];
@@ -508,6 +503,17 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
     const uint32_t sub = warp & 3;  // TMEM sub-partition this warp may access
     const int part = int(warp - 2) / 4;  // column slice
     Epilogue<EPI> epi{&tmC, &p, smem + STG1_OFF + (warp - 2) * C::NB * STG_BYTES, lane};
+    if constexpr (EPI == EPI_BF16_BIAS) {
+      // fused a4: the bias lives in the staging region (the a4 path stores directly, not via TMA)
+      if (p.stage_on && p.N * 2 <= C::STG) {
+        const int t = int(threadIdx.x) - 64;  // epilogue threads 0 .. 32 * EPI_WARPS - 1
+        uint32_t* dst = reinterpret_cast<uint32_t*>(smem + STG1_OFF);
+        const uint32_t* src = reinterpret_cast<const uint32_t*>(p.bias);
+        for (int i = t; i < p.N / 2; i += 32 * EPI_WARPS) dst[i] = __ldg(src + i);
+        ptx::bar_sync(1, 32 * EPI_WARPS);
+        epi.sbias = ptx::smem_u32(smem + STG1_OFF);
+      }
+    }
     int acc = 0;
     uint32_t acc_phase = 0;
     for (int t = blockIdx.x; t < num_work; t += gridDim.x) {
@@ -648,6 +654,17 @@ gemm2_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__
     const uint32_t sub = warp & 3;
     const int part = int(warp - 2) / 4;  // column slice
     Epilogue<EPI> epi{&tmC, &p, smem + STG2_OFF + (warp - 2) * C::NB * STG_BYTES, lane};
+    if constexpr (EPI == EPI_BF16_BIAS) {
+      // fused a4: the bias lives in the staging region (the a4 path stores directly, not via TMA)
+      if (p.stage_on && p.N * 2 <= C::STG) {
+        const int t = int(threadIdx.x) - 64;  // epilogue threads 0 .. 32 * EPI_WARPS - 1
+        uint32_t* dst = reinterpret_cast<uint32_t*>(smem + STG2_OFF);
+        const uint32_t* src = reinterpret_cast<const uint32_t*>(p.bias);
+        for (int i = t; i < p.N / 2; i += 32 * EPI_WARPS) dst[i] = __ldg(src + i);
+        ptx::bar_sync(1, 32 * EPI_WARPS);
+        epi.sbias = ptx::smem_u32(smem + STG2_OFF);
+      }
+    }
     int acc = 0;
     uint32_t acc_phase = 0;
     for (int t = pair; t < num_work; t += n_pairs) {

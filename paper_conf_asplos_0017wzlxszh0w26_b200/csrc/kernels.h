@@ -37,6 +37,7 @@ struct StageParams {
   int64_t scratch_page_bytes, scratch_layer_off;
   int64_t head_bytes;
   int32_t n_req;             // requests of the plan (q_info rows)
+  int64_t off_rowreq;        // [M] request of every suffix row (the fused QKV epilogue's lookup)
 };
 
 // ------------------------------------------------------------------------ tcgen05 GEMM

@@ -340,6 +340,7 @@ void build_plan(const Pool& pool, int32_t group, int32_t kv_heads,
   im.off_tok = reserve_at(plan.M);
   im.off_pos = reserve_at(plan.M);
   im.off_rseg = reserve_at(plan.M);
+  im.off_rowreq = reserve_at(plan.M);
   im.off_qinfo = reserve_at(int64_t(B) * 8);
   im.off_pages = reserve_at(plan.n_pages_padded);
   im.off_kmeta = reserve_at(int64_t(plan.n_pages_padded) * kPageTokens * 2);
@@ -352,6 +353,7 @@ void build_plan(const Pool& pool, int32_t group, int32_t kv_heads,
       v[im.off_tok + qp.token_off + t] = qp.tokens[t];
       v[im.off_pos + qp.token_off + t] = qp.pos[t];
       v[im.off_rseg + qp.token_off + t] = qp.seg[t];
+      v[im.off_rowreq + qp.token_off + t] = b;
     }
     int32_t* qi = &v[im.off_qinfo + int64_t(b) * 8];
     qi[0] = qp.token_off; qi[1] = qp.S; qi[2] = qp.qtile0; qi[3] = qp.n_qtiles;

@@ -42,6 +42,7 @@ struct PlanRequest {
 struct PlanImage {
   std::vector<int32_t> buf;
   int64_t off_tok = 0, off_pos = 0, off_rseg = 0;   // [M]
+  int64_t off_rowreq = 0;                           // [M] request index of every suffix row
   int64_t off_qinfo = 0;                            // [B][8]
   int64_t off_pages = 0;                            // [n_pages_padded_total]
   int64_t off_kmeta = 0;                            // [16 * n_pages_padded_total][2]
