@@ -39,7 +39,7 @@ constexpr int A_BYTES = 128 * BK * 2;           // 16 KB: 128 rows of A per CTA
 // profiles/r1_gemm_raster.txt); BAT_GEMM_GROUP_M / _SWIGLU override
 constexpr int GROUP_M = 1;
 constexpr int GROUP_M_SWIGLU = 32;       // 1-CTA SwiGLU kernel (128-row M-tiles)
-constexpr int GROUP_M_SWIGLU_PAIR = 16;  // CTA-pair SwiGLU kernel (256-row M-tiles; 4: 1% slower)
+constexpr int GROUP_M_SWIGLU_PAIR = 32;  // CTA-pair SwiGLU kernel (256-row M-tiles; profiles/r2_gemm_epilogue.txt (k))
 // Epilogue warps per CTA: 4 (one per TMEM lane quarter) or 8 (two per quarter, splitting the
 // accumulator's columns).  The SwiGLU GEMM (short K = hidden, MUFU-heavy epilogue) runs 8 and
 // gains 5% over 4; the others keep 4 warps and one more ring stage (their K loops are long or
@@ -737,8 +737,8 @@ void launch_gemm(int epi, const CUtensorMap& tmA, const CUtensorMap& tmB, const 
   if (!p.hints) p.hints = hints;
   // SwiGLU on CTA pairs by default (BAT_GEMM_SWIGLU_PAIR=0: 1-CTA 128-row tiles): 8 epilogue warps
   // and MUFU ex2 / rcp silu, 1,202 -> 1,375-1,389 TFLOP/s in the configs[2] step against the 1-CTA
-  // kernel with the same epilogue (profiles/r2_gemm_epilogue.txt); rasterisation groups of 16 pair
-  // M-tiles (4,096 rows) or 32 1-CTA M-tiles, evict_last weight loads (the 55 MB of gate/up
+  // kernel with the same epilogue (profiles/r2_gemm_epilogue.txt); rasterisation groups of 32 pair
+  // M-tiles (8,192 rows) or 32 1-CTA M-tiles, evict_last weight loads (the 55 MB of gate/up
   // weights are re-streamed once per group; profiles/r1_gemm_raster.txt)
   static const char* sp_env = std::getenv("BAT_GEMM_SWIGLU_PAIR");
   static const bool swiglu_pair = !(sp_env && sp_env[0] == '0');
