@@ -290,9 +290,11 @@ BAT_API bat_status bat_plan_export(bat_plan plan, int32_t b, int32_t field, int3
  *   BAT_PFD_KPAGES    int32 [n_ktiles*8]: page id each k-tile's loader copies (pool page >= 0,
  *                     -(s+1) suffix scratch page s, INT32_MIN the all-zero pad page), or
  *                     BAT_PFD_NOT_LOADED for a tile no work item lists (skipped)
+ *   BAT_PFD_STAGE     int32 [S][3]: where the fused QKV epilogue (a4) stores suffix row t, from the
+ *                     device row map: {global q-tile, suffix page id (as KPAGES), slot in the page}
  * BAT_E_STATE if the device image is inconsistent: KV heads with different lists, a (q-tile,
  * k-tile) pair listed twice, a partial tile without a mask, out-of-range indices. */
-enum { BAT_PFD_VIS = 0, BAT_PFD_VIS_LAST = 1, BAT_PFD_KPAGES = 2 };
+enum { BAT_PFD_VIS = 0, BAT_PFD_VIS_LAST = 1, BAT_PFD_KPAGES = 2, BAT_PFD_STAGE = 3 };
 #define BAT_PFD_NOT_LOADED (-2147483647)
 BAT_API bat_status bat_plan_export_device(bat_plan plan, int32_t b, int32_t field, void* out, int64_t cap,
                                           int64_t* count);

@@ -374,16 +374,16 @@ def bat_plan_export(plan: int, b: int, field: int) -> np.ndarray:
     return out[: n.value]
 
 
-BAT_PFD_VIS, BAT_PFD_VIS_LAST, BAT_PFD_KPAGES = range(3)
+BAT_PFD_VIS, BAT_PFD_VIS_LAST, BAT_PFD_KPAGES, BAT_PFD_STAGE = range(4)
 BAT_PFD_NOT_LOADED = -2147483647
 
 
 def bat_plan_export_device(plan: int, b: int, field: int) -> np.ndarray:
     """The device image of a bat_plan_build plan decoded as the attention kernel reads it:
-    VIS / VIS_LAST uint8 [S][n_ktiles*128]; KPAGES int32 [n_ktiles*8]."""
+    VIS / VIS_LAST uint8 [S][n_ktiles*128]; KPAGES int32 [n_ktiles*8]; STAGE int32 [S][3]."""
     n = c_int64()
     _check(lib().bat_plan_export_device(plan, b, field, None, 0, byref(n)))
-    out = np.zeros(max(n.value, 1), dtype=np.int32 if field == BAT_PFD_KPAGES else np.uint8)
+    out = np.zeros(max(n.value, 1), dtype=np.int32 if field in (BAT_PFD_KPAGES, BAT_PFD_STAGE) else np.uint8)
     _check(lib().bat_plan_export_device(plan, b, field, out.ctypes.data_as(c_void_p), len(out), byref(n)))
     return out[: n.value]
 

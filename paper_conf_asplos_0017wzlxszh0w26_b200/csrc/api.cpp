@@ -1163,7 +1163,7 @@ bat_status bat_plan_export_device(bat_plan plan, int32_t b, int32_t field, void*
     BAT_REQUIRE(plan && plan->dev_img, "plan built with bat_plan_build");
     const Plan& pl = plan->plan;
     BAT_REQUIRE(b >= 0 && b < int32_t(pl.q.size()), "request index");
-    BAT_REQUIRE(field >= BAT_PFD_VIS && field <= BAT_PFD_KPAGES, "field");
+    BAT_REQUIRE(field >= BAT_PFD_VIS && field <= BAT_PFD_STAGE, "field");
     const PlanImage& im = pl.img;
     if (plan->dev_copy.empty()) {
       DeviceGuard dg(plan->device);
@@ -1172,6 +1172,28 @@ bat_status bat_plan_export_device(bat_plan plan, int32_t b, int32_t field, void*
     }
     const std::vector<int32_t>& I = plan->dev_copy;
     const QueryPlan& q = pl.q[b];
+    if (field == BAT_PFD_STAGE) {
+      // the fused QKV epilogue's per-row lookups (k_gemm.cu Epilogue::stage_row), decoded from the
+      // device image: row -> request (row map) -> q_info -> q-tile, suffix page (spages), slot
+      std::vector<int32_t> st(size_t(q.S) * 3);
+      const int32_t tok_off = I[size_t(im.off_qinfo + int64_t(b) * 8)];
+      for (int32_t t = 0; t < q.S; ++t) {
+        const int64_t row = int64_t(tok_off) + t;
+        const int32_t rb = I[size_t(im.off_rowreq + row)];
+        if (rb != b) fail(BAT_E_STATE, "row map names another request");
+        const int32_t* qi = &I[size_t(im.off_qinfo + int64_t(rb) * 8)];
+        const int32_t tt = int32_t(row - qi[0]);
+        st[size_t(t) * 3 + 0] = qi[2] + tt / pl.qt;
+        st[size_t(t) * 3 + 1] = I[size_t(im.off_spages + int64_t(qi[6] + tt / kPageTokens) * 4 + 3)];
+        st[size_t(t) * 3 + 2] = tt % kPageTokens;
+      }
+      if (count) *count = int64_t(st.size());
+      if (out) {
+        BAT_REQUIRE(cap >= int64_t(st.size()), "cap too small");
+        std::copy(st.begin(), st.end(), static_cast<int32_t*>(out));
+      }
+      return;
+    }
     const int64_t n_cols = int64_t(q.n_ktiles) * kKtile;
     const bool last = field == BAT_PFD_VIS_LAST;
     const int64_t off_work = last ? im.off_work_last : im.off_work;

@@ -13,7 +13,9 @@ Asserted for every request of the batch:
   * KPAGES: a k-tile is loaded iff some q-tile of the request has a visible pair in it (exact
     block-skip), with the oracle's page ids (prefix pages from the pool index, suffix scratch
     pages, the all-zero page as 8-page padding);
-  * every KV head sees the same lists (checked inside the export: BAT_E_STATE otherwise).
+  * every KV head sees the same lists (checked inside the export: BAT_E_STATE otherwise);
+  * STAGE: the destinations the fused QKV epilogue (a4) derives for every suffix row from the
+    device row map — global q-tile, suffix page, slot — equal the oracle's.
 Batches: configs[1] exactly as bench.py builds it (64 IP requests, |U| = 512, 100 Zipf items),
 configs[2] (64 requests, 200 items, lognormal |U|, larger-side rule -> mixed UP/IP), and small
 mixed batches with RE requests, headers, ragged multi-page items, GQA groups 6 / 7 and d = 64."""
@@ -80,10 +82,17 @@ def _check_batch(B, cfg, queries, n_pages):
     n_listed = n_partial_rows = 0
     try:
         sp = 0
+        qtile0 = 0
         for b, q in enumerate(queries):
             ref = oplan.plan_query(q, ep, group, sp)
             sp += (ref["S"] + 15) // 16
             S, qt = ref["S"], oplan.qtile_tokens(group)
+            # the fused QKV epilogue's per-row destinations (row map -> q-tile, suffix page, slot)
+            t = np.arange(S)
+            want_st = np.stack([qtile0 + t // qt, ref["pages"][ref["n_prefix_pages"] + t // 16], t % 16], axis=1)
+            got_st = B.bat_plan_export_device(plan, b, B.BAT_PFD_STAGE).reshape(S, 3)
+            assert np.array_equal(got_st, want_st), (b, "a4 destinations", np.argwhere(got_st != want_st)[:5])
+            qtile0 += (S + qt - 1) // qt
             n_kt = ref["tile_state"].shape[1]
             want = np.zeros((S, n_kt * 128), np.uint8)
             want[:, : ref["vis"].shape[1]] = ref["vis"]
